@@ -1,0 +1,236 @@
+"""Python front-end of the CPU fp64 oracle (oracle.c).
+
+TEST INFRASTRUCTURE ONLY: imported by tests/, __graft_entry__.smoke() and
+bench.py's cpu_baseline / --impl reference leg, never by the product package.
+It shares no code with the CUDA path; it only reads the synthetic inputs of
+paper_conf_ipps_acharyas25_b200.synth (a generator with no method arithmetic).
+
+All arithmetic happens in oracle.c; this module marshals numpy arrays.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+from concurrent.futures import ThreadPoolExecutor
+from typing import Dict, List, Optional, Sequence
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+SRC = os.path.join(HERE, "oracle.c")
+LIB = os.path.join(HERE, "liboracle.so")
+
+OK, RANGE, SELF_LOOP, CYCLE = 0, -2, -3, -4
+F = 80
+FEAT_DTYPE = np.dtype([("op", "<u2"), ("dtype", "u1"), ("kind", "u1"), ("dims", "<u4", (4,))])
+
+_lock = threading.Lock()
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c with gcc (-ffp-contract=off: no FMA contraction)."""
+    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < max(
+            os.path.getmtime(SRC), os.path.getmtime(os.path.join(HERE, "oracle.h"))):
+        tmp = LIB + ".tmp%d" % os.getpid()
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC",
+                               "-shared", "-Wall", "-o", tmp, SRC, "-lm"])
+        os.replace(tmp, LIB)
+    return LIB
+
+
+class _Cfg(ctypes.Structure):
+    _fields_ = [("L", ctypes.c_int), ("d", ctypes.c_int), ("H", ctypes.c_int),
+                ("d_ff", ctypes.c_int), ("pool", ctypes.c_int), ("ln_eps", ctypes.c_double)]
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            build()
+            L = ctypes.CDLL(LIB)
+            P = ctypes.c_void_p
+            i32, i64, dbl = ctypes.c_int, ctypes.c_int64, ctypes.c_double
+            L.orc_validate.argtypes = [i32, i32, P, P]
+            L.orc_validate.restype = i32
+            L.orc_depth.argtypes = [i32, i32, P, P, P]
+            L.orc_row_words.argtypes = [i32]
+            L.orc_row_words.restype = i32
+            L.orc_reach.argtypes = [i32, i32, P, P, P]
+            L.orc_mask.argtypes = [i32, P, P]
+            L.orc_tiles.argtypes = [i32, P, P]
+            L.orc_tiles.restype = i64
+            L.orc_blob_floats.argtypes = [P]
+            L.orc_blob_floats.restype = ctypes.c_long
+            L.orc_features.argtypes = [i32, P, P]
+            L.orc_embed.argtypes = [P, P, i32, P, P, P]
+            L.orc_attention.argtypes = [P, P, i32, i32, P, P, P]
+            L.orc_layer.argtypes = [P, P, i32, i32, P, P, P]
+            L.orc_readout.argtypes = [P, P, i32, P]
+            L.orc_readout.restype = dbl
+            L.orc_forward.argtypes = [P, P, i32, i32, P, P, P, P, P]
+            L.orc_forward.restype = i32
+            L.orc_plan_T.argtypes = [i64, P, P, P, P, i64, P]
+            L.orc_argmin.argtypes = [i64, P]
+            L.orc_argmin.restype = i64
+            _lib = L
+    return _lib
+
+
+def _p(a: Optional[np.ndarray]):
+    return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _i32(a) -> np.ndarray:
+    return np.ascontiguousarray(a, dtype=np.int32)
+
+
+def _feats(f) -> np.ndarray:
+    return np.ascontiguousarray(f, dtype=FEAT_DTYPE)
+
+
+def cfg(model_cfg: dict) -> _Cfg:
+    return _Cfg(model_cfg["num_layers"], model_cfg["d_model"], model_cfg["num_heads"],
+                model_cfg["d_ff"], model_cfg.get("pool", 0), float(model_cfg.get("ln_eps", 1e-5)))
+
+
+# ---- graph steps -----------------------------------------------------------
+def validate(n, src, dst) -> int:
+    s, d = _i32(src), _i32(dst)
+    return lib().orc_validate(n, len(s), _p(s), _p(d))
+
+
+def depth(n, src, dst) -> np.ndarray:
+    s, d = _i32(src), _i32(dst)
+    out = np.zeros(n, np.int32)
+    lib().orc_depth(n, len(s), _p(s), _p(d), _p(out))
+    return out
+
+
+def row_words(n: int) -> int:
+    return 2 * ((n + 127) // 128)
+
+
+def reach(n, src, dst) -> np.ndarray:
+    """Closure bitsets [n, W] uint64 (layout of include/predtop.h)."""
+    s, d = _i32(src), _i32(dst)
+    out = np.zeros((n, row_words(n)), np.uint64)
+    lib().orc_reach(n, len(s), _p(s), _p(d), _p(out))
+    return out
+
+
+def mask(n, R: np.ndarray) -> np.ndarray:
+    R = np.ascontiguousarray(R, np.uint64)
+    out = np.zeros_like(R)
+    lib().orc_mask(n, _p(R), _p(out))
+    return out
+
+
+def tiles(n, M: np.ndarray):
+    M = np.ascontiguousarray(M, np.uint64)
+    T = (n + 127) // 128
+    cls = np.zeros(T * T, np.uint8)
+    pairs = lib().orc_tiles(n, _p(M), _p(cls))
+    return cls, int(pairs)
+
+
+def bits_to_dense(B: np.ndarray, n: int) -> np.ndarray:
+    """[n, W] uint64 bitset rows -> dense bool [n, n] (bit u%64 of word u/64)."""
+    by = np.ascontiguousarray(B).view(np.uint8).reshape(B.shape[0], -1)
+    return np.unpackbits(by, axis=1, bitorder="little")[:, :n].astype(bool)
+
+
+# ---- model steps -----------------------------------------------------------
+def blob_floats(model_cfg) -> int:
+    c = cfg(model_cfg)
+    return lib().orc_blob_floats(ctypes.byref(c))
+
+
+def features(n, feats) -> np.ndarray:
+    f = _feats(feats)
+    out = np.zeros((n, F), np.float64)
+    lib().orc_features(n, _p(f), _p(out))
+    return out
+
+
+def embed(model_cfg, blob, n, feats, dep) -> np.ndarray:
+    c = cfg(model_cfg)
+    b = np.ascontiguousarray(blob, np.float32)
+    out = np.zeros((n, model_cfg["d_model"]), np.float64)
+    lib().orc_embed(ctypes.byref(c), _p(b), n, _p(_feats(feats)), _p(_i32(dep)), _p(out))
+    return out
+
+
+def attention(model_cfg, blob, layer, n, M, x) -> np.ndarray:
+    c = cfg(model_cfg)
+    b = np.ascontiguousarray(blob, np.float32)
+    x = np.ascontiguousarray(x, np.float64)
+    out = np.zeros((n, model_cfg["d_model"]), np.float64)
+    lib().orc_attention(ctypes.byref(c), _p(b), layer, n, _p(np.ascontiguousarray(M, np.uint64)),
+                        _p(x), _p(out))
+    return out
+
+
+def layer(model_cfg, blob, li, n, M, x) -> np.ndarray:
+    c = cfg(model_cfg)
+    b = np.ascontiguousarray(blob, np.float32)
+    x = np.ascontiguousarray(x, np.float64)
+    out = np.zeros_like(x)
+    lib().orc_layer(ctypes.byref(c), _p(b), li, n, _p(np.ascontiguousarray(M, np.uint64)),
+                    _p(x), _p(out))
+    return out
+
+
+def readout(model_cfg, blob, n, x) -> float:
+    c = cfg(model_cfg)
+    b = np.ascontiguousarray(blob, np.float32)
+    return float(lib().orc_readout(ctypes.byref(c), _p(b), n, _p(np.ascontiguousarray(x, np.float64))))
+
+
+def forward(model_cfg, blob, n, src, dst, feats, taps: bool = False):
+    """One stage graph -> (status, latency, taps or None)."""
+    c = cfg(model_cfg)
+    b = np.ascontiguousarray(blob, np.float32)
+    s, d = _i32(src), _i32(dst)
+    y = np.zeros(1, np.float64)
+    t = np.zeros((model_cfg["num_layers"] + 1, n, model_cfg["d_model"]), np.float64) if taps else None
+    st = lib().orc_forward(ctypes.byref(c), _p(b), n, len(s), _p(s), _p(d), _p(_feats(feats)),
+                           _p(y), _p(t))
+    return st, float(y[0]), t
+
+
+def forward_batch(model_cfg, blob, batch, graphs: Optional[Sequence[int]] = None,
+                  threads: Optional[int] = None) -> np.ndarray:
+    """Latency of every graph (or the listed ones) of a synth.StageBatch, one
+    graph per worker thread (ctypes releases the GIL)."""
+    gs = list(range(batch.num_graphs)) if graphs is None else list(graphs)
+    threads = threads or (os.cpu_count() or 1)
+    lib()
+
+    def one(g):
+        n, s, d, f = batch.graph(g)
+        return forward(model_cfg, blob, n, s, d, f)[1]
+
+    if threads <= 1 or len(gs) <= 1:
+        return np.asarray([one(g) for g in gs], np.float64)
+    with ThreadPoolExecutor(threads) as ex:
+        return np.asarray(list(ex.map(one, gs)), np.float64)
+
+
+# ---- pipeline formula ------------------------------------------------------
+def plan_T(plan_ptr, plan_stage, microbatches, stage_latency) -> np.ndarray:
+    pp = np.ascontiguousarray(plan_ptr, np.int64)
+    ps = np.ascontiguousarray(plan_stage, np.int32)
+    B = np.ascontiguousarray(microbatches, np.int32)
+    t = np.ascontiguousarray(stage_latency, np.float32)
+    T = np.zeros(len(pp) - 1, np.float64)
+    lib().orc_plan_T(len(pp) - 1, _p(pp), _p(ps), _p(B), _p(t), len(t), _p(T))
+    return T
+
+
+def argmin(T) -> int:
+    T = np.ascontiguousarray(T, np.float64)
+    return int(lib().orc_argmin(len(T), _p(T)))

@@ -1,0 +1,450 @@
+/*
+ * oracle.c -- plain CPU fp64 oracle of the PredTOP prediction path.
+ * TEST INFRASTRUCTURE ONLY (see oracle.h).  Slow and obviously correct:
+ * one graph at a time, textbook loops, no blocking, fusion or reordering.
+ * Compile with -ffp-contract=off (no FMA contraction; Eqn 4 rounding rule R13).
+ */
+#include "oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ------------------------------------------------------------------------ */
+/* Graph checks ("DL models are often represented as DAGs"; the stage  */
+/* graph of SIV-B2).  Precedence: RANGE, then SELF_LOOP, then CYCLE.   */
+/* Cycle test: iterative DFS with white/grey/black colouring.                 */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  int* off; /* n+1 */
+  int* adj; /* e   */
+} orc_csr;
+
+static orc_csr build_csr(int n, int e, const int32_t* from, const int32_t* to) {
+  orc_csr g;
+  g.off = (int*)calloc((size_t)n + 1, sizeof(int));
+  g.adj = (int*)malloc(sizeof(int) * (size_t)(e > 0 ? e : 1));
+  for (int i = 0; i < e; ++i) g.off[from[i] + 1]++;
+  for (int v = 0; v < n; ++v) g.off[v + 1] += g.off[v];
+  int* fill = (int*)malloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+  for (int v = 0; v < n; ++v) fill[v] = g.off[v];
+  for (int i = 0; i < e; ++i) g.adj[fill[from[i]]++] = to[i];
+  free(fill);
+  return g;
+}
+static void free_csr(orc_csr* g) { free(g->off); free(g->adj); }
+
+int orc_validate(int n, int e, const int32_t* src, const int32_t* dst) {
+  for (int i = 0; i < e; ++i)
+    if (src[i] < 0 || src[i] >= n || dst[i] < 0 || dst[i] >= n) return ORC_RANGE;
+  for (int i = 0; i < e; ++i)
+    if (src[i] == dst[i]) return ORC_SELF_LOOP;
+  orc_csr succ = build_csr(n, e, src, dst);
+  char* colour = (char*)calloc((size_t)n + 1, 1); /* 0 white, 1 grey, 2 black */
+  int* stack = (int*)malloc(sizeof(int) * ((size_t)n + 1));
+  int* next = (int*)malloc(sizeof(int) * ((size_t)n + 1)); /* next successor index */
+  int status = ORC_OK;
+  for (int r = 0; r < n && status == ORC_OK; ++r) {
+    if (colour[r]) continue;
+    int sp = 0;
+    stack[sp++] = r;
+    colour[r] = 1;
+    next[r] = succ.off[r];
+    while (sp > 0 && status == ORC_OK) {
+      int v = stack[sp - 1];
+      if (next[v] < succ.off[v + 1]) {
+        int w = succ.adj[next[v]++];
+        if (colour[w] == 1) status = ORC_CYCLE;   /* back edge */
+        else if (colour[w] == 0) {
+          colour[w] = 1;
+          next[w] = succ.off[w];
+          stack[sp++] = w;
+        }
+      } else {
+        colour[v] = 2;
+        --sp;
+      }
+    }
+  }
+  free(colour); free(stack); free(next); free_csr(&succ);
+  return status;
+}
+
+/* ------------------------------------------------------------------------ */
+/* DAGPE depth ("using the depth of the nodes as the positional        */
+/* encoding"; reading R4): depth(v) = 0 if v has no predecessor, otherwise    */
+/* 1 + max_{p in pred(v)} depth(p).  Memoised recursion over predecessors,   */
+/* written with an explicit stack.  Requires an acyclic graph.               */
+/* ------------------------------------------------------------------------ */
+void orc_depth(int n, int e, const int32_t* src, const int32_t* dst, int32_t* depth) {
+  orc_csr pred = build_csr(n, e, dst, src);
+  int* stack = (int*)malloc(sizeof(int) * ((size_t)n + (size_t)e + 1));
+  for (int v = 0; v < n; ++v) depth[v] = -1;
+  for (int r = 0; r < n; ++r) {
+    if (depth[r] >= 0) continue;
+    int sp = 0;
+    stack[sp++] = r;
+    while (sp > 0) {
+      int v = stack[sp - 1];
+      int ready = 1;
+      for (int i = pred.off[v]; i < pred.off[v + 1]; ++i) {
+        int p = pred.adj[i];
+        if (depth[p] < 0) { stack[sp++] = p; ready = 0; }
+      }
+      if (!ready) continue;
+      int best = -1; /* max over predecessors; -1 + 1 = 0 for a source */
+      for (int i = pred.off[v]; i < pred.off[v + 1]; ++i)
+        if (depth[pred.adj[i]] > best) best = depth[pred.adj[i]];
+      depth[v] = best + 1;
+      --sp;
+    }
+  }
+  free(stack); free_csr(&pred);
+}
+
+/* ------------------------------------------------------------------------ */
+/* DAGRA reachability ("a node n will attend to another node m if and  */
+/* only if there exists a path from m to n or vice versa"; P:145 k = inf).   */
+/* R[v] = { u != v : v reaches u by a directed path of >= 1 edge }, one      */
+/* iterative DFS along successors per v.  Layout (include/predtop.h): row v  */
+/* is W = 2*ceil(n/128) uint64 words, bit u%64 of word u/64; padding 0.      */
+/* ------------------------------------------------------------------------ */
+int orc_row_words(int n) { return 2 * ((n + 127) / 128); }
+
+void orc_reach(int n, int e, const int32_t* src, const int32_t* dst, uint64_t* R) {
+  int W = orc_row_words(n);
+  memset(R, 0, sizeof(uint64_t) * (size_t)n * (size_t)W);
+  orc_csr succ = build_csr(n, e, src, dst);
+  char* seen = (char*)malloc((size_t)n + 1);
+  int* stack = (int*)malloc(sizeof(int) * ((size_t)e + (size_t)n + 1));
+  for (int v = 0; v < n; ++v) {
+    memset(seen, 0, (size_t)n);
+    int sp = 0;
+    for (int i = succ.off[v]; i < succ.off[v + 1]; ++i) stack[sp++] = succ.adj[i];
+    while (sp > 0) {
+      int u = stack[--sp];
+      if (seen[u]) continue;
+      seen[u] = 1;
+      for (int i = succ.off[u]; i < succ.off[u + 1]; ++i)
+        if (!seen[succ.adj[i]]) stack[sp++] = succ.adj[i];
+    }
+    for (int u = 0; u < n; ++u)
+      if (seen[u] && u != v) R[(size_t)v * W + (size_t)(u / 64)] |= (uint64_t)1 << (u % 64);
+  }
+  free(seen); free(stack); free_csr(&succ);
+}
+
+static int bit(const uint64_t* B, int W, int row, int col) {
+  return (int)((B[(size_t)row * W + (size_t)(col / 64)] >> (col % 64)) & 1u);
+}
+
+/* Eqn 1 mask: M(u,v) = 0 (allowed) iff u in N_inf(v).  With     */
+/* P:135 "or vice versa" the relation is symmetric (R3), and a node attends  */
+/* to itself (R2): allowed(u,v) = [u == v] or R[u][v] or R[v][u].            */
+void orc_mask(int n, const uint64_t* R, uint64_t* M) {
+  int W = orc_row_words(n);
+  memset(M, 0, sizeof(uint64_t) * (size_t)n * (size_t)W);
+  for (int u = 0; u < n; ++u)
+    for (int v = 0; v < n; ++v)
+      if (u == v || bit(R, W, u, v) || bit(R, W, v, u))
+        M[(size_t)u * W + (size_t)(v / 64)] |= (uint64_t)1 << (v % 64);
+}
+
+/* Block classes of M over 128x128 tiles (clipped to n): 0 no allowed pair,   */
+/* 2 all allowed, 1 otherwise.  Returns |A| = number of allowed pairs.       */
+int64_t orc_tiles(int n, const uint64_t* M, uint8_t* cls) {
+  int W = orc_row_words(n);
+  int T = (n + 127) / 128;
+  int64_t total = 0;
+  for (int qt = 0; qt < T; ++qt)
+    for (int kt = 0; kt < T; ++kt) {
+      int64_t cnt = 0, cells = 0;
+      for (int u = qt * 128; u < n && u < qt * 128 + 128; ++u)
+        for (int v = kt * 128; v < n && v < kt * 128 + 128; ++v) {
+          cells++;
+          cnt += bit(M, W, u, v);
+        }
+      if (cls) cls[qt * T + kt] = (uint8_t)(cnt == 0 ? 0 : (cnt == cells ? 2 : 1));
+      total += cnt;
+    }
+  return total;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Weight blob walk (order documented in include/predtop.h).                 */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  const float *W_in, *b_in;
+  const float *H1, *c1, *H2, *c2, *w_o, *c_o;
+} orc_top;
+typedef struct {
+  const float *Wqkv, *bqkv, *Wo, *bo, *g1, *be1, *W1, *b1, *W2, *b2, *g2, *be2;
+} orc_lw;
+
+static long layer_floats(const orc_cfg* c) {
+  long d = c->d, f = c->d_ff;
+  return 3 * d * d + 3 * d + d * d + d + 2 * d + f * d + f + d * f + d + 2 * d;
+}
+
+long orc_blob_floats(const orc_cfg* c) {
+  long d = c->d;
+  return d * ORC_F + d + (long)c->L * layer_floats(c) + 2 * (d * d + d) + d + 1;
+}
+
+static orc_lw layer_weights(const orc_cfg* c, const float* blob, int l) {
+  long d = c->d, f = c->d_ff;
+  const float* p = blob + d * ORC_F + d + (long)l * layer_floats(c);
+  orc_lw w;
+  w.Wqkv = p; p += 3 * d * d;
+  w.bqkv = p; p += 3 * d;
+  w.Wo = p; p += d * d;
+  w.bo = p; p += d;
+  w.g1 = p; p += d;
+  w.be1 = p; p += d;
+  w.W1 = p; p += f * d;
+  w.b1 = p; p += f;
+  w.W2 = p; p += d * f;
+  w.b2 = p; p += d;
+  w.g2 = p; p += d;
+  w.be2 = p;
+  return w;
+}
+
+static orc_top top_weights(const orc_cfg* c, const float* blob) {
+  long d = c->d;
+  orc_top t;
+  t.W_in = blob;
+  t.b_in = blob + d * ORC_F;
+  const float* p = blob + d * ORC_F + d + (long)c->L * layer_floats(c);
+  t.H1 = p; p += d * d;
+  t.c1 = p; p += d;
+  t.H2 = p; p += d * d;
+  t.c2 = p; p += d;
+  t.w_o = p; p += d;
+  t.c_o = p;
+  return t;
+}
+
+/* y[r][o] = b[o] + sum_i W[o][i] x[r][i]   (PyTorch Linear, W is [out][in]) */
+static void linear(int rows, int in, int out, const double* x, const float* W, const float* b,
+                   double* y) {
+  for (int r = 0; r < rows; ++r)
+    for (int o = 0; o < out; ++o) {
+      double s = b ? (double)b[o] : 0.0;
+      for (int i = 0; i < in; ++i) s += (double)W[(size_t)o * in + i] * x[(size_t)r * in + i];
+      y[(size_t)r * out + o] = s;
+    }
+}
+
+/* LayerNorm over the last dim, biased variance, affine (R7: eps from cfg). */
+static void layer_norm(int rows, int d, const double* z, const float* g, const float* b,
+                       double eps, double* y) {
+  for (int r = 0; r < rows; ++r) {
+    const double* zr = z + (size_t)r * d;
+    double mean = 0.0;
+    for (int i = 0; i < d; ++i) mean += zr[i];
+    mean /= d;
+    double var = 0.0;
+    for (int i = 0; i < d; ++i) var += (zr[i] - mean) * (zr[i] - mean);
+    var /= d;
+    double inv = 1.0 / sqrt(var + eps);
+    for (int i = 0; i < d; ++i) y[(size_t)r * d + i] = (zr[i] - mean) * inv * (double)g[i] + (double)b[i];
+  }
+}
+
+/* ------------------------------------------------------------------------ */
+/* Node features, Table I + log scaling, reading R9:     */
+/* f = [onehot(op) 64 | ln(1+dim_j) j<4 | onehot(dtype) 8 | onehot(kind) 4]. */
+/* Out-of-vocabulary ids give an all-zero one-hot block.                      */
+/* ------------------------------------------------------------------------ */
+void orc_features(int n, const orc_feat* feats, double* f) {
+  memset(f, 0, sizeof(double) * (size_t)n * ORC_F);
+  for (int v = 0; v < n; ++v) {
+    double* fv = f + (size_t)v * ORC_F;
+    if (feats[v].op < ORC_NUM_OPS) fv[feats[v].op] = 1.0;
+    for (int j = 0; j < ORC_NUM_DIMS; ++j) fv[ORC_NUM_OPS + j] = log1p((double)feats[v].dims[j]);
+    if (feats[v].dtype < ORC_NUM_DTYPES) fv[ORC_NUM_OPS + ORC_NUM_DIMS + feats[v].dtype] = 1.0;
+    if (feats[v].kind < ORC_NUM_KINDS)
+      fv[ORC_NUM_OPS + ORC_NUM_DIMS + ORC_NUM_DTYPES + feats[v].kind] = 1.0;
+  }
+}
+
+/* x0 = W_in f(v) + b_in + PE(depth(v)).  PE is the sinusoidal encoding of   */
+/* [34] applied to the depth (reading R5):                            */
+/*   PE[2i] = sin(depth * w_i), PE[2i+1] = cos(depth * w_i),                 */
+/*   w_i = 10000^(-2i/d).                                                    */
+void orc_embed(const orc_cfg* c, const float* blob, int n, const orc_feat* feats,
+               const int32_t* depth, double* x0) {
+  int d = c->d;
+  orc_top t = top_weights(c, blob);
+  double* f = (double*)malloc(sizeof(double) * (size_t)n * ORC_F);
+  orc_features(n, feats, f);
+  linear(n, ORC_F, d, f, t.W_in, t.b_in, x0);
+  for (int v = 0; v < n; ++v)
+    for (int i = 0; 2 * i < d; ++i) {
+      double w = pow(10000.0, -(2.0 * i) / d);
+      x0[(size_t)v * d + 2 * i] += sin(depth[v] * w);
+      if (2 * i + 1 < d) x0[(size_t)v * d + 2 * i + 1] += cos(depth[v] * w);
+    }
+  free(f);
+}
+
+/* ------------------------------------------------------------------------ */
+/* Eqn 1 with V (reading R1): per head h,                         */
+/*   O_h = softmax(Q_h K_h^T / sqrt(d_h) + M) V_h,  M in {0, -inf}.          */
+/* Softmax is the plain two-pass form over the allowed set (max, exp, sum).  */
+/* Output: concat_h O_h, [n][d].                                             */
+/* ------------------------------------------------------------------------ */
+void orc_attention(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
+                   const double* x, double* concat_out) {
+  int d = c->d, H = c->H, dh = c->d / c->H;
+  int W = orc_row_words(n);
+  orc_lw w = layer_weights(c, blob, layer);
+  double* qkv = (double*)malloc(sizeof(double) * (size_t)n * 3 * d);
+  linear(n, d, 3 * d, x, w.Wqkv, w.bqkv, qkv);
+  double* s = (double*)malloc(sizeof(double) * (size_t)n);
+  double scale = 1.0 / sqrt((double)dh);
+  for (int h = 0; h < H; ++h)
+    for (int u = 0; u < n; ++u) {
+      const double* q = qkv + (size_t)u * 3 * d + h * dh;
+      double mx = -INFINITY;
+      for (int v = 0; v < n; ++v) {
+        if (!bit(M, W, u, v)) continue;
+        const double* k = qkv + (size_t)v * 3 * d + d + h * dh;
+        double acc = 0.0;
+        for (int j = 0; j < dh; ++j) acc += q[j] * k[j];
+        s[v] = acc * scale;
+        if (s[v] > mx) mx = s[v];
+      }
+      double sum = 0.0;
+      for (int v = 0; v < n; ++v)
+        if (bit(M, W, u, v)) { s[v] = exp(s[v] - mx); sum += s[v]; }
+      double* o = concat_out + (size_t)u * d + h * dh;
+      for (int j = 0; j < dh; ++j) o[j] = 0.0;
+      for (int v = 0; v < n; ++v) {
+        if (!bit(M, W, u, v)) continue;
+        const double* vv = qkv + (size_t)v * 3 * d + 2 * d + h * dh;
+        double p = s[v] / sum;
+        for (int j = 0; j < dh; ++j) o[j] += p * vv[j];
+      }
+    }
+  free(qkv); free(s);
+}
+
+/* DAG Transformer layer (Fig. 4; reading R6, post-LN encoder  */
+/* layer of [34] with ReLU FFN):                                             */
+/*   h = LN1(x + W_o a + b_o),  x' = LN2(h + W_2 ReLU(W_1 h + b_1) + b_2).   */
+void orc_layer(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
+               const double* x_in, double* x_out) {
+  int d = c->d, f = c->d_ff;
+  orc_lw w = layer_weights(c, blob, layer);
+  double* a = (double*)malloc(sizeof(double) * (size_t)n * d);
+  double* z = (double*)malloc(sizeof(double) * (size_t)n * d);
+  double* h = (double*)malloc(sizeof(double) * (size_t)n * d);
+  double* u = (double*)malloc(sizeof(double) * (size_t)n * f);
+  orc_attention(c, blob, layer, n, M, x_in, a);
+  linear(n, d, d, a, w.Wo, w.bo, z);
+  for (long i = 0; i < (long)n * d; ++i) z[i] += x_in[i];
+  layer_norm(n, d, z, w.g1, w.be1, c->ln_eps, h);
+  linear(n, d, f, h, w.W1, w.b1, u);
+  for (long i = 0; i < (long)n * f; ++i) u[i] = u[i] > 0.0 ? u[i] : 0.0;
+  linear(n, f, d, u, w.W2, w.b2, z);
+  for (long i = 0; i < (long)n * d; ++i) z[i] += h[i];
+  layer_norm(n, d, z, w.g2, w.be2, c->ln_eps, x_out);
+  free(a); free(z); free(h); free(u);
+}
+
+/* Readout: global add pool, Eqn 2: x_i = sum_n x_n^i (mean if the   */
+/* R11 flag is set), then "linear layers each with ReLU activation, and      */
+/* finally ... the output layer" (reading R10: two hidden layers of   */
+/* width d, output Linear(d -> 1), no output activation).                     */
+double orc_readout(const orc_cfg* c, const float* blob, int n, const double* x) {
+  int d = c->d;
+  orc_top t = top_weights(c, blob);
+  double* g = (double*)calloc((size_t)d, sizeof(double));
+  double* z1 = (double*)malloc(sizeof(double) * (size_t)d);
+  double* z2 = (double*)malloc(sizeof(double) * (size_t)d);
+  for (int v = 0; v < n; ++v)
+    for (int j = 0; j < d; ++j) g[j] += x[(size_t)v * d + j];
+  if (c->pool == 1)
+    for (int j = 0; j < d; ++j) g[j] /= n;
+  linear(1, d, d, g, t.H1, t.c1, z1);
+  for (int j = 0; j < d; ++j) z1[j] = z1[j] > 0.0 ? z1[j] : 0.0;
+  linear(1, d, d, z1, t.H2, t.c2, z2);
+  for (int j = 0; j < d; ++j) z2[j] = z2[j] > 0.0 ? z2[j] : 0.0;
+  double y;
+  linear(1, d, 1, z2, t.w_o, t.c_o, &y);
+  free(g); free(z1); free(z2);
+  return y;
+}
+
+/* Whole black-box stage predictor for one stage graph.          */
+/* taps (nullable): (L+1) x n x d doubles: x0, then x after each layer.      */
+/* Returns the validation status; y = NaN for an invalid graph.              */
+int orc_forward(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
+                const int32_t* dst, const orc_feat* feats, double* y, double* taps) {
+  int st = orc_validate(n, e, src, dst);
+  if (st != ORC_OK) { *y = NAN; return st; }
+  int d = c->d, W = orc_row_words(n);
+  int32_t* depth = (int32_t*)malloc(sizeof(int32_t) * (size_t)n);
+  uint64_t* R = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)n * W);
+  uint64_t* M = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)n * W);
+  double* x = (double*)malloc(sizeof(double) * (size_t)n * d);
+  double* x2 = (double*)malloc(sizeof(double) * (size_t)n * d);
+  orc_depth(n, e, src, dst, depth);
+  orc_reach(n, e, src, dst, R);
+  orc_mask(n, R, M);
+  orc_embed(c, blob, n, feats, depth, x);
+  if (taps) memcpy(taps, x, sizeof(double) * (size_t)n * d);
+  for (int l = 0; l < c->L; ++l) {
+    orc_layer(c, blob, l, n, M, x, x2);
+    double* tmp = x; x = x2; x2 = tmp;
+    if (taps) memcpy(taps + (size_t)(l + 1) * n * d, x, sizeof(double) * (size_t)n * d);
+  }
+  *y = orc_readout(c, blob, n, x);
+  free(depth); free(R); free(M); free(x); free(x2);
+  return ORC_OK;
+}
+
+/* ------------------------------------------------------------------------ */
+/* White-box pipeline model, Eqn 4 (definitions):              */
+/*   T = sum_{i=1..S} t_i + (B - 1) * max_j t_j                              */
+/* Reading R13 (canonical fp64 order): sort the plan's fp32 latencies        */
+/* ascending, sum them in fp64 left to right, m = max, T = sum + (B-1)*m.    */
+/* Invalid plan (S < 1, S > 64, B < 1, stage index out of range) -> NaN.     */
+/* ------------------------------------------------------------------------ */
+void orc_plan_T(int64_t P, const int64_t* plan_ptr, const int32_t* plan_stage,
+                const int32_t* B, const float* t, int64_t num_stages, double* T) {
+  float buf[64];
+  for (int64_t p = 0; p < P; ++p) {
+    int64_t S = plan_ptr[p + 1] - plan_ptr[p];
+    int ok = S >= 1 && S <= 64 && B[p] >= 1;
+    for (int64_t i = 0; ok && i < S; ++i) {
+      int32_t s = plan_stage[plan_ptr[p] + i];
+      if (s < 0 || s >= num_stages) ok = 0;
+    }
+    if (!ok) { T[p] = NAN; continue; }
+    for (int64_t i = 0; i < S; ++i) buf[i] = t[plan_stage[plan_ptr[p] + i]];
+    for (int64_t i = 1; i < S; ++i) { /* insertion sort, ascending */
+      float key = buf[i];
+      int64_t j = i - 1;
+      while (j >= 0 && buf[j] > key) { buf[j + 1] = buf[j]; --j; }
+      buf[j + 1] = key;
+    }
+    double sum = 0.0;
+    for (int64_t i = 0; i < S; ++i) sum += (double)buf[i];
+    double m = (double)buf[S - 1];
+    double prod = (double)(B[p] - 1) * m;
+    T[p] = sum + prod;
+  }
+}
+
+/* argmin by (T, index) (R13); NaN never chosen; all NaN -> -1. */
+int64_t orc_argmin(int64_t n, const double* T) {
+  int64_t best = -1;
+  for (int64_t i = 0; i < n; ++i) {
+    if (isnan(T[i])) continue;
+    if (best < 0 || T[i] < T[best]) best = i;
+  }
+  return best;
+}

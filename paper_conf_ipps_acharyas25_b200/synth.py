@@ -1,0 +1,763 @@
+"""Seeded synthetic inputs for the PredTOP prediction path.
+
+INPUT GENERATION ONLY.  This module draws stage graphs, node records, model
+weights and pipeline plans; it contains none of the method's arithmetic (no
+depth, reachability, attention, pooling or pipeline formula).  It is the one
+module shared by the CUDA path (tests / bench) and the CPU oracle (tests), as
+allowed by DESIGN.md "input recipe".
+
+Everything is integer-deterministic: a counter-based splitmix64 stream keyed by
+(config seed, purpose, graph id) so any graph, shard or subset regenerates
+bit-identically on any host.
+
+Recipe (DESIGN.md section "Synthetic inputs"):
+  * Stage graphs are fwd+bwd training stages of a GPT-3 / GShard-MoE
+    transformer, built the way the paper builds them from Jaxpr (SIV-B2):
+    each equation is an operator node, parameters / boundary activations are
+    input nodes, constants are literal nodes, gradients / activations leaving
+    the stage are output nodes (Table I node types), edges are data
+    dependencies.  Pruned ops (reshape, convert_element_type)
+    are never emitted.
+  * A stage is a contiguous slice of the forward op tape of several layers plus
+    its reverse-mode backward ("stages of different sizes").
+  * The slice length is chosen so the node count lands on a per-graph target
+    drawn from the config's range; the remainder is padded by splicing
+    elementwise ops onto random edges.
+  * Shapes follow Table IV (read in DESIGN.md): GPT-3 1.3B hidden
+    2048, seq 1024, 32 heads; MoE 2.6B hidden 768, seq 1024, 16 heads,
+    16 experts.  Microbatch in {1,2,4,8}, model-parallel split in {1,2,4}.
+"""
+from __future__ import annotations
+
+import dataclasses
+from typing import Dict, List, Optional, Sequence, Tuple
+
+import numpy as np
+
+MASK64 = (1 << 64) - 1
+GOLDEN = 0x9E3779B97F4A7C15
+
+# --------------------------------------------------------------------------
+# Vocabularies (Table I one-hot slots; sizes fixed by include/predtop.h)
+# --------------------------------------------------------------------------
+NUM_OPS, NUM_DIMS, NUM_DTYPES, NUM_KINDS = 64, 4, 8, 4
+NUM_FEATURES = NUM_OPS + NUM_DIMS + NUM_DTYPES + NUM_KINDS
+
+OPS = [
+    "dot_general", "add", "sub", "mul", "div", "neg", "exp", "log", "tanh",
+    "logistic", "rsqrt", "sqrt", "integer_pow", "erf", "max", "min",
+    "reduce_sum", "reduce_max", "reduce_min", "argmax", "broadcast_in_dim",
+    "transpose", "select_n", "eq", "lt", "gt", "and", "or", "not", "iota",
+    "one_hot", "cumsum", "gather", "scatter_add", "dynamic_slice",
+    "dynamic_update_slice", "concatenate", "pad", "clamp", "abs", "sign",
+    "square", "pow", "stop_gradient", "copy", "rng_bit_generator",
+    "all_reduce", "all_gather", "reduce_scatter", "ppermute", "psum",
+    "custom_jvp_call", "pjit", "while", "cond", "sort", "top_k", "cumprod",
+    "reduce_precision", "exp2", "log1p", "expm1", "atan2", "other",
+]
+assert len(OPS) == NUM_OPS, len(OPS)
+OP = {n: i for i, n in enumerate(OPS)}
+DTYPES = ["f32", "f16", "bf16", "i32", "bool", "u32", "i64", "f64"]
+DT = {n: i for i, n in enumerate(DTYPES)}
+KIND_INPUT, KIND_LITERAL, KIND_OPERATOR, KIND_OUTPUT = 0, 1, 2, 3
+
+FEAT_DTYPE = np.dtype([("op", "<u2"), ("dtype", "u1"), ("kind", "u1"), ("dims", "<u4", (4,))])
+assert FEAT_DTYPE.itemsize == 20
+
+_PAD_OPS = ["add", "mul", "sub", "copy", "max", "exp", "tanh", "neg", "abs", "select_n"]
+
+
+# --------------------------------------------------------------------------
+# Counter-based RNG (splitmix64)
+# --------------------------------------------------------------------------
+def splitmix64(x: int) -> int:
+    x = (x + GOLDEN) & MASK64
+    z = x
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & MASK64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & MASK64
+    return z ^ (z >> 31)
+
+
+def _splitmix64_np(x: np.ndarray) -> np.ndarray:
+    x = x.astype(np.uint64) + np.uint64(GOLDEN)
+    z = x
+    z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+    z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+    return z ^ (z >> np.uint64(31))
+
+
+class CounterRng:
+    """Stream `key` of seed `seed`: value i = splitmix64(base + i * GOLDEN)."""
+
+    def __init__(self, seed: int, *key: int):
+        b = splitmix64(seed & MASK64)
+        for k in key:
+            b = splitmix64((b ^ (k & MASK64)) & MASK64)
+        self.base = b
+        self.ctr = 0
+
+    def u64(self) -> int:
+        self.ctr += 1
+        return splitmix64((self.base + self.ctr * GOLDEN) & MASK64)
+
+    def uniform(self) -> float:
+        return (self.u64() >> 11) * (1.0 / (1 << 53))
+
+    def randint(self, lo: int, hi: int) -> int:
+        """Integer in [lo, hi)."""
+        return lo + self.u64() % (hi - lo)
+
+    def choice(self, seq: Sequence):
+        return seq[self.randint(0, len(seq))]
+
+    def uniform_array(self, n: int) -> np.ndarray:
+        """n doubles in [0, 1) (vectorised, advances the counter by n)."""
+        with np.errstate(over="ignore"):
+            idx = np.arange(self.ctr + 1, self.ctr + 1 + n, dtype=np.uint64)
+            x = np.uint64(self.base) + idx * np.uint64(GOLDEN)
+            v = _splitmix64_np(x)
+        self.ctr += n
+        return (v >> np.uint64(11)).astype(np.float64) * (1.0 / (1 << 53))
+
+    def permutation(self, n: int) -> np.ndarray:
+        keys = self.uniform_array(n)
+        return np.argsort(keys, kind="stable").astype(np.int64)
+
+
+# --------------------------------------------------------------------------
+# Forward op tape of a transformer (records) -- shapes from Table IV
+# --------------------------------------------------------------------------
+@dataclasses.dataclass
+class _Rec:
+    op: str
+    dtype: str
+    dims: Tuple[int, ...]
+    ins: List[Tuple]  # ("rec", idx) | ("param", dims, dtype) | ("lit", dtype)
+
+
+class _Tape:
+    def __init__(self):
+        self.recs: List[_Rec] = []
+
+    def rec(self, op, dtype, dims, ins):
+        self.recs.append(_Rec(op, dtype, tuple(int(d) for d in dims), list(ins)))
+        return ("rec", len(self.recs) - 1)
+
+
+def _P(dims, dtype="f16"):
+    return ("param", tuple(int(d) for d in dims), dtype)
+
+
+def _L(dtype="f32"):
+    return ("lit", dtype)
+
+
+def _ln(t: _Tape, x, B, S, Hd):
+    s = t.rec("reduce_sum", "f32", [B, S], [x])
+    m = t.rec("div", "f32", [B, S], [s, _L()])
+    c = t.rec("sub", "f32", [B, S, Hd], [x, m])
+    sq = t.rec("integer_pow", "f32", [B, S, Hd], [c])
+    v = t.rec("reduce_sum", "f32", [B, S], [sq])
+    v2 = t.rec("div", "f32", [B, S], [v, _L()])
+    ve = t.rec("add", "f32", [B, S], [v2, _L()])
+    r = t.rec("rsqrt", "f32", [B, S], [ve])
+    n = t.rec("mul", "f32", [B, S, Hd], [c, r])
+    g = t.rec("mul", "f16", [B, S, Hd], [n, _P([Hd])])
+    return t.rec("add", "f16", [B, S, Hd], [g, _P([Hd])])
+
+
+def _dense(t: _Tape, x, din, dout, dims_out):
+    y = t.rec("dot_general", "f16", dims_out, [x, _P([din, dout])])
+    return t.rec("add", "f16", dims_out, [y, _P([dout])])
+
+
+def _gelu(t: _Tape, x, dims):
+    c3 = t.rec("integer_pow", "f16", dims, [x])
+    c4 = t.rec("mul", "f16", dims, [c3, _L("f16")])
+    c5 = t.rec("add", "f16", dims, [x, c4])
+    c6 = t.rec("mul", "f16", dims, [c5, _L("f16")])
+    c7 = t.rec("tanh", "f16", dims, [c6])
+    c8 = t.rec("add", "f16", dims, [c7, _L("f16")])
+    c9 = t.rec("mul", "f16", dims, [x, c8])
+    return t.rec("mul", "f16", dims, [c9, _L("f16")])
+
+
+def _attention(t: _Tape, x, B, S, Hd, nh):
+    h = _ln(t, x, B, S, Hd)
+    q = _dense(t, h, Hd, Hd, [B, S, Hd])
+    k = _dense(t, h, Hd, Hd, [B, S, Hd])
+    v = _dense(t, h, Hd, Hd, [B, S, Hd])
+    s = t.rec("dot_general", "f16", [B, nh, S, S], [q, k])
+    s2 = t.rec("mul", "f16", [B, nh, S, S], [s, _L("f16")])
+    mx = t.rec("reduce_max", "f32", [B, nh, S], [s2])
+    sb = t.rec("sub", "f32", [B, nh, S, S], [s2, mx])
+    e = t.rec("exp", "f32", [B, nh, S, S], [sb])
+    z = t.rec("reduce_sum", "f32", [B, nh, S], [e])
+    p = t.rec("div", "f16", [B, nh, S, S], [e, z])
+    o = t.rec("dot_general", "f16", [B, S, Hd], [p, v])
+    a = _dense(t, o, Hd, Hd, [B, S, Hd])
+    return t.rec("add", "f16", [B, S, Hd], [x, a])
+
+
+def _gpt_layer(t: _Tape, x, B, S, Hd, nh):
+    x1 = _attention(t, x, B, S, Hd, nh)
+    h2 = _ln(t, x1, B, S, Hd)
+    F = 4 * Hd
+    f1 = _dense(t, h2, Hd, F, [B, S, F])
+    g = _gelu(t, f1, [B, S, F])
+    f2 = _dense(t, g, F, Hd, [B, S, Hd])
+    return t.rec("add", "f16", [B, S, Hd], [x1, f2])
+
+
+def _moe_layer(t: _Tape, x, B, S, Hd, nh, E, cap):
+    x1 = _attention(t, x, B, S, Hd, nh)
+    h2 = _ln(t, x1, B, S, Hd)
+    gate = t.rec("dot_general", "f32", [B, S, E], [h2, _P([Hd, E], "f32")])
+    gm = t.rec("reduce_max", "f32", [B, S], [gate])
+    gs = t.rec("sub", "f32", [B, S, E], [gate, gm])
+    ge = t.rec("exp", "f32", [B, S, E], [gs])
+    gz = t.rec("reduce_sum", "f32", [B, S], [ge])
+    gp = t.rec("div", "f32", [B, S, E], [ge, gz])
+    top = t.rec("argmax", "i32", [B, S], [gp])
+    oh = t.rec("one_hot", "bool", [B, S, E], [top, _L("i32")])
+    disp = t.rec("mul", "f16", [B, S, E], [gp, oh])
+    F = 4 * Hd
+    outs = []
+    for _ in range(E):
+        xe = t.rec("dot_general", "f16", [cap, Hd], [h2, disp])
+        f1 = _dense(t, xe, Hd, F, [cap, F])
+        g = _gelu(t, f1, [cap, F])
+        f2 = _dense(t, g, F, Hd, [cap, Hd])
+        outs.append(t.rec("mul", "f16", [B, S, Hd], [f2, disp]))
+    acc = outs[0]
+    for o in outs[1:]:
+        acc = t.rec("add", "f16", [B, S, Hd], [acc, o])
+    return t.rec("add", "f16", [B, S, Hd], [x1, acc])
+
+
+_TAPE_CACHE: Dict[Tuple, _Tape] = {}
+
+
+def _tape(style: str, mb: int, split: int, n_layers: int) -> _Tape:
+    key = (style, mb, split, n_layers)
+    if key in _TAPE_CACHE:
+        return _TAPE_CACHE[key]
+    t = _Tape()
+    S = 1024
+    if style == "gpt":   # GPT-3 1.3B (Table IV): hidden 2048, 32 heads
+        Hd, nh = 2048 // split, 32 // split
+        x = t.rec("gather", "f16", [mb, S, Hd], [_P([51200 // split, Hd]), _L("i32")])
+        for _ in range(n_layers):
+            x = _gpt_layer(t, x, mb, S, Hd, nh)
+    elif style == "moe":  # GShard MoE 2.6B (Table IV): hidden 768, 16 heads, 16 experts
+        Hd, nh = 768 // split, 16 // split
+        x = t.rec("gather", "f16", [mb, S, Hd], [_P([32000 // split, Hd]), _L("i32")])
+        for li in range(n_layers):
+            if li % 2 == 1:
+                x = _moe_layer(t, x, mb, S, Hd, nh, 16, 2048 // split)
+            else:
+                x = _gpt_layer(t, x, mb, S, Hd, nh)
+    else:
+        raise ValueError(style)
+    _TAPE_CACHE[key] = t
+    return t
+
+
+# --------------------------------------------------------------------------
+# Stage graph = forward slice + reverse-mode backward
+# --------------------------------------------------------------------------
+class _GraphBuilder:
+    def __init__(self):
+        self.op: List[int] = []
+        self.dt: List[int] = []
+        self.kind: List[int] = []
+        self.dims: List[Tuple[int, ...]] = []
+        self.src: List[int] = []
+        self.dst: List[int] = []
+
+    def node(self, op, dtype, kind, dims, ins=()):
+        v = len(self.op)
+        self.op.append(OP[op])
+        self.dt.append(DT[dtype])
+        self.kind.append(kind)
+        self.dims.append(tuple(dims)[:4])
+        for u in ins:
+            self.src.append(u)
+            self.dst.append(v)
+        return v
+
+    def __len__(self):
+        return len(self.op)
+
+
+def _grad_nodes(gb: _GraphBuilder, r: _Rec, f: int, ins: List[int], kinds: List[str],
+                g: int) -> List[Optional[int]]:
+    """Backward of one forward record r (node f, input nodes ins) given the
+    gradient node g of its output.  Returns one gradient node per input (None
+    when the input gets no gradient).  Literal inputs get none."""
+    out: List[Optional[int]] = [None] * len(ins)
+    dt = r.dtype
+    op = r.op
+    for i, (u, k) in enumerate(zip(ins, kinds)):
+        if k == "lit":
+            continue
+        dims_u = gb.dims[u]
+        other = ins[1 - i] if len(ins) == 2 else None
+        if op == "add":
+            t = g
+        elif op == "sub":
+            t = g if i == 0 else gb.node("neg", dt, KIND_OPERATOR, dims_u, [g])
+        elif op == "mul":
+            t = gb.node("mul", dt, KIND_OPERATOR, dims_u, [g, other])
+        elif op == "div":
+            if i == 0:
+                t = gb.node("div", dt, KIND_OPERATOR, dims_u, [g, other])
+            else:
+                t1 = gb.node("mul", dt, KIND_OPERATOR, gb.dims[f], [g, f])
+                t2 = gb.node("div", dt, KIND_OPERATOR, gb.dims[f], [t1, u])
+                t = gb.node("neg", dt, KIND_OPERATOR, dims_u, [t2])
+        elif op == "dot_general":
+            if i == 0:
+                t = gb.node("dot_general", dt, KIND_OPERATOR, dims_u, [g, other])
+            else:
+                t = gb.node("dot_general", dt, KIND_OPERATOR, dims_u, [other, g])
+        elif op == "exp":
+            t = gb.node("mul", dt, KIND_OPERATOR, dims_u, [g, f])
+        elif op == "tanh":
+            t1 = gb.node("mul", dt, KIND_OPERATOR, dims_u, [f, f])
+            lit = gb.node("other", dt, KIND_LITERAL, ())
+            t2 = gb.node("sub", dt, KIND_OPERATOR, dims_u, [lit, t1])
+            t = gb.node("mul", dt, KIND_OPERATOR, dims_u, [g, t2])
+        elif op == "rsqrt":
+            t1 = gb.node("div", dt, KIND_OPERATOR, dims_u, [f, u])
+            lit = gb.node("other", dt, KIND_LITERAL, ())
+            t2 = gb.node("mul", dt, KIND_OPERATOR, dims_u, [t1, lit])
+            t = gb.node("mul", dt, KIND_OPERATOR, dims_u, [g, t2])
+        elif op == "integer_pow":
+            lit = gb.node("other", dt, KIND_LITERAL, ())
+            t1 = gb.node("mul", dt, KIND_OPERATOR, dims_u, [u, lit])
+            t = gb.node("mul", dt, KIND_OPERATOR, dims_u, [g, t1])
+        elif op == "reduce_sum":
+            t = gb.node("broadcast_in_dim", dt, KIND_OPERATOR, dims_u, [g])
+        elif op == "reduce_max":
+            t1 = gb.node("eq", "bool", KIND_OPERATOR, dims_u, [u, f])
+            t = gb.node("select_n", dt, KIND_OPERATOR, dims_u, [t1, g])
+        elif op == "gather":
+            t = gb.node("scatter_add", dt, KIND_OPERATOR, dims_u, [g])
+        else:  # argmax, one_hot, ...: not differentiable
+            continue
+        if k == "param" and op in ("add", "mul") and t is not None:
+            # broadcast parameter (bias / LN gamma, beta): reduce over batch dims
+            t = gb.node("reduce_sum", dt, KIND_OPERATOR, dims_u, [t])
+        out[i] = t
+    return out
+
+
+def _build_stage(tape: _Tape, start: int, m: int) -> _GraphBuilder:
+    gb = _GraphBuilder()
+    recs = tape.recs
+    end = start + m
+    node_of: Dict[int, int] = {}      # forward record -> node
+    ext: Dict[int, int] = {}          # record outside the slice -> boundary input node
+    in_nodes: Dict[int, List[int]] = {}
+    in_kinds: Dict[int, List[str]] = {}
+    params: List[int] = []
+    boundary_in: List[int] = []
+    for ri in range(start, end):
+        r = recs[ri]
+        ins, kinds = [], []
+        for ref in r.ins:
+            if ref[0] == "rec":
+                j = ref[1]
+                if j >= start:
+                    ins.append(node_of[j])
+                else:
+                    if j not in ext:
+                        ext[j] = gb.node("other", recs[j].dtype, KIND_INPUT, recs[j].dims)
+                        boundary_in.append(ext[j])
+                    ins.append(ext[j])
+                kinds.append("act")
+            elif ref[0] == "param":
+                p = gb.node("other", ref[2], KIND_INPUT, ref[1])
+                params.append(p)
+                ins.append(p)
+                kinds.append("param")
+            else:
+                ins.append(gb.node("other", ref[1], KIND_LITERAL, ()))
+                kinds.append("lit")
+        node_of[ri] = gb.node(r.op, r.dtype, KIND_OPERATOR, r.dims, ins)
+        in_nodes[ri], in_kinds[ri] = ins, kinds
+    # stage outputs: records consumed after the slice (or the last record)
+    consumed_later = set()
+    for rj in range(end, len(recs)):
+        for ref in recs[rj].ins:
+            if ref[0] == "rec" and start <= ref[1] < end:
+                consumed_later.add(ref[1])
+    consumed_later.add(end - 1)
+    grad: Dict[int, int] = {}
+    for ri in sorted(consumed_later):
+        f = node_of[ri]
+        gb.node("other", recs[ri].dtype, KIND_OUTPUT, recs[ri].dims, [f])  # activation out
+        grad[f] = gb.node("other", recs[ri].dtype, KIND_INPUT, recs[ri].dims)  # upstream grad in
+    for ri in range(end - 1, start - 1, -1):
+        f = node_of[ri]
+        if f not in grad:
+            continue
+        gs = _grad_nodes(gb, recs[ri], f, in_nodes[ri], in_kinds[ri], grad[f])
+        for u, t in zip(in_nodes[ri], gs):
+            if t is None:
+                continue
+            if u in grad:
+                grad[u] = gb.node("add", recs[ri].dtype, KIND_OPERATOR, gb.dims[u], [grad[u], t])
+            else:
+                grad[u] = t
+    for p in params + boundary_in:
+        if p in grad:
+            gb.node("other", DTYPES[gb.dt[p]], KIND_OUTPUT, gb.dims[p], [grad[p]])
+    return gb
+
+
+@dataclasses.dataclass
+class StageBatch:
+    """Packed batch of stage DAGs in the layout of include/predtop.h."""
+    node_ptr: np.ndarray   # int64 [G+1]
+    edge_ptr: np.ndarray   # int64 [G+1]
+    src: np.ndarray        # int32 [E] graph-local
+    dst: np.ndarray        # int32 [E] graph-local
+    feats: np.ndarray      # FEAT_DTYPE [N_tot]
+
+    @property
+    def num_graphs(self) -> int:
+        return len(self.node_ptr) - 1
+
+    @property
+    def sizes(self) -> np.ndarray:
+        return np.diff(self.node_ptr)
+
+    def graph(self, g: int):
+        """(N, src, dst, feats) of graph g (views)."""
+        n0, n1 = int(self.node_ptr[g]), int(self.node_ptr[g + 1])
+        e0, e1 = int(self.edge_ptr[g]), int(self.edge_ptr[g + 1])
+        return n1 - n0, self.src[e0:e1], self.dst[e0:e1], self.feats[n0:n1]
+
+    def subset(self, graphs: Sequence[int]) -> "StageBatch":
+        return pack_graphs([self.graph(int(g)) for g in graphs])
+
+
+def pack_graphs(graphs: Sequence[Tuple]) -> StageBatch:
+    """graphs: iterable of (N, src, dst, feats)."""
+    ns = [int(g[0]) for g in graphs]
+    es = [len(g[1]) for g in graphs]
+    node_ptr = np.zeros(len(ns) + 1, np.int64)
+    node_ptr[1:] = np.cumsum(ns)
+    edge_ptr = np.zeros(len(es) + 1, np.int64)
+    edge_ptr[1:] = np.cumsum(es)
+    src = np.concatenate([np.asarray(g[1], np.int32) for g in graphs]) if graphs else np.zeros(0, np.int32)
+    dst = np.concatenate([np.asarray(g[2], np.int32) for g in graphs]) if graphs else np.zeros(0, np.int32)
+    feats = np.concatenate([np.asarray(g[3], FEAT_DTYPE) for g in graphs]) if graphs else np.zeros(0, FEAT_DTYPE)
+    return StageBatch(node_ptr, edge_ptr, src.astype(np.int32), dst.astype(np.int32), feats)
+
+
+def _feats_of(gb: _GraphBuilder) -> np.ndarray:
+    f = np.zeros(len(gb), FEAT_DTYPE)
+    f["op"] = gb.op
+    f["dtype"] = gb.dt
+    f["kind"] = gb.kind
+    d = np.zeros((len(gb), 4), np.uint32)
+    for i, dims in enumerate(gb.dims):
+        if dims:
+            d[i, :len(dims)] = dims
+    f["dims"] = d
+    return f
+
+
+_SIZE_CACHE: Dict[Tuple, int] = {}
+
+
+def _stage_size(tape_key, tape, start, m) -> int:
+    k = (tape_key, start, m)
+    if k not in _SIZE_CACHE:
+        _SIZE_CACHE[k] = len(_build_stage(tape, start, m))
+    return _SIZE_CACHE[k]
+
+
+def _pad_to(gb: _GraphBuilder, target: int, rng: CounterRng):
+    """Splice elementwise ops onto random edges until len(gb) == target, then
+    relabel into a topological construction order."""
+    n0 = len(gb)
+    key = [(i, 0) for i in range(n0)]
+    ctr = 1
+    while len(gb) < target:
+        # only edges whose destination is an original node (keeps key order topological)
+        while True:
+            e = rng.randint(0, len(gb.src))
+            if gb.dst[e] < n0:
+                break
+        u, v = gb.src[e], gb.dst[e]
+        w = gb.node(rng.choice(_PAD_OPS), DTYPES[gb.dt[u]], KIND_OPERATOR, gb.dims[u], [u])
+        gb.src[e] = w  # u -> w -> v
+        key.append((key[u][0], ctr))
+        ctr += 1
+    order = sorted(range(len(gb)), key=lambda i: key[i])
+    newid = np.empty(len(gb), np.int64)
+    newid[order] = np.arange(len(gb))
+    gb.op = [gb.op[i] for i in order]
+    gb.dt = [gb.dt[i] for i in order]
+    gb.kind = [gb.kind[i] for i in order]
+    gb.dims = [gb.dims[i] for i in order]
+    gb.src = [int(newid[s]) for s in gb.src]
+    gb.dst = [int(newid[d]) for d in gb.dst]
+
+
+def stage_graph(style: str, n_target: int, seed: int, gid: int):
+    """One synthetic stage DAG with exactly n_target nodes: (N, src, dst, feats)."""
+    rng = CounterRng(seed, 0x5747, gid)
+    mb = rng.choice([1, 2, 4, 8])
+    split = rng.choice([1, 2, 4])
+    per_layer = 52 if style == "gpt" else 300
+    n_layers = max(4, (n_target // (3 * per_layer)) + 4)
+    tape_key = (style, mb, split, n_layers)
+    tape = _tape(style, mb, split, n_layers)
+    start = rng.randint(1, per_layer + 1)
+    # largest slice length whose stage fits in n_target (sizes are monotone enough;
+    # walk down from a generous upper estimate)
+    lo, hi = 1, min(len(tape.recs) - start, max(2, n_target))
+    while lo < hi:  # binary search for the largest m with size <= target
+        mid = (lo + hi + 1) // 2
+        if _stage_size(tape_key, tape, start, mid) <= n_target:
+            lo = mid
+        else:
+            hi = mid - 1
+    gb = _build_stage(tape, start, lo)
+    if len(gb) > n_target:
+        raise RuntimeError("stage template larger than target")
+    _pad_to(gb, n_target, rng)
+    return n_target, np.asarray(gb.src, np.int32), np.asarray(gb.dst, np.int32), _feats_of(gb)
+
+
+# --------------------------------------------------------------------------
+# Hand-made tiny graphs (config 0) and structured test graphs
+# --------------------------------------------------------------------------
+def _rand_feats(n: int, rng: CounterRng, kinds=None) -> np.ndarray:
+    f = np.zeros(n, FEAT_DTYPE)
+    for i in range(n):
+        f[i]["op"] = rng.randint(0, NUM_OPS)
+        f[i]["dtype"] = rng.randint(0, NUM_DTYPES)
+        f[i]["kind"] = rng.randint(0, NUM_KINDS) if kinds is None else kinds[i]
+        rank = rng.randint(0, 5)
+        for j in range(rank):
+            f[i]["dims"][j] = rng.choice([1, 2, 4, 8, 16, 128, 768, 1024, 2048, 8192, 51200])
+    return f
+
+
+def chain(n: int):
+    s = np.arange(n - 1, dtype=np.int32)
+    return s, s + 1
+
+
+def diamond_chains(n: int):
+    """s -> two parallel chains -> t (n >= 4)."""
+    k = (n - 2) // 2
+    src, dst = [], []
+    a = list(range(1, 1 + k))
+    b = list(range(1 + k, n - 1))
+    t = n - 1
+    for ch in (a, b):
+        if not ch:
+            continue
+        src.append(0); dst.append(ch[0])
+        for x, y in zip(ch[:-1], ch[1:]):
+            src.append(x); dst.append(y)
+        src.append(ch[-1]); dst.append(t)
+    return np.asarray(src, np.int32), np.asarray(dst, np.int32)
+
+
+def star(n: int):
+    return np.zeros(n - 1, np.int32), np.arange(1, n, dtype=np.int32)
+
+
+def chain_with_skips(n: int):
+    s, d = chain(n)
+    return np.concatenate([s, [0, 3]]).astype(np.int32), np.concatenate([d, [5, n - 1]]).astype(np.int32)
+
+
+def tiny_batch(seed: int = 0) -> StageBatch:
+    """configs[0]: chain of 8, diamond of 10, fan-out star of 16, 12-node chain with skips."""
+    rng = CounterRng(seed, 0x7171)
+    gs = []
+    for n, (s, d) in [(8, chain(8)), (10, diamond_chains(10)), (16, star(16)), (12, chain_with_skips(12))]:
+        gs.append((n, s, d, _rand_feats(n, rng)))
+    return pack_graphs(gs)
+
+
+def random_dag(n: int, p_edge: float, rng: CounterRng, relabel: bool = True):
+    """Random DAG on n nodes: edge i->j (i<j in a hidden order) with prob p."""
+    src, dst = [], []
+    for j in range(n):
+        for i in range(j):
+            if rng.uniform() < p_edge:
+                src.append(i); dst.append(j)
+    src = np.asarray(src, np.int64); dst = np.asarray(dst, np.int64)
+    if relabel and n > 0:
+        perm = rng.permutation(n)
+        src, dst = perm[src], perm[dst]
+    return src.astype(np.int32), dst.astype(np.int32)
+
+
+def relabel(n: int, src, dst, feats, perm: np.ndarray):
+    """Node v becomes perm[v]."""
+    inv = np.empty(n, np.int64)
+    inv[perm] = np.arange(n)
+    return (perm[np.asarray(src)].astype(np.int32), perm[np.asarray(dst)].astype(np.int32),
+            np.asarray(feats)[inv])
+
+
+# --------------------------------------------------------------------------
+# Benchmark configurations (BASELINE.json configs)
+# --------------------------------------------------------------------------
+CONFIG_SEEDS = {"tiny": 0, "gpt": 1, "moe": 2, "16k": 3, "sweep": 4}
+N_RANGE = {"gpt": (270, 330), "moe": (1350, 1650)}
+
+
+def graph_sizes(config: str, num_graphs: int, seed: Optional[int] = None) -> np.ndarray:
+    seed = CONFIG_SEEDS[config] if seed is None else seed
+    lo, hi = N_RANGE[config]
+    return np.asarray([CounterRng(seed, 0x517E, g).randint(lo, hi + 1) for g in range(num_graphs)],
+                      np.int64)
+
+
+def stage_batch(config: str, num_graphs: int, first_graph: int = 0,
+                seed: Optional[int] = None) -> StageBatch:
+    """Graphs [first_graph, first_graph+num_graphs) of a config ('gpt', 'moe', '16k').
+    Graph g depends only on (seed, g), so shards regenerate identically."""
+    seed = CONFIG_SEEDS[config] if seed is None else seed
+    gs = []
+    for g in range(first_graph, first_graph + num_graphs):
+        if config == "16k":
+            gs.append(stage_graph("gpt", 16384, seed, g))
+        else:
+            n = int(CounterRng(seed, 0x517E, g).randint(N_RANGE[config][0], N_RANGE[config][1] + 1))
+            gs.append(stage_graph(config, n, seed, g))
+    return pack_graphs(gs)
+
+
+# --------------------------------------------------------------------------
+# Model configuration and weights (reading R14 in DESIGN.md)
+# --------------------------------------------------------------------------
+# head_scale / out_bias (R14): the synthetic weights are untrained, so the raw
+# head output w_o . z2 has an arbitrary sign and a scale that grows with the
+# sum-pooled graph size.  These per-config constants (chosen once from a sample
+# of the raw outputs, then frozen) map the outputs to positive, latency-like
+# values of O(1-10) without letting the output bias dominate.
+MODEL_CONFIGS = {
+    "tiny": dict(num_layers=1, d_model=32, num_heads=2, d_ff=128, pool=0, ln_eps=1e-5,
+                 head_scale=1.0, out_bias=4.0, seed=100),
+    "paper": dict(num_layers=4, d_model=64, num_heads=4, d_ff=256, pool=0, ln_eps=1e-5,
+                  head_scale=-0.03, out_bias=0.0, seed=101),
+    "gpt": dict(num_layers=4, d_model=128, num_heads=8, d_ff=512, pool=0, ln_eps=1e-5,
+                head_scale=0.25, out_bias=1.0, seed=102),
+    "moe": dict(num_layers=4, d_model=256, num_heads=8, d_ff=1024, pool=0, ln_eps=1e-5,
+                head_scale=0.007, out_bias=0.0, seed=103),
+    "16k": dict(num_layers=4, d_model=128, num_heads=8, d_ff=512, pool=0, ln_eps=1e-5,
+                head_scale=0.25, out_bias=1.0, seed=104),
+}
+
+
+def weight_shapes(cfg: dict) -> List[Tuple[str, Tuple[int, ...]]]:
+    """Names and shapes in the blob order of include/predtop.h."""
+    d, dff, F = cfg["d_model"], cfg["d_ff"], NUM_FEATURES
+    out = [("W_in", (d, F)), ("b_in", (d,))]
+    for l in range(cfg["num_layers"]):
+        out += [(f"L{l}.W_qkv", (3 * d, d)), (f"L{l}.b_qkv", (3 * d,)),
+                (f"L{l}.W_o", (d, d)), (f"L{l}.b_o", (d,)),
+                (f"L{l}.ln1_g", (d,)), (f"L{l}.ln1_b", (d,)),
+                (f"L{l}.W_1", (dff, d)), (f"L{l}.b_1", (dff,)),
+                (f"L{l}.W_2", (d, dff)), (f"L{l}.b_2", (d,)),
+                (f"L{l}.ln2_g", (d,)), (f"L{l}.ln2_b", (d,))]
+    out += [("H_1", (d, d)), ("c_1", (d,)), ("H_2", (d, d)), ("c_2", (d,)),
+            ("w_o", (1, d)), ("c_o", (1,))]
+    return out
+
+
+def model_weights(cfg: dict, seed: Optional[int] = None, head_scale: Optional[float] = None,
+                  out_bias: Optional[float] = None) -> Dict[str, np.ndarray]:
+    """R14: Xavier-uniform Linear weights, U(+-0.05) biases, LN gamma 1+U(+-0.05),
+    beta U(+-0.05); head output weight x head_scale, output bias out_bias.
+    Every value is rounded once to the nearest fp16 (so fp16 device storage is
+    exact) and returned as float32."""
+    seed = cfg.get("seed", 100) if seed is None else seed
+    head_scale = cfg.get("head_scale", 0.1) if head_scale is None else head_scale
+    out_bias = cfg.get("out_bias", 1.0) if out_bias is None else out_bias
+    rng = CounterRng(seed, 0x3E16)
+    w = {}
+    for name, shape in weight_shapes(cfg):
+        n = int(np.prod(shape))
+        u = rng.uniform_array(n) * 2.0 - 1.0
+        base = name.split(".")[-1]
+        if base.startswith(("W_", "H_")) or base == "w_o":
+            fan_out, fan_in = shape
+            a = np.sqrt(6.0 / (fan_in + fan_out))
+            v = u * a
+            if base == "w_o":
+                v = v * head_scale
+        elif base.endswith("_g"):
+            v = 1.0 + 0.05 * u
+        elif base == "c_o":
+            v = np.full(n, out_bias)
+        else:  # biases, LN beta
+            v = 0.05 * u
+        w[name] = v.astype(np.float16).astype(np.float32).reshape(shape)
+    return w
+
+
+def pack_weights(cfg: dict, w: Dict[str, np.ndarray]) -> np.ndarray:
+    return np.concatenate([np.ascontiguousarray(w[n], np.float32).ravel() for n, _ in weight_shapes(cfg)])
+
+
+# --------------------------------------------------------------------------
+# Pipeline plans (D8)
+# --------------------------------------------------------------------------
+@dataclasses.dataclass
+class PlanSet:
+    plan_ptr: np.ndarray      # int64 [P+1]
+    plan_stage: np.ndarray    # int32 [sum S]
+    microbatches: np.ndarray  # int32 [P]
+
+    @property
+    def num_plans(self) -> int:
+        return len(self.plan_ptr) - 1
+
+
+def owned_plans(num_graphs: int, stages_per_plan: int, microbatches: int) -> PlanSet:
+    """Owned mode: plan p uses stage graphs [S*p, S*p + S)."""
+    P = num_graphs // stages_per_plan
+    ptr = np.arange(P + 1, dtype=np.int64) * stages_per_plan
+    return PlanSet(ptr, np.arange(P * stages_per_plan, dtype=np.int32),
+                   np.full(P, microbatches, np.int32))
+
+
+def sweep_plans(num_plans: int, seed: int = 4, first_plan: int = 0) -> Tuple[PlanSet, np.ndarray]:
+    """Plan sweep: S ~ U{2..8}, B ~ U{1,4,16,64}; plans own their stages.
+    Returns the plan set and each plan's first global stage id (plan p's stage
+    graphs are global ids [first, first + S_p))."""
+    S = np.empty(num_plans, np.int64)
+    B = np.empty(num_plans, np.int32)
+    for i in range(num_plans):
+        r = CounterRng(seed, 0x9A17, first_plan + i)
+        S[i] = r.randint(2, 9)
+        B[i] = (1, 4, 16, 64)[r.randint(0, 4)]
+    ptr = np.zeros(num_plans + 1, np.int64)
+    ptr[1:] = np.cumsum(S)
+    return PlanSet(ptr, np.arange(ptr[-1], dtype=np.int32), B), ptr[:-1].copy()
+
+
+def random_plans(num_plans: int, num_stages: int, seed: int, max_s: int = 8,
+                 bs=(1, 2, 3, 4, 16, 64)) -> PlanSet:
+    """Plans over a shared stage table (stages may repeat across plans)."""
+    r = CounterRng(seed, 0x9A18)
+    S = [r.randint(1, max_s + 1) for _ in range(num_plans)]
+    ptr = np.zeros(num_plans + 1, np.int64)
+    ptr[1:] = np.cumsum(S)
+    st = np.asarray([r.randint(0, num_stages) for _ in range(int(ptr[-1]))], np.int32)
+    B = np.asarray([r.choice(bs) for _ in range(num_plans)], np.int32)
+    return PlanSet(ptr, st, B)
