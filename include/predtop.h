@@ -42,6 +42,12 @@
 #include <stddef.h>
 #include <stdint.h>
 
+#if defined(__GNUC__)
+#define PREDTOP_API __attribute__((visibility("default")))
+#else
+#define PREDTOP_API
+#endif
+
 #ifdef __cplusplus
 extern "C" {
 #endif
@@ -115,7 +121,7 @@ typedef struct predtop_model_s* predtop_model;
 
 /* Bytes of device workspace predtop_build_dag needs for `desc` (256-byte
  * aligned base required).  0 on invalid desc. */
-size_t predtop_build_dag_workspace(const predtop_batch_desc* desc);
+PREDTOP_API size_t predtop_build_dag_workspace(const predtop_batch_desc* desc);
 
 /* Validate every graph, compute node depth and the reachability closure.
  *  - Validation, in this precedence per graph: RANGE (an endpoint outside
@@ -143,7 +149,7 @@ size_t predtop_build_dag_workspace(const predtop_batch_desc* desc);
  * graph.  With PREDTOP_NO_SYNC it returns PREDTOP_OK after enqueueing, and
  * predtop_dag_status() reports later; graphs with an error get a NaN latency
  * from predtop_stage_forward. */
-predtop_status predtop_build_dag(const predtop_batch_desc* desc,
+PREDTOP_API predtop_status predtop_build_dag(const predtop_batch_desc* desc,
                                  const int64_t* node_ptr, const int64_t* edge_ptr,
                                  const int32_t* edge_src, const int32_t* edge_dst,
                                  const predtop_node_feat* feats,
@@ -153,30 +159,30 @@ predtop_status predtop_build_dag(const predtop_batch_desc* desc,
 
 /* Synchronises `cuda_stream` and returns the build status of `dag` (and the
  * lowest bad graph via [host] first_bad_graph, nullable). */
-predtop_status predtop_dag_status(predtop_dag dag, int32_t* first_bad_graph, void* cuda_stream);
+PREDTOP_API predtop_status predtop_dag_status(predtop_dag dag, int32_t* first_bad_graph, void* cuda_stream);
 
 /* Number of uint64 words predtop_reachability writes:
  * sum_g N_g * W_g with W_g = 2 * ceil(N_g / 128).  [host] result. */
-predtop_status predtop_dag_reach_words(predtop_dag dag, int64_t* words, void* cuda_stream);
+PREDTOP_API predtop_status predtop_dag_reach_words(predtop_dag dag, int64_t* words, void* cuda_stream);
 
 /* Copy the closure R to bits_out (device, uint64).  Layout: graph g starts at
  * word offset sum_{h<g} N_h * W_h; row v (caller order) of graph g is W_g
  * words; bit (u % 64) of word (u / 64) of row v is 1 iff v ~> u by >= 1 edge.
  * Padding bits (u >= N_g) are 0.  Rows are 16-byte aligned. */
-predtop_status predtop_reachability(predtop_dag dag, uint64_t* bits_out, void* cuda_stream);
+PREDTOP_API predtop_status predtop_reachability(predtop_dag dag, uint64_t* bits_out, void* cuda_stream);
 
 /* Same layout, for the attention mask M = R | R^T | I (debug / tests). */
-predtop_status predtop_debug_mask(predtop_dag dag, uint64_t* bits_out, void* cuda_stream);
+PREDTOP_API predtop_status predtop_debug_mask(predtop_dag dag, uint64_t* bits_out, void* cuda_stream);
 
 /* Per-graph block structure of M (debug / tests):
  *  tile_class_out: graph g starts at offset sum_{h<g} T_h^2, T_h = ceil(N_h/128);
  *    entry (qt * T_g + kt) for the 128x128 tile of rows [128qt,..) x cols [128kt,..)
  *    (clipped to N_g): 0 = no allowed pair, 2 = every pair allowed, 1 = otherwise.
  *  pairs_out[G]: |A_g| = popcount(M_g) = N_g + 2 |R_g|.   Both device, nullable. */
-predtop_status predtop_debug_tiles(predtop_dag dag, uint8_t* tile_class_out,
+PREDTOP_API predtop_status predtop_debug_tiles(predtop_dag dag, uint8_t* tile_class_out,
                                    int64_t* pairs_out, void* cuda_stream);
 
-void predtop_dag_destroy(predtop_dag dag);
+PREDTOP_API void predtop_dag_destroy(predtop_dag dag);
 
 /* ---------------------------------------------------------------------------
  * DAG-Transformer latency model (SIV-B5).  One model per mesh /
@@ -215,24 +221,24 @@ typedef struct {
  *   H_1 [d][d] c_1 [d]  H_2 [d][d] c_2 [d]  w_o [d]  c_o [1]
  * The per-layer GEMM weights (W_qkv, W_o, W_1, W_2) are stored on the device
  * as fp16; values that are not fp16-representable are rounded to nearest. */
-size_t predtop_model_weight_floats(const predtop_model_config* cfg); /* blob length in floats */
-size_t predtop_model_device_bytes(const predtop_model_config* cfg);  /* device weight bytes */
+PREDTOP_API size_t predtop_model_weight_floats(const predtop_model_config* cfg); /* blob length in floats */
+PREDTOP_API size_t predtop_model_device_bytes(const predtop_model_config* cfg);  /* device weight bytes */
 
 /* Validates cfg, converts and uploads the blob into caller-allocated device
  * memory (>= predtop_model_device_bytes, 256-byte aligned).  Synchronous. */
-predtop_status predtop_model_create(const predtop_model_config* cfg,
+PREDTOP_API predtop_status predtop_model_create(const predtop_model_config* cfg,
                                     const float* weights_host, size_t num_floats,
                                     void* device_weights, size_t device_bytes,
                                     predtop_model* out);
-void predtop_model_destroy(predtop_model model);
+PREDTOP_API void predtop_model_destroy(predtop_model model);
 
 /* Device workspace bytes for predtop_stage_forward(model, dag). */
-size_t predtop_stage_forward_workspace(predtop_model model, predtop_dag dag);
+PREDTOP_API size_t predtop_stage_forward_workspace(predtop_model model, predtop_dag dag);
 
 /* latency_out[G] (device, fp32): predicted stage latency of every graph.
  * Deterministic: each graph's value is bit-identical whatever the batch
  * composition, order or size (no split-K, no float atomics). */
-predtop_status predtop_stage_forward(predtop_model model, predtop_dag dag,
+PREDTOP_API predtop_status predtop_stage_forward(predtop_model model, predtop_dag dag,
                                      void* workspace, size_t ws_bytes,
                                      float* latency_out, void* cuda_stream);
 
@@ -240,7 +246,7 @@ predtop_status predtop_stage_forward(predtop_model model, predtop_dag dag,
  * embedding + PE), fp32 [N_tot][d] device.  Valid after predtop_stage_forward
  * ran with the same workspace only for layer = L-1 (the final x); other layers
  * are recomputed by this call. */
-predtop_status predtop_debug_node_embeddings(predtop_model model, predtop_dag dag,
+PREDTOP_API predtop_status predtop_debug_node_embeddings(predtop_model model, predtop_dag dag,
                                              void* workspace, size_t ws_bytes, int32_t layer,
                                              float* x_out, void* cuda_stream);
 
@@ -260,8 +266,8 @@ predtop_status predtop_debug_node_embeddings(predtop_model model, predtop_dag da
  *  flags: PREDTOP_NO_SYNC or 0 (sync mode returns INVALID_ARG for a bad plan,
  *  and the lowest bad plan index via [host] first_bad_plan, nullable). */
 #define PREDTOP_MAX_PLAN_STAGES 64
-size_t predtop_plan_latency_workspace(void);
-predtop_status predtop_plan_latency(int64_t num_plans, const int64_t* plan_ptr,
+PREDTOP_API size_t predtop_plan_latency_workspace(void);
+PREDTOP_API predtop_status predtop_plan_latency(int64_t num_plans, const int64_t* plan_ptr,
                                     const int32_t* plan_stage, const int32_t* microbatches,
                                     const float* stage_latency, int64_t num_stages,
                                     double* T_out, void* workspace, size_t ws_bytes,
@@ -271,17 +277,27 @@ predtop_status predtop_plan_latency(int64_t num_plans, const int64_t* plan_ptr,
 /* best_out[1] (device int64) = argmin_p T[p] with ties to the lower index
  * (ranking by (T, plan id), R13).  NaN entries are never chosen unless all
  * are NaN (then -1).  workspace >= predtop_plan_argmin_workspace(n). */
-size_t predtop_plan_argmin_workspace(int64_t num_plans);
-predtop_status predtop_plan_argmin(int64_t num_plans, const double* T, int64_t* best_out,
+PREDTOP_API size_t predtop_plan_argmin_workspace(int64_t num_plans);
+PREDTOP_API predtop_status predtop_plan_argmin(int64_t num_plans, const double* T, int64_t* best_out,
                                    void* workspace, size_t ws_bytes, void* cuda_stream);
 
 /* Misc. */
-const char* predtop_status_string(predtop_status s);
-const char* predtop_last_error(void); /* thread-local */
-int predtop_abi_version(void);
+PREDTOP_API const char* predtop_status_string(predtop_status s);
+PREDTOP_API const char* predtop_last_error(void); /* thread-local */
+PREDTOP_API int predtop_abi_version(void);
 /* Number of kernels this library has launched in this process (all entry
  * points).  Lets callers count launches inside a timed region. */
-int64_t predtop_launch_count(void);
+PREDTOP_API int64_t predtop_launch_count(void);
+
+/* Optional per-kernel timing.  When enabled, every launch site records a CUDA
+ * event pair on its launching stream.  predtop_profile_read synchronises on
+ * the recorded events, writes the accumulated milliseconds and launch counts
+ * per kernel kind (ms[k], launches[k], k < min(max_kinds, kinds)), resets the
+ * accumulators and returns the number of kinds; predtop_profile_kind_name(k)
+ * names kind k.  [host] arrays, nullable. */
+PREDTOP_API void predtop_profile_enable(int on);
+PREDTOP_API int predtop_profile_read(double* ms, int64_t* launches, int max_kinds);
+PREDTOP_API const char* predtop_profile_kind_name(int kind);
 
 #ifdef __cplusplus
 }

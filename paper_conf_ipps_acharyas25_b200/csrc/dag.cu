@@ -1,0 +1,418 @@
+// dag.cu -- stage-DAG preprocessing on the device (predtop_build_dag).
+//
+//  k_meta      per-graph sizes, size checks, prefix offsets (one CTA)
+//  k_depth     K1: range / self-loop check, successor CSR, level-synchronous
+//              Kahn (P:137 DAGPE depth = Kahn level = longest path from a
+//              source; a graph whose Kahn order misses a node has a cycle)
+//  k_closure   K2: packed-bitset transitive closure R[v] = OR_{w in succ(v)}
+//              (R[w] | {w}), level-synchronous from the deepest level up
+//              (P:135 DAGRA, P:145 k = infinity); one CTA per (graph, column
+//              slice), the slice of all rows resident in shared memory
+//  k_mask      K3: M = R | R^T | I with warp-ballot 32x32 bit transposes and
+//              popcounts per 128x128 tile
+//  k_classify  tile classes (empty / partial / full) and |A| per graph
+//  k_work      attention work list (graph, 128-row q-tile)
+#include <algorithm>
+#include <climits>
+
+#include "internal.h"
+
+namespace predtop {
+
+template <class T>
+__device__ T block_excl_scan(T v, T* total, T* sh /*[32]*/) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  T x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    T y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) sh[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    T w = lane < nw ? sh[lane] : T(0);
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      T y = __shfl_up_sync(0xffffffffu, w, o);
+      if (lane >= o) w += y;
+    }
+    sh[lane] = w;
+  }
+  __syncthreads();
+  T base = wid > 0 ? sh[wid - 1] : T(0);
+  *total = sh[nw - 1];
+  __syncthreads();
+  return base + x - v;
+}
+
+__global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
+  __shared__ int64_t sh64[32];
+  int64_t carry_rows = 0, carry_tiles = 0, carry_q = 0;
+  for (int base = 0; base < G; base += blockDim.x) {
+    const int g = base + threadIdx.x;
+    int64_t rows = 0, tiles = 0, q = 0;
+    if (g < G) {
+      const int64_t n = d.node_ptr[g + 1] - d.node_ptr[g];
+      const int64_t e = d.edge_ptr[g + 1] - d.edge_ptr[g];
+      int st = PREDTOP_OK;
+      if (n < 1 || n > max_nodes || n > PREDTOP_MAX_NODES) st = PREDTOP_ERR_TOO_LARGE;
+      else if (e < 0) st = PREDTOP_ERR_INVALID_ARG;
+      d.status[g] = st;
+      d.num_levels[g] = 0;
+      d.pairs[g] = 0;
+      if (st == PREDTOP_OK) {
+        const int64_t T = (n + 127) / 128;
+        rows = n * 2 * T;
+        tiles = T * T;
+        q = T;
+      }
+    }
+    int64_t tot;
+    int64_t ex = block_excl_scan<int64_t>(rows, &tot, sh64);
+    if (g < G) d.row_off[g] = carry_rows + ex;
+    carry_rows += tot;
+    ex = block_excl_scan<int64_t>(tiles, &tot, sh64);
+    if (g < G) d.tile_off[g] = carry_tiles + ex;
+    carry_tiles += tot;
+    ex = block_excl_scan<int64_t>(q, &tot, sh64);
+    if (g < G) d.qtile_off[g] = (int32_t)(carry_q + ex);
+    carry_q += tot;
+  }
+  if (threadIdx.x == 0) {
+    d.row_off[G] = carry_rows;
+    d.tile_off[G] = carry_tiles;
+    d.qtile_off[G] = (int32_t)carry_q;
+    int first = INT_MAX;
+    for (int g = 0; g < G && first == INT_MAX; ++g) {
+      // lowest graph with a size error (device-detected errors lower it later)
+      if (d.status[g] != PREDTOP_OK) first = g;
+    }
+    *d.first_bad = first;
+  }
+}
+
+// K1: validation + successor CSR + Kahn levels / depth.  One CTA per graph.
+__global__ void __launch_bounds__(256) k_depth(DagDev d) {
+  const int g = blockIdx.x;
+  if (d.status[g] != PREDTOP_OK) return;
+  __shared__ int s_err, s_tail;
+  __shared__ int32_t sh32[32];
+  const int64_t n0 = d.node_ptr[g];
+  const int N = (int)(d.node_ptr[g + 1] - n0);
+  const int64_t e0 = d.edge_ptr[g];
+  const int E = (int)(d.edge_ptr[g + 1] - e0);
+  int32_t* indeg = d.indeg + n0;
+  int32_t* soff = d.succ_off + n0 + g;   // N+1
+  int32_t* lptr = d.level_ptr + n0 + g;  // N+1 (first used as fill cursor)
+  int32_t* succ = d.succ + e0;
+  int32_t* topo = d.topo + n0;
+  int32_t* depth = d.depth + n0;
+  const int32_t* src = d.src + e0;
+  const int32_t* dst = d.dst + e0;
+  const int tid = threadIdx.x, nt = blockDim.x;
+
+  if (tid == 0) { s_err = 0; s_tail = 0; soff[0] = 0; }
+  for (int v = tid; v < N; v += nt) { indeg[v] = 0; soff[v + 1] = 0; }
+  __syncthreads();
+  for (int e = tid; e < E; e += nt) {
+    const int s = src[e], t = dst[e];
+    if (s < 0 || s >= N || t < 0 || t >= N) atomicOr(&s_err, 1);
+    else if (s == t) atomicOr(&s_err, 2);
+    else {
+      atomicAdd(&indeg[t], 1);
+      atomicAdd(&soff[s + 1], 1);
+    }
+  }
+  __syncthreads();
+  if (s_err) {
+    if (tid == 0) {
+      d.status[g] = (s_err & 1) ? PREDTOP_ERR_RANGE : PREDTOP_ERR_SELF_LOOP;
+      atomicMin(d.first_bad, g);
+    }
+    for (int v = tid; v < N; v += nt) depth[v] = -1;
+    return;
+  }
+  // inclusive scan of out-degrees -> soff[1..N]
+  int32_t carry = 0;
+  for (int base = 0; base < N; base += nt) {
+    const int v = base + tid;
+    const int32_t c = v < N ? soff[v + 1] : 0;
+    int32_t tot;
+    const int32_t ex = block_excl_scan<int32_t>(c, &tot, sh32);
+    if (v < N) soff[v + 1] = carry + ex + c;
+    carry += tot;
+  }
+  __syncthreads();
+  for (int v = tid; v < N; v += nt) lptr[v] = soff[v];
+  __syncthreads();
+  for (int e = tid; e < E; e += nt) {
+    const int pos = atomicAdd(&lptr[src[e]], 1);
+    succ[pos] = dst[e];
+  }
+  __syncthreads();
+  // Kahn, level synchronous: a node enters level l+1 when its last
+  // predecessor (at level l) is retired, so its level is 1 + max pred level.
+  for (int v = tid; v < N; v += nt)
+    if (indeg[v] == 0) {
+      const int p = atomicAdd(&s_tail, 1);
+      topo[p] = v;
+      depth[v] = 0;
+    }
+  __syncthreads();
+  int lb = 0, le = s_tail, level = 0;
+  if (tid == 0) lptr[0] = 0;
+  while (lb < le) {
+    for (int i = lb + tid; i < le; i += nt) {
+      const int v = topo[i];
+      for (int k = soff[v]; k < soff[v + 1]; ++k) {
+        const int w = succ[k];
+        if (atomicSub(&indeg[w], 1) == 1) {
+          const int p = atomicAdd(&s_tail, 1);
+          topo[p] = w;
+          depth[w] = level + 1;
+        }
+      }
+    }
+    __syncthreads();
+    lb = le;  // level `level` spans topo[lptr[level] .. lptr[level+1])
+    le = s_tail;
+    ++level;
+    if (tid == 0) lptr[level] = lb;
+    __syncthreads();
+  }
+  if (tid == 0) d.num_levels[g] = level;
+  if (le != N) {
+    if (tid == 0) {
+      d.status[g] = PREDTOP_ERR_CYCLE;
+      atomicMin(d.first_bad, g);
+    }
+    for (int v = tid; v < N; v += nt) depth[v] = -1;
+  }
+}
+
+// K2: closure.  grid = (G, slices); dynamic smem `smem_bytes`.
+__global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  const int g = blockIdx.x, slice = blockIdx.y;
+  const int64_t n0 = d.node_ptr[g];
+  const int N = (int)(d.node_ptr[g + 1] - n0);
+  const int st = d.status[g];
+  if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;  // no rows
+  const int W = 2 * ((N + 127) / 128);
+  uint64_t* Rg = d.R + d.row_off[g];
+  const int tid = threadIdx.x, nt = blockDim.x;
+  // Column slicing: CW words of every row resident in shared memory.
+  const int L = d.num_levels[g];
+  const int E = (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]);
+  const size_t csr_bytes = align_up((size_t)4 * ((size_t)N + (N + 1) + E + (L + 1)), 16);
+  int CW = (int)min((int64_t)W, (int64_t)smem_bytes / (8 * (int64_t)N));
+  bool csr_in_smem = false;
+  if ((int64_t)smem_bytes > (int64_t)csr_bytes) {
+    const int cw2 = (int)min((int64_t)W, ((int64_t)smem_bytes - (int64_t)csr_bytes) / (8 * (int64_t)N));
+    if (cw2 >= 1 && (W + cw2 - 1) / cw2 <= (int)gridDim.y) { CW = cw2; csr_in_smem = true; }
+  }
+  const bool global_mode = CW < 1;
+  if (global_mode) CW = max(1, (W + (int)gridDim.y - 1) / (int)gridDim.y);
+  const int word0 = slice * CW;
+  if (word0 >= W) return;
+  const int nw = min(CW, W - word0);
+  if (st != PREDTOP_OK) {  // device-detected error: rows are defined as zero
+    for (int64_t it = tid; it < (int64_t)N * nw; it += nt)
+      Rg[(it / nw) * W + word0 + it % nw] = 0;
+    return;
+  }
+  const int32_t* topo = d.topo + n0;
+  const int32_t* soff = d.succ_off + n0 + g;
+  const int32_t* succ = d.succ + d.edge_ptr[g];
+  const int32_t* lptr = d.level_ptr + n0 + g;
+  uint64_t* Rs;
+  int64_t rs;  // row stride of Rs in words
+  if (csr_in_smem) {
+    int32_t* s_topo = (int32_t*)sm;
+    int32_t* s_soff = s_topo + N;
+    int32_t* s_succ = s_soff + (N + 1);
+    int32_t* s_lptr = s_succ + E;
+    for (int i = tid; i < N; i += nt) s_topo[i] = topo[i];
+    for (int i = tid; i <= N; i += nt) s_soff[i] = soff[i];
+    for (int i = tid; i < E; i += nt) s_succ[i] = succ[i];
+    for (int i = tid; i <= L; i += nt) s_lptr[i] = lptr[i];
+    topo = s_topo; soff = s_soff; succ = s_succ; lptr = s_lptr;
+  }
+  if (global_mode) {
+    Rs = Rg + word0;
+    rs = W;
+  } else {
+    Rs = (uint64_t*)(sm + (csr_in_smem ? csr_bytes : 0));
+    rs = CW;
+  }
+  for (int64_t it = tid; it < (int64_t)N * nw; it += nt) Rs[(it / nw) * rs + it % nw] = 0;
+  __syncthreads();
+  for (int level = L - 1; level >= 0; --level) {
+    const int lb = lptr[level], le = lptr[level + 1];
+    const int items = (le - lb) * nw;
+    for (int it = tid; it < items; it += nt) {
+      const int v = topo[lb + it / nw];
+      const int j = it % nw;
+      const int word = word0 + j;
+      uint64_t acc = 0;
+      for (int k = soff[v]; k < soff[v + 1]; ++k) {
+        const int w = succ[k];
+        acc |= Rs[(int64_t)w * rs + j];
+        if ((w >> 6) == word) acc |= 1ull << (w & 63);
+      }
+      Rs[(int64_t)v * rs + j] = acc;
+    }
+    __syncthreads();
+  }
+  if (!global_mode)
+    for (int64_t it = tid; it < (int64_t)N * nw; it += nt)
+      Rg[(it / nw) * W + word0 + it % nw] = Rs[(it / nw) * rs + it % nw];
+}
+
+// K3: M = R | R^T | I and per-tile popcounts.  grid = (G, YB), 8 warps.
+__global__ void __launch_bounds__(256) k_mask(DagDev d) {
+  const int g = blockIdx.x;
+  const int st = d.status[g];
+  if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
+  const int64_t n0 = d.node_ptr[g];
+  const int N = (int)(d.node_ptr[g + 1] - n0);
+  const int W = 2 * ((N + 127) / 128);
+  const int T = (N + 127) / 128;
+  const uint32_t* R32 = reinterpret_cast<const uint32_t*>(d.R + d.row_off[g]);
+  uint32_t* M32 = reinterpret_cast<uint32_t*>(d.M + d.row_off[g]);
+  int32_t* cnt = d.tile_cnt + d.tile_off[g];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+  const int NB = (N + 31) / 32;
+  const int64_t W32 = 2 * (int64_t)W;  // row stride in 32-bit words
+  for (int ur = blockIdx.y; ur < NB; ur += gridDim.y) {
+    const int U0 = ur * 32;
+    const int u = U0 + lane;
+    for (int vr = warp; vr < 2 * W; vr += nwarp) {
+      const int V0 = vr * 32;  // covers padding columns too (M padding must be 0)
+      const uint32_t direct = (u < N) ? R32[(int64_t)u * W32 + vr] : 0u;
+      const int vrow = V0 + lane;
+      const uint32_t x = (vrow < N) ? R32[(int64_t)vrow * W32 + ur] : 0u;
+      uint32_t t = 0;
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const uint32_t b = __ballot_sync(0xffffffffu, (x >> i) & 1u);
+        if (lane == i) t = b;
+      }
+      uint32_t m = direct | t;
+      if (U0 == V0 && u < N) m |= 1u << lane;
+      if (u >= N) m = 0;
+      if (u < N) M32[(int64_t)u * W32 + vr] = m;
+      int c = __popc(m);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+      if (lane == 0 && c && V0 < N) atomicAdd(&cnt[(U0 / 128) * T + V0 / 128], c);
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_classify(DagDev d) {
+  const int g = blockIdx.x;
+  const int st = d.status[g];
+  if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
+  __shared__ unsigned long long s_pairs;
+  const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+  const int T = (N + 127) / 128;
+  const int32_t* cnt = d.tile_cnt + d.tile_off[g];
+  uint8_t* cls = d.tile_cls + d.tile_off[g];
+  if (threadIdx.x == 0) s_pairs = 0;
+  __syncthreads();
+  unsigned long long local = 0;
+  for (int t = threadIdx.x; t < T * T; t += blockDim.x) {
+    const int qt = t / T, kt = t % T;
+    const int64_t cells = (int64_t)min(128, N - qt * 128) * min(128, N - kt * 128);
+    const int c = cnt[t];
+    cls[t] = (uint8_t)(c == 0 ? 0 : (c == cells ? 2 : 1));
+    local += (unsigned long long)c;
+  }
+  atomicAdd(&s_pairs, local);  // integer: order-independent
+  __syncthreads();
+  if (threadIdx.x == 0) d.pairs[g] = (int64_t)s_pairs;
+}
+
+__global__ void k_work(DagDev d) {
+  const int g = blockIdx.x;
+  const int st = d.status[g];
+  if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
+  const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+  const int T = (N + 127) / 128;
+  for (int qt = threadIdx.x; qt < T; qt += blockDim.x) d.work[d.qtile_off[g] + qt] = make_int2(g, qt);
+}
+
+__global__ void k_copy_words(const int64_t* total, const uint64_t* from, uint64_t* to) {
+  const int64_t n = *total;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    to[i] = from[i];
+}
+
+predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
+  const predtop_batch_desc& b = dag->desc;
+  const DagDev& d = dag->d;
+  const int G = b.num_graphs;
+  PT_CUDA_TRY(cudaMemsetAsync(d.tile_cnt, 0, sizeof(int32_t) * (size_t)dag->tiles_bound, st));
+{
+    ProfScope _p(PK_DAG_META, st);
+    k_meta<<<1, 1024, 0, st>>>(d, G, b.max_nodes);
+    PT_LAUNCH_CHECK();
+  }
+{
+    ProfScope _p(PK_DAG_DEPTH, st);
+    k_depth<<<G, 256, 0, st>>>(d);
+    PT_LAUNCH_CHECK();
+  }
+  // closure: shared memory for a column slice of all rows of the largest graph
+  // (+ its CSR when it fits); several CTAs per SM for small graphs.
+  const int64_t maxN = b.max_nodes;
+  const int64_t Wmax = dag->max_words;
+  int64_t want = maxN * Wmax * 8 + 4 * (4 * maxN + 8) + 16;  // R slice + CSR (E ~ 2N)
+  int smem = (int)std::min<int64_t>(want, 200 * 1024);
+  smem = (int)align_up((size_t)smem, 1024);
+  PT_CUDA_TRY(cudaFuncSetAttribute(k_closure, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   200 * 1024));
+  int64_t cw = std::max<int64_t>(1, std::min<int64_t>(Wmax, (int64_t)smem / (8 * maxN)));
+  int64_t slices = ceil_div(Wmax, cw);
+  if ((int64_t)smem < 8 * maxN) slices = std::min<int64_t>(ceil_div(Wmax, 2), 65535);  // global mode
+  dim3 gc(G, (unsigned)std::max<int64_t>(1, slices));
+{
+    ProfScope _p(PK_DAG_CLOSURE, st);
+    k_closure<<<gc, 256, smem, st>>>(d, smem);
+    PT_LAUNCH_CHECK();
+  }
+  const int NBmax = (int)ceil_div(maxN, 32);
+  dim3 gm(G, (unsigned)std::min(NBmax, 64));
+{
+    ProfScope _p(PK_DAG_MASK, st);
+    k_mask<<<gm, 256, 0, st>>>(d);
+    PT_LAUNCH_CHECK();
+  }
+{
+    ProfScope _p(PK_DAG_CLASSIFY, st);
+    k_classify<<<G, 256, 0, st>>>(d);
+    PT_LAUNCH_CHECK();
+  }
+{
+    ProfScope _p(PK_DAG_WORK, st);
+    k_work<<<G, 128, 0, st>>>(d);
+    PT_LAUNCH_CHECK();
+  }
+  return PREDTOP_OK;
+}
+
+predtop_status dag_copy_bits(const predtop_dag_s* dag, const uint64_t* from, uint64_t* to,
+                             cudaStream_t st) {
+  const int G = dag->desc.num_graphs;
+{
+    ProfScope _p(PK_COPY, st);
+    k_copy_words<<<592, 256, 0, st>>>(dag->d.row_off + G, from, to);
+    PT_LAUNCH_CHECK();
+  }
+  return PREDTOP_OK;
+}
+
+}  // namespace predtop

@@ -1,0 +1,162 @@
+// embed_readout.cu -- node embedding (Table I features + DAGPE) and the
+// graph readout (global add pool + MLP head), both fp32 on CUDA cores.
+//
+// K4  x0[v] = b_in + W_in[:,op] + sum_j ln(1+dims_j) W_in[:,64+j]
+//           + W_in[:,68+dtype] + W_in[:,76+kind] + PE(depth v)
+//     (Table I; log scaling P:167; DAGPE P:137, sinusoidal PE of
+//      [34] over the depth, reading R5).  The one-hot product is a row gather
+//      of the transposed W_in; the PE comes from a per-call table indexed by
+//      depth, computed in fp64 (angles up to ~1e4 rad for deep graphs).
+// K8  g = sum_n x_n (Eqn 2; mean if pool = MEAN), then
+//     y = w_o . ReLU(H_2 ReLU(H_1 g + c_1) + c_2) + c_o
+//     One CTA per graph, fixed summation order: deterministic per graph.
+#include "internal.h"
+
+namespace predtop {
+
+__global__ void k_pe_table(float* pe, int rows, int d) {
+  const int half = d / 2;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (int64_t)rows * half;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int depth = (int)(i / half), k = (int)(i % half);
+    const double w = pow(10000.0, -(2.0 * k) / d);
+    double s, c;
+    sincos((double)depth * w, &s, &c);
+    pe[(int64_t)depth * d + 2 * k] = (float)s;
+    pe[(int64_t)depth * d + 2 * k + 1] = (float)c;
+  }
+}
+
+predtop_status pe_table_launch(float* pe, int rows, int d, cudaStream_t st) {
+  const int64_t n = (int64_t)rows * (d / 2);
+  const int blocks = (int)std::min<int64_t>(ceil_div(n, 256), 148 * 8);
+{
+    ProfScope _p(PK_PE, st);
+    k_pe_table<<<blocks, 256, 0, st>>>(pe, rows, d);
+    PT_LAUNCH_CHECK();
+  }
+  return PREDTOP_OK;
+}
+
+template <int D>
+__global__ void __launch_bounds__(256) k_embed(const float* __restrict__ WT, const float* __restrict__ b,
+                                               const predtop_node_feat* __restrict__ feats,
+                                               const int32_t* __restrict__ depth,
+                                               const float* __restrict__ pe, int64_t n_tot,
+                                               float* __restrict__ x32, __half* __restrict__ x16) {
+  constexpr int PER = D / 32;  // columns per lane
+  const int lane = threadIdx.x & 31;
+  const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t v = warp0; v < n_tot; v += nwarps) {
+    const predtop_node_feat f = feats[v];
+    int dep = depth[v];
+    if (dep < 0) dep = 0;  // invalid graph: latency is NaN anyway
+    float l[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) l[j] = log1pf((float)f.dims[j]);
+    const float* rop = f.op < PREDTOP_NUM_OPS ? WT + (size_t)f.op * D : nullptr;
+    const float* rdt = f.dtype < PREDTOP_NUM_DTYPES ? WT + (size_t)(68 + f.dtype) * D : nullptr;
+    const float* rkd = f.kind < PREDTOP_NUM_KINDS ? WT + (size_t)(76 + f.kind) * D : nullptr;
+    const float* rpe = pe + (size_t)dep * D;
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int c = k * 32 + lane;
+      float acc = b[c];
+      if (rop) acc += rop[c];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc += l[j] * WT[(size_t)(64 + j) * D + c];
+      if (rdt) acc += rdt[c];
+      if (rkd) acc += rkd[c];
+      acc += rpe[c];
+      x32[v * D + c] = acc;
+      x16[v * D + c] = __float2half_rn(acc);
+    }
+  }
+}
+
+predtop_status embed_launch(const predtop_model_s* m, const predtop_dag_s* dag, const float* pe,
+                            float* x32, __half* x16, cudaStream_t st) {
+  const int64_t n = dag->desc.total_nodes;
+  const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 8), 148 * 16));
+  const DagDev& d = dag->d;
+  ProfScope _p(PK_EMBED, st);
+#define PT_EMBED(D)                                                                  \
+  case D:                                                                            \
+    k_embed<D><<<blocks, 256, 0, st>>>(m->W_inT, m->b_in, d.feats, d.depth, pe, n, x32, x16); \
+    break;
+  switch (m->cfg.d_model) {
+    PT_EMBED(32)
+    PT_EMBED(64)
+    PT_EMBED(128)
+    PT_EMBED(256)
+    default: set_error("unsupported d_model"); return PREDTOP_ERR_UNSUPPORTED;
+  }
+#undef PT_EMBED
+  PT_LAUNCH_CHECK();
+  return PREDTOP_OK;
+}
+
+// ---------------------------------------------------------------- readout
+template <int D>
+__global__ void __launch_bounds__(D) k_readout(const float* __restrict__ x32,
+                                               const int64_t* __restrict__ node_ptr,
+                                               const int32_t* __restrict__ status, int pool_mean,
+                                               const float* __restrict__ H1T, const float* __restrict__ c1,
+                                               const float* __restrict__ H2T, const float* __restrict__ c2,
+                                               const float* __restrict__ w_o, const float* __restrict__ c_o,
+                                               float* __restrict__ latency) {
+  __shared__ float sg[D], sz[D], red[D / 32];
+  const int g = blockIdx.x, c = threadIdx.x;
+  if (status[g] != PREDTOP_OK) {
+    if (c == 0) latency[g] = __int_as_float(0x7fc00000);  // NaN
+    return;
+  }
+  const int64_t n0 = node_ptr[g], n1 = node_ptr[g + 1];
+  float s = 0.f;
+  for (int64_t v = n0; v < n1; ++v) s += x32[v * D + c];  // Eqn 2, node order
+  if (pool_mean) s /= (float)(n1 - n0);
+  sg[c] = s;
+  __syncthreads();
+  float z = c1[c];
+  for (int i = 0; i < D; ++i) z += H1T[i * D + c] * sg[i];
+  sz[c] = fmaxf(z, 0.f);
+  __syncthreads();
+  z = c2[c];
+  for (int i = 0; i < D; ++i) z += H2T[i * D + c] * sz[i];
+  z = fmaxf(z, 0.f);
+  float p = w_o[c] * z;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(0xffffffffu, p, o);
+  if ((c & 31) == 0) red[c >> 5] = p;
+  __syncthreads();
+  if (c == 0) {
+    float y = 0.f;
+    for (int w = 0; w < D / 32; ++w) y += red[w];
+    latency[g] = y + c_o[0];
+  }
+}
+
+predtop_status readout_launch(const predtop_model_s* m, const predtop_dag_s* dag, const float* x32,
+                              float* latency, cudaStream_t st) {
+  const int G = dag->desc.num_graphs;
+  const DagDev& d = dag->d;
+  ProfScope _p(PK_READOUT, st);
+#define PT_READ(D)                                                                       \
+  case D:                                                                                \
+    k_readout<D><<<G, D, 0, st>>>(x32, d.node_ptr, d.status, m->cfg.pool, m->H1T, m->c1, \
+                                  m->H2T, m->c2, m->w_o, m->c_o, latency);               \
+    break;
+  switch (m->cfg.d_model) {
+    PT_READ(32)
+    PT_READ(64)
+    PT_READ(128)
+    PT_READ(256)
+    default: set_error("unsupported d_model"); return PREDTOP_ERR_UNSUPPORTED;
+  }
+#undef PT_READ
+  PT_LAUNCH_CHECK();
+  return PREDTOP_OK;
+}
+
+}  // namespace predtop

@@ -1,0 +1,133 @@
+// internal.h -- handle structs and launcher prototypes shared by the .cu files
+// of libpredtop.  Not part of the ABI.
+#pragma once
+#include <cuda.h>
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include <vector>
+
+#include "common.cuh"
+
+namespace predtop {
+
+// Device views of a built batch of stage DAGs (all carved from the caller's
+// build_dag workspace, except the borrowed input arrays).
+struct DagDev {
+  // borrowed inputs
+  const int64_t* node_ptr;
+  const int64_t* edge_ptr;
+  const int32_t* src;
+  const int32_t* dst;
+  const predtop_node_feat* feats;
+  // per graph
+  int32_t* status;     // [G]   predtop_status of the graph
+  int32_t* num_levels; // [G]
+  int64_t* row_off;    // [G+1] word offset of the graph's bitset rows (prefix of N_g*W_g)
+  int64_t* tile_off;   // [G+1] prefix of T_g^2
+  int32_t* qtile_off;  // [G+1] prefix of T_g (attention work items)
+  int64_t* pairs;      // [G]   |A_g|
+  int32_t* first_bad;  // [1]   lowest bad graph (INT_MAX if none)
+  // per node / edge
+  int32_t* depth;      // [N_tot] caller order
+  int32_t* topo;       // [N_tot] graph-local ids by level
+  int32_t* level_ptr;  // [N_tot + G] graph g at node_ptr[g] + g
+  int32_t* succ_off;   // [N_tot + G] graph g at node_ptr[g] + g
+  int32_t* succ;       // [E]  graph-local successor lists
+  int32_t* indeg;      // [N_tot]
+  // bitsets and tiles
+  uint64_t* R;         // [sum N_g W_g]
+  uint64_t* M;         // [sum N_g W_g]
+  int32_t* tile_cnt;   // [sum T_g^2]
+  uint8_t* tile_cls;   // [sum T_g^2]
+  int2* work;          // [qtile bound] (graph, q-tile) attention work items
+};
+
+}  // namespace predtop
+
+struct predtop_dag_s {
+  predtop_batch_desc desc;
+  predtop::DagDev d;
+  int64_t words_bound;  // upper bound of sum N_g W_g
+  int64_t tiles_bound;  // upper bound of sum T_g^2
+  int64_t qtiles_bound; // upper bound of sum T_g
+  int32_t max_words;    // 2*ceil(max_nodes/128)
+};
+
+namespace predtop {
+
+constexpr int kMaxLayers = 16;
+
+struct LayerDev {
+  __half* Wqkv;  // [3d][d]
+  float* bqkv;   // [3d]
+  __half* Wo;    // [d][d]
+  float* bo;
+  float* g1;
+  float* be1;
+  __half* W1;    // [dff][d]
+  float* b1;
+  __half* W2;    // [d][dff]
+  float* b2;
+  float* g2;
+  float* be2;
+  CUtensorMap tm_qkv, tm_o, tm_1, tm_2;  // B-operand TMA maps
+};
+
+}  // namespace predtop
+
+struct predtop_model_s {
+  predtop_model_config cfg;
+  float* W_inT;  // [F][d] (transposed: one-hot rows are gathers)
+  float* b_in;   // [d]
+  predtop::LayerDev layer[predtop::kMaxLayers];
+  float* H1T;    // [d][d] transposed (in-major)
+  float* c1;
+  float* H2T;
+  float* c2;
+  float* w_o;    // [d]
+  float* c_o;    // [1]
+  int bn_qkv, bn_ff1;  // GEMM N-tile widths
+};
+
+namespace predtop {
+
+// ---- dag.cu
+predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st);
+predtop_status dag_copy_bits(const predtop_dag_s* dag, const uint64_t* from, uint64_t* to,
+                             cudaStream_t st);
+
+// ---- tma.cu
+bool encode_tma_2d_f16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
+                       uint32_t box_inner, uint32_t box_outer);
+
+// ---- gemm.cu
+enum GemmEpi { EPI_BIAS_F16 = 0, EPI_BIAS_RELU_F16 = 1, EPI_BIAS_RESID_LN = 2 };
+struct GemmArgs {
+  int M, K, N;           // rows, reduction, total output columns
+  const float* bias;     // [N]
+  __half* out16;         // [M][N]
+  float* out32;          // [M][N]   (LN epilogue)
+  const float* resid32;  // [M][N]   (LN epilogue; may alias out32)
+  const float* gamma;
+  const float* beta;
+  float eps;
+};
+predtop_status gemm_launch(const CUtensorMap* tmA, const CUtensorMap* tmB, int bn, int epi,
+                           const GemmArgs& a, cudaStream_t st);
+int gemm_pick_bn(int N);
+
+// ---- embed.cu / readout.cu / attention.cu / plan.cu
+predtop_status pe_table_launch(float* pe, int max_depth, int d, cudaStream_t st);
+predtop_status embed_launch(const predtop_model_s* m, const predtop_dag_s* dag, const float* pe,
+                            float* x32, __half* x16, cudaStream_t st);
+predtop_status attention_launch(const predtop_dag_s* dag, int d, int H, const __half* qkv,
+                                __half* out, cudaStream_t st);
+predtop_status readout_launch(const predtop_model_s* m, const predtop_dag_s* dag, const float* x32,
+                              float* latency, cudaStream_t st);
+predtop_status plan_launch(int64_t P, const int64_t* plan_ptr, const int32_t* plan_stage,
+                           const int32_t* B, const float* t, int64_t num_stages, double* T,
+                           int64_t* first_bad, cudaStream_t st);
+predtop_status argmin_launch(int64_t n, const double* T, int64_t* best, cudaStream_t st);
+
+}  // namespace predtop

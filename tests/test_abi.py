@@ -1,0 +1,94 @@
+"""C-ABI contract checks that need no GPU: the library builds for sm_100a,
+loads, exports every symbol include/predtop.h declares (and nothing else),
+carries tcgen05 / TMA instructions, and host-side validation and the no-GPU
+path fail loudly instead of falling back."""
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+from paper_conf_ipps_acharyas25_b200 import build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "predtop.h")
+
+
+@pytest.fixture(scope="module")
+def libpath():
+    return build.build_library()
+
+
+def _declared():
+    txt = open(HEADER).read()
+    return sorted(set(re.findall(r"^PREDTOP_API [^;(]*?\b(predtop_\w+)\(", txt, flags=re.M)))
+
+
+def test_exports_match_header(libpath):
+    decl = _declared()
+    assert len(decl) >= 20
+    out = subprocess.run(["nm", "-D", "--defined-only", libpath], capture_output=True, text=True).stdout
+    exported = sorted({l.split()[-1] for l in out.splitlines() if " T " in l})
+    assert exported == decl
+    L = ctypes.CDLL(libpath)
+    for name in decl:
+        assert hasattr(L, name), name
+
+
+def test_sass_is_blackwell_native(libpath):
+    sass = subprocess.run(["cuobjdump", "-sass", libpath], capture_output=True, text=True).stdout
+    assert "UTCHMMA" in sass        # tcgen05.mma
+    assert "UTMALDG" in sass        # TMA tile loads
+    assert "LDTM" in sass           # tcgen05.ld (TMEM -> registers)
+    assert "sm_100a" in subprocess.run(["cuobjdump", "-lelf", libpath], capture_output=True,
+                                       text=True).stdout
+
+
+def test_host_validation_without_gpu(libpath):
+    from paper_conf_ipps_acharyas25_b200 import predtop as pt
+    L = pt.lib()
+    assert L.predtop_abi_version() == 1
+    assert L.predtop_status_string(-4) == b"graph has a cycle"
+    d = pt.BatchDesc(0, 1, 0, 0, 0)
+    assert L.predtop_build_dag_workspace(ctypes.byref(d)) == 0          # G < 1
+    d = pt.BatchDesc(3, 10, 2, 0, 0)
+    assert L.predtop_build_dag_workspace(ctypes.byref(d)) == 0          # N_tot < G
+    d = pt.BatchDesc(4, 330, 1200, 1700, 0)
+    assert L.predtop_build_dag_workspace(ctypes.byref(d)) > 1200 * 6 * 8 * 2
+    h = ctypes.c_void_p()
+    st = L.predtop_build_dag(ctypes.byref(d), None, None, None, None, None, None, 0, None,
+                             ctypes.byref(h), None, None)
+    assert st == pt.INVALID_ARG and not h.value
+    cfg = pt.ModelConfig(4, 128, 8, 512, 0, 1e-5)
+    assert L.predtop_model_weight_floats(ctypes.byref(cfg)) > 0
+    bad = pt.ModelConfig(4, 96, 8, 512, 0, 1e-5)                        # d_h = 12
+    assert L.predtop_model_weight_floats(ctypes.byref(bad)) == 0
+    assert L.predtop_plan_latency(-1, None, None, None, None, 0, None, None, 0, 0, None, None) == pt.INVALID_ARG
+
+
+def test_weight_blob_size_matches_generator(libpath):
+    from paper_conf_ipps_acharyas25_b200 import predtop as pt, synth
+    for name, c in synth.MODEL_CONFIGS.items():
+        cfg = pt.ModelConfig(c["num_layers"], c["d_model"], c["num_heads"], c["d_ff"], 0, 1e-5)
+        n = pt.lib().predtop_model_weight_floats(ctypes.byref(cfg))
+        assert n == len(synth.pack_weights(c, synth.model_weights(c))), name
+
+
+def test_no_gpu_fails_loudly(libpath):
+    """Without a CUDA device, work-launching calls return PREDTOP_ERR_CUDA."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    from paper_conf_ipps_acharyas25_b200 import predtop as pt
+    L = pt.lib()
+    d = pt.BatchDesc(1, 4, 4, 3, 0)
+    ws = ctypes.create_string_buffer(L.predtop_build_dag_workspace(ctypes.byref(d)) + 256)
+    base = (ctypes.addressof(ws) + 255) // 256 * 256
+    dummy = ctypes.c_void_p(base)
+    h = ctypes.c_void_p()
+    st = L.predtop_build_dag(ctypes.byref(d), dummy, dummy, dummy, dummy, dummy, dummy,
+                             L.predtop_build_dag_workspace(ctypes.byref(d)), None, ctypes.byref(h),
+                             None, None)
+    assert st == pt.CUDA
+    assert b"device" in L.predtop_last_error()

@@ -1,0 +1,124 @@
+"""GPU parity of the DAG-Transformer forward (predtop_stage_forward) against the
+CPU fp64 oracle, per graph relative error <= 2e-3 (BASELINE.json north star),
+plus layer-wise taps (localisation), determinism and shard invariance
+(per-graph outputs bit-identical whatever the batch composition)."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_ipps_acharyas25_b200 import synth
+
+pytestmark = pytest.mark.gpu
+TOL = 2e-3
+
+
+@pytest.fixture(scope="module")
+def pt():
+    from paper_conf_ipps_acharyas25_b200 import build, predtop
+    build.build_library()
+    assert torch.cuda.is_available()
+    return predtop
+
+
+def _model(pt, name, **kw):
+    cfg = dict(synth.MODEL_CONFIGS[name])
+    cfg.update(kw)
+    blob = synth.pack_weights(cfg, synth.model_weights(cfg))
+    return cfg, blob, pt.Model(cfg, blob)
+
+
+def _gpu_latency(pt, model, batch):
+    dag = pt.Dag(pt.DeviceBatch.from_host(batch))
+    assert dag.status == pt.OK
+    y = model.forward(dag)
+    torch.cuda.synchronize()
+    return y.cpu().numpy().astype(np.float64), dag
+
+
+def _rel(a, b):
+    return np.abs(a - b) / np.abs(b)
+
+
+@pytest.mark.parametrize("name, batch_fn", [
+    ("tiny", lambda: synth.tiny_batch()),
+    ("paper", lambda: synth.stage_batch("gpt", 12, seed=11)),
+    ("gpt", lambda: synth.stage_batch("gpt", 24)),
+    ("moe", lambda: synth.stage_batch("moe", 3)),
+])
+def test_latency_parity(pt, oracle_mod, name, batch_fn):
+    cfg, blob, model = _model(pt, name)
+    batch = batch_fn()
+    y, _ = _gpu_latency(pt, model, batch)
+    want = oracle_mod.forward_batch(cfg, blob, batch)
+    err = _rel(y, want)
+    print(f"{name}: max rel err {err.max():.3e} median {np.median(err):.3e}")
+    assert np.isfinite(y).all()
+    assert err.max() <= TOL
+
+
+def test_mean_pool_and_relabelled(pt, oracle_mod):
+    cfg, blob, model = _model(pt, "gpt", pool=1)
+    b = synth.stage_batch("gpt", 4, first_graph=300)
+    gs = []
+    for g in range(b.num_graphs):
+        n, s, d, f = b.graph(g)
+        s2, d2, f2 = synth.relabel(n, s, d, f, synth.CounterRng(5, g).permutation(n))
+        gs.append((n, s2, d2, f2))
+    rb = synth.pack_graphs(gs)
+    y, _ = _gpu_latency(pt, model, rb)
+    want = oracle_mod.forward_batch(cfg, blob, rb)
+    assert _rel(y, want).max() <= TOL
+
+
+def test_layer_taps(pt, oracle_mod):
+    """Embedding (fp32) and per-layer node embeddings against the oracle taps."""
+    cfg, blob, model = _model(pt, "gpt")
+    b = synth.stage_batch("gpt", 3, first_graph=50)
+    dag = pt.Dag(pt.DeviceBatch.from_host(b))
+    taps = [oracle_mod.forward(cfg, blob, *b.graph(g), taps=True)[2] for g in range(3)]
+    for layer in range(-1, cfg["num_layers"]):
+        x = model.node_embeddings(dag, layer).cpu().numpy()
+        want = np.concatenate([t[layer + 1] for t in taps])
+        err = np.abs(x - want).max()
+        print(f"layer {layer}: max abs err {err:.3e}")
+        assert err < (1e-4 if layer < 0 else 5e-2)
+
+
+def test_determinism_and_shard_invariance(pt):
+    cfg, blob, model = _model(pt, "gpt")
+    full = synth.stage_batch("gpt", 40)
+    y1, _ = _gpu_latency(pt, model, full)
+    y2, _ = _gpu_latency(pt, model, full)
+    np.testing.assert_array_equal(y1, y2)
+    idx = [39, 3, 17, 8, 22]
+    ys, _ = _gpu_latency(pt, model, full.subset(idx))
+    np.testing.assert_array_equal(ys, y1[idx])
+
+
+def test_invalid_graph_nan_others_exact(pt):
+    cfg, blob, model = _model(pt, "tiny")
+    tb = synth.tiny_batch()
+    gs = [tb.graph(g) for g in range(4)]
+    f = gs[0][3]
+    bad = (8, np.array([0, 1, 2], np.int32), np.array([1, 2, 0], np.int32), f)
+    b2 = synth.pack_graphs(gs[:2] + [bad] + gs[2:])
+    dag = pt.Dag(pt.DeviceBatch.from_host(b2), no_sync=True)
+    y = model.forward(dag).cpu().numpy()
+    yref, _ = _gpu_latency(pt, model, tb)
+    assert np.isnan(y[2])
+    np.testing.assert_array_equal(np.delete(y, 2), yref)
+
+
+@pytest.mark.slow
+def test_full_gpt_config_sampled(pt, oracle_mod):
+    """configs[1] at full size (1024 graphs, the bench launch configuration);
+    oracle on a sample of graphs."""
+    cfg, blob, model = _model(pt, "gpt")
+    batch = synth.stage_batch("gpt", 1024)
+    y, _ = _gpu_latency(pt, model, batch)
+    assert np.isfinite(y).all()
+    sample = list(range(0, 1024, 37)) + [1023]
+    want = oracle_mod.forward_batch(cfg, blob, batch, graphs=sample)
+    err = _rel(y[sample], want)
+    print(f"gpt full: max rel err {err.max():.3e} median {np.median(err):.3e}")
+    assert err.max() <= TOL
