@@ -363,7 +363,7 @@ def main():
             roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                     "frac": ach / peaks["hbm_gbs"]}
         else:
-            clk = clk_mhz = (clk.summary()["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0))
+            clk_mhz = (clk.summary()["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0))
             peak = MUFU_EX2_PER_CLK_SM * NUM_SMS * clk_mhz * 1e6 / 1e9
             ach = units / sec / 1e9
             tflops = 4.0 * d * A / sec / 1e12

@@ -4,12 +4,19 @@
 //   FFN-1                 D = ReLU(H W_1^T + b_1)            -> fp16
 //   O-proj / FFN-2 + LN   x' = LN(resid + A W^T + b)*g + be  -> fp32 + fp16
 //
-// One CTA computes a 128 x BN tile: TMA streams 128 x KCH (A) and BN x KCH
-// (B) fp16 tiles into a 2-stage shared-memory ring (128B/64B swizzle, the UMMA
-// K-major canonical layout), one elected thread issues tcgen05.mma
-// (M=128, N=BN, K=16, fp32 accumulate in TMEM), and all four warps run the
-// epilogue straight out of TMEM (tcgen05.ld, thread i <-> row i).  The LN
-// epilogue needs the whole row in one CTA, so it runs with BN = d.
+// Persistent, warp-specialised kernel, one CTA per SM:
+//   warp 0      TMA producer: 128 x KCH (A) and BN x KCH (B) fp16 tiles into an
+//               S-stage shared-memory ring (128B/64B swizzle = the UMMA K-major
+//               canonical layout)
+//   warp 1      MMA issuer: one elected thread issues tcgen05.mma
+//               (M=128, N=BN, K=16, fp32 accumulate) into one of TWO TMEM
+//               accumulators, so tile i+1's MMAs overlap tile i's epilogue
+//   warps 2..5  epilogue: tcgen05.ld (thread <-> row), bias / ReLU / residual
+//               + LayerNorm in registers, swizzled staging tile in shared
+//               memory, TMA bulk-tensor store (coalesced, ragged tail clipped
+//               by the tensor map).  The LN epilogue TMA-loads the fp32
+//               residual tile into the same staging buffer and writes the
+//               result back in place.
 #include <algorithm>
 
 #include "internal.h"
@@ -19,206 +26,323 @@ namespace predtop {
 
 namespace {
 
-constexpr int kStages = 2;
-constexpr int kThreads = 128;
+constexpr int kThreads = 192;   // 6 warps
+constexpr int kEpiThreads = 128;
+constexpr int kSmemBudget = 225 * 1024;
 
 template <int BN>
-constexpr uint32_t tmem_cols() {
-  return BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : BN <= 256 ? 256 : 512;
+constexpr uint32_t tmem_cols2() {  // two accumulators of BN fp32 columns
+  return 2 * BN <= 32 ? 32 : 2 * BN <= 64 ? 64 : 2 * BN <= 128 ? 128 : 2 * BN <= 256 ? 256 : 512;
 }
 
-template <int BN, int KCH>
-constexpr int smem_bytes() {
-  return kStages * (128 * KCH * 2 + BN * KCH * 2) + 1024;
-}
+template <int BN, int KCH, int EPI>
+struct Cfg {
+  static constexpr int A_BYTES = 128 * KCH * 2;
+  static constexpr int B_BYTES = BN * KCH * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int OUT16_BOX = BN % 64 == 0 ? 64 : 32;           // f16 store box (elements)
+  static constexpr int OUT32_BYTES = EPI == EPI_BIAS_RESID_LN ? 128 * BN * 4 : 0;
+  // LN with a wide row (d = 256): no room for a separate fp16 staging tile next
+  // to the fp32 one and a 2-stage ring; the fp16 copy is then stored directly.
+  static constexpr bool F16_DIRECT =
+      EPI == EPI_BIAS_RESID_LN && 128 * BN * 6 + 2 * STAGE_BYTES + 1024 > kSmemBudget;
+  static constexpr int OUT16_BYTES = F16_DIRECT ? 0 : 128 * BN * 2;
+  static constexpr int STAGING = OUT16_BYTES + OUT32_BYTES;
+  static constexpr int STAGES_FIT = (kSmemBudget - STAGING - 1024) / STAGE_BYTES;
+  static constexpr int STAGES = STAGES_FIT > 4 ? 4 : STAGES_FIT;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + STAGING + 1024;
+  static_assert(STAGES >= 2, "shared memory budget");
+};
 
 __device__ __forceinline__ uint32_t pack_half2(float a, float b) {
   __half2 h = __floats2half2_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
+// Byte offset of 16-byte chunk `chunk` of row `r` inside a swizzled TMA box
+// whose rows are `RB` bytes (128 -> SWIZZLE_128B, 64 -> SWIZZLE_64B).
+template <int RB>
+__device__ __forceinline__ uint32_t swz(int r, int chunk) {
+  constexpr int mask = RB == 128 ? 7 : 3;
+  const uint32_t off = (uint32_t)r * RB + (uint32_t)chunk * 16;
+  return off ^ (((off >> 7) & mask) << 4);
+}
+
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void epi_bar() {  // named barrier over the 4 epilogue warps
+  asm volatile("bar.sync 1, %0;" ::"n"(kEpiThreads) : "memory");
+}
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* smem, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(sm100::smem_u32(smem)), "r"(c0), "r"(c1)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() {
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sm100::smem_u32(bar)) : "memory");
+}
+
+struct Maps {
+  CUtensorMap a, b, out16, x32;  // x32: residual load + fp32 store (LN epilogue)
+};
+
 template <int BN, int KCH, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
-    k_gemm(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-           GemmArgs args) {
-  constexpr int SW = KCH * 2;  // swizzle bytes = row bytes of a K chunk
-  constexpr int A_BYTES = 128 * KCH * 2;
-  constexpr int B_BYTES = BN * KCH * 2;
-  constexpr uint32_t NCOLS = tmem_cols<BN>();
+    k_gemm(const __grid_constant__ Maps maps, GemmArgs args) {
+  using C = Cfg<BN, KCH, EPI>;
+  constexpr int SW = KCH * 2;
+  constexpr int S = C::STAGES;
+  constexpr uint32_t NCOLS = tmem_cols2<BN>();
   extern __shared__ unsigned char dsm[];
   unsigned char* base = (unsigned char*)(((uintptr_t)dsm + 1023) & ~(uintptr_t)1023);
-  unsigned char* sA = base;
-  unsigned char* sB = base + kStages * A_BYTES;
-  __shared__ __align__(8) uint64_t full_bar[kStages], empty_bar[kStages], acc_bar;
+  unsigned char* ring = base;
+  unsigned char* st16 = base + S * C::STAGE_BYTES;       // f16 output staging
+  unsigned char* st32 = st16 + C::OUT16_BYTES;           // fp32 residual / output staging
+  __shared__ __align__(8) uint64_t full_bar[S], empty_bar[S], tfull[2], tempty[2], resid_bar;
   __shared__ uint32_t tmem_slot;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m0 = blockIdx.x * 128;
-  const int n0 = blockIdx.y * BN;
+  const int ntn = args.N / BN;
+  const int ntiles = (int)ceil_div(args.M, 128) * ntn;
   const int KC = args.K / KCH;
 
   if (threadIdx.x == 0) {
-    sm100::tma_prefetch(&tmA);
-    sm100::tma_prefetch(&tmB);
-    for (int s = 0; s < kStages; ++s) {
+    sm100::tma_prefetch(&maps.a);
+    sm100::tma_prefetch(&maps.b);
+    sm100::tma_prefetch(&maps.out16);
+    if (EPI == EPI_BIAS_RESID_LN) sm100::tma_prefetch(&maps.x32);
+    for (int s = 0; s < S; ++s) {
       sm100::mbar_init(&full_bar[s], 1);
       sm100::mbar_init(&empty_bar[s], 1);
     }
-    sm100::mbar_init(&acc_bar, 1);
+    for (int a = 0; a < 2; ++a) {
+      sm100::mbar_init(&tfull[a], 1);
+      sm100::mbar_init(&tempty[a], kEpiThreads);
+    }
+    sm100::mbar_init(&resid_bar, 1);
     sm100::fence_mbar_init();
   }
-  if (warp == 2) sm100::tmem_alloc<NCOLS>(&tmem_slot);
+  if (warp == 1) sm100::tmem_alloc<NCOLS>(&tmem_slot);
   sm100::tc_fence_before();
   __syncthreads();
   sm100::tc_fence_after();
   const uint32_t tmem = tmem_slot;
 
-  if (warp == 0 && lane == 0) {
-    // ---- TMA producer
-    for (int kc = 0; kc < KC; ++kc) {
-      const int s = kc % kStages;
-      if (kc >= kStages) sm100::mbar_wait(&empty_bar[s], ((kc / kStages) - 1) & 1);
-      sm100::mbar_arrive_expect_tx(&full_bar[s], A_BYTES + B_BYTES);
-      sm100::tma_load_2d(sA + s * A_BYTES, &tmA, &full_bar[s], kc * KCH, m0);
-      sm100::tma_load_2d(sB + s * B_BYTES, &tmB, &full_bar[s], kc * KCH, n0);
-    }
-  } else if (warp == 1 && lane == 0) {
-    // ---- MMA issuer (single thread)
-    constexpr uint32_t idesc = sm100::make_idesc_f16(128, BN);
-    for (int kc = 0; kc < KC; ++kc) {
-      const int s = kc % kStages;
-      sm100::mbar_wait(&full_bar[s], (kc / kStages) & 1);
-      sm100::tc_fence_after();
-      const uint32_t a0 = sm100::smem_u32(sA + s * A_BYTES);
-      const uint32_t b0 = sm100::smem_u32(sB + s * B_BYTES);
-#pragma unroll
-      for (int kk = 0; kk < KCH / 16; ++kk) {
-        const uint64_t ad = sm100::make_sdesc<SW>(a0 + kk * 32);
-        const uint64_t bd = sm100::make_sdesc<SW>(b0 + kk * 32);
-        sm100::mma_f16_ss(tmem, ad, bd, idesc, (kc | kk) != 0);
-      }
-      sm100::mma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs finish
-    }
-    sm100::mma_commit(&acc_bar);  // accumulator complete
-  }
-  __syncwarp();
-
-  // ---- epilogue: thread (warp w, lane l) owns output row m0 + 32w + l
-  sm100::mbar_wait(&acc_bar, 0);
-  sm100::tc_fence_after();
-  const int row = m0 + warp * 32 + lane;
-  const bool valid = row < args.M;
-  const uint32_t t_row = tmem + ((uint32_t)(warp * 32) << 16);
-  float v[16];
-
-  if constexpr (EPI == EPI_BIAS_F16 || EPI == EPI_BIAS_RELU_F16) {
-    __half* out = args.out16 + (size_t)row * args.N + n0;
-#pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      sm100::tmem_ld16(t_row + c, v);
-      if (valid) {
-        uint32_t p[8];
-#pragma unroll
-        for (int j = 0; j < 16; j += 2) {
-          float x0 = v[j] + __ldg(args.bias + n0 + c + j);
-          float x1 = v[j + 1] + __ldg(args.bias + n0 + c + j + 1);
-          if (EPI == EPI_BIAS_RELU_F16) { x0 = fmaxf(x0, 0.f); x1 = fmaxf(x1, 0.f); }
-          p[j / 2] = pack_half2(x0, x1);
+  if (warp == 0) {
+    if (lane == 0) {  // ---------------- TMA producer
+      int it = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
+        for (int kc = 0; kc < KC; ++kc, ++it) {
+          const int s = it % S;
+          sm100::mbar_wait(&empty_bar[s], ((it / S) & 1) ^ 1);
+          unsigned char* sa = ring + s * C::STAGE_BYTES;
+          sm100::mbar_arrive_expect_tx(&full_bar[s], C::STAGE_BYTES);
+          sm100::tma_load_2d(sa, &maps.a, &full_bar[s], kc * KCH, m0);
+          sm100::tma_load_2d(sa + C::A_BYTES, &maps.b, &full_bar[s], kc * KCH, n0);
         }
-        uint4* o = reinterpret_cast<uint4*>(out + c);
-        o[0] = make_uint4(p[0], p[1], p[2], p[3]);
-        o[1] = make_uint4(p[4], p[5], p[6], p[7]);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---------------- MMA issuer
+      constexpr uint32_t idesc = sm100::make_idesc_f16(128, BN);
+      int it = 0, local = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++local) {
+        const int acc = local & 1;
+        sm100::mbar_wait(&tempty[acc], ((local >> 1) & 1) ^ 1);
+        sm100::tc_fence_after();
+        const uint32_t d_tmem = tmem + (uint32_t)(acc * BN);
+        for (int kc = 0; kc < KC; ++kc, ++it) {
+          const int s = it % S;
+          sm100::mbar_wait(&full_bar[s], (it / S) & 1);
+          sm100::tc_fence_after();
+          const uint32_t a0 = sm100::smem_u32(ring + s * C::STAGE_BYTES);
+          const uint32_t b0 = a0 + C::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < KCH / 16; ++kk)
+            sm100::mma_f16_ss(d_tmem, sm100::make_sdesc<SW>(a0 + kk * 32),
+                              sm100::make_sdesc<SW>(b0 + kk * 32), idesc, (kc | kk) != 0);
+          sm100::mma_commit(&empty_bar[s]);
+        }
+        sm100::mma_commit(&tfull[acc]);
       }
     }
   } else {
-    // LN(resid + acc + bias): three passes over the row (mean, variance,
-    // normalise + store), re-reading TMEM and the fp32 residual each pass.
-    const float* res = args.resid32 + (size_t)row * BN;
-    float sum = 0.f;
-#pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      sm100::tmem_ld16(t_row + c, v);
-      if (valid) {
+    // ---------------- epilogue warps 2..5: TMEM lane quarter q = warp % 4
+    const int q = warp & 3;
+    const int r = q * 32 + lane;  // row within the tile
+    const bool leader = (warp == 2 && lane == 0);
+    int local = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++local) {
+      const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
+      const int acc = local & 1;
+      // staging buffers free again? (previous tile's TMA stores have read them)
+      if (leader) bulk_wait_read0();
+      epi_bar();
+      if (EPI == EPI_BIAS_RESID_LN) {
+        if (leader) {
+          sm100::mbar_arrive_expect_tx(&resid_bar, C::OUT32_BYTES);
 #pragma unroll
-        for (int j = 0; j < 16; ++j) sum += v[j] + __ldg(args.bias + c + j) + res[c + j];
-      }
-    }
-    const float mean = sum * (1.0f / BN);
-    float sq = 0.f;
-#pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      sm100::tmem_ld16(t_row + c, v);
-      if (valid) {
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const float z = v[j] + __ldg(args.bias + c + j) + res[c + j] - mean;
-          sq += z * z;
+          for (int b = 0; b < BN / 32; ++b)
+            sm100::tma_load_2d(st32 + b * 16384, &maps.x32, &resid_bar, n0 + b * 32, m0);
         }
       }
-    }
-    const float rstd = rsqrtf(sq * (1.0f / BN) + args.eps);
-    float* o32 = args.out32 + (size_t)row * BN;
-    __half* o16 = args.out16 + (size_t)row * BN;
+      sm100::mbar_wait(&tfull[acc], (local >> 1) & 1);
+      sm100::tc_fence_after();
+      const uint32_t t_row = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * BN);
+      float v[16];
+      if constexpr (EPI == EPI_BIAS_F16 || EPI == EPI_BIAS_RELU_F16) {
 #pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      sm100::tmem_ld16(t_row + c, v);
-      if (valid) {
-        float y[16];
+        for (int c = 0; c < BN; c += 16) {
+          sm100::tmem_ld16(t_row + c, v);
+          uint32_t p[8];
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const float z = v[j] + __ldg(args.bias + c + j) + res[c + j] - mean;
-          y[j] = z * rstd * __ldg(args.gamma + c + j) + __ldg(args.beta + c + j);
+          for (int j = 0; j < 16; j += 2) {
+            float x0 = v[j] + __ldg(args.bias + n0 + c + j);
+            float x1 = v[j + 1] + __ldg(args.bias + n0 + c + j + 1);
+            if (EPI == EPI_BIAS_RELU_F16) { x0 = fmaxf(x0, 0.f); x1 = fmaxf(x1, 0.f); }
+            p[j / 2] = pack_half2(x0, x1);
+          }
+          constexpr int RB = C::OUT16_BOX * 2;
+          unsigned char* box = st16 + (c / C::OUT16_BOX) * (128 * RB);
+          const int ch = (c % C::OUT16_BOX) / 8;
+          *reinterpret_cast<uint4*>(box + swz<RB>(r, ch)) = make_uint4(p[0], p[1], p[2], p[3]);
+          *reinterpret_cast<uint4*>(box + swz<RB>(r, ch + 1)) = make_uint4(p[4], p[5], p[6], p[7]);
         }
-        float4* q = reinterpret_cast<float4*>(o32 + c);
+        sm100::tc_fence_before();
+        mbar_arrive(&tempty[acc]);  // accumulator may be overwritten now
+      } else {
+        sm100::mbar_wait(&resid_bar, local & 1);
+        // pass 1: v = acc + bias + resid (written back in place), row sum
+        float sum = 0.f;
+#pragma unroll 1
+        for (int c = 0; c < BN; c += 16) {
+          sm100::tmem_ld16(t_row + c, v);
+          unsigned char* box = st32 + (c / 32) * 16384;
 #pragma unroll
-        for (int j = 0; j < 4; ++j) q[j] = make_float4(y[4 * j], y[4 * j + 1], y[4 * j + 2], y[4 * j + 3]);
-        uint32_t p[8];
+          for (int k = 0; k < 4; ++k) {
+            float4* p = reinterpret_cast<float4*>(box + swz<128>(r, (c % 32) / 4 + k));
+            float4 x = *p;
+            x.x += v[4 * k + 0] + __ldg(args.bias + c + 4 * k + 0);
+            x.y += v[4 * k + 1] + __ldg(args.bias + c + 4 * k + 1);
+            x.z += v[4 * k + 2] + __ldg(args.bias + c + 4 * k + 2);
+            x.w += v[4 * k + 3] + __ldg(args.bias + c + 4 * k + 3);
+            sum += (x.x + x.y) + (x.z + x.w);
+            *p = x;
+          }
+        }
+        sm100::tc_fence_before();
+        mbar_arrive(&tempty[acc]);
+        const float mean = sum * (1.0f / BN);
+        float sq = 0.f;
+#pragma unroll 4
+        for (int c4 = 0; c4 < BN / 4; ++c4) {
+          const float4 x = *reinterpret_cast<const float4*>(st32 + (c4 / 8) * 16384 + swz<128>(r, c4 % 8));
+          const float a = x.x - mean, b = x.y - mean, cc = x.z - mean, d = x.w - mean;
+          sq += (a * a + b * b) + (cc * cc + d * d);
+        }
+        const float rstd = rsqrtf(sq * (1.0f / BN) + args.eps);
+        constexpr int RB = C::OUT16_BOX * 2;
+#pragma unroll 2
+        for (int c8 = 0; c8 < BN / 8; ++c8) {  // 8 columns per iteration
+          float y[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) p[j] = pack_half2(y[2 * j], y[2 * j + 1]);
-        uint4* h = reinterpret_cast<uint4*>(o16 + c);
-        h[0] = make_uint4(p[0], p[1], p[2], p[3]);
-        h[1] = make_uint4(p[4], p[5], p[6], p[7]);
+          for (int h = 0; h < 2; ++h) {
+            const int c4 = 2 * c8 + h;
+            float4* p = reinterpret_cast<float4*>(st32 + (c4 / 8) * 16384 + swz<128>(r, c4 % 8));
+            float4 x = *p;
+            const int c = 4 * c4;
+            x.x = (x.x - mean) * rstd * __ldg(args.gamma + c + 0) + __ldg(args.beta + c + 0);
+            x.y = (x.y - mean) * rstd * __ldg(args.gamma + c + 1) + __ldg(args.beta + c + 1);
+            x.z = (x.z - mean) * rstd * __ldg(args.gamma + c + 2) + __ldg(args.beta + c + 2);
+            x.w = (x.w - mean) * rstd * __ldg(args.gamma + c + 3) + __ldg(args.beta + c + 3);
+            *p = x;
+            y[4 * h + 0] = x.x; y[4 * h + 1] = x.y; y[4 * h + 2] = x.z; y[4 * h + 3] = x.w;
+          }
+          const int c = 8 * c8;
+          const uint4 pk = make_uint4(pack_half2(y[0], y[1]), pack_half2(y[2], y[3]),
+                                      pack_half2(y[4], y[5]), pack_half2(y[6], y[7]));
+          if constexpr (C::F16_DIRECT) {
+            if (m0 + r < args.M)
+              *reinterpret_cast<uint4*>(args.out16 + (size_t)(m0 + r) * args.N + c) = pk;
+          } else {
+            unsigned char* box = st16 + (c / C::OUT16_BOX) * (128 * RB);
+            *reinterpret_cast<uint4*>(box + swz<RB>(r, (c % C::OUT16_BOX) / 8)) = pk;
+          }
+        }
+      }
+      fence_proxy_async();  // staging writes -> visible to the TMA (async proxy)
+      epi_bar();
+      if (leader) {
+        constexpr int nb16 = C::F16_DIRECT ? 0 : BN / C::OUT16_BOX;
+#pragma unroll
+        for (int b = 0; b < nb16; ++b)
+          tma_store_2d(&maps.out16, st16 + b * (128 * C::OUT16_BOX * 2), n0 + b * C::OUT16_BOX, m0);
+        if (EPI == EPI_BIAS_RESID_LN) {
+#pragma unroll
+          for (int b = 0; b < BN / 32; ++b) tma_store_2d(&maps.x32, st32 + b * 16384, n0 + b * 32, m0);
+        }
+        bulk_commit();
       }
     }
+    if (leader) bulk_wait0();
   }
-
+  __syncwarp();
   sm100::tc_fence_before();
   __syncthreads();
-  if (warp == 2) sm100::tmem_dealloc<NCOLS>(tmem);
+  if (warp == 1) sm100::tmem_dealloc<NCOLS>(tmem);
 }
 
+int g_num_sms = 0;
+
 template <int BN, int KCH, int EPI>
-predtop_status launch_t(const CUtensorMap* tmA, const CUtensorMap* tmB, const GemmArgs& a,
-                        cudaStream_t st) {
-  constexpr int smem = smem_bytes<BN, KCH>();
-  PT_CUDA_TRY(cudaFuncSetAttribute(k_gemm<BN, KCH, EPI>,
-                                   cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  dim3 grid((unsigned)ceil_div(a.M, 128), (unsigned)(a.N / BN));
-  k_gemm<BN, KCH, EPI><<<grid, kThreads, smem, st>>>(*tmA, *tmB, a);
+predtop_status launch_t(const Maps& maps, const GemmArgs& a, cudaStream_t st) {
+  using C = Cfg<BN, KCH, EPI>;
+  PT_CUDA_TRY(cudaFuncSetAttribute(k_gemm<BN, KCH, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   C::SMEM));
+  if (!g_num_sms) {
+    int dev = 0;
+    PT_CUDA_TRY(cudaGetDevice(&dev));
+    PT_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
+  }
+  const int64_t tiles = ceil_div(a.M, 128) * (a.N / BN);
+  const int grid = (int)std::min<int64_t>(tiles, g_num_sms);
+  k_gemm<BN, KCH, EPI><<<grid, kThreads, C::SMEM, st>>>(maps, a);
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;
 }
 
 template <int BN, int KCH>
-predtop_status launch_epi(int epi, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                          const GemmArgs& a, cudaStream_t st) {
+predtop_status launch_epi(int epi, const Maps& m, const GemmArgs& a, cudaStream_t st) {
   switch (epi) {
-    case EPI_BIAS_F16: return launch_t<BN, KCH, EPI_BIAS_F16>(tmA, tmB, a, st);
-    case EPI_BIAS_RELU_F16: return launch_t<BN, KCH, EPI_BIAS_RELU_F16>(tmA, tmB, a, st);
-    default: return launch_t<BN, KCH, EPI_BIAS_RESID_LN>(tmA, tmB, a, st);
+    case EPI_BIAS_F16: return launch_t<BN, KCH, EPI_BIAS_F16>(m, a, st);
+    case EPI_BIAS_RELU_F16: return launch_t<BN, KCH, EPI_BIAS_RELU_F16>(m, a, st);
+    default:
+      if constexpr (BN == 32 || BN == 64 || BN == 128 || BN == 256) {
+        return launch_t<BN, KCH, EPI_BIAS_RESID_LN>(m, a, st);
+      } else {
+        set_error("LN epilogue supports d in {32, 64, 128, 256}");
+        return PREDTOP_ERR_UNSUPPORTED;
+      }
   }
 }
 
 template <int KCH>
-predtop_status launch_bn(int bn, int epi, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                         const GemmArgs& a, cudaStream_t st) {
+predtop_status launch_bn(int bn, int epi, const Maps& m, const GemmArgs& a, cudaStream_t st) {
   switch (bn) {
-    case 32: return launch_epi<32, KCH>(epi, tmA, tmB, a, st);
-    case 64: return launch_epi<64, KCH>(epi, tmA, tmB, a, st);
-    case 96: return launch_epi<96, KCH>(epi, tmA, tmB, a, st);
-    case 128: return launch_epi<128, KCH>(epi, tmA, tmB, a, st);
-    case 192: return launch_epi<192, KCH>(epi, tmA, tmB, a, st);
-    case 256: return launch_epi<256, KCH>(epi, tmA, tmB, a, st);
+    case 32: return launch_epi<32, KCH>(epi, m, a, st);
+    case 64: return launch_epi<64, KCH>(epi, m, a, st);
+    case 96: return launch_epi<96, KCH>(epi, m, a, st);
+    case 128: return launch_epi<128, KCH>(epi, m, a, st);
+    case 192: return launch_epi<192, KCH>(epi, m, a, st);
+    case 256: return launch_epi<256, KCH>(epi, m, a, st);
     default:
       set_error("unsupported GEMM tile width %d", bn);
       return PREDTOP_ERR_UNSUPPORTED;
@@ -228,7 +352,7 @@ predtop_status launch_bn(int bn, int epi, const CUtensorMap* tmA, const CUtensor
 }  // namespace
 
 // Output tile width for N total columns: the widest of {256,192,128,96,64,32}
-// dividing N with N/BN tiles (<= 256 keeps TMEM <= 256 columns).
+// dividing N (<= 256: two fp32 accumulators fit the 512 TMEM columns).
 int gemm_pick_bn(int N) {
   const int cands[] = {256, 192, 128, 96, 64, 32};
   for (int c : cands)
@@ -243,8 +367,22 @@ predtop_status gemm_launch(const CUtensorMap* tmA, const CUtensorMap* tmB, int b
     set_error("LN epilogue needs the whole row in one tile (bn=%d, N=%d)", bn, a.N);
     return PREDTOP_ERR_UNSUPPORTED;
   }
-  if (a.K % 64 == 0) return launch_bn<64>(bn, epi, tmA, tmB, a, st);
-  if (a.K == 32) return launch_bn<32>(bn, epi, tmA, tmB, a, st);
+  Maps m;
+  m.a = *tmA;
+  m.b = *tmB;
+  // output / residual maps over the caller's buffers
+  if (!encode_tma_2d(&m.out16, a.out16, 2, a.N, a.M, bn % 64 == 0 ? 64 : 32, 128)) return PREDTOP_ERR_CUDA;
+  if (epi == EPI_BIAS_RESID_LN) {
+    if (a.out32 != a.resid32) {
+      set_error("LN epilogue updates the residual in place (out32 must equal resid32)");
+      return PREDTOP_ERR_UNSUPPORTED;
+    }
+    if (!encode_tma_2d(&m.x32, a.out32, 4, a.N, a.M, 32, 128)) return PREDTOP_ERR_CUDA;
+  } else {
+    m.x32 = m.out16;
+  }
+  if (a.K % 64 == 0) return launch_bn<64>(bn, epi, m, a, st);
+  if (a.K == 32) return launch_bn<32>(bn, epi, m, a, st);
   set_error("unsupported GEMM K=%d", a.K);
   return PREDTOP_ERR_UNSUPPORTED;
 }

@@ -98,6 +98,8 @@ predtop_status dag_copy_bits(const predtop_dag_s* dag, const uint64_t* from, uin
                              cudaStream_t st);
 
 // ---- tma.cu
+bool encode_tma_2d(CUtensorMap* map, const void* base, int elem_bytes, uint64_t inner,
+                   uint64_t outer, uint32_t box_inner, uint32_t box_outer);
 bool encode_tma_2d_f16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
                        uint32_t box_inner, uint32_t box_outer);
 

@@ -22,32 +22,42 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   return fn;
 }
 
-// Row-major fp16 matrix [outer][inner] -> tiles of box_outer rows x box_inner
-// columns, swizzled to match the UMMA K-major canonical layout
-// (128B swizzle for 64-element rows, 64B for 32-element rows).  Out-of-bounds
-// rows read as zero.
-bool encode_tma_2d_f16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
-                       uint32_t box_inner, uint32_t box_outer) {
+// Row-major matrix [outer][inner] of 2-byte (fp16) or 4-byte (fp32) elements
+// -> tiles of box_outer rows x box_inner columns.  The shared-memory side uses
+// the swizzle matching the box row size (128 B -> SWIZZLE_128B, the UMMA
+// K-major canonical layout; 64 B -> 64B; 32 B -> 32B).  Out-of-bounds rows read
+// as zero and are clipped on stores.
+bool encode_tma_2d(CUtensorMap* map, const void* base, int elem_bytes, uint64_t inner,
+                   uint64_t outer, uint32_t box_inner, uint32_t box_outer) {
   auto enc = get_encode();
   if (!enc) {
     set_error("cuTensorMapEncodeTiled unavailable (no CUDA driver)");
     return false;
   }
   cuuint64_t dims[2] = {inner, outer};
-  cuuint64_t strides[1] = {inner * 2};
+  cuuint64_t strides[1] = {inner * (cuuint64_t)elem_bytes};
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
-  CUtensorMapSwizzle sw =
-      box_inner * 2 == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
-  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), dims, strides,
-                   box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  const uint32_t rb = box_inner * (uint32_t)elem_bytes;
+  CUtensorMapSwizzle sw = rb == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                          : rb == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                          : rb == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                     : CU_TENSOR_MAP_SWIZZLE_NONE;
+  CUtensorMapDataType dt = elem_bytes == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  CUresult r = enc(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d): inner=%llu outer=%llu box=%ux%u", (int)r,
               (unsigned long long)inner, (unsigned long long)outer, box_inner, box_outer);
     return false;
   }
   return true;
+}
+
+bool encode_tma_2d_f16(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
+                       uint32_t box_inner, uint32_t box_outer) {
+  return encode_tma_2d(map, base, 2, inner, outer, box_inner, box_outer);
 }
 
 }  // namespace predtop

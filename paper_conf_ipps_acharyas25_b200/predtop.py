@@ -77,6 +77,9 @@ _SIGS = {
     "predtop_last_error": (ctypes.c_char_p, []),
     "predtop_abi_version": (ctypes.c_int, []),
     "predtop_launch_count": (_I64, []),
+    "predtop_profile_enable": (None, [ctypes.c_int]),
+    "predtop_profile_read": (ctypes.c_int, [_P, _P, ctypes.c_int]),
+    "predtop_profile_kind_name": (ctypes.c_char_p, [ctypes.c_int]),
 }
 
 
