@@ -374,7 +374,7 @@ def main():
     names = [L.predtop_profile_kind_name(i).decode() for i in range(nk)]
     prof = {names[i]: {"ms_per_step": kms[i] / prof_steps, "launches_per_step": kcnt[i] / prof_steps}
             for i in range(nk) if kcnt[i]}
-    step_ms_prof = sum(ms_prof) / prof_steps
+    step_ms_prof = total_ms / args.steps  # shares relative to the headline (graph) step time
     for k in prof:
         prof[k]["share"] = prof[k]["ms_per_step"] / step_ms_prof
 
@@ -392,6 +392,7 @@ def main():
         "gemm_oproj_ln": ("tensor", 2.0 * Ntot * d * d),
         "gemm_ffn1": ("tensor", 2.0 * Ntot * d * dff),
         "gemm_ffn2_ln": ("tensor", 2.0 * Ntot * dff * d),
+        "layer_tail": ("tensor", 2.0 * Ntot * (d * d + 2 * d * dff)),
         "attention": ("alu", float(H) * A),  # exps per launch (MUFU-bound)
         "dag_closure": ("hbm", 8.0 * words + 8.0 * E),
         "dag_mask": ("hbm", 3 * 8.0 * words),

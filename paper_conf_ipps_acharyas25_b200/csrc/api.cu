@@ -385,7 +385,8 @@ predtop_status predtop_model_create(const predtop_model_config* cfg, const float
     bool ok = encode_tma_2d_f16(&L.tm_qkv, L.Wqkv, d, 3 * d, kch_for(d), m->bn_qkv) &&
               encode_tma_2d_f16(&L.tm_o, L.Wo, d, d, kch_for(d), d) &&
               encode_tma_2d_f16(&L.tm_1, L.W1, d, f, kch_for(d), m->bn_ff1) &&
-              encode_tma_2d_f16(&L.tm_2, L.W2, f, d, kch_for(f), d);
+              encode_tma_2d_f16(&L.tm_2, L.W2, f, d, kch_for(f), d) &&
+              (f < 128 || encode_tma_2d_f16(&L.tm_1c, L.W1, d, f, kch_for(d), 128));
     if (!ok) {
       delete m;
       return PREDTOP_ERR_CUDA;
@@ -400,6 +401,16 @@ void predtop_model_destroy(predtop_model model) { delete model; }
 size_t predtop_stage_forward_workspace(predtop_model model, predtop_dag dag) {
   if (!model || !dag) return 0;
   return carve_fwd(model, dag, nullptr, nullptr);
+}
+
+// The fused layer tail (layer.cu) covers d in {64, 128}; PREDTOP_UNFUSED=1 forces
+// the three-GEMM path (tests compare the two).
+static bool use_fused_tail(int d, int dff) {
+  static const bool unfused = [] {
+    const char* e = getenv("PREDTOP_UNFUSED");
+    return e && e[0] == '1';
+  }();
+  return !unfused && layer_tail_supported(d, dff);
 }
 
 static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, size_t ws_bytes,
@@ -434,6 +445,11 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
       if ((s = gemm_launch(&tm_x16, &L.tm_qkv, m->bn_qkv, EPI_BIAS_F16, a, st)) != PREDTOP_OK) return s;
     }
     if ((s = attention_launch(dag, d, H, w.qkv, w.att, st)) != PREDTOP_OK) return s;
+    if (use_fused_tail(d, f)) {
+      ProfScope _p(PK_LAYER_TAIL, st);
+      if ((s = layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st)) != PREDTOP_OK) return s;
+      continue;
+    }
     a = GemmArgs{};
     a.M = M; a.K = d; a.N = d; a.bias = L.bo; a.resid32 = w.x32; a.out32 = w.x32; a.out16 = w.x16;
     a.gamma = L.g1; a.beta = L.be1; a.eps = m->cfg.ln_eps;

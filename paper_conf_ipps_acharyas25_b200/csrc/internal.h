@@ -71,7 +71,8 @@ struct LayerDev {
   float* b2;
   float* g2;
   float* be2;
-  CUtensorMap tm_qkv, tm_o, tm_1, tm_2;  // B-operand TMA maps
+  CUtensorMap tm_qkv, tm_o, tm_1, tm_2;  // B-operand TMA maps (unfused GEMMs)
+  CUtensorMap tm_1c;                     // W_1 in 128-row chunks (fused layer tail)
 };
 
 }  // namespace predtop
@@ -131,5 +132,10 @@ predtop_status plan_launch(int64_t P, const int64_t* plan_ptr, const int32_t* pl
                            const int32_t* B, const float* t, int64_t num_stages, double* T,
                            int64_t* first_bad, cudaStream_t st);
 predtop_status argmin_launch(int64_t n, const double* T, int64_t* best, cudaStream_t st);
+
+// ---- layer.cu (fused O-proj + LN1 + FFN + LN2)
+bool layer_tail_supported(int d, int dff);
+predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
+                                 __half* x16, int M, cudaStream_t st);
 
 }  // namespace predtop

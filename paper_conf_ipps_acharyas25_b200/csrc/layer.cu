@@ -1,0 +1,377 @@
+// layer.cu -- K7: the post-attention half of the DAG-Transformer layer
+// (Fig. 4; reading R6, post-LN encoder layer of [34]) as ONE
+// persistent tcgen05 kernel per 128-row tile:
+//     h  = LN1(x + att W_o^T + b_o)
+//     x' = LN2(h + ReLU(h W_1^T + b_1) W_2^T + b_2)
+// The d_ff-wide hidden activation never leaves the SM: it is produced in
+// 128-column chunks into TMEM, turned into an fp16 UMMA operand in shared
+// memory by the epilogue warps, and consumed by the FFN-2 MMAs that
+// accumulate x' in TMEM.  HBM traffic per row: att (2d B) + x (4d B) in,
+// x' (4d + 2d B) out.
+//
+// Roles (10 warps, one CTA per SM, persistent over row tiles):
+//   warp 0      TMA producer: att tile, fp32 residual tile, and the weight
+//               tiles (W_o, W_1 chunk, W_2 chunk; 64-wide K slices) through a
+//               ring, in exactly the order the MMA warp consumes them
+//   warp 1      MMA issuer (one thread): O-proj -> acc_o; FFN-1 chunk j ->
+//               acc_f[j%2] (double buffered, so chunk j+1 overlaps the ReLU
+//               epilogue of chunk j); FFN-2 chunk j -> acc_out (accumulated)
+//   warps 2..9  epilogue: LN1 (acc_o + b_o + x -> h fp32 in place, h fp16 as
+//               the FFN-1 A operand), ReLU(acc_f + b_1) -> fp16 A operand of
+//               FFN-2, LN2 (acc_out + b_2 + h) -> x' fp32 / fp16, TMA stores
+// TMEM columns: acc_o [0,D) | acc_f0 [D,D+128) | acc_f1 [D+128,D+256) |
+//               acc_out [D+256, 2D+256)   (512 at D = 128)
+#include <algorithm>
+
+#include "internal.h"
+#include "sm100.cuh"
+
+namespace predtop {
+
+namespace {
+
+constexpr int kThreads = 320;
+constexpr int kEpi = 256;
+constexpr int FC = 128;  // FFN chunk (hidden columns per chunk)
+constexpr int kSub = 128 * 128;  // bytes of one [128 rows x 64 fp16] or [128 x 32 fp32] sub-tile
+
+template <int D>
+struct TailCfg {
+  static constexpr int X32 = 128 * D * 4;   // residual / h / x' fp32 tile
+  static constexpr int SA = 128 * 128 * 2;  // att tile [128 x D] and ReLU chunk 0 [128 x 128]
+  static constexpr int SP1 = 128 * 128 * 2; // ReLU chunk 1
+  static constexpr int SH = 128 * D * 2;    // h fp16 (FFN-1 A operand) / x' fp16 staging
+  static constexpr int SLOT = (D > FC ? D : FC) * 64 * 2;
+  static constexpr int FIXED = X32 + SA + SP1 + SH + 1024;
+  static constexpr int RS_FIT = (224 * 1024 - FIXED) / SLOT;
+  static constexpr int RS = RS_FIT > 6 ? 6 : RS_FIT;
+  static constexpr int SMEM = FIXED + RS * SLOT;
+  static constexpr uint32_t TMEM_COLS = 512;
+  static_assert(RS >= 2, "smem budget");
+};
+
+struct TailMaps {
+  CUtensorMap att, x32, x16, wo, w1, w2;
+};
+
+struct TailArgs {
+  int M, dff;
+  const float *bo, *g1, *be1, *b1, *b2, *g2, *be2;
+  float eps;
+};
+
+template <int D>
+__global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constant__ TailMaps mp, TailArgs args) {
+  using C = TailCfg<D>;
+  constexpr int RS = C::RS;
+  constexpr int KD = D / 64;  // 64-wide K slices of d
+  extern __shared__ unsigned char dsm[];
+  unsigned char* base = (unsigned char*)(((uintptr_t)dsm + 1023) & ~(uintptr_t)1023);
+  unsigned char* sX = base;                 // fp32 [128 x D], D/32 sub-tiles
+  unsigned char* sA = sX + C::X32;          // att / ReLU chunk buffer 0
+  unsigned char* sP1 = sA + C::SA;          // ReLU chunk buffer 1
+  unsigned char* sH = sP1 + C::SP1;         // h fp16 / x' fp16
+  unsigned char* ring = sH + C::SH;
+  __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
+  __shared__ __align__(8) uint64_t a_full, a_free, x_full, x_free, o_full, o_empty, h_ready;
+  __shared__ __align__(8) uint64_t f_full[2], f_empty[2], p_ready[2], p_free[2], out_full, out_empty;
+  __shared__ uint32_t tmem_slot;
+  __shared__ float red_a[2][128], red_b[2][128];
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ntiles = (int)ceil_div(args.M, 128);
+  const int NJ = args.dff / FC;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < RS; ++s) {
+      sm100::mbar_init(&ring_full[s], 1);
+      sm100::mbar_init(&ring_empty[s], 1);
+    }
+    uint64_t* singles[] = {&a_full, &a_free, &x_full, &x_free, &o_full, &o_empty, &h_ready,
+                           &f_full[0], &f_full[1], &f_empty[0], &f_empty[1], &p_ready[0], &p_ready[1],
+                           &p_free[0], &p_free[1], &out_full, &out_empty};
+    for (uint64_t* b : singles) sm100::mbar_init(b, 1);
+    sm100::fence_mbar_init();
+  }
+  if (warp == 1) sm100::tmem_alloc<C::TMEM_COLS>(&tmem_slot);
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::tc_fence_after();
+  const uint32_t tmem = tmem_slot;
+  const uint32_t acc_o = tmem, acc_out = tmem + D + 2 * FC;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ------------------------------------------ TMA producer
+      sm100::tma_prefetch(&mp.att);
+      sm100::tma_prefetch(&mp.x32);
+      sm100::tma_prefetch(&mp.wo);
+      sm100::tma_prefetch(&mp.w1);
+      sm100::tma_prefetch(&mp.w2);
+      int it = 0;
+      auto load_w = [&](const CUtensorMap* m, int c0, int c1, int rows) {
+        const int s = it % RS;
+        sm100::mbar_wait(&ring_empty[s], ((it / RS) & 1) ^ 1);
+        sm100::mbar_arrive_expect_tx(&ring_full[s], rows * 128);
+        sm100::tma_load_2d(ring + s * C::SLOT, m, &ring_full[s], c0, c1);
+        ++it;
+      };
+      int i = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        const int m0 = t * 128;
+        sm100::mbar_wait(&a_free, (i & 1) ^ 1);
+        sm100::mbar_arrive_expect_tx(&a_full, 128 * D * 2);
+        for (int b = 0; b < KD; ++b) sm100::tma_load_2d(sA + b * kSub, &mp.att, &a_full, b * 64, m0);
+        for (int kc = 0; kc < KD; ++kc) load_w(&mp.wo, kc * 64, 0, D);
+        sm100::mbar_wait(&x_free, i & 1);
+        sm100::mbar_arrive_expect_tx(&x_full, 128 * D * 4);
+        for (int b = 0; b < D / 32; ++b) sm100::tma_load_2d(sX + b * kSub, &mp.x32, &x_full, b * 32, m0);
+        for (int j = 0; j < 2 && j < NJ; ++j)
+          for (int kc = 0; kc < KD; ++kc) load_w(&mp.w1, kc * 64, j * FC, FC);
+        for (int j = 0; j < NJ; ++j) {
+          for (int kc = 0; kc < FC / 64; ++kc) load_w(&mp.w2, j * FC + kc * 64, 0, D);
+          if (j + 2 < NJ)
+            for (int kc = 0; kc < KD; ++kc) load_w(&mp.w1, kc * 64, (j + 2) * FC, FC);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ------------------------------------------ MMA issuer
+      constexpr uint32_t id_D = sm100::make_idesc_f16(128, D);
+      constexpr uint32_t id_F = sm100::make_idesc_f16(128, FC);
+      int it = 0;
+      // consume `nk` ring slots: D[tmem] (+)= A (64-wide K slices at a_base + kc*kSub) * slot^T
+      auto mma_ring = [&](uint32_t d_tmem, uint32_t a_base, int nk, uint32_t idesc, bool first) {
+        for (int kc = 0; kc < nk; ++kc, ++it) {
+          const int s = it % RS;
+          sm100::mbar_wait(&ring_full[s], (it / RS) & 1);
+          sm100::tc_fence_after();
+          const uint32_t b0 = sm100::smem_u32(ring + s * C::SLOT);
+          const uint32_t a0 = a_base + kc * kSub;
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            sm100::mma_f16_ss(d_tmem, sm100::make_sdesc<128>(a0 + kk * 32),
+                              sm100::make_sdesc<128>(b0 + kk * 32), idesc, !(first && kc == 0 && kk == 0));
+          sm100::mma_commit(&ring_empty[s]);
+        }
+      };
+      const uint32_t aA = sm100::smem_u32(sA), aP1 = sm100::smem_u32(sP1), aH = sm100::smem_u32(sH);
+      int i = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        const int cbase = i * NJ;  // global FFN chunk counter of this tile's chunk 0
+        auto ffn1 = [&](int j) {
+          const int b = j & 1, u = (cbase + j) >> 1;
+          sm100::mbar_wait(&f_empty[b], (u & 1) ^ 1);
+          sm100::tc_fence_after();
+          mma_ring(tmem + D + b * FC, aH, KD, id_F, true);
+          sm100::mma_commit(&f_full[b]);
+        };
+        sm100::mbar_wait(&a_full, i & 1);
+        sm100::mbar_wait(&o_empty, (i & 1) ^ 1);
+        sm100::tc_fence_after();
+        mma_ring(acc_o, aA, KD, id_D, true);  // O-proj
+        sm100::mma_commit(&o_full);
+        sm100::mbar_wait(&h_ready, i & 1);
+        sm100::tc_fence_after();
+        for (int j = 0; j < 2 && j < NJ; ++j) ffn1(j);
+        for (int j = 0; j < NJ; ++j) {
+          const int b = j & 1, u = (cbase + j) >> 1;
+          sm100::mbar_wait(&p_ready[b], u & 1);
+          if (j == 0) sm100::mbar_wait(&out_empty, (i & 1) ^ 1);
+          sm100::tc_fence_after();
+          mma_ring(acc_out, b ? aP1 : aA, FC / 64, id_D, j == 0);  // FFN-2 chunk j
+          sm100::mma_commit(&p_free[b]);
+          if (j == NJ - 2) sm100::mma_commit(&a_free);  // last read of sA this tile
+          if (j + 2 < NJ) ffn1(j + 2);
+        }
+        sm100::mma_commit(&out_full);
+      }
+    }
+  } else {
+    // ------------------------------------------ epilogue warps 2..9
+    const int q = warp & 3, half = (warp - 2) >> 2;
+    const int r = q * 32 + lane;
+    const uint32_t lrow = (uint32_t)(q * 32) << 16;
+    const bool leader = (warp == 2 && lane == 0);
+    float v[16];
+    // LayerNorm of the row r over D columns, this thread doing columns
+    // [half*D/2, +D/2): z (in sX, fp32, in place) -> y; y also to sH as fp16.
+    auto layer_norm = [&](float sum, const float* g, const float* be) {
+      red_a[half][r] = sum;
+      sm100::named_bar<kEpi>(1);
+      const float mean = (red_a[0][r] + red_a[1][r]) * (1.0f / D);
+      float sq = 0.f;
+#pragma unroll 4
+      for (int c4 = half * D / 8; c4 < (half + 1) * D / 8; ++c4) {
+        const float4 x = *reinterpret_cast<const float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
+        const float a = x.x - mean, b = x.y - mean, cc = x.z - mean, d = x.w - mean;
+        sq += (a * a + b * b) + (cc * cc + d * d);
+      }
+      red_b[half][r] = sq;
+      sm100::named_bar<kEpi>(1);
+      const float rstd = rsqrtf((red_b[0][r] + red_b[1][r]) * (1.0f / D) + args.eps);
+#pragma unroll 2
+      for (int c8 = half * D / 16; c8 < (half + 1) * D / 16; ++c8) {
+        float y[8];
+#pragma unroll
+        for (int h2 = 0; h2 < 2; ++h2) {
+          const int c4 = 2 * c8 + h2;
+          float4* p = reinterpret_cast<float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
+          float4 x = *p;
+          const float4 gm = __ldg(reinterpret_cast<const float4*>(g) + c4);
+          const float4 bt = __ldg(reinterpret_cast<const float4*>(be) + c4);
+          x.x = (x.x - mean) * rstd * gm.x + bt.x;
+          x.y = (x.y - mean) * rstd * gm.y + bt.y;
+          x.z = (x.z - mean) * rstd * gm.z + bt.z;
+          x.w = (x.w - mean) * rstd * gm.w + bt.w;
+          *p = x;
+          y[4 * h2] = x.x; y[4 * h2 + 1] = x.y; y[4 * h2 + 2] = x.z; y[4 * h2 + 3] = x.w;
+        }
+        const int c = 8 * c8;
+        *reinterpret_cast<uint4*>(sH + (c / 64) * kSub + sm100::swz<128>(r, (c % 64) / 8)) =
+            make_uint4(sm100::pack_half2(y[0], y[1]), sm100::pack_half2(y[2], y[3]),
+                       sm100::pack_half2(y[4], y[5]), sm100::pack_half2(y[6], y[7]));
+      }
+    };
+    // z = acc (TMEM) + bias + sX (fp32), written back to sX; returns the partial row sum
+    auto add_residual = [&](uint32_t acc, const float* bias) {
+      float sum = 0.f;
+#pragma unroll 1
+      for (int c = half * D / 2; c < (half + 1) * D / 2; c += 16) {
+        sm100::tmem_ld16(acc + lrow + c, v);
+        unsigned char* box = sX + (c / 32) * kSub;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          float4* p = reinterpret_cast<float4*>(box + sm100::swz<128>(r, (c % 32) / 4 + k));
+          const float4 b = __ldg(reinterpret_cast<const float4*>(bias + c) + k);
+          float4 x = *p;
+          x.x += v[4 * k + 0] + b.x;
+          x.y += v[4 * k + 1] + b.y;
+          x.z += v[4 * k + 2] + b.z;
+          x.w += v[4 * k + 3] + b.w;
+          sum += (x.x + x.y) + (x.z + x.w);
+          *p = x;
+        }
+      }
+      return sum;
+    };
+    int i = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const int m0 = t * 128;
+      const int cbase = i * NJ;
+      // previous tile's stores have read sX / sH -> the residual of this tile may land
+      if (leader) sm100::bulk_wait_read0();
+      sm100::named_bar<kEpi>(1);
+      if (leader) sm100::mbar_arrive(&x_free);
+      // ---- LN1
+      sm100::mbar_wait(&o_full, i & 1);
+      sm100::mbar_wait(&x_full, i & 1);
+      sm100::tc_fence_after();
+      const float s1 = add_residual(acc_o, args.bo);
+      sm100::tc_fence_before();
+      layer_norm(s1, args.g1, args.be1);
+      sm100::fence_proxy_async();
+      sm100::named_bar<kEpi>(1);
+      if (leader) {
+        sm100::mbar_arrive(&o_empty);
+        sm100::mbar_arrive(&h_ready);
+      }
+      // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 operand buffer
+      for (int j = 0; j < NJ; ++j) {
+        const int b = j & 1, u = (cbase + j) >> 1;
+        sm100::mbar_wait(&f_full[b], u & 1);
+        sm100::mbar_wait(&p_free[b], (u & 1) ^ 1);
+        sm100::tc_fence_after();
+        unsigned char* P = b ? sP1 : sA;
+        const uint32_t accf = tmem + D + b * FC + lrow;
+        const float* b1 = args.b1 + j * FC;
+#pragma unroll 1
+        for (int c = half * FC / 2; c < (half + 1) * FC / 2; c += 16) {
+          sm100::tmem_ld16(accf + c, v);
+          uint32_t pk[8];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const float4 bb = __ldg(reinterpret_cast<const float4*>(b1 + c) + k);
+            pk[2 * k] = sm100::pack_half2(fmaxf(v[4 * k] + bb.x, 0.f), fmaxf(v[4 * k + 1] + bb.y, 0.f));
+            pk[2 * k + 1] = sm100::pack_half2(fmaxf(v[4 * k + 2] + bb.z, 0.f), fmaxf(v[4 * k + 3] + bb.w, 0.f));
+          }
+          unsigned char* sub = P + (c / 64) * kSub;
+          *reinterpret_cast<uint4*>(sub + sm100::swz<128>(r, (c % 64) / 8)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+          *reinterpret_cast<uint4*>(sub + sm100::swz<128>(r, (c % 64) / 8 + 1)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+        }
+        sm100::tc_fence_before();
+        sm100::fence_proxy_async();
+        sm100::named_bar<kEpi>(1);
+        if (leader) {
+          sm100::mbar_arrive(&f_empty[b]);
+          sm100::mbar_arrive(&p_ready[b]);
+        }
+      }
+      // ---- LN2 and stores
+      sm100::mbar_wait(&out_full, i & 1);
+      sm100::tc_fence_after();
+      const float s2 = add_residual(acc_out, args.b2);
+      sm100::tc_fence_before();
+      layer_norm(s2, args.g2, args.be2);
+      sm100::fence_proxy_async();
+      sm100::named_bar<kEpi>(1);
+      if (leader) {
+        sm100::mbar_arrive(&out_empty);
+        for (int b = 0; b < D / 32; ++b) sm100::tma_store_2d(&mp.x32, sX + b * kSub, b * 32, m0);
+        for (int b = 0; b < KD; ++b) sm100::tma_store_2d(&mp.x16, sH + b * kSub, b * 64, m0);
+        sm100::bulk_commit();
+      }
+    }
+    if (leader) sm100::bulk_wait0();
+  }
+  __syncwarp();
+  sm100::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) sm100::tmem_dealloc<C::TMEM_COLS>(tmem);
+}
+
+int g_sms = 0;
+
+template <int D>
+predtop_status launch_d(const TailMaps& mp, const TailArgs& a, cudaStream_t st) {
+  using C = TailCfg<D>;
+  static bool attr_done = false;
+  if (!attr_done) {
+    PT_CUDA_TRY(cudaFuncSetAttribute(k_layer_tail<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+    attr_done = true;
+  }
+  if (!g_sms) {
+    int dev = 0;
+    PT_CUDA_TRY(cudaGetDevice(&dev));
+    PT_CUDA_TRY(cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev));
+  }
+  const int grid = (int)std::min<int64_t>(ceil_div(a.M, 128), g_sms);
+  k_layer_tail<D><<<grid, kThreads, C::SMEM, st>>>(mp, a);
+  PT_LAUNCH_CHECK();
+  return PREDTOP_OK;
+}
+
+}  // namespace
+
+bool layer_tail_supported(int d, int dff) { return (d == 64 || d == 128) && dff % (2 * FC) == 0; }
+
+predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
+                                 __half* x16, int M, cudaStream_t st) {
+  const int d = m->cfg.d_model, dff = m->cfg.d_ff;
+  if (!layer_tail_supported(d, dff)) {
+    set_error("fused layer tail needs d in {64,128} and d_ff %% 256 == 0");
+    return PREDTOP_ERR_UNSUPPORTED;
+  }
+  if (M <= 0) return PREDTOP_OK;
+  const LayerDev& L = m->layer[l];
+  TailMaps mp;
+  if (!encode_tma_2d(&mp.att, att, 2, d, M, 64, 128) || !encode_tma_2d(&mp.x32, x32, 4, d, M, 32, 128) ||
+      !encode_tma_2d(&mp.x16, x16, 2, d, M, 64, 128))
+    return PREDTOP_ERR_CUDA;
+  mp.wo = L.tm_o;
+  mp.w1 = L.tm_1c;
+  mp.w2 = L.tm_2;
+  TailArgs a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps};
+  return d == 128 ? launch_d<128>(mp, a, st) : launch_d<64>(mp, a, st);
+}
+
+}  // namespace predtop
