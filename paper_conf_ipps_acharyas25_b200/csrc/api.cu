@@ -31,7 +31,7 @@ static inline cudaStream_t S(void* s) { return reinterpret_cast<cudaStream_t>(s)
 
 // ------------------------------------------------------------ DAG workspace
 struct DagBounds {
-  int64_t words, tiles, qtiles;
+  int64_t words, tiles, qtiles, bflags;
   int32_t max_words;
 };
 
@@ -45,6 +45,7 @@ static bool dag_bounds(const predtop_batch_desc* b, DagBounds* o) {
   o->words = b->total_nodes * 2 * T;
   o->qtiles = ceil_div(b->total_nodes, 128) + b->num_graphs;
   o->tiles = o->qtiles * T;
+  o->bflags = (ceil_div(b->total_nodes, 16) + b->num_graphs) * ceil_div(maxn, 64);
   return true;
 }
 
@@ -71,6 +72,8 @@ static size_t carve_dag(const predtop_batch_desc* b, const DagBounds& bd, void* 
   t.tile_cnt = c.take<int32_t>(bd.tiles);
   t.tile_cls = c.take<uint8_t>(bd.tiles);
   t.work = c.take<int2>(bd.qtiles);
+  t.bflag_off = c.take<int64_t>(G + 1);
+  t.bflag = c.take<uint8_t>(bd.bflags);
   if (d) *d = t;
   return align_up(c.used, 256);
 }
@@ -241,6 +244,7 @@ predtop_status predtop_build_dag(const predtop_batch_desc* desc, const int64_t* 
   dag->words_bound = bd.words;
   dag->tiles_bound = bd.tiles;
   dag->qtiles_bound = bd.qtiles;
+  dag->bflags_bound = bd.bflags;
   dag->max_words = bd.max_words;
   *out = dag;
   predtop_status st = dag_build_launch(dag, S(cuda_stream));

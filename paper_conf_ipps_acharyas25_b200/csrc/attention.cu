@@ -71,16 +71,30 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
-// The 16 mask bits a thread needs from one 64-key word: for n-tile nt (8 keys)
-// and element u, key nt*8 + 2*tq + u  ->  bit 2*nt + u of the result.
-__device__ __forceinline__ uint32_t thread_bits(uint64_t word, int tq) {
-  uint64_t w = (word >> (2 * tq)) & 0x0303030303030303ull;
-  w = (w | (w >> 6)) & 0x000F000F000F000Full;
-  w = (w | (w >> 12)) & 0x000000FF000000FFull;
-  return (uint32_t)(w | (w >> 24)) & 0xFFFFu;
+// Zero-accumulator variant (first k-step): C = 0 without zeroing registers.
+__device__ __forceinline__ void mma16816_z(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%10,%10,%10,%10};"
+      : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1), "f"(0.f));
+}
+__device__ __forceinline__ void ldsm_x2_t(uint32_t addr, uint32_t& r0, uint32_t& r1) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0,%1}, [%2];"
+               : "=r"(r0), "=r"(r1)
+               : "r"(addr));
 }
 
 constexpr int kChunk = 64;
+
+// Keys are permuted inside each 64-key chunk: mask bit b (key b of the chunk)
+// is stored in shared-memory row p(b) = 8*((b%16)/2) + 2*(b/16) + b%2.  Then
+// the m16n8 fragment element (n-tile nt, column 2*tq+u) of a thread holds
+// key b = 16*tq + 2*nt + u, i.e. a thread's 16 mask bits are the contiguous
+// bits [16*tq, 16*tq+16) of the word, bit 2*nt+u.  16-row block j (n-tiles
+// 2j, 2j+1) covers the mask bits 0x000F000F000F000F << 4j.  Softmax and PV
+// are invariant under a consistent permutation of K and V rows.
+__device__ __forceinline__ int key_row(int b) { return ((b & 15) >> 1) * 8 + 2 * (b >> 4) + (b & 1); }
 
 template <int DH>
 struct Attn {
@@ -88,42 +102,52 @@ struct Attn {
   static constexpr int KS = DH / 16;    // k-steps for QK^T
   static constexpr int DN = DH / 8;     // n-tiles of the output
   static constexpr int CHUNK_HALVES = kChunk * PITCH;
+  static constexpr int BLK = 16 * PITCH * 2;  // bytes of a 16-key block
 
   uint32_t qa[KS][4];
   float o[DN][4];
-  float m_a, m_b, l_a, l_b;
+  float osum[4];  // P x (ones column of V): row sums l, [0] row a, [2] row b
+  float m_a, m_b;
   float scale;
+  uint32_t kl, vl, vl1;  // per-lane ldmatrix byte offsets
+
+  __device__ __forceinline__ void init(int lane) {
+    const int r8 = lane & 7;
+    kl = (uint32_t)(((((lane >> 4) & 1) * 8 + r8) * PITCH + ((lane >> 3) & 1) * 8) * 2);
+    vl = (uint32_t)(((((lane >> 3) & 1) * 8 + r8) * PITCH + ((lane >> 4) & 1) * 8) * 2);
+    vl1 = (uint32_t)(((((lane >> 3) & 1) * 8 + r8) * PITCH + DH) * 2);
+#pragma unroll
+    for (int i = 0; i < DN; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
+    osum[0] = osum[1] = osum[2] = osum[3] = 0.f;
+    m_a = m_b = -INFINITY;
+  }
 
   // One 64-key chunk for the warp's 16 rows.  kbase/vbase: shared addresses of
-  // the chunk's K and V; mwa/mwb: mask words of rows a/b (0 for absent rows).
+  // the chunk's (permuted) K and V rows; mwa/mwb: mask words of rows a/b.
+  // fl: block flags of (warp's 16-row group, chunk) from the DAG build
+  // (k_bflags): bit j = block j has an allowed pair, bit 4+j = fully allowed.
   __device__ __forceinline__ void chunk(uint32_t kbase, uint32_t vbase, uint64_t mwa, uint64_t mwb,
-                                        bool va, bool vb, int lane) {
-    const int tq = lane & 3;
-    uint32_t act = 0, full = 0;
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const uint32_t ba = (uint32_t)(mwa >> (16 * j)) & 0xffffu;
-      const uint32_t bb = (uint32_t)(mwb >> (16 * j)) & 0xffffu;
-      if (__any_sync(0xffffffffu, (ba | bb) != 0u)) act |= 1u << j;
-      const bool f = (!va || ba == 0xffffu) && (!vb || bb == 0xffffu);
-      if (__all_sync(0xffffffffu, f)) full |= 1u << j;
-    }
+                                        uint32_t fl, int tq) {
+    const uint32_t act = fl & 15u, full = fl >> 4;
     if (!act) return;
-    const uint32_t ta = thread_bits(mwa, tq), tb = thread_bits(mwb, tq);
+    const uint32_t ta = (uint32_t)(mwa >> (16 * tq)) & 0xffffu;
+    const uint32_t tb = (uint32_t)(mwb >> (16 * tq)) & 0xffffu;
     float s[8][4];
+    float mx_a = -INFINITY, mx_b = -INFINITY;  // raw row maxima over the active blocks
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-#pragma unroll
-      for (int u = 0; u < 2; ++u) s[2 * j + u][0] = s[2 * j + u][1] = s[2 * j + u][2] = s[2 * j + u][3] = 0.f;
       if (act & (1u << j)) {
 #pragma unroll
         for (int ks = 0; ks < KS; ++ks) {
-          const int r = 16 * j + ((lane >> 4) & 1) * 8 + (lane & 7);
-          const int col = ks * 16 + ((lane >> 3) & 1) * 8;
           uint32_t b0, b1, b2, b3;
-          ldsm_x4(kbase + (uint32_t)((r * PITCH + col) * 2), b0, b1, b2, b3);
-          mma16816(s[2 * j], qa[ks], b0, b1);
-          mma16816(s[2 * j + 1], qa[ks], b2, b3);
+          ldsm_x4(kbase + kl + j * BLK + ks * 32, b0, b1, b2, b3);
+          if (ks == 0) {
+            mma16816_z(s[2 * j], qa[ks], b0, b1);
+            mma16816_z(s[2 * j + 1], qa[ks], b2, b3);
+          } else {
+            mma16816(s[2 * j], qa[ks], b0, b1);
+            mma16816(s[2 * j + 1], qa[ks], b2, b3);
+          }
         }
         if (!(full & (1u << j))) {  // partial block: masked scores -> -inf
 #pragma unroll
@@ -135,35 +159,35 @@ struct Attn {
             if (!((tb >> (e + 1)) & 1u)) s[2 * j + u][3] = -INFINITY;
           }
         }
-      }
-    }
-    float mx_a = -INFINITY, mx_b = -INFINITY;
-#pragma unroll
-    for (int nt = 0; nt < 8; ++nt) {
-      if (act & (1u << (nt >> 1))) {
-        mx_a = fmaxf(mx_a, fmaxf(s[nt][0], s[nt][1]));
-        mx_b = fmaxf(mx_b, fmaxf(s[nt][2], s[nt][3]));
+        mx_a = fmaxf(mx_a, fmaxf(fmaxf(s[2 * j][0], s[2 * j][1]), fmaxf(s[2 * j + 1][0], s[2 * j + 1][1])));
+        mx_b = fmaxf(mx_b, fmaxf(fmaxf(s[2 * j][2], s[2 * j][3]), fmaxf(s[2 * j + 1][2], s[2 * j + 1][3])));
       }
     }
     mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 1));
     mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 2));
     mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 1));
     mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 2));
-    const float mn_a = fmaxf(m_a, mx_a * scale), mn_b = fmaxf(m_b, mx_b * scale);
-    const float mu_a = mn_a == -INFINITY ? 0.f : mn_a;
-    const float mu_b = mn_b == -INFINITY ? 0.f : mn_b;
-    if (mn_a != m_a || mn_b != m_b) {  // rescale only when a running max moved
-      const float al_a = ex2(m_a - mu_a), al_b = ex2(m_b - mu_b);
-      l_a *= al_a;
-      l_b *= al_b;
+    mx_a *= scale;
+    mx_b *= scale;
+    // Lazy rescaling: the reference m only moves when a row maximum exceeds it
+    // by more than 8 (log2 units), so P = exp2(s - m) <= 256 stays exact in
+    // fp16 and fp32; the final O / l is unchanged.
+    if (__any_sync(0xffffffffu, mx_a > m_a + 8.f || mx_b > m_b + 8.f)) {
+      const float mn_a = fmaxf(m_a, mx_a), mn_b = fmaxf(m_b, mx_b);
+      const float al_a = ex2(m_a - (mn_a == -INFINITY ? 0.f : mn_a));
+      const float al_b = ex2(m_b - (mn_b == -INFINITY ? 0.f : mn_b));
 #pragma unroll
       for (int i = 0; i < DN; ++i) {
         o[i][0] *= al_a; o[i][1] *= al_a;
         o[i][2] *= al_b; o[i][3] *= al_b;
       }
+      osum[0] *= al_a; osum[1] *= al_a;
+      osum[2] *= al_b; osum[3] *= al_b;
       m_a = mn_a;
       m_b = mn_b;
     }
+    const float mu_a = m_a == -INFINITY ? 0.f : m_a;
+    const float mu_b = m_b == -INFINITY ? 0.f : m_b;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       if (!(act & (1u << j))) continue;
@@ -171,24 +195,19 @@ struct Attn {
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
         const int nt = 2 * j + u;
-        const float p0 = ex2(fmaf(s[nt][0], scale, -mu_a));
-        const float p1 = ex2(fmaf(s[nt][1], scale, -mu_a));
-        const float p2 = ex2(fmaf(s[nt][2], scale, -mu_b));
-        const float p3 = ex2(fmaf(s[nt][3], scale, -mu_b));
-        l_a += p0 + p1;
-        l_b += p2 + p3;
-        pa[2 * u + 0] = pack_h2(p0, p1);
-        pa[2 * u + 1] = pack_h2(p2, p3);
+        pa[2 * u + 0] = pack_h2(ex2(fmaf(s[nt][0], scale, -mu_a)), ex2(fmaf(s[nt][1], scale, -mu_a)));
+        pa[2 * u + 1] = pack_h2(ex2(fmaf(s[nt][2], scale, -mu_b)), ex2(fmaf(s[nt][3], scale, -mu_b)));
       }
 #pragma unroll
       for (int dn = 0; dn < DN; dn += 2) {
-        const int r = 16 * j + ((lane >> 3) & 1) * 8 + (lane & 7);
-        const int col = dn * 8 + ((lane >> 4) & 1) * 8;
         uint32_t b0, b1, b2, b3;
-        ldsm_x4_t(vbase + (uint32_t)((r * PITCH + col) * 2), b0, b1, b2, b3);
+        ldsm_x4_t(vbase + vl + j * BLK + dn * 16, b0, b1, b2, b3);
         mma16816(o[dn], pa, b0, b1);
         mma16816(o[dn + 1], pa, b2, b3);
       }
+      uint32_t c0, c1;
+      ldsm_x2_t(vbase + vl1 + j * BLK, c0, c1);
+      mma16816(osum, pa, c0, c1);
     }
   }
 };
@@ -226,6 +245,8 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   const bool warp_live = qt * 128 + warp * 16 < N;
   const uint64_t* Ma = Mg + (int64_t)(va ? ra : 0) * W;
   const uint64_t* Mb = Mg + (int64_t)(vb ? rb : 0) * W;
+  // block flags of this warp's 16-row group, one byte per chunk (k_bflags)
+  const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)(warp_live ? qt * 8 + warp : 0) * nchunks;
 
   constexpr int SEGS = kChunk * DH / 8;  // 16-byte segments per matrix per chunk
   auto load_chunks = [&](int c0, int c1, int buf0) {
@@ -235,7 +256,7 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
       const int mat = rem / SEGS, r = (rem % SEGS) / (DH / 8), seg = rem % (DH / 8);
       const int key = (c0 + cc) * kChunk + r;
       const __half* src = (mat ? Vg : Kg) + (int64_t)(key < N ? key : 0) * ld3 + seg * 8;
-      __half* dst = (mat ? sV : sK) + (size_t)(buf0 + cc) * A::CHUNK_HALVES + r * A::PITCH + seg * 8;
+      __half* dst = (mat ? sV : sK) + (size_t)(buf0 + cc) * A::CHUNK_HALVES + key_row(r) * A::PITCH + seg * 8;
       cp_async16(static_cast<uint32_t>(__cvta_generic_to_shared(dst)), src, key < N);
     }
     cp_commit();
@@ -243,10 +264,10 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
 
   A st;
   st.scale = 1.4426950408889634f * rsqrtf((float)DH);  // log2(e)/sqrt(d_h)
-#pragma unroll
-  for (int i = 0; i < A::DN; ++i) st.o[i][0] = st.o[i][1] = st.o[i][2] = st.o[i][3] = 0.f;
-  st.m_a = st.m_b = -INFINITY;
-  st.l_a = st.l_b = 0.f;
+  st.init(lane);
+  // V padding columns [DH, DH+8) hold ones: the PV MMA then yields the row sums
+  for (int rr = threadIdx.x; rr < nbuf * kChunk; rr += blockDim.x)
+    *reinterpret_cast<uint4*>(sV + (size_t)rr * A::PITCH + DH) = make_uint4(0x3C003C00u, 0x3C003C00u, 0x3C003C00u, 0x3C003C00u);
 
   if (RESIDENT) load_chunks(0, nchunks, 0);
   else load_chunks(0, 1, 0);
@@ -270,7 +291,7 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
       const uint64_t nwa = (c + 1 < nchunks && va) ? Ma[c + 1] : 0ull;
       const uint64_t nwb = (c + 1 < nchunks && vb) ? Mb[c + 1] : 0ull;
       st.chunk(kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2),
-               mwa, mwb, va, vb, lane);
+               mwa, mwb, Fw[c], tq);
       mwa = nwa;
       mwb = nwb;
     }
@@ -289,18 +310,14 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
       __syncthreads();
       if (warp_live)
         st.chunk(kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2),
-                 mwa, mwb, va, vb, lane);
+                 mwa, mwb, Fw[c], tq);
       __syncthreads();
       mwa = nwa;
       mwb = nwb;
     }
     if (!warp_live) return;
   }
-  float l_a = st.l_a, l_b = st.l_b;
-  l_a += __shfl_xor_sync(0xffffffffu, l_a, 1);
-  l_a += __shfl_xor_sync(0xffffffffu, l_a, 2);
-  l_b += __shfl_xor_sync(0xffffffffu, l_b, 1);
-  l_b += __shfl_xor_sync(0xffffffffu, l_b, 2);
+  const float l_a = st.osum[0], l_b = st.osum[2];
   const float ia = l_a > 0.f ? 1.f / l_a : 0.f, ib = l_b > 0.f ? 1.f / l_b : 0.f;
   __half* Og = out + n0 * dmodel + h * DH;
 #pragma unroll

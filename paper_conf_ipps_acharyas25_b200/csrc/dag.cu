@@ -46,12 +46,21 @@ __device__ T block_excl_scan(T v, T* total, T* sh /*[32]*/) {
   return base + x - v;
 }
 
+// Graphs with N <= sc.sn nodes and E <= sc.se edges take the fused one-warp-
+// per-graph path (k_dag_small); the multi-kernel path below skips them.
+struct SmallCfg {
+  int sn, se, slot;  // node / edge capacity of a warp slot, slot bytes
+};
+__host__ __device__ inline bool is_small(int N, int E, const SmallCfg& sc) {
+  return N <= sc.sn && E <= sc.se;
+}
+
 __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
   __shared__ int64_t sh64[32];
-  int64_t carry_rows = 0, carry_tiles = 0, carry_q = 0;
+  int64_t carry_rows = 0, carry_tiles = 0, carry_q = 0, carry_f = 0;
   for (int base = 0; base < G; base += blockDim.x) {
     const int g = base + threadIdx.x;
-    int64_t rows = 0, tiles = 0, q = 0;
+    int64_t rows = 0, tiles = 0, q = 0, fl = 0;
     if (g < G) {
       const int64_t n = d.node_ptr[g + 1] - d.node_ptr[g];
       const int64_t e = d.edge_ptr[g + 1] - d.edge_ptr[g];
@@ -66,6 +75,7 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
         rows = n * 2 * T;
         tiles = T * T;
         q = T;
+        fl = ((n + 15) / 16) * ((n + 63) / 64);
       }
     }
     int64_t tot;
@@ -78,6 +88,9 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
     ex = block_excl_scan<int64_t>(q, &tot, sh64);
     if (g < G) d.qtile_off[g] = (int32_t)(carry_q + ex);
     carry_q += tot;
+    ex = block_excl_scan<int64_t>(fl, &tot, sh64);
+    if (g < G) d.bflag_off[g] = carry_f + ex;
+    carry_f += tot;
   }
   // lowest graph with a size error (device-detected errors lower it later)
   __shared__ int s_first;
@@ -90,14 +103,16 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
     d.row_off[G] = carry_rows;
     d.tile_off[G] = carry_tiles;
     d.qtile_off[G] = (int32_t)carry_q;
+    d.bflag_off[G] = carry_f;
     *d.first_bad = s_first;
   }
 }
 
 // K1: validation + successor CSR + Kahn levels / depth.  One CTA per graph.
-__global__ void __launch_bounds__(256) k_depth(DagDev d) {
+__global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc) {
   const int g = blockIdx.x;
   if (d.status[g] != PREDTOP_OK) return;
+  if (is_small((int)(d.node_ptr[g + 1] - d.node_ptr[g]), (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
   __shared__ int s_err, s_tail;
   __shared__ int32_t sh32[32];
   const int64_t n0 = d.node_ptr[g];
@@ -194,11 +209,12 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d) {
 }
 
 // K2: closure.  grid = (G, slices); dynamic smem `smem_bytes`.
-__global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes) {
+__global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, SmallCfg sc) {
   extern __shared__ __align__(16) unsigned char sm[];
   const int g = blockIdx.x, slice = blockIdx.y;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
+  if (is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
   const int st = d.status[g];
   if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;  // no rows
   const int W = 2 * ((N + 127) / 128);
@@ -273,12 +289,13 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes) {
 }
 
 // K3: M = R | R^T | I and per-tile popcounts.  grid = (G, YB), 8 warps.
-__global__ void __launch_bounds__(256) k_mask(DagDev d) {
+__global__ void __launch_bounds__(256) k_mask(DagDev d, SmallCfg sc) {
   const int g = blockIdx.x;
   const int st = d.status[g];
   if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
+  if (is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
   const int W = 2 * ((N + 127) / 128);
   const int T = (N + 127) / 128;
   const uint32_t* R32 = reinterpret_cast<const uint32_t*>(d.R + d.row_off[g]);
@@ -303,7 +320,7 @@ __global__ void __launch_bounds__(256) k_mask(DagDev d) {
       }
       uint32_t m = direct | t;
       if (U0 == V0 && u < N) m |= 1u << lane;
-      if (u >= N) m = 0;
+      if (u >= N || st != PREDTOP_OK) m = 0;  // invalid graph: M defined as zero
       if (u < N) M32[(int64_t)u * W32 + vr] = m;
       int c = __popc(m);
 #pragma unroll
@@ -313,12 +330,13 @@ __global__ void __launch_bounds__(256) k_mask(DagDev d) {
   }
 }
 
-__global__ void __launch_bounds__(256) k_classify(DagDev d) {
+__global__ void __launch_bounds__(256) k_classify(DagDev d, SmallCfg sc) {
   const int g = blockIdx.x;
   const int st = d.status[g];
   if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
   __shared__ unsigned long long s_pairs;
   const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+  if (is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
   const int T = (N + 127) / 128;
   const int32_t* cnt = d.tile_cnt + d.tile_off[g];
   uint8_t* cls = d.tile_cls + d.tile_off[g];
@@ -337,13 +355,223 @@ __global__ void __launch_bounds__(256) k_classify(DagDev d) {
   if (threadIdx.x == 0) d.pairs[g] = (int64_t)s_pairs;
 }
 
-__global__ void k_work(DagDev d) {
+__global__ void k_work(DagDev d, SmallCfg sc) {
   const int g = blockIdx.x;
   const int st = d.status[g];
   if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
   const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+  if (is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
   const int T = (N + 127) / 128;
   for (int qt = threadIdx.x; qt < T; qt += blockDim.x) d.work[d.qtile_off[g] + qt] = make_int2(g, qt);
+}
+
+
+// ---------------------------------------------------------------------------
+// Fused small-graph path: one warp per graph does K1 + K2 + K3 in shared
+// memory (validation, successor CSR, Kahn depth, closure, mask, tile classes,
+// |A|, attention work items) with __syncwarp between levels instead of CTA
+// barriers.  GPT-size stage graphs (N ~ 300) need ~25 KB per warp.
+__device__ __forceinline__ size_t small_int_bytes(const SmallCfg& sc) {
+  return align_up((size_t)4 * (4 * (size_t)sc.sn + 2 + sc.se + 24), 16);
+}
+
+__global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc) {
+  extern __shared__ __align__(16) unsigned char sm_small[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int g = blockIdx.x * 4 + warp;
+  if (g >= G || d.status[g] != PREDTOP_OK) return;
+  const int64_t n0 = d.node_ptr[g];
+  const int N = (int)(d.node_ptr[g + 1] - n0);
+  const int64_t e0 = d.edge_ptr[g];
+  const int E = (int)(d.edge_ptr[g + 1] - e0);
+  if (!is_small(N, E, sc)) return;
+  unsigned char* slot = sm_small + (size_t)warp * sc.slot;
+  int* indeg = reinterpret_cast<int*>(slot);
+  int* soff = indeg + sc.sn;        // N+1
+  int* succ = soff + sc.sn + 1;     // E
+  int* topo = succ + sc.se;         // N
+  int* lptr = topo + sc.sn;         // N+1 (first the fill cursor)
+  int* tcnt = lptr + sc.sn + 1;     // 16 tile counts (T <= 4)
+  int* ctr = tcnt + 16;             // Kahn queue tail
+  uint64_t* R = reinterpret_cast<uint64_t*>(slot + small_int_bytes(sc));
+  const int W = 2 * ((N + 127) / 128), T = (N + 127) / 128;
+  const int32_t* src = d.src + e0;
+  const int32_t* dst = d.dst + e0;
+  int32_t* depth = d.depth + n0;
+  uint64_t* Rg = d.R + d.row_off[g];
+  uint32_t* M32 = reinterpret_cast<uint32_t*>(d.M + d.row_off[g]);
+  uint8_t* cls = d.tile_cls + d.tile_off[g];
+
+  for (int v = lane; v < N; v += 32) { indeg[v] = 0; soff[v + 1] = 0; }
+  if (lane < 16) tcnt[lane] = 0;
+  if (lane == 0) { soff[0] = 0; *ctr = 0; }
+  __syncwarp();
+  bool rng = false, self = false;
+  for (int e = lane; e < E; e += 32) {
+    const int s = src[e], t = dst[e];
+    if (s < 0 || s >= N || t < 0 || t >= N) rng = true;
+    else if (s == t) self = true;
+    else {
+      atomicAdd(&indeg[t], 1);
+      atomicAdd(&soff[s + 1], 1);
+    }
+  }
+  rng = __any_sync(0xffffffffu, rng);
+  self = __any_sync(0xffffffffu, self);
+  int status = rng ? PREDTOP_ERR_RANGE : self ? PREDTOP_ERR_SELF_LOOP : PREDTOP_OK;
+  __syncwarp();
+  int level = 0;
+  if (status == PREDTOP_OK) {
+    int carry = 0;  // inclusive scan of out-degrees
+    for (int base = 0; base < N; base += 32) {
+      const int v = base + lane;
+      int x = v < N ? soff[v + 1] : 0;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      if (v < N) soff[v + 1] = carry + x;
+      carry += __shfl_sync(0xffffffffu, x, 31);
+    }
+    __syncwarp();
+    for (int v = lane; v < N; v += 32) lptr[v] = soff[v];
+    __syncwarp();
+    for (int e = lane; e < E; e += 32) succ[atomicAdd(&lptr[src[e]], 1)] = dst[e];
+    __syncwarp();
+    // Kahn, level synchronous (P:137 depth = 1 + max predecessor depth)
+    int tail = 0;
+    for (int base = 0; base < N; base += 32) {
+      const int v = base + lane;
+      const bool z = v < N && indeg[v] == 0;
+      const uint32_t bal = __ballot_sync(0xffffffffu, z);
+      if (z) {
+        topo[tail + __popc(bal & ((1u << lane) - 1u))] = v;
+        depth[v] = 0;
+      }
+      tail += __popc(bal);
+    }
+    if (lane == 0) { *ctr = tail; lptr[0] = 0; }
+    __syncwarp();
+    int lb = 0, le = tail;
+    while (lb < le) {
+      for (int i = lb + lane; i < le; i += 32) {
+        const int v = topo[i];
+        for (int k = soff[v]; k < soff[v + 1]; ++k) {
+          const int w = succ[k];
+          if (atomicSub(&indeg[w], 1) == 1) {
+            topo[atomicAdd(ctr, 1)] = w;
+            depth[w] = level + 1;
+          }
+        }
+      }
+      __syncwarp();
+      lb = le;
+      le = *reinterpret_cast<volatile int*>(ctr);
+      ++level;
+      if (lane == 0) lptr[level] = lb;
+      __syncwarp();
+    }
+    if (le != N) status = PREDTOP_ERR_CYCLE;
+  }
+  if (lane == 0) d.num_levels[g] = level;
+  if (status != PREDTOP_OK) {
+    if (lane == 0) {
+      d.status[g] = status;
+      atomicMin(d.first_bad, g);
+    }
+    for (int v = lane; v < N; v += 32) depth[v] = -1;
+    for (int64_t i = lane; i < (int64_t)N * W; i += 32) Rg[i] = 0;
+    for (int64_t i = lane; i < (int64_t)N * 2 * W; i += 32) M32[i] = 0;
+    for (int t = lane; t < T * T; t += 32) cls[t] = 0;
+    return;
+  }
+  // closure R[v] = OR_{w in succ(v)} (R[w] | {w}), deepest level first
+  for (int i = lane; i < N * W; i += 32) R[i] = 0;
+  __syncwarp();
+  for (int l = level - 1; l >= 0; --l) {
+    const int lb = lptr[l], le = lptr[l + 1];
+    for (int it = lane; it < (le - lb) * W; it += 32) {
+      const int v = topo[lb + it / W], j = it % W;
+      uint64_t acc = 0;
+      for (int k = soff[v]; k < soff[v + 1]; ++k) {
+        const int w = succ[k];
+        acc |= R[w * W + j];
+        if ((w >> 6) == j) acc |= 1ull << (w & 63);
+      }
+      R[v * W + j] = acc;
+    }
+    __syncwarp();
+  }
+  for (int i = lane; i < N * W; i += 32) Rg[i] = R[i];
+  // mask M = R | R^T | I (32x32 ballot transposes) and per-tile counts
+  const uint32_t* R32 = reinterpret_cast<const uint32_t*>(R);
+  const int W32 = 2 * W, NB = (N + 31) / 32;
+  for (int ur = 0; ur < NB; ++ur) {
+    const int U0 = ur * 32, u = U0 + lane;
+    for (int vr = 0; vr < W32; ++vr) {
+      const int V0 = vr * 32, vrow = V0 + lane;
+      const uint32_t direct = u < N ? R32[u * W32 + vr] : 0u;
+      const uint32_t x = vrow < N ? R32[vrow * W32 + ur] : 0u;
+      uint32_t t = 0;
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const uint32_t b = __ballot_sync(0xffffffffu, (x >> i) & 1u);
+        if (lane == i) t = b;
+      }
+      uint32_t m = direct | t;
+      if (U0 == V0 && u < N) m |= 1u << lane;
+      if (u < N) M32[(int64_t)u * W32 + vr] = m;
+      else m = 0;
+      int c = __popc(m);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+      if (lane == 0 && V0 < N) tcnt[(U0 / 128) * T + V0 / 128] += c;
+    }
+  }
+  __syncwarp();
+  long long pairs = 0;
+  for (int t = lane; t < T * T; t += 32) {
+    const int qt = t / T, kt = t % T;
+    const int cells = min(128, N - qt * 128) * min(128, N - kt * 128);
+    const int c = tcnt[t];
+    cls[t] = (uint8_t)(c == 0 ? 0 : (c == cells ? 2 : 1));
+    pairs += c;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) pairs += __shfl_xor_sync(0xffffffffu, pairs, o);
+  if (lane == 0) d.pairs[g] = pairs;
+  for (int qt = lane; qt < T; qt += 32) d.work[d.qtile_off[g] + qt] = make_int2(g, qt);
+}
+
+// Block flags for the attention kernel: for every 16-row group rg and 64-key
+// chunk c, bit j (j < 4) = some row of the group has an allowed key in the
+// permuted 16-key block j (mask bits 0x000F000F000F000F << 4j, attention.cu),
+// bit 4+j = every row of the group allows every key of block j.
+__global__ void __launch_bounds__(128) k_bflags(DagDev d) {
+  const int g = blockIdx.x;
+  if (d.status[g] == PREDTOP_ERR_TOO_LARGE || d.status[g] == PREDTOP_ERR_INVALID_ARG) return;
+  const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+  const int W = 2 * ((N + 127) / 128), nch = (N + 63) / 64, ng = (N + 15) / 16;
+  const uint64_t* Mg = d.M + d.row_off[g];
+  uint8_t* out = d.bflag + d.bflag_off[g];
+  for (int it = threadIdx.x; it < ng * nch; it += blockDim.x) {
+    const int rg = it / nch, c = it % nch;
+    uint64_t o = 0, a = ~0ull;
+    for (int r = rg * 16; r < min(N, rg * 16 + 16); ++r) {
+      const uint64_t w = Mg[(int64_t)r * W + c];
+      o |= w;
+      a &= w;
+    }
+    uint32_t f = 0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint64_t MJ = 0x000F000F000F000Full << (4 * j);
+      if (o & MJ) f |= 1u << j;
+      if ((a & MJ) == MJ) f |= 16u << j;
+    }
+    out[it] = (uint8_t)f;
+  }
 }
 
 __global__ void k_copy_words(const int64_t* total, const uint64_t* from, uint64_t* to) {
@@ -363,9 +591,29 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
     k_meta<<<1, 1024, 0, st>>>(d, G, b.max_nodes);
     PT_LAUNCH_CHECK();
   }
+  // small-graph capacity: graphs up to 512 nodes (and <= 4 edges/node) run fused
+  SmallCfg sc{0, 0, 0};
+  if (b.max_nodes <= 512) {
+    sc.sn = b.max_nodes;
+    sc.se = 4 * b.max_nodes;
+    const size_t ib = align_up((size_t)4 * (4 * (size_t)sc.sn + 2 + sc.se + 24), 16);
+    sc.slot = (int)align_up(ib + (size_t)sc.sn * 2 * ceil_div(sc.sn, 128) * 8, 16);
+  }
+  const bool all_small_possible = sc.sn > 0;
+  if (all_small_possible) {
+    static int attr_small = 0;
+    if (attr_small < 4 * sc.slot) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_dag_small, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       std::max(4 * sc.slot, 48 * 1024)));
+      attr_small = std::max(4 * sc.slot, 48 * 1024);
+    }
+    ProfScope _p(PK_DAG_SMALL, st);
+    k_dag_small<<<(unsigned)ceil_div(G, 4), 128, 4 * sc.slot, st>>>(d, G, sc);
+    PT_LAUNCH_CHECK();
+  }
 {
     ProfScope _p(PK_DAG_DEPTH, st);
-    k_depth<<<G, 256, 0, st>>>(d);
+    k_depth<<<G, 256, 0, st>>>(d, sc);
     PT_LAUNCH_CHECK();
   }
   // closure: shared memory for a column slice of all rows of the largest graph
@@ -387,24 +635,29 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
   dim3 gc(G, (unsigned)std::max<int64_t>(1, slices));
 {
     ProfScope _p(PK_DAG_CLOSURE, st);
-    k_closure<<<gc, 256, smem, st>>>(d, smem);
+    k_closure<<<gc, 256, smem, st>>>(d, smem, sc);
     PT_LAUNCH_CHECK();
   }
   const int NBmax = (int)ceil_div(maxN, 32);
   dim3 gm(G, (unsigned)std::min(NBmax, 64));
 {
     ProfScope _p(PK_DAG_MASK, st);
-    k_mask<<<gm, 256, 0, st>>>(d);
+    k_mask<<<gm, 256, 0, st>>>(d, sc);
     PT_LAUNCH_CHECK();
   }
 {
     ProfScope _p(PK_DAG_CLASSIFY, st);
-    k_classify<<<G, 256, 0, st>>>(d);
+    k_classify<<<G, 256, 0, st>>>(d, sc);
     PT_LAUNCH_CHECK();
   }
 {
     ProfScope _p(PK_DAG_WORK, st);
-    k_work<<<G, 128, 0, st>>>(d);
+    k_work<<<G, 128, 0, st>>>(d, sc);
+    PT_LAUNCH_CHECK();
+  }
+  {
+    ProfScope _p(PK_DAG_FLAGS, st);
+    k_bflags<<<G, 128, 0, st>>>(d);
     PT_LAUNCH_CHECK();
   }
   return PREDTOP_OK;

@@ -41,6 +41,9 @@ struct DagDev {
   int32_t* tile_cnt;   // [sum T_g^2]
   uint8_t* tile_cls;   // [sum T_g^2]
   int2* work;          // [qtile bound] (graph, q-tile) attention work items
+  int64_t* bflag_off;  // [G+1] prefix of ceil(N/16) * ceil(N/64)
+  uint8_t* bflag;      // per (16-row group, 64-key chunk): bits 0-3 block has an allowed
+                       // pair, bits 4-7 block fully allowed (permuted 16-key blocks, attention.cu)
 };
 
 }  // namespace predtop
@@ -51,6 +54,7 @@ struct predtop_dag_s {
   int64_t words_bound;  // upper bound of sum N_g W_g
   int64_t tiles_bound;  // upper bound of sum T_g^2
   int64_t qtiles_bound; // upper bound of sum T_g
+  int64_t bflags_bound; // upper bound of sum ceil(N/16) ceil(N/64)
   int32_t max_words;    // 2*ceil(max_nodes/128)
 };
 
