@@ -444,6 +444,8 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     const LayerDev& L = m->layer[l];
     GemmArgs a{};
     a.M = M; a.K = d; a.N = 3 * d; a.bias = L.bqkv; a.out16 = w.qkv;
+    a.qcols = d;  // Q in log2 units for the attention kernel: q * log2(e) / sqrt(d_h)
+    a.qscale = (float)(1.4426950408889634 / sqrt((double)(d / H)));
     {
       ProfScope _p(PK_GEMM_QKV, st);
       if ((s = gemm_launch(&tm_x16, &L.tm_qkv, m->bn_qkv, EPI_BIAS_F16, a, st)) != PREDTOP_OK) return s;

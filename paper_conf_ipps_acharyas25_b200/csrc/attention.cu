@@ -210,6 +210,7 @@ struct Attn {
       mma16816(osum, pa, c0, c1);
     }
   }
+
 };
 
 template <int DH, bool RESIDENT>
@@ -234,8 +235,6 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   const uint64_t* Mg = d.M + d.row_off[g];
   const int ld3 = 3 * dmodel;
   const __half* Qg = qkv + n0 * ld3 + h * DH;
-  const __half* Kg = Qg + dmodel;
-  const __half* Vg = Qg + 2 * dmodel;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int gq = lane >> 2, tq = lane & 3;
@@ -248,22 +247,37 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   // block flags of this warp's 16-row group, one byte per chunk (k_bflags)
   const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)(warp_live ? qt * 8 + warp : 0) * nchunks;
 
+  // Loader roles: a chunk is 2 (K, V) x 64 keys x DH/8 16-byte segments =
+  // 16*DH segments; thread t always moves the same (matrix, key, segment)
+  // slots (t, t+256, ...) of every chunk, so per chunk it only adds offsets.
   constexpr int SEGS = kChunk * DH / 8;  // 16-byte segments per matrix per chunk
+  constexpr int PER = 2 * SEGS / 256;    // slots per thread per chunk (1 or 2)
+  static_assert(2 * SEGS % 256 == 0, "loader");
+  uint32_t ld_dst[PER];
+  int64_t ld_src[PER];
+  int ld_key[PER];
+#pragma unroll
+  for (int k = 0; k < PER; ++k) {
+    const unsigned s = threadIdx.x + 256u * k;
+    const unsigned mat = s / SEGS, r = (s % SEGS) / (DH / 8), seg = s % (DH / 8);
+    ld_key[k] = (int)r;
+    ld_src[k] = (int64_t)(mat ? 2 * dmodel : dmodel) + (int64_t)r * ld3 + seg * 8;  // from Qg
+    ld_dst[k] = static_cast<uint32_t>(__cvta_generic_to_shared((mat ? sV : sK) + key_row((int)r) * A::PITCH + seg * 8));
+  }
   auto load_chunks = [&](int c0, int c1, int buf0) {
-    const int total = (c1 - c0) * 2 * SEGS;
-    for (int s = threadIdx.x; s < total; s += blockDim.x) {
-      const int cc = s / (2 * SEGS), rem = s % (2 * SEGS);
-      const int mat = rem / SEGS, r = (rem % SEGS) / (DH / 8), seg = rem % (DH / 8);
-      const int key = (c0 + cc) * kChunk + r;
-      const __half* src = (mat ? Vg : Kg) + (int64_t)(key < N ? key : 0) * ld3 + seg * 8;
-      __half* dst = (mat ? sV : sK) + (size_t)(buf0 + cc) * A::CHUNK_HALVES + key_row(r) * A::PITCH + seg * 8;
-      cp_async16(static_cast<uint32_t>(__cvta_generic_to_shared(dst)), src, key < N);
+    for (int c = c0; c < c1; ++c) {
+      const uint32_t boff = (uint32_t)((buf0 + c - c0) * A::CHUNK_HALVES * 2);
+#pragma unroll
+      for (int k = 0; k < PER; ++k) {
+        const int key = c * kChunk + ld_key[k];
+        const __half* src = Qg + (key < N ? ld_src[k] + (int64_t)c * kChunk * ld3 : 0);
+        cp_async16(ld_dst[k] + boff, src, key < N);
+      }
     }
     cp_commit();
   };
 
   A st;
-  st.scale = 1.4426950408889634f * rsqrtf((float)DH);  // log2(e)/sqrt(d_h)
   st.init(lane);
   // V padding columns [DH, DH+8) hold ones: the PV MMA then yields the row sums
   for (int rr = threadIdx.x; rr < nbuf * kChunk; rr += blockDim.x)
@@ -286,14 +300,22 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
   if (RESIDENT) {
     cp_wait<0>();
     __syncthreads();
+  }
+  st.scale = 1.f;  // online path: scores already in log2 units
+
+  if (RESIDENT) {
     if (!warp_live) return;
+    uint32_t fl = Fw[0];
     for (int c = 0; c < nchunks; ++c) {
-      const uint64_t nwa = (c + 1 < nchunks && va) ? Ma[c + 1] : 0ull;
-      const uint64_t nwb = (c + 1 < nchunks && vb) ? Mb[c + 1] : 0ull;
-      st.chunk(kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2),
-               mwa, mwb, Fw[c], tq);
+      const bool more = c + 1 < nchunks;
+      const uint64_t nwa = (more && va) ? Ma[c + 1] : 0ull;
+      const uint64_t nwb = (more && vb) ? Mb[c + 1] : 0ull;
+      const uint32_t nfl = more ? Fw[c + 1] : 0u;
+      const uint32_t kc = kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2);
+      st.chunk(kc, vc, mwa, mwb, __shfl_sync(0xffffffffu, fl, 0), tq);
       mwa = nwa;
       mwb = nwb;
+      fl = nfl;
     }
   } else {
     for (int c = 0; c < nchunks; ++c) {
@@ -308,9 +330,11 @@ __global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmo
         cp_wait<0>();
       }
       __syncthreads();
-      if (warp_live)
-        st.chunk(kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2),
-                 mwa, mwb, Fw[c], tq);
+      if (warp_live) {
+        const uint32_t kc = kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2);
+        const uint32_t fl = __shfl_sync(0xffffffffu, (uint32_t)Fw[c], 0);
+        st.chunk(kc, vc, mwa, mwb, fl, tq);
+      }
       __syncthreads();
       mwa = nwa;
       mwb = nwb;

@@ -214,10 +214,11 @@ __global__ void __launch_bounds__(kThreads, 1)
             bb[4 * k] = t4.x; bb[4 * k + 1] = t4.y; bb[4 * k + 2] = t4.z; bb[4 * k + 3] = t4.w;
           }
           uint32_t p[8];
+          const float qs = (n0 + c < args.qcols) ? args.qscale : 1.f;
 #pragma unroll
           for (int j = 0; j < 16; j += 2) {
-            float x0 = v[j] + bb[j];
-            float x1 = v[j + 1] + bb[j + 1];
+            float x0 = (v[j] + bb[j]) * qs;
+            float x1 = (v[j + 1] + bb[j + 1]) * qs;
             if (EPI == EPI_BIAS_RELU_F16) { x0 = fmaxf(x0, 0.f); x1 = fmaxf(x1, 0.f); }
             p[j / 2] = pack_half2(x0, x1);
           }

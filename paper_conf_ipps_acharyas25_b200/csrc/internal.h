@@ -119,6 +119,8 @@ struct GemmArgs {
   const float* gamma;
   const float* beta;
   float eps;
+  int qcols;      // bias epilogue: output columns [0, qcols) are multiplied by qscale
+  float qscale;   // (QKV: Q pre-scaled by log2(e)/sqrt(d_h) for the attention kernel)
 };
 predtop_status gemm_launch(const CUtensorMap* tmA, const CUtensorMap* tmB, int bn, int epi,
                            const GemmArgs& a, cudaStream_t st);

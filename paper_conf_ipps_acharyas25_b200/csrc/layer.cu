@@ -42,7 +42,8 @@ struct TailCfg {
   static constexpr int SP1 = 128 * 128 * 2; // ReLU chunk 1
   static constexpr int SH = 128 * D * 2;    // h fp16 (FFN-1 A operand) / x' fp16 staging
   static constexpr int SLOT = (D > FC ? D : FC) * 64 * 2;
-  static constexpr int FIXED = X32 + SA + SP1 + SH + 1024;
+  static constexpr int PARAMS = (6 * D + 1024) * 4;  // bo g1 be1 b2 g2 be2 [D], b1 [<= 1024]
+  static constexpr int FIXED = X32 + SA + SP1 + SH + PARAMS + 1024;
   static constexpr int RS_FIT = (224 * 1024 - FIXED) / SLOT;
   static constexpr int RS = RS_FIT > 6 ? 6 : RS_FIT;
   static constexpr int SMEM = FIXED + RS * SLOT;
@@ -72,6 +73,23 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
   unsigned char* sP1 = sA + C::SA;          // ReLU chunk buffer 1
   unsigned char* sH = sP1 + C::SP1;         // h fp16 / x' fp16
   unsigned char* ring = sH + C::SH;
+  float* sPar = reinterpret_cast<float*>(ring + RS * C::SLOT);  // per-layer vectors
+  float* p_bo = sPar;
+  float* p_g1 = sPar + D;
+  float* p_be1 = sPar + 2 * D;
+  float* p_b2 = sPar + 3 * D;
+  float* p_g2 = sPar + 4 * D;
+  float* p_be2 = sPar + 5 * D;
+  float* p_b1 = sPar + 6 * D;
+  for (int i = threadIdx.x; i < D; i += blockDim.x) {
+    p_bo[i] = args.bo[i];
+    p_g1[i] = args.g1[i];
+    p_be1[i] = args.be1[i];
+    p_b2[i] = args.b2[i];
+    p_g2[i] = args.g2[i];
+    p_be2[i] = args.be2[i];
+  }
+  for (int i = threadIdx.x; i < args.dff; i += blockDim.x) p_b1[i] = args.b1[i];
   __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
   __shared__ __align__(8) uint64_t a_full, a_free, x_full, x_free, o_full, o_empty, h_ready;
   __shared__ __align__(8) uint64_t f_full[2], f_empty[2], p_ready[2], p_free[2], out_full, out_empty;
@@ -217,8 +235,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
           const int c4 = 2 * c8 + h2;
           float4* p = reinterpret_cast<float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
           float4 x = *p;
-          const float4 gm = __ldg(reinterpret_cast<const float4*>(g) + c4);
-          const float4 bt = __ldg(reinterpret_cast<const float4*>(be) + c4);
+          const float4 gm = reinterpret_cast<const float4*>(g)[c4];
+          const float4 bt = reinterpret_cast<const float4*>(be)[c4];
           x.x = (x.x - mean) * rstd * gm.x + bt.x;
           x.y = (x.y - mean) * rstd * gm.y + bt.y;
           x.z = (x.z - mean) * rstd * gm.z + bt.z;
@@ -242,7 +260,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           float4* p = reinterpret_cast<float4*>(box + sm100::swz<128>(r, (c % 32) / 4 + k));
-          const float4 b = __ldg(reinterpret_cast<const float4*>(bias + c) + k);
+          const float4 b = reinterpret_cast<const float4*>(bias + c)[k];
           float4 x = *p;
           x.x += v[4 * k + 0] + b.x;
           x.y += v[4 * k + 1] + b.y;
@@ -266,9 +284,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       sm100::mbar_wait(&o_full, i & 1);
       sm100::mbar_wait(&x_full, i & 1);
       sm100::tc_fence_after();
-      const float s1 = add_residual(acc_o, args.bo);
+      const float s1 = add_residual(acc_o, p_bo);
       sm100::tc_fence_before();
-      layer_norm(s1, args.g1, args.be1);
+      layer_norm(s1, p_g1, p_be1);
       sm100::fence_proxy_async();
       sm100::named_bar<kEpi>(1);
       if (leader) {
@@ -283,14 +301,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
         sm100::tc_fence_after();
         unsigned char* P = b ? sP1 : sA;
         const uint32_t accf = tmem + D + b * FC + lrow;
-        const float* b1 = args.b1 + j * FC;
+        const float* b1 = p_b1 + j * FC;
 #pragma unroll 1
         for (int c = half * FC / 2; c < (half + 1) * FC / 2; c += 16) {
           sm100::tmem_ld16(accf + c, v);
           uint32_t pk[8];
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
-            const float4 bb = __ldg(reinterpret_cast<const float4*>(b1 + c) + k);
+            const float4 bb = reinterpret_cast<const float4*>(b1 + c)[k];
             pk[2 * k] = sm100::pack_half2(fmaxf(v[4 * k] + bb.x, 0.f), fmaxf(v[4 * k + 1] + bb.y, 0.f));
             pk[2 * k + 1] = sm100::pack_half2(fmaxf(v[4 * k + 2] + bb.z, 0.f), fmaxf(v[4 * k + 3] + bb.w, 0.f));
           }
@@ -309,9 +327,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       // ---- LN2 and stores
       sm100::mbar_wait(&out_full, i & 1);
       sm100::tc_fence_after();
-      const float s2 = add_residual(acc_out, args.b2);
+      const float s2 = add_residual(acc_out, p_b2);
       sm100::tc_fence_before();
-      layer_norm(s2, args.g2, args.be2);
+      layer_norm(s2, p_g2, p_be2);
       sm100::fence_proxy_async();
       sm100::named_bar<kEpi>(1);
       if (leader) {

@@ -644,18 +644,22 @@ def stage_batch(config: str, num_graphs: int, first_graph: int = 0,
 # --------------------------------------------------------------------------
 # Model configuration and weights (reading R14 in DESIGN.md)
 # --------------------------------------------------------------------------
-# head_scale / out_bias (R14): the synthetic weights are untrained, so the raw
-# head output w_o . z2 has an arbitrary sign and a scale that grows with the
-# sum-pooled graph size.  These per-config constants (chosen once from a sample
-# of the raw outputs, then frozen) map the outputs to positive, latency-like
-# values of O(1-10) without letting the output bias dominate.
+# head_scale / out_bias (R14, R17): the synthetic weights are
+# untrained, so the raw head output w_o . z2 has an arbitrary sign and a scale
+# that grows with the sum-pooled graph size.  These per-config constants map
+# the outputs to positive, latency-like values bounded away from zero (the
+# per-graph relative error of the north star is ill-conditioned near 0)
+# without letting the output bias dominate.  Chosen once from the raw-output
+# distribution (gpt: 256 graphs, mean 17.9, std 8.0, min -4.7, max 34.8;
+# paper: 128 graphs, mean -161, std 27; moe: 12 graphs, mean 815, std 119) so
+# that y >= ~2 down to mean - 4 std, then frozen.
 MODEL_CONFIGS = {
     "tiny": dict(num_layers=1, d_model=32, num_heads=2, d_ff=128, pool=0, ln_eps=1e-5,
                  head_scale=1.0, out_bias=4.0, seed=100),
     "paper": dict(num_layers=4, d_model=64, num_heads=4, d_ff=256, pool=0, ln_eps=1e-5,
-                  head_scale=-0.03, out_bias=0.0, seed=101),
+                  head_scale=-0.03, out_bias=0.5, seed=101),
     "gpt": dict(num_layers=4, d_model=128, num_heads=8, d_ff=512, pool=0, ln_eps=1e-5,
-                head_scale=0.25, out_bias=1.0, seed=102),
+                head_scale=0.25, out_bias=5.5, seed=102),
     "moe": dict(num_layers=4, d_model=256, num_heads=8, d_ff=1024, pool=0, ln_eps=1e-5,
                 head_scale=0.007, out_bias=0.0, seed=103),
     "16k": dict(num_layers=4, d_model=128, num_heads=8, d_ff=512, pool=0, ln_eps=1e-5,
