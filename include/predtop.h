@@ -32,7 +32,12 @@
  *  - Pointers: array arguments are DEVICE pointers unless marked [host].
  *    All device work is stream-ordered on `cuda_stream` (a cudaStream_t,
  *    NULL = legacy default stream).  Input arrays are only read during the
- *    call's stream-ordered work; nothing keeps a reference to them.
+ *    call's stream-ordered work, except that a predtop_dag keeps node_ptr,
+ *    edge_ptr and feats (and depth_out) by reference for the later
+ *    predtop_stage_forward calls on it.
+ *  - CUDA graphs: with PREDTOP_NO_SYNC every call is stream-capturable (no
+ *    host synchronisation, no allocation), so a whole prediction step can be
+ *    captured once and replayed (bench.py does).
  *  - There is no CPU fallback: without a usable sm_100 device every call that
  *    launches work returns PREDTOP_ERR_CUDA.
  */

@@ -214,7 +214,7 @@ struct Attn {
 };
 
 template <int DH, bool RESIDENT>
-__global__ void __launch_bounds__(256, 2) k_attn(DagDev d, int G, int H, int dmodel,
+__global__ void __launch_bounds__(256, DH == 16 ? 3 : 2) k_attn(DagDev d, int G, int H, int dmodel,
                                                  const __half* __restrict__ qkv,
                                                  __half* __restrict__ out) {
   using A = Attn<DH>;

@@ -288,6 +288,21 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
       Rg[(it / nw) * W + word0 + it % nw] = Rs[(it / nw) * rs + it % nw];
 }
 
+// 32x32 bit-matrix transpose across a warp: lane i holds row i (bit j =
+// column j) on entry and column i (bit j = row j) on exit.  Five butterfly
+// stages of shuffles with swap masks (instead of 32 ballots).
+__device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
+#pragma unroll
+  for (int k = 0; k < 5; ++k) {
+    const int sh = 16 >> k;
+    const uint32_t m = k == 0 ? 0x0000FFFFu : k == 1 ? 0x00FF00FFu : k == 2 ? 0x0F0F0F0Fu
+                     : k == 3 ? 0x33333333u : 0x55555555u;
+    const uint32_t y = __shfl_xor_sync(0xffffffffu, x, sh);
+    x = (lane & sh) ? ((x & ~m) | ((y >> sh) & m)) : ((x & m) | ((y << sh) & ~m));
+  }
+  return x;
+}
+
 // K3: M = R | R^T | I and per-tile popcounts.  grid = (G, YB), 8 warps.
 __global__ void __launch_bounds__(256) k_mask(DagDev d, SmallCfg sc) {
   const int g = blockIdx.x;
@@ -312,12 +327,7 @@ __global__ void __launch_bounds__(256) k_mask(DagDev d, SmallCfg sc) {
       const uint32_t direct = (u < N) ? R32[(int64_t)u * W32 + vr] : 0u;
       const int vrow = V0 + lane;
       const uint32_t x = (vrow < N) ? R32[(int64_t)vrow * W32 + ur] : 0u;
-      uint32_t t = 0;
-#pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        const uint32_t b = __ballot_sync(0xffffffffu, (x >> i) & 1u);
-        if (lane == i) t = b;
-      }
+      const uint32_t t = transpose32(x, lane);
       uint32_t m = direct | t;
       if (U0 == V0 && u < N) m |= 1u << lane;
       if (u >= N || st != PREDTOP_OK) m = 0;  // invalid graph: M defined as zero
@@ -513,12 +523,7 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
       const int V0 = vr * 32, vrow = V0 + lane;
       const uint32_t direct = u < N ? R32[u * W32 + vr] : 0u;
       const uint32_t x = vrow < N ? R32[vrow * W32 + ur] : 0u;
-      uint32_t t = 0;
-#pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        const uint32_t b = __ballot_sync(0xffffffffu, (x >> i) & 1u);
-        if (lane == i) t = b;
-      }
+      const uint32_t t = transpose32(x, lane);
       uint32_t m = direct | t;
       if (U0 == V0 && u < N) m |= 1u << lane;
       if (u < N) M32[(int64_t)u * W32 + vr] = m;
