@@ -76,5 +76,30 @@ def build_library(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_variant(name: str, extra_flags, verbose: bool = False) -> str:
+    """Debug build (e.g. name='trace', extra_flags=['-DPREDTOP_TRACE']) into
+    lib/libpredtop_<name>.so; load it with PREDTOP_LIB=<path>."""
+    obj_dir = os.path.join(PKG, "build_obj_" + name)
+    os.makedirs(obj_dir, exist_ok=True)
+    os.makedirs(LIB_DIR, exist_ok=True)
+    nvcc = _nvcc()
+
+    def compile_one(src):
+        obj = os.path.join(obj_dir, os.path.basename(src)[:-3] + ".o")
+        r = subprocess.run([nvcc] + NVFLAGS + list(extra_flags) + ["-c", src, "-o", obj],
+                           capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")
+        return obj
+
+    with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
+        objs = list(ex.map(compile_one, _sources()))
+    out = os.path.join(LIB_DIR, f"libpredtop_{name}.so")
+    r = subprocess.run([nvcc] + ARCH + ["-shared", "-o", out] + objs + ["-lcudart"], capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
+    return out
+
+
 if __name__ == "__main__":
     print(build_library(force="--force" in sys.argv, verbose=True))

@@ -132,89 +132,94 @@ struct Attn {
     if (!act) return;
     const uint32_t ta = (uint32_t)(mwa >> (16 * tq)) & 0xffffu;
     const uint32_t tb = (uint32_t)(mwb >> (16 * tq)) & 0xffffu;
-    float s[8][4];
-    float mx_a = -INFINITY, mx_b = -INFINITY;  // raw row maxima over the active blocks
+    // two 32-key phases (blocks 2ph, 2ph+1): half the live score registers
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      if (act & (1u << j)) {
+    for (int ph = 0; ph < 2; ++ph) {
+      const uint32_t pact = (act >> (2 * ph)) & 3u;
+      if (!pact) continue;
+      float s[4][4];
+      float mx_a = -INFINITY, mx_b = -INFINITY;  // row maxima over the active blocks
+#pragma unroll
+      for (int jj = 0; jj < 2; ++jj) {
+        const int j = 2 * ph + jj;
+        if (!(act & (1u << j))) continue;
 #pragma unroll
         for (int ks = 0; ks < KS; ++ks) {
           uint32_t b0, b1, b2, b3;
           ldsm_x4(kbase + kl + j * BLK + ks * 32, b0, b1, b2, b3);
           if (ks == 0) {
-            mma16816_z(s[2 * j], qa[ks], b0, b1);
-            mma16816_z(s[2 * j + 1], qa[ks], b2, b3);
+            mma16816_z(s[2 * jj], qa[ks], b0, b1);
+            mma16816_z(s[2 * jj + 1], qa[ks], b2, b3);
           } else {
-            mma16816(s[2 * j], qa[ks], b0, b1);
-            mma16816(s[2 * j + 1], qa[ks], b2, b3);
+            mma16816(s[2 * jj], qa[ks], b0, b1);
+            mma16816(s[2 * jj + 1], qa[ks], b2, b3);
           }
         }
         if (!(full & (1u << j))) {  // partial block: masked scores -> -inf
 #pragma unroll
           for (int u = 0; u < 2; ++u) {
             const int e = 2 * (2 * j + u);
-            if (!((ta >> e) & 1u)) s[2 * j + u][0] = -INFINITY;
-            if (!((ta >> (e + 1)) & 1u)) s[2 * j + u][1] = -INFINITY;
-            if (!((tb >> e) & 1u)) s[2 * j + u][2] = -INFINITY;
-            if (!((tb >> (e + 1)) & 1u)) s[2 * j + u][3] = -INFINITY;
+            if (!((ta >> e) & 1u)) s[2 * jj + u][0] = -INFINITY;
+            if (!((ta >> (e + 1)) & 1u)) s[2 * jj + u][1] = -INFINITY;
+            if (!((tb >> e) & 1u)) s[2 * jj + u][2] = -INFINITY;
+            if (!((tb >> (e + 1)) & 1u)) s[2 * jj + u][3] = -INFINITY;
           }
         }
-        mx_a = fmaxf(mx_a, fmaxf(fmaxf(s[2 * j][0], s[2 * j][1]), fmaxf(s[2 * j + 1][0], s[2 * j + 1][1])));
-        mx_b = fmaxf(mx_b, fmaxf(fmaxf(s[2 * j][2], s[2 * j][3]), fmaxf(s[2 * j + 1][2], s[2 * j + 1][3])));
+        mx_a = fmaxf(mx_a, fmaxf(fmaxf(s[2 * jj][0], s[2 * jj][1]), fmaxf(s[2 * jj + 1][0], s[2 * jj + 1][1])));
+        mx_b = fmaxf(mx_b, fmaxf(fmaxf(s[2 * jj][2], s[2 * jj][3]), fmaxf(s[2 * jj + 1][2], s[2 * jj + 1][3])));
       }
-    }
-    mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 1));
-    mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 2));
-    mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 1));
-    mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 2));
-    mx_a *= scale;
-    mx_b *= scale;
-    // Lazy rescaling: the reference m only moves when a row maximum exceeds it
-    // by more than 8 (log2 units), so P = exp2(s - m) <= 256 stays exact in
-    // fp16 and fp32; the final O / l is unchanged.
-    if (__any_sync(0xffffffffu, mx_a > m_a + 8.f || mx_b > m_b + 8.f)) {
-      const float mn_a = fmaxf(m_a, mx_a), mn_b = fmaxf(m_b, mx_b);
-      const float al_a = ex2(m_a - (mn_a == -INFINITY ? 0.f : mn_a));
-      const float al_b = ex2(m_b - (mn_b == -INFINITY ? 0.f : mn_b));
+      mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 1));
+      mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 2));
+      mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 1));
+      mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 2));
+      // Lazy rescaling: the reference m only moves when a row maximum exceeds
+      // it by more than 8 (log2 units; Q is pre-scaled), so P = exp2(s - m)
+      // <= 256 stays exact in fp16 and fp32; the final O / l is unchanged.
+      if (__any_sync(0xffffffffu, mx_a > m_a + 8.f || mx_b > m_b + 8.f)) {
+        const float mn_a = fmaxf(m_a, mx_a), mn_b = fmaxf(m_b, mx_b);
+        const float al_a = ex2(m_a - (mn_a == -INFINITY ? 0.f : mn_a));
+        const float al_b = ex2(m_b - (mn_b == -INFINITY ? 0.f : mn_b));
 #pragma unroll
-      for (int i = 0; i < DN; ++i) {
-        o[i][0] *= al_a; o[i][1] *= al_a;
-        o[i][2] *= al_b; o[i][3] *= al_b;
+        for (int i = 0; i < DN; ++i) {
+          o[i][0] *= al_a; o[i][1] *= al_a;
+          o[i][2] *= al_b; o[i][3] *= al_b;
+        }
+        osum[0] *= al_a; osum[1] *= al_a;
+        osum[2] *= al_b; osum[3] *= al_b;
+        m_a = mn_a;
+        m_b = mn_b;
       }
-      osum[0] *= al_a; osum[1] *= al_a;
-      osum[2] *= al_b; osum[3] *= al_b;
-      m_a = mn_a;
-      m_b = mn_b;
-    }
-    const float mu_a = m_a == -INFINITY ? 0.f : m_a;
-    const float mu_b = m_b == -INFINITY ? 0.f : m_b;
+      const float mu_a = m_a == -INFINITY ? 0.f : m_a;
+      const float mu_b = m_b == -INFINITY ? 0.f : m_b;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      if (!(act & (1u << j))) continue;
-      uint32_t pa[4];
+      for (int jj = 0; jj < 2; ++jj) {
+        const int j = 2 * ph + jj;
+        if (!(act & (1u << j))) continue;
+        uint32_t pa[4];
 #pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int nt = 2 * j + u;
-        pa[2 * u + 0] = pack_h2(ex2(fmaf(s[nt][0], scale, -mu_a)), ex2(fmaf(s[nt][1], scale, -mu_a)));
-        pa[2 * u + 1] = pack_h2(ex2(fmaf(s[nt][2], scale, -mu_b)), ex2(fmaf(s[nt][3], scale, -mu_b)));
+        for (int u = 0; u < 2; ++u) {
+          const int nt = 2 * jj + u;
+          pa[2 * u + 0] = pack_h2(ex2(s[nt][0] - mu_a), ex2(s[nt][1] - mu_a));
+          pa[2 * u + 1] = pack_h2(ex2(s[nt][2] - mu_b), ex2(s[nt][3] - mu_b));
+        }
+#pragma unroll
+        for (int dn = 0; dn < DN; dn += 2) {
+          uint32_t b0, b1, b2, b3;
+          ldsm_x4_t(vbase + vl + j * BLK + dn * 16, b0, b1, b2, b3);
+          mma16816(o[dn], pa, b0, b1);
+          mma16816(o[dn + 1], pa, b2, b3);
+        }
+        uint32_t c0, c1;
+        ldsm_x2_t(vbase + vl1 + j * BLK, c0, c1);
+        mma16816(osum, pa, c0, c1);
       }
-#pragma unroll
-      for (int dn = 0; dn < DN; dn += 2) {
-        uint32_t b0, b1, b2, b3;
-        ldsm_x4_t(vbase + vl + j * BLK + dn * 16, b0, b1, b2, b3);
-        mma16816(o[dn], pa, b0, b1);
-        mma16816(o[dn + 1], pa, b2, b3);
-      }
-      uint32_t c0, c1;
-      ldsm_x2_t(vbase + vl1 + j * BLK, c0, c1);
-      mma16816(osum, pa, c0, c1);
     }
   }
 
 };
 
 template <int DH, bool RESIDENT>
-__global__ void __launch_bounds__(256, DH == 16 ? 3 : 2) k_attn(DagDev d, int G, int H, int dmodel,
+__global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G, int H, int dmodel,
                                                  const __half* __restrict__ qkv,
                                                  __half* __restrict__ out) {
   using A = Attn<DH>;

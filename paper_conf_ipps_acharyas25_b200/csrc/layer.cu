@@ -28,6 +28,24 @@
 
 namespace predtop {
 
+#ifdef PREDTOP_TRACE
+// Debug timeline of CTA 0 (first 16 tiles): %globaltimer at phase boundaries.
+__device__ unsigned long long g_tail_trace[16][16];
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TTRACE(i, k) \
+  do {               \
+    if (leader && blockIdx.x == 0 && (i) < 16) g_tail_trace[i][k] = gtime(); \
+  } while (0)
+#else
+#define TTRACE(i, k) \
+  do {               \
+  } while (0)
+#endif
+
 namespace {
 
 constexpr int kThreads = 320;
@@ -277,12 +295,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       const int m0 = t * 128;
       const int cbase = i * NJ;
       // previous tile's stores have read sX / sH -> the residual of this tile may land
+      TTRACE(i, 0);
       if (leader) sm100::bulk_wait_read0();
       sm100::named_bar<kEpi>(1);
       if (leader) sm100::mbar_arrive(&x_free);
+      TTRACE(i, 1);
       // ---- LN1
       sm100::mbar_wait(&o_full, i & 1);
+      TTRACE(i, 2);
       sm100::mbar_wait(&x_full, i & 1);
+      TTRACE(i, 3);
       sm100::tc_fence_after();
       const float s1 = add_residual(acc_o, p_bo);
       sm100::tc_fence_before();
@@ -293,11 +315,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
         sm100::mbar_arrive(&o_empty);
         sm100::mbar_arrive(&h_ready);
       }
+      TTRACE(i, 4);
       // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 operand buffer
       for (int j = 0; j < NJ; ++j) {
         const int b = j & 1, u = (cbase + j) >> 1;
         sm100::mbar_wait(&f_full[b], u & 1);
         sm100::mbar_wait(&p_free[b], (u & 1) ^ 1);
+        TTRACE(i, 5 + 2 * (j & 3));
         sm100::tc_fence_after();
         unsigned char* P = b ? sP1 : sA;
         const uint32_t accf = tmem + D + b * FC + lrow;
@@ -323,9 +347,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
           sm100::mbar_arrive(&f_empty[b]);
           sm100::mbar_arrive(&p_ready[b]);
         }
+        TTRACE(i, 6 + 2 * (j & 3));
       }
       // ---- LN2 and stores
       sm100::mbar_wait(&out_full, i & 1);
+      TTRACE(i, 13);
       sm100::tc_fence_after();
       const float s2 = add_residual(acc_out, p_b2);
       sm100::tc_fence_before();
@@ -338,6 +364,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
         for (int b = 0; b < KD; ++b) sm100::tma_store_2d(&mp.x16, sH + b * kSub, b * 64, m0);
         sm100::bulk_commit();
       }
+      TTRACE(i, 14);
     }
     if (leader) sm100::bulk_wait0();
   }
@@ -393,3 +420,9 @@ predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* 
 }
 
 }  // namespace predtop
+
+#ifdef PREDTOP_TRACE
+extern "C" PREDTOP_API int predtop_debug_tail_trace(unsigned long long* out) {
+  return cudaMemcpyFromSymbol(out, predtop::g_tail_trace, sizeof(predtop::g_tail_trace)) == cudaSuccess ? 0 : -7;
+}
+#endif

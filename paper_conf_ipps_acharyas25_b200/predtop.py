@@ -21,7 +21,7 @@ import torch
 from . import build as _build
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = _build.LIB
+LIB_PATH = os.environ.get("PREDTOP_LIB", _build.LIB)  # override: debug builds (tools/)
 
 OK, INVALID_ARG, RANGE, SELF_LOOP, CYCLE, TOO_LARGE, WORKSPACE, CUDA, UNSUPPORTED = \
     0, -1, -2, -3, -4, -5, -6, -7, -8
