@@ -66,6 +66,11 @@ __device__ __forceinline__ void cp_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N));
 }
 
+__device__ __forceinline__ float dot_h2(uint32_t a, uint32_t b) {
+  const float2 x = __half22float2(*reinterpret_cast<const __half2*>(&a));
+  const float2 y = __half22float2(*reinterpret_cast<const __half2*>(&b));
+  return x.x * y.x + x.y * y.y;
+}
 __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   __half2 h = __floats2half2_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
@@ -78,6 +83,16 @@ __device__ __forceinline__ void mma16816_z(float (&d)[4], const uint32_t (&a)[4]
       "{%10,%10,%10,%10};"
       : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
       : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1), "f"(0.f));
+}
+// D = A*B + C with an explicit accumulator input (QK^T: C = -m or -inf).
+__device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1,
+                                           const float (&c)[4]) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%10,%11,%12,%13};"
+      : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1), "f"(c[0]), "f"(c[1]), "f"(c[2]),
+        "f"(c[3]));
 }
 __device__ __forceinline__ void ldsm_x2_t(uint32_t addr, uint32_t& r0, uint32_t& r1) {
   asm volatile("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0,%1}, [%2];"
@@ -108,7 +123,6 @@ struct Attn {
   float o[DN][4];
   float osum[4];  // P x (ones column of V): row sums l, [0] row a, [2] row b
   float m_a, m_b;
-  float scale;
   uint32_t kl, vl, vl1;  // per-lane ldmatrix byte offsets
 
   __device__ __forceinline__ void init(int lane) {
@@ -119,66 +133,83 @@ struct Attn {
 #pragma unroll
     for (int i = 0; i < DN; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
     osum[0] = osum[1] = osum[2] = osum[3] = 0.f;
-    m_a = m_b = -INFINITY;
+    m_a = m_b = 0.f;  // set to the diagonal score by the kernel
   }
 
   // One 64-key chunk for the warp's 16 rows.  kbase/vbase: shared addresses of
-  // the chunk's (permuted) K and V rows; mwa/mwb: mask words of rows a/b.
-  // fl: block flags of (warp's 16-row group, chunk) from the DAG build
-  // (k_bflags): bit j = block j has an allowed pair, bit 4+j = fully allowed.
-  __device__ __forceinline__ void chunk(uint32_t kbase, uint32_t vbase, uint64_t mwa, uint64_t mwb,
-                                        uint32_t fl, int tq) {
+  // the chunk's (permuted) K and V rows; mk: this thread's 16 mask bits of
+  // row a (bits 0-15) and of row b (bits 16-31); fl: block flags of (warp's
+  // 16-row group, chunk) from the DAG build (k_bflags): bit j = block j has an
+  // allowed pair, bit 4+j = all pairs allowed.
+  //
+  // The mask and the running reference m enter through the accumulator input
+  // of the QK^T MMA: C = -m (allowed) or -inf (masked), so the MMA returns
+  // s - m directly and P = exp2(S) needs no subtraction and no select.
+  __device__ __forceinline__ void chunk(uint32_t kbase, uint32_t vbase, uint32_t mk, uint32_t fl) {
     const uint32_t act = fl & 15u, full = fl >> 4;
     if (!act) return;
-    const uint32_t ta = (uint32_t)(mwa >> (16 * tq)) & 0xffffu;
-    const uint32_t tb = (uint32_t)(mwb >> (16 * tq)) & 0xffffu;
     // two 32-key phases (blocks 2ph, 2ph+1): half the live score registers
 #pragma unroll
     for (int ph = 0; ph < 2; ++ph) {
-      const uint32_t pact = (act >> (2 * ph)) & 3u;
-      if (!pact) continue;
+      if (!((act >> (2 * ph)) & 3u)) continue;
+      const float nma = -m_a, nmb = -m_b;
       float s[4][4];
-      float mx_a = -INFINITY, mx_b = -INFINITY;  // row maxima over the active blocks
+      float mx = -INFINITY;  // max of s - m over both rows (overflow check only)
 #pragma unroll
       for (int jj = 0; jj < 2; ++jj) {
         const int j = 2 * ph + jj;
         if (!(act & (1u << j))) continue;
+        float c[2][4];
+        if (full & (1u << j)) {
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            c[u][0] = nma; c[u][1] = nma;
+            c[u][2] = nmb; c[u][3] = nmb;
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {
+            const int e = 2 * (2 * j + u);
+            c[u][0] = ((mk >> e) & 1u) ? nma : -INFINITY;
+            c[u][1] = ((mk >> (e + 1)) & 1u) ? nma : -INFINITY;
+            c[u][2] = ((mk >> (e + 16)) & 1u) ? nmb : -INFINITY;
+            c[u][3] = ((mk >> (e + 17)) & 1u) ? nmb : -INFINITY;
+          }
+        }
 #pragma unroll
         for (int ks = 0; ks < KS; ++ks) {
           uint32_t b0, b1, b2, b3;
           ldsm_x4(kbase + kl + j * BLK + ks * 32, b0, b1, b2, b3);
           if (ks == 0) {
-            mma16816_z(s[2 * jj], qa[ks], b0, b1);
-            mma16816_z(s[2 * jj + 1], qa[ks], b2, b3);
+            mma16816_c(s[2 * jj], qa[ks], b0, b1, c[0]);
+            mma16816_c(s[2 * jj + 1], qa[ks], b2, b3, c[1]);
           } else {
             mma16816(s[2 * jj], qa[ks], b0, b1);
             mma16816(s[2 * jj + 1], qa[ks], b2, b3);
           }
         }
-        if (!(full & (1u << j))) {  // partial block: masked scores -> -inf
-#pragma unroll
-          for (int u = 0; u < 2; ++u) {
-            const int e = 2 * (2 * j + u);
-            if (!((ta >> e) & 1u)) s[2 * jj + u][0] = -INFINITY;
-            if (!((ta >> (e + 1)) & 1u)) s[2 * jj + u][1] = -INFINITY;
-            if (!((tb >> e) & 1u)) s[2 * jj + u][2] = -INFINITY;
-            if (!((tb >> (e + 1)) & 1u)) s[2 * jj + u][3] = -INFINITY;
-          }
-        }
-        mx_a = fmaxf(mx_a, fmaxf(fmaxf(s[2 * jj][0], s[2 * jj][1]), fmaxf(s[2 * jj + 1][0], s[2 * jj + 1][1])));
-        mx_b = fmaxf(mx_b, fmaxf(fmaxf(s[2 * jj][2], s[2 * jj][3]), fmaxf(s[2 * jj + 1][2], s[2 * jj + 1][3])));
+        const float* x = s[2 * jj];
+        const float* y = s[2 * jj + 1];
+        mx = fmaxf(fmaxf(mx, fmaxf(x[0], x[1])), fmaxf(fmaxf(x[2], x[3]), fmaxf(y[0], y[1])));
+        mx = fmaxf(mx, fmaxf(y[2], y[3]));
       }
-      mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 1));
-      mx_a = fmaxf(mx_a, __shfl_xor_sync(0xffffffffu, mx_a, 2));
-      mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 1));
-      mx_b = fmaxf(mx_b, __shfl_xor_sync(0xffffffffu, mx_b, 2));
-      // Lazy rescaling: the reference m only moves when a row maximum exceeds
-      // it by more than 8 (log2 units; Q is pre-scaled), so P = exp2(s - m)
-      // <= 256 stays exact in fp16 and fp32; the final O / l is unchanged.
-      if (__any_sync(0xffffffffu, mx_a > m_a + 8.f || mx_b > m_b + 8.f)) {
-        const float mn_a = fmaxf(m_a, mx_a), mn_b = fmaxf(m_b, mx_b);
-        const float al_a = ex2(m_a - (mn_a == -INFINITY ? 0.f : mn_a));
-        const float al_b = ex2(m_b - (mn_b == -INFINITY ? 0.f : mn_b));
+      // Lazy rescaling: m starts at the row's diagonal score (always allowed,
+      // M includes I) and only moves when a score exceeds it by more than 8
+      // (log2 units), so P = exp2(s - m) <= 256 stays exact in fp16.
+      if (__any_sync(0xffffffffu, mx > 8.f)) {
+        float ma = -INFINITY, mb = -INFINITY;
+#pragma unroll
+        for (int jj = 0; jj < 2; ++jj) {
+          if (!(act & (1u << (2 * ph + jj)))) continue;
+          ma = fmaxf(ma, fmaxf(fmaxf(s[2 * jj][0], s[2 * jj][1]), fmaxf(s[2 * jj + 1][0], s[2 * jj + 1][1])));
+          mb = fmaxf(mb, fmaxf(fmaxf(s[2 * jj][2], s[2 * jj][3]), fmaxf(s[2 * jj + 1][2], s[2 * jj + 1][3])));
+        }
+        ma = fmaxf(ma, __shfl_xor_sync(0xffffffffu, ma, 1));
+        ma = fmaxf(ma, __shfl_xor_sync(0xffffffffu, ma, 2));
+        mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, 1));
+        mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, 2));
+        const float da = ma > 8.f ? ma : 0.f, db = mb > 8.f ? mb : 0.f;
+        const float al_a = ex2(-da), al_b = ex2(-db);
 #pragma unroll
         for (int i = 0; i < DN; ++i) {
           o[i][0] *= al_a; o[i][1] *= al_a;
@@ -186,11 +217,14 @@ struct Attn {
         }
         osum[0] *= al_a; osum[1] *= al_a;
         osum[2] *= al_b; osum[3] *= al_b;
-        m_a = mn_a;
-        m_b = mn_b;
+        m_a += da;
+        m_b += db;
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) {
+          s[nt][0] -= da; s[nt][1] -= da;
+          s[nt][2] -= db; s[nt][3] -= db;
+        }
       }
-      const float mu_a = m_a == -INFINITY ? 0.f : m_a;
-      const float mu_b = m_b == -INFINITY ? 0.f : m_b;
 #pragma unroll
       for (int jj = 0; jj < 2; ++jj) {
         const int j = 2 * ph + jj;
@@ -199,8 +233,8 @@ struct Attn {
 #pragma unroll
         for (int u = 0; u < 2; ++u) {
           const int nt = 2 * jj + u;
-          pa[2 * u + 0] = pack_h2(ex2(s[nt][0] - mu_a), ex2(s[nt][1] - mu_a));
-          pa[2 * u + 1] = pack_h2(ex2(s[nt][2] - mu_b), ex2(s[nt][3] - mu_b));
+          pa[2 * u + 0] = pack_h2(ex2(s[nt][0]), ex2(s[nt][1]));
+          pa[2 * u + 1] = pack_h2(ex2(s[nt][2]), ex2(s[nt][3]));
         }
 #pragma unroll
         for (int dn = 0; dn < DN; dn += 2) {
@@ -298,7 +332,36 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
     st.qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0 + 8) : 0u;
     st.qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0 + 8) : 0u;
   }
-  uint64_t mwa = va ? Ma[0] : 0ull, mwb = vb ? Mb[0] : 0ull;
+  // reference m of each row: its diagonal score q.k (M includes I, so the
+  // row max is >= it; with lazy rescaling m stays within 8 of the max)
+  {
+    float sa = 0.f, sb = 0.f;
+#pragma unroll
+    for (int ks = 0; ks < A::KS; ++ks) {
+      const int k0 = dmodel + ks * 16 + 2 * tq;
+      const uint32_t ka0 = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0) : 0u;
+      const uint32_t ka2 = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0 + 8) : 0u;
+      const uint32_t kb0 = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0) : 0u;
+      const uint32_t kb2 = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0 + 8) : 0u;
+      sa += dot_h2(st.qa[ks][0], ka0) + dot_h2(st.qa[ks][2], ka2);
+      sb += dot_h2(st.qa[ks][1], kb0) + dot_h2(st.qa[ks][3], kb2);
+    }
+    sa += __shfl_xor_sync(0xffffffffu, sa, 1);
+    sa += __shfl_xor_sync(0xffffffffu, sa, 2);
+    sb += __shfl_xor_sync(0xffffffffu, sb, 1);
+    sb += __shfl_xor_sync(0xffffffffu, sb, 2);
+    st.m_a = sa;
+    st.m_b = sb;
+  }
+  // this thread's 16 mask bits of rows a / b in chunk c: 16-bit piece tq of the word
+  const uint16_t* Ma16 = reinterpret_cast<const uint16_t*>(Ma) + tq;
+  const uint16_t* Mb16 = reinterpret_cast<const uint16_t*>(Mb) + tq;
+  auto mask_bits = [&](int c) -> uint32_t {
+    const uint32_t lo = va ? (uint32_t)Ma16[4 * c] : 0u;
+    const uint32_t hi = vb ? (uint32_t)Mb16[4 * c] : 0u;
+    return lo | (hi << 16);
+  };
+  uint32_t mk = mask_bits(0);
   const uint32_t kb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sK));
   const uint32_t vb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sV));
 
@@ -306,30 +369,26 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
     cp_wait<0>();
     __syncthreads();
   }
-  st.scale = 1.f;  // online path: scores already in log2 units
 
   if (RESIDENT) {
     if (!warp_live) return;
     uint32_t fl = Fw[0];
     for (int c = 0; c < nchunks; ++c) {
       const bool more = c + 1 < nchunks;
-      const uint64_t nwa = (more && va) ? Ma[c + 1] : 0ull;
-      const uint64_t nwb = (more && vb) ? Mb[c + 1] : 0ull;
+      const uint32_t nmk = more ? mask_bits(c + 1) : 0u;
       const uint32_t nfl = more ? Fw[c + 1] : 0u;
       const uint32_t kc = kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2);
-      st.chunk(kc, vc, mwa, mwb, __shfl_sync(0xffffffffu, fl, 0), tq);
-      mwa = nwa;
-      mwb = nwb;
+      st.chunk(kc, vc, mk, __shfl_sync(0xffffffffu, fl, 0));
+      mk = nmk;
       fl = nfl;
     }
   } else {
     for (int c = 0; c < nchunks; ++c) {
       const int buf = c & 1;
-      uint64_t nwa = 0ull, nwb = 0ull;
+      uint32_t nmk = 0u;
       if (c + 1 < nchunks) {
         load_chunks(c + 1, c + 2, buf ^ 1);
-        nwa = va ? Ma[c + 1] : 0ull;
-        nwb = vb ? Mb[c + 1] : 0ull;
+        nmk = mask_bits(c + 1);
         cp_wait<1>();
       } else {
         cp_wait<0>();
@@ -338,11 +397,10 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
       if (warp_live) {
         const uint32_t kc = kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2);
         const uint32_t fl = __shfl_sync(0xffffffffu, (uint32_t)Fw[c], 0);
-        st.chunk(kc, vc, mwa, mwb, fl, tq);
+        st.chunk(kc, vc, mk, fl);
       }
       __syncthreads();
-      mwa = nwa;
-      mwb = nwb;
+      mk = nmk;
     }
     if (!warp_live) return;
   }

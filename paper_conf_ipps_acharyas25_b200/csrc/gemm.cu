@@ -101,7 +101,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   constexpr int S = C::STAGES;
   constexpr uint32_t NCOLS = tmem_cols2<BN>();
   extern __shared__ unsigned char dsm[];
-  unsigned char* base = (unsigned char*)(((uintptr_t)dsm + 1023) & ~(uintptr_t)1023);
+  unsigned char* base = sm100::align1024(dsm);
   unsigned char* ring = base;
   unsigned char* st16 = base + S * C::STAGE_BYTES;       // f16 output staging
   unsigned char* st32 = st16 + C::OUT16_BYTES;           // fp32 residual / output staging

@@ -40,7 +40,16 @@ __device__ __forceinline__ unsigned long long gtime() {
   do {               \
     if (leader && blockIdx.x == 0 && (i) < 16) g_tail_trace[i][k] = gtime(); \
   } while (0)
+// per-warp clock64 at 4 points of FFN chunk 1 of tile 4 (CTA 0)
+__device__ long long g_tail_trace2[4][8];
+#define TTRACEW(i, j, k) \
+  do {                   \
+    if (lane == 0 && blockIdx.x == 0 && (i) == 4 && (j) == 1) g_tail_trace2[k][warp - 2] = clock64(); \
+  } while (0)
 #else
+#define TTRACEW(i, j, k) \
+  do {                   \
+  } while (0)
 #define TTRACE(i, k) \
   do {               \
   } while (0)
@@ -85,7 +94,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
   constexpr int RS = C::RS;
   constexpr int KD = D / 64;  // 64-wide K slices of d
   extern __shared__ unsigned char dsm[];
-  unsigned char* base = (unsigned char*)(((uintptr_t)dsm + 1023) & ~(uintptr_t)1023);
+  unsigned char* base = sm100::align1024(dsm);
   unsigned char* sX = base;                 // fp32 [128 x D], D/32 sub-tiles
   unsigned char* sA = sX + C::X32;          // att / ReLU chunk buffer 0
   unsigned char* sP1 = sA + C::SA;          // ReLU chunk buffer 1
@@ -228,67 +237,60 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
     const int r = q * 32 + lane;
     const uint32_t lrow = (uint32_t)(q * 32) << 16;
     const bool leader = (warp == 2 && lane == 0);
-    float v[16];
-    // LayerNorm of the row r over D columns, this thread doing columns
-    // [half*D/2, +D/2): z (in sX, fp32, in place) -> y; y also to sH as fp16.
-    auto layer_norm = [&](float sum, const float* g, const float* be) {
+    constexpr int DH2 = D / 2;  // columns of the row handled by this thread
+    // One LayerNorm block of row r, this thread doing columns [half*D/2, +D/2),
+    // register resident: z = acc (TMEM) + bias + sX (fp32 residual), mean and
+    // variance over the two halves through red_a / red_b, then
+    // y = (z - mean) * rstd * g + be  ->  sX (fp32, in place) and sH (fp16).
+    auto ln_block = [&](uint32_t acc, const float* bias, const float* g, const float* be) {
+      float z[DH2];
+      sm100::tmem_ld<DH2>(acc + lrow + half * DH2, z);
+      sm100::tc_fence_before();
+      float sum = 0.f;
+#pragma unroll
+      for (int k = 0; k < DH2 / 4; ++k) {
+        const int c4 = half * DH2 / 4 + k;
+        const float4 x = *reinterpret_cast<const float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
+        const float4 bb = reinterpret_cast<const float4*>(bias)[c4];
+        z[4 * k + 0] = x.x + (z[4 * k + 0] + bb.x);
+        z[4 * k + 1] = x.y + (z[4 * k + 1] + bb.y);
+        z[4 * k + 2] = x.z + (z[4 * k + 2] + bb.z);
+        z[4 * k + 3] = x.w + (z[4 * k + 3] + bb.w);
+        sum += (z[4 * k] + z[4 * k + 1]) + (z[4 * k + 2] + z[4 * k + 3]);
+      }
       red_a[half][r] = sum;
       sm100::named_bar<kEpi>(1);
       const float mean = (red_a[0][r] + red_a[1][r]) * (1.0f / D);
       float sq = 0.f;
-#pragma unroll 4
-      for (int c4 = half * D / 8; c4 < (half + 1) * D / 8; ++c4) {
-        const float4 x = *reinterpret_cast<const float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
-        const float a = x.x - mean, b = x.y - mean, cc = x.z - mean, d = x.w - mean;
+#pragma unroll
+      for (int k = 0; k < DH2 / 4; ++k) {
+        const float a = z[4 * k] - mean, b = z[4 * k + 1] - mean, cc = z[4 * k + 2] - mean, d = z[4 * k + 3] - mean;
         sq += (a * a + b * b) + (cc * cc + d * d);
       }
       red_b[half][r] = sq;
       sm100::named_bar<kEpi>(1);
       const float rstd = rsqrtf((red_b[0][r] + red_b[1][r]) * (1.0f / D) + args.eps);
-#pragma unroll 2
-      for (int c8 = half * D / 16; c8 < (half + 1) * D / 16; ++c8) {
+#pragma unroll
+      for (int k8 = 0; k8 < DH2 / 8; ++k8) {
         float y[8];
 #pragma unroll
         for (int h2 = 0; h2 < 2; ++h2) {
-          const int c4 = 2 * c8 + h2;
-          float4* p = reinterpret_cast<float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
-          float4 x = *p;
+          const int k = 2 * k8 + h2, c4 = half * DH2 / 4 + k;
           const float4 gm = reinterpret_cast<const float4*>(g)[c4];
           const float4 bt = reinterpret_cast<const float4*>(be)[c4];
-          x.x = (x.x - mean) * rstd * gm.x + bt.x;
-          x.y = (x.y - mean) * rstd * gm.y + bt.y;
-          x.z = (x.z - mean) * rstd * gm.z + bt.z;
-          x.w = (x.w - mean) * rstd * gm.w + bt.w;
-          *p = x;
-          y[4 * h2] = x.x; y[4 * h2 + 1] = x.y; y[4 * h2 + 2] = x.z; y[4 * h2 + 3] = x.w;
+          float4 o;
+          o.x = (z[4 * k + 0] - mean) * rstd * gm.x + bt.x;
+          o.y = (z[4 * k + 1] - mean) * rstd * gm.y + bt.y;
+          o.z = (z[4 * k + 2] - mean) * rstd * gm.z + bt.z;
+          o.w = (z[4 * k + 3] - mean) * rstd * gm.w + bt.w;
+          *reinterpret_cast<float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8)) = o;
+          y[4 * h2] = o.x; y[4 * h2 + 1] = o.y; y[4 * h2 + 2] = o.z; y[4 * h2 + 3] = o.w;
         }
-        const int c = 8 * c8;
+        const int c = half * DH2 + 8 * k8;
         *reinterpret_cast<uint4*>(sH + (c / 64) * kSub + sm100::swz<128>(r, (c % 64) / 8)) =
             make_uint4(sm100::pack_half2(y[0], y[1]), sm100::pack_half2(y[2], y[3]),
                        sm100::pack_half2(y[4], y[5]), sm100::pack_half2(y[6], y[7]));
       }
-    };
-    // z = acc (TMEM) + bias + sX (fp32), written back to sX; returns the partial row sum
-    auto add_residual = [&](uint32_t acc, const float* bias) {
-      float sum = 0.f;
-#pragma unroll 1
-      for (int c = half * D / 2; c < (half + 1) * D / 2; c += 16) {
-        sm100::tmem_ld16(acc + lrow + c, v);
-        unsigned char* box = sX + (c / 32) * kSub;
-#pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          float4* p = reinterpret_cast<float4*>(box + sm100::swz<128>(r, (c % 32) / 4 + k));
-          const float4 b = reinterpret_cast<const float4*>(bias + c)[k];
-          float4 x = *p;
-          x.x += v[4 * k + 0] + b.x;
-          x.y += v[4 * k + 1] + b.y;
-          x.z += v[4 * k + 2] + b.z;
-          x.w += v[4 * k + 3] + b.w;
-          sum += (x.x + x.y) + (x.z + x.w);
-          *p = x;
-        }
-      }
-      return sum;
     };
     int i = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
@@ -306,9 +308,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       sm100::mbar_wait(&x_full, i & 1);
       TTRACE(i, 3);
       sm100::tc_fence_after();
-      const float s1 = add_residual(acc_o, p_bo);
-      sm100::tc_fence_before();
-      layer_norm(s1, p_g1, p_be1);
+      ln_block(acc_o, p_bo, p_g1, p_be1);
       sm100::fence_proxy_async();
       sm100::named_bar<kEpi>(1);
       if (leader) {
@@ -322,26 +322,33 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
         sm100::mbar_wait(&f_full[b], u & 1);
         sm100::mbar_wait(&p_free[b], (u & 1) ^ 1);
         TTRACE(i, 5 + 2 * (j & 3));
+        TTRACEW(i, j, 0);
         sm100::tc_fence_after();
         unsigned char* P = b ? sP1 : sA;
         const uint32_t accf = tmem + D + b * FC + lrow;
         const float* b1 = p_b1 + j * FC;
-#pragma unroll 1
-        for (int c = half * FC / 2; c < (half + 1) * FC / 2; c += 16) {
-          sm100::tmem_ld16(accf + c, v);
+        float v[FC / 2];
+        sm100::tmem_ld<FC / 2>(accf + half * FC / 2, v);
+        TTRACEW(i, j, 1);
+#pragma unroll
+        for (int g16 = 0; g16 < FC / 32; ++g16) {
+          const int c = half * FC / 2 + 16 * g16;
           uint32_t pk[8];
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             const float4 bb = reinterpret_cast<const float4*>(b1 + c)[k];
-            pk[2 * k] = sm100::pack_half2(fmaxf(v[4 * k] + bb.x, 0.f), fmaxf(v[4 * k + 1] + bb.y, 0.f));
-            pk[2 * k + 1] = sm100::pack_half2(fmaxf(v[4 * k + 2] + bb.z, 0.f), fmaxf(v[4 * k + 3] + bb.w, 0.f));
+            const float* w = v + 16 * g16 + 4 * k;
+            pk[2 * k] = sm100::pack_half2(fmaxf(w[0] + bb.x, 0.f), fmaxf(w[1] + bb.y, 0.f));
+            pk[2 * k + 1] = sm100::pack_half2(fmaxf(w[2] + bb.z, 0.f), fmaxf(w[3] + bb.w, 0.f));
           }
           unsigned char* sub = P + (c / 64) * kSub;
           *reinterpret_cast<uint4*>(sub + sm100::swz<128>(r, (c % 64) / 8)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
           *reinterpret_cast<uint4*>(sub + sm100::swz<128>(r, (c % 64) / 8 + 1)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
         }
+        TTRACEW(i, j, 2);
         sm100::tc_fence_before();
         sm100::fence_proxy_async();
+        TTRACEW(i, j, 3);
         sm100::named_bar<kEpi>(1);
         if (leader) {
           sm100::mbar_arrive(&f_empty[b]);
@@ -353,9 +360,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       sm100::mbar_wait(&out_full, i & 1);
       TTRACE(i, 13);
       sm100::tc_fence_after();
-      const float s2 = add_residual(acc_out, p_b2);
-      sm100::tc_fence_before();
-      layer_norm(s2, p_g2, p_be2);
+      ln_block(acc_out, p_b2, p_g2, p_be2);
       sm100::fence_proxy_async();
       sm100::named_bar<kEpi>(1);
       if (leader) {
@@ -423,6 +428,7 @@ predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* 
 
 #ifdef PREDTOP_TRACE
 extern "C" PREDTOP_API int predtop_debug_tail_trace(unsigned long long* out) {
-  return cudaMemcpyFromSymbol(out, predtop::g_tail_trace, sizeof(predtop::g_tail_trace)) == cudaSuccess ? 0 : -7;
+  if (cudaMemcpyFromSymbol(out, predtop::g_tail_trace, sizeof(predtop::g_tail_trace)) != cudaSuccess) return -7;
+  return cudaMemcpyFromSymbol(out + 256, predtop::g_tail_trace2, sizeof(predtop::g_tail_trace2)) == cudaSuccess ? 0 : -7;
 }
 #endif

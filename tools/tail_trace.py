@@ -26,16 +26,21 @@ def main():
     for _ in range(3):
         m.forward(dag, ws, lat)
     torch.cuda.synchronize()
-    buf = (ctypes.c_ulonglong * 256)()
+    buf = (ctypes.c_ulonglong * 288)()
     pt.lib().predtop_debug_tail_trace.argtypes = [ctypes.c_void_p]
     assert pt.lib().predtop_debug_tail_trace(ctypes.cast(buf, ctypes.c_void_p)) == 0
-    t = np.frombuffer(buf, dtype=np.uint64).reshape(16, 16).astype(np.int64)
+    raw = np.frombuffer(buf, dtype=np.uint64).astype(np.int64)
+    t = raw[:256].reshape(16, 16)
+    w = raw[256:].reshape(4, 8)
     t0 = t[0, 0]
     print("tile " + " ".join(f"{n:>9s}" for n in NAMES))
     for i in range(12):
         print(f"{i:4d} " + " ".join(f"{(t[i, k] - t0) / 1000:9.2f}" for k in range(15)))
     d = np.diff(t[:12, :15], axis=1).mean(0) / 1000
     print("mean phase durations (us):", " ".join(f"{NAMES[k + 1]}:{d[k]:.2f}" for k in range(14)))
+    w0 = w[0].min()
+    for k, n in enumerate(["after waits", "after tmem_ld", "after stores", "after fences"]):
+        print(f"chunk1 tile4 {n:14s} (clk, per epilogue warp):", " ".join(f"{x - w0:6d}" for x in w[k]))
 
 
 if __name__ == "__main__":
