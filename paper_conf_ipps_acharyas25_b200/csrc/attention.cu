@@ -102,6 +102,12 @@ __device__ __forceinline__ void ldsm_x2_t(uint32_t addr, uint32_t& r0, uint32_t&
 
 constexpr int kChunk = 64;
 
+// flag nibble f (bit j = block j fully allowed) -> the thread's mask bits of
+// those blocks in rows a (bits 0-15) and b (bits 16-31): nibble j of each half
+__constant__ uint32_t c_full_bits[16] = {
+    0x00000000u, 0x000F000Fu, 0x00F000F0u, 0x00FF00FFu, 0x0F000F00u, 0x0F0F0F0Fu, 0x0FF00FF0u, 0x0FFF0FFFu,
+    0xF000F000u, 0xF00FF00Fu, 0xF0F0F0F0u, 0xF0FFF0FFu, 0xFF00FF00u, 0xFF0FFF0Fu, 0xFFF0FFF0u, 0xFFFFFFFFu};
+
 // Keys are permuted inside each 64-key chunk: mask bit b (key b of the chunk)
 // is stored in shared-memory row p(b) = 8*((b%16)/2) + 2*(b/16) + b%2.  Then
 // the m16n8 fragment element (n-tile nt, column 2*tq+u) of a thread holds
@@ -121,15 +127,14 @@ struct Attn {
 
   uint32_t qa[KS][4];
   float o[DN][4];
-  float osum[4];  // P x (ones column of V): row sums l, [0] row a, [2] row b
+  float osum[4];  // P x ones (tensor-core row sums l): [0] row a, [2] row b
   float m_a, m_b;
-  uint32_t kl, vl, vl1;  // per-lane ldmatrix byte offsets
+  uint32_t kl, vl;  // per-lane ldmatrix byte offsets
 
   __device__ __forceinline__ void init(int lane) {
     const int r8 = lane & 7;
     kl = (uint32_t)(((((lane >> 4) & 1) * 8 + r8) * PITCH + ((lane >> 3) & 1) * 8) * 2);
     vl = (uint32_t)(((((lane >> 3) & 1) * 8 + r8) * PITCH + ((lane >> 4) & 1) * 8) * 2);
-    vl1 = (uint32_t)(((((lane >> 3) & 1) * 8 + r8) * PITCH + DH) * 2);
 #pragma unroll
     for (int i = 0; i < DN; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
     osum[0] = osum[1] = osum[2] = osum[3] = 0.f;
@@ -146,8 +151,11 @@ struct Attn {
   // of the QK^T MMA: C = -m (allowed) or -inf (masked), so the MMA returns
   // s - m directly and P = exp2(S) needs no subtraction and no select.
   __device__ __forceinline__ void chunk(uint32_t kbase, uint32_t vbase, uint32_t mk, uint32_t fl) {
-    const uint32_t act = fl & 15u, full = fl >> 4;
+    const uint32_t act = fl & 15u;
     if (!act) return;
+    // fully allowed blocks (flag bits 4-7): set all of the thread's bits of
+    // those blocks -- one select per score either way, no second code path
+    mk |= c_full_bits[(fl >> 4) & 15u];
     // two 32-key phases (blocks 2ph, 2ph+1): half the live score registers
 #pragma unroll
     for (int ph = 0; ph < 2; ++ph) {
@@ -160,21 +168,13 @@ struct Attn {
         const int j = 2 * ph + jj;
         if (!(act & (1u << j))) continue;
         float c[2][4];
-        if (full & (1u << j)) {
 #pragma unroll
-          for (int u = 0; u < 2; ++u) {
-            c[u][0] = nma; c[u][1] = nma;
-            c[u][2] = nmb; c[u][3] = nmb;
-          }
-        } else {
-#pragma unroll
-          for (int u = 0; u < 2; ++u) {
-            const int e = 2 * (2 * j + u);
-            c[u][0] = ((mk >> e) & 1u) ? nma : -INFINITY;
-            c[u][1] = ((mk >> (e + 1)) & 1u) ? nma : -INFINITY;
-            c[u][2] = ((mk >> (e + 16)) & 1u) ? nmb : -INFINITY;
-            c[u][3] = ((mk >> (e + 17)) & 1u) ? nmb : -INFINITY;
-          }
+        for (int u = 0; u < 2; ++u) {
+          const int e = 2 * (2 * j + u);
+          c[u][0] = ((mk >> e) & 1u) ? nma : -INFINITY;
+          c[u][1] = ((mk >> (e + 1)) & 1u) ? nma : -INFINITY;
+          c[u][2] = ((mk >> (e + 16)) & 1u) ? nmb : -INFINITY;
+          c[u][3] = ((mk >> (e + 17)) & 1u) ? nmb : -INFINITY;
         }
 #pragma unroll
         for (int ks = 0; ks < KS; ++ks) {
@@ -243,9 +243,8 @@ struct Attn {
           mma16816(o[dn], pa, b0, b1);
           mma16816(o[dn + 1], pa, b2, b3);
         }
-        uint32_t c0, c1;
-        ldsm_x2_t(vbase + vl1 + j * BLK, c0, c1);
-        mma16816(osum, pa, c0, c1);
+        // row sums l: P x (16 x 8 all-ones B operand, constant fragments)
+        mma16816(osum, pa, 0x3C003C00u, 0x3C003C00u);
       }
     }
   }
@@ -318,9 +317,6 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
 
   A st;
   st.init(lane);
-  // V padding columns [DH, DH+8) hold ones: the PV MMA then yields the row sums
-  for (int rr = threadIdx.x; rr < nbuf * kChunk; rr += blockDim.x)
-    *reinterpret_cast<uint4*>(sV + (size_t)rr * A::PITCH + DH) = make_uint4(0x3C003C00u, 0x3C003C00u, 0x3C003C00u, 0x3C003C00u);
 
   if (RESIDENT) load_chunks(0, nchunks, 0);
   else load_chunks(0, 1, 0);
