@@ -317,30 +317,33 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
 
   A st;
   st.init(lane);
-
-  if (RESIDENT) load_chunks(0, nchunks, 0);
-  else load_chunks(0, 1, 0);
+  // Q fragments and the K words of the rows' own keys (for the reference m)
+  // are requested before the K/V copies so their latency overlaps them
+  uint32_t kw[A::KS][4];
 #pragma unroll
   for (int ks = 0; ks < A::KS; ++ks) {
     const int k0 = ks * 16 + 2 * tq;
-    st.qa[ks][0] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0) : 0u;
-    st.qa[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0) : 0u;
-    st.qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0 + 8) : 0u;
-    st.qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0 + 8) : 0u;
+    const __half* qa_p = Qg + (int64_t)ra * ld3 + k0;
+    const __half* qb_p = Qg + (int64_t)rb * ld3 + k0;
+    st.qa[ks][0] = va ? *reinterpret_cast<const uint32_t*>(qa_p) : 0u;
+    st.qa[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(qb_p) : 0u;
+    st.qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + 8) : 0u;
+    st.qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + 8) : 0u;
+    kw[ks][0] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel) : 0u;
+    kw[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel) : 0u;
+    kw[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel + 8) : 0u;
+    kw[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel + 8) : 0u;
   }
+  if (RESIDENT) load_chunks(0, nchunks, 0);
+  else load_chunks(0, 1, 0);
   // reference m of each row: its diagonal score q.k (M includes I, so the
   // row max is >= it; with lazy rescaling m stays within 8 of the max)
   {
     float sa = 0.f, sb = 0.f;
 #pragma unroll
     for (int ks = 0; ks < A::KS; ++ks) {
-      const int k0 = dmodel + ks * 16 + 2 * tq;
-      const uint32_t ka0 = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0) : 0u;
-      const uint32_t ka2 = va ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)ra * ld3 + k0 + 8) : 0u;
-      const uint32_t kb0 = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0) : 0u;
-      const uint32_t kb2 = vb ? *reinterpret_cast<const uint32_t*>(Qg + (int64_t)rb * ld3 + k0 + 8) : 0u;
-      sa += dot_h2(st.qa[ks][0], ka0) + dot_h2(st.qa[ks][2], ka2);
-      sb += dot_h2(st.qa[ks][1], kb0) + dot_h2(st.qa[ks][3], kb2);
+      sa += dot_h2(st.qa[ks][0], kw[ks][0]) + dot_h2(st.qa[ks][2], kw[ks][2]);
+      sb += dot_h2(st.qa[ks][1], kw[ks][1]) + dot_h2(st.qa[ks][3], kw[ks][3]);
     }
     sa += __shfl_xor_sync(0xffffffffu, sa, 1);
     sa += __shfl_xor_sync(0xffffffffu, sa, 2);
@@ -352,12 +355,11 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
   // this thread's 16 mask bits of rows a / b in chunk c: 16-bit piece tq of the word
   const uint16_t* Ma16 = reinterpret_cast<const uint16_t*>(Ma) + tq;
   const uint16_t* Mb16 = reinterpret_cast<const uint16_t*>(Mb) + tq;
-  auto mask_bits = [&](int c) -> uint32_t {
-    const uint32_t lo = va ? (uint32_t)Ma16[4 * c] : 0u;
-    const uint32_t hi = vb ? (uint32_t)Mb16[4 * c] : 0u;
-    return lo | (hi << 16);
-  };
-  uint32_t mk = mask_bits(0);
+  // raw 16-bit pieces, combined only where used: the loads of chunk c+1 are
+  // issued before chunk c and their latency hides behind it
+  auto mask_lo = [&](int c) -> uint32_t { return va ? (uint32_t)Ma16[4 * c] : 0u; };
+  auto mask_hi = [&](int c) -> uint32_t { return vb ? (uint32_t)Mb16[4 * c] : 0u; };
+  uint32_t mlo = mask_lo(0), mhi = mask_hi(0);
   const uint32_t kb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sK));
   const uint32_t vb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sV));
 
@@ -371,20 +373,22 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
     uint32_t fl = Fw[0];
     for (int c = 0; c < nchunks; ++c) {
       const bool more = c + 1 < nchunks;
-      const uint32_t nmk = more ? mask_bits(c + 1) : 0u;
+      const uint32_t nlo = more ? mask_lo(c + 1) : 0u, nhi = more ? mask_hi(c + 1) : 0u;
       const uint32_t nfl = more ? Fw[c + 1] : 0u;
       const uint32_t kc = kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2);
-      st.chunk(kc, vc, mk, __shfl_sync(0xffffffffu, fl, 0));
-      mk = nmk;
+      st.chunk(kc, vc, mlo | (mhi << 16), __shfl_sync(0xffffffffu, fl, 0));
+      mlo = nlo;
+      mhi = nhi;
       fl = nfl;
     }
   } else {
     for (int c = 0; c < nchunks; ++c) {
       const int buf = c & 1;
-      uint32_t nmk = 0u;
+      uint32_t nlo = 0u, nhi = 0u;
       if (c + 1 < nchunks) {
         load_chunks(c + 1, c + 2, buf ^ 1);
-        nmk = mask_bits(c + 1);
+        nlo = mask_lo(c + 1);
+        nhi = mask_hi(c + 1);
         cp_wait<1>();
       } else {
         cp_wait<0>();
@@ -393,10 +397,11 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
       if (warp_live) {
         const uint32_t kc = kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2);
         const uint32_t fl = __shfl_sync(0xffffffffu, (uint32_t)Fw[c], 0);
-        st.chunk(kc, vc, mk, fl);
+        st.chunk(kc, vc, mlo | (mhi << 16), fl);
       }
       __syncthreads();
-      mk = nmk;
+      mlo = nlo;
+      mhi = nhi;
     }
     if (!warp_live) return;
   }
@@ -448,6 +453,10 @@ predtop_status attention_launch(const predtop_dag_s* dag, int d, int H, const __
     return PREDTOP_ERR_TOO_LARGE;
   }
   ProfScope _p(PK_ATTN, st);
+  // PREDTOP_ATTN_TC=1: the tcgen05/TMEM variant (attention_tc.cu); measured
+  // slower than this kernel on the GPT workload, so opt-in
+  const char* tc = getenv("PREDTOP_ATTN_TC");
+  if (tc && tc[0] == '1' && attention_tc_supported(dag, d, H)) return attention_tc_launch(dag, d, H, qkv, out, st);
   if (dh == 16) return launch_dh<16>(dag, d, H, qkv, out, st, (unsigned)blocks);
   if (dh == 32) return launch_dh<32>(dag, d, H, qkv, out, st, (unsigned)blocks);
   set_error("unsupported head dim %d", dh);

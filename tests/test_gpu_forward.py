@@ -56,6 +56,24 @@ def test_latency_parity(pt, oracle_mod, name, batch_fn):
     assert err.max() <= TOL
 
 
+@pytest.mark.parametrize("name, batch_fn", [
+    ("paper", lambda: synth.stage_batch("gpt", 12, seed=11)),
+    ("gpt", lambda: synth.stage_batch("gpt", 24)),
+    ("gpt", lambda: synth.tiny_batch()),
+])
+def test_latency_parity_tcgen05_attention(pt, oracle_mod, name, batch_fn, monkeypatch):
+    """The opt-in tcgen05/TMEM attention kernel (attention_tc.cu, d_h = 16)."""
+    monkeypatch.setenv("PREDTOP_ATTN_TC", "1")
+    cfg, blob, model = _model(pt, name)
+    batch = batch_fn()
+    y, _ = _gpu_latency(pt, model, batch)
+    want = oracle_mod.forward_batch(cfg, blob, batch)
+    err = _rel(y, want)
+    print(f"{name} (tcgen05 attention): max rel err {err.max():.3e}")
+    assert np.isfinite(y).all()
+    assert err.max() <= TOL
+
+
 def test_mean_pool_and_relabelled(pt, oracle_mod):
     cfg, blob, model = _model(pt, "gpt", pool=1)
     b = synth.stage_batch("gpt", 4, first_graph=300)

@@ -16,6 +16,7 @@ import oracle  # noqa: E402
 from paper_conf_ipps_acharyas25_b200 import synth  # noqa: E402
 
 POINTS = ["x16", "qkv", "P", "att", "h16", "relu"]
+EX16 = os.environ.get("EX16") == "1"
 
 
 def r16(t, on):
@@ -39,8 +40,17 @@ def forward(cfg, w, n, s, d, f, off=()):
             sl = slice(hh * dh, (hh + 1) * dh)
             sc = (q[:, sl] @ k[:, sl].T) / np.sqrt(dh)
             sc = sc.masked_fill(~M, float("-inf"))
-            p = torch.exp(sc - sc.max(1, keepdim=True).values)
-            p16 = r16(p, on["P"])
+            if EX16:
+                # kernel v9 candidate: exp2 on fp16 arguments (ex2.approx.f16x2):
+                # m = diagonal score unless the row max exceeds it by > 8
+                l2 = sc * np.log2(np.e)
+                mx = l2.max(1, keepdim=True).values
+                dg = torch.diagonal(l2).unsqueeze(1)
+                m = torch.where(mx > dg + 8, mx, dg)
+                p16 = torch.exp2((l2 - m).half().float()).half().float()
+            else:
+                p = torch.exp(sc - sc.max(1, keepdim=True).values)
+                p16 = r16(p, on["P"])
             att[:, sl] = (p16 @ v[:, sl]) / p16.sum(1, keepdim=True)
         att = r16(att, on["att"])
         z = x + att @ g("W_o").T + g("b_o")
