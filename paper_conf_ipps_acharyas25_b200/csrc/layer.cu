@@ -41,15 +41,34 @@ __device__ __forceinline__ unsigned long long gtime() {
     if (leader && blockIdx.x == 0 && (i) < 16) g_tail_trace[i][k] = gtime(); \
   } while (0)
 // per-warp clock64 at 4 points of FFN chunk 1 of tile 4 (CTA 0)
-__device__ long long g_tail_trace2[4][8];
+__device__ long long g_tail_trace2[4][16];
+// MMA warp, tiles 2..9 of CTA 0: total clocks spent waiting on [0] ring_full,
+// [1] p_ready, [2] h_ready, [3] a_full, [4] o_empty / out_empty; [5] tile span
+__device__ long long g_tail_trace3[8];
+#define TWAIT(k, stmt)                                                   \
+  do {                                                                   \
+    const long long t0_ = clock64();                                     \
+    stmt;                                                                \
+    if (blockIdx.x == 0 && tile_i >= 2 && tile_i < 10) g_tail_trace3[k] += clock64() - t0_; \
+  } while (0)
 #define TTRACEW(i, j, k) \
   do {                   \
     if (lane == 0 && blockIdx.x == 0 && (i) == 4 && (j) == 1) g_tail_trace2[k][warp - 2] = clock64(); \
   } while (0)
 #else
+// MMA warp, tiles 2..9 of CTA 0: total clocks spent waiting on [0] ring_full,
+// [1] p_ready, [2] h_ready, [3] a_full, [4] o_empty / out_empty; [5] tile span
+__device__ long long g_tail_trace3[8];
+#define TWAIT(k, stmt)                                                   \
+  do {                                                                   \
+    const long long t0_ = clock64();                                     \
+    stmt;                                                                \
+    if (blockIdx.x == 0 && tile_i >= 2 && tile_i < 10) g_tail_trace3[k] += clock64() - t0_; \
+  } while (0)
 #define TTRACEW(i, j, k) \
   do {                   \
   } while (0)
+#define TWAIT(k, stmt) stmt
 #define TTRACE(i, k) \
   do {               \
   } while (0)
@@ -57,20 +76,23 @@ __device__ long long g_tail_trace2[4][8];
 
 namespace {
 
-constexpr int kThreads = 320;
-constexpr int kEpi = 256;
+#ifndef PREDTOP_TAIL_GROUPS
+#define PREDTOP_TAIL_GROUPS 4
+#endif
+constexpr int kGroups = PREDTOP_TAIL_GROUPS;  // column groups of the epilogue (x 4 warps each)
+constexpr int kEpi = 128 * kGroups;           // epilogue threads
+constexpr int kThreads = 64 + kEpi;
 constexpr int FC = 128;  // FFN chunk (hidden columns per chunk)
 constexpr int kSub = 128 * 128;  // bytes of one [128 rows x 64 fp16] or [128 x 32 fp32] sub-tile
 
 template <int D>
 struct TailCfg {
   static constexpr int X32 = 128 * D * 4;   // residual / h / x' fp32 tile
-  static constexpr int SA = 128 * 128 * 2;  // att tile [128 x D] and ReLU chunk 0 [128 x 128]
-  static constexpr int SP1 = 128 * 128 * 2; // ReLU chunk 1
+  static constexpr int SA = 128 * D * 2;    // att tile [128 x D] (O-proj A operand)
   static constexpr int SH = 128 * D * 2;    // h fp16 (FFN-1 A operand) / x' fp16 staging
   static constexpr int SLOT = (D > FC ? D : FC) * 64 * 2;
   static constexpr int PARAMS = (6 * D + 1024) * 4;  // bo g1 be1 b2 g2 be2 [D], b1 [<= 1024]
-  static constexpr int FIXED = X32 + SA + SP1 + SH + PARAMS + 1024;
+  static constexpr int FIXED = X32 + SA + SH + PARAMS + 1024;
   static constexpr int RS_FIT = (224 * 1024 - FIXED) / SLOT;
   static constexpr int RS = RS_FIT > 6 ? 6 : RS_FIT;
   static constexpr int SMEM = FIXED + RS * SLOT;
@@ -96,9 +118,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
   extern __shared__ unsigned char dsm[];
   unsigned char* base = sm100::align1024(dsm);
   unsigned char* sX = base;                 // fp32 [128 x D], D/32 sub-tiles
-  unsigned char* sA = sX + C::X32;          // att / ReLU chunk buffer 0
-  unsigned char* sP1 = sA + C::SA;          // ReLU chunk buffer 1
-  unsigned char* sH = sP1 + C::SP1;         // h fp16 / x' fp16
+  unsigned char* sA = sX + C::X32;          // att
+  unsigned char* sH = sA + C::SA;           // h fp16 / x' fp16
   unsigned char* ring = sH + C::SH;
   float* sPar = reinterpret_cast<float*>(ring + RS * C::SLOT);  // per-layer vectors
   float* p_bo = sPar;
@@ -119,9 +140,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
   for (int i = threadIdx.x; i < args.dff; i += blockDim.x) p_b1[i] = args.b1[i];
   __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
   __shared__ __align__(8) uint64_t a_full, a_free, x_full, x_free, o_full, o_empty, h_ready;
-  __shared__ __align__(8) uint64_t f_full[2], f_empty[2], p_ready[2], p_free[2], out_full, out_empty;
+  __shared__ __align__(8) uint64_t f_full[2], p_ready[2], out_full, out_empty;
   __shared__ uint32_t tmem_slot;
-  __shared__ float red_a[2][128], red_b[2][128];
+  __shared__ float red_a[kGroups][128], red_b[kGroups][128];
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ntiles = (int)ceil_div(args.M, 128);
@@ -133,8 +154,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       sm100::mbar_init(&ring_empty[s], 1);
     }
     uint64_t* singles[] = {&a_full, &a_free, &x_full, &x_free, &o_full, &o_empty, &h_ready,
-                           &f_full[0], &f_full[1], &f_empty[0], &f_empty[1], &p_ready[0], &p_ready[1],
-                           &p_free[0], &p_free[1], &out_full, &out_empty};
+                           &f_full[0], &f_full[1], &p_ready[0], &p_ready[1],
+                           &out_full, &out_empty};
     for (uint64_t* b : singles) sm100::mbar_init(b, 1);
     sm100::fence_mbar_init();
   }
@@ -184,11 +205,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
       constexpr uint32_t id_D = sm100::make_idesc_f16(128, D);
       constexpr uint32_t id_F = sm100::make_idesc_f16(128, FC);
       int it = 0;
+      int tile_i = 0;
+      (void)tile_i;
       // consume `nk` ring slots: D[tmem] (+)= A (64-wide K slices at a_base + kc*kSub) * slot^T
       auto mma_ring = [&](uint32_t d_tmem, uint32_t a_base, int nk, uint32_t idesc, bool first) {
         for (int kc = 0; kc < nk; ++kc, ++it) {
           const int s = it % RS;
-          sm100::mbar_wait(&ring_full[s], (it / RS) & 1);
+          TWAIT(0, sm100::mbar_wait(&ring_full[s], (it / RS) & 1));
           sm100::tc_fence_after();
           const uint32_t b0 = sm100::smem_u32(ring + s * C::SLOT);
           const uint32_t a0 = a_base + kc * kSub;
@@ -199,57 +222,84 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
           sm100::mma_commit(&ring_empty[s]);
         }
       };
-      const uint32_t aA = sm100::smem_u32(sA), aP1 = sm100::smem_u32(sP1), aH = sm100::smem_u32(sH);
+      // FFN-2 with A = P from TMEM: the epilogue leaves ReLU(chunk) as fp16
+      // pairs in the first FG/2 columns of each group's FG-column slice of
+      // acc_f[b]; K-step ks (16 hidden units) sits at column pcol(ks).
+      constexpr int FG = FC / kGroups;
+      auto mma_ring_ts = [&](uint32_t d_tmem, uint32_t p_tmem, int nk, uint32_t idesc, bool first) {
+        for (int kc = 0; kc < nk; ++kc, ++it) {
+          const int s = it % RS;
+          TWAIT(0, sm100::mbar_wait(&ring_full[s], (it / RS) & 1));
+          sm100::tc_fence_after();
+          const uint32_t b0 = sm100::smem_u32(ring + s * C::SLOT);
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {
+            const int ks = 4 * kc + kk;
+            const uint32_t pcol = (uint32_t)((ks / (FG / 16)) * FG + (ks % (FG / 16)) * 8);
+            sm100::mma_f16_ts(d_tmem, p_tmem + pcol, sm100::make_sdesc<128>(b0 + kk * 32), idesc,
+                              !(first && kc == 0 && kk == 0));
+          }
+          sm100::mma_commit(&ring_empty[s]);
+        }
+      };
+      const uint32_t aA = sm100::smem_u32(sA), aH = sm100::smem_u32(sH);
       int i = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
         const int cbase = i * NJ;  // global FFN chunk counter of this tile's chunk 0
+        // FFN-1 of chunk j into acc_f[j&1].  It overwrites the P of chunk j-2,
+        // which FFN-2 of chunk j-2 reads from TMEM; that MMA was issued earlier
+        // by this thread, and tcgen05.mma executes in issue order.
         auto ffn1 = [&](int j) {
-          const int b = j & 1, u = (cbase + j) >> 1;
-          sm100::mbar_wait(&f_empty[b], (u & 1) ^ 1);
-          sm100::tc_fence_after();
-          mma_ring(tmem + D + b * FC, aH, KD, id_F, true);
-          sm100::mma_commit(&f_full[b]);
+          mma_ring(tmem + D + (j & 1) * FC, aH, KD, id_F, true);
+          sm100::mma_commit(&f_full[j & 1]);
         };
-        sm100::mbar_wait(&a_full, i & 1);
-        sm100::mbar_wait(&o_empty, (i & 1) ^ 1);
+        tile_i = i;
+#ifdef PREDTOP_TRACE
+        const long long tspan0 = clock64();
+#endif
+        TWAIT(3, sm100::mbar_wait(&a_full, i & 1));
+        TWAIT(4, sm100::mbar_wait(&o_empty, (i & 1) ^ 1));
         sm100::tc_fence_after();
         mma_ring(acc_o, aA, KD, id_D, true);  // O-proj
         sm100::mma_commit(&o_full);
-        sm100::mbar_wait(&h_ready, i & 1);
+        sm100::mma_commit(&a_free);  // sA read: the next att tile may land
+        TWAIT(2, sm100::mbar_wait(&h_ready, i & 1));
         sm100::tc_fence_after();
         for (int j = 0; j < 2 && j < NJ; ++j) ffn1(j);
         for (int j = 0; j < NJ; ++j) {
           const int b = j & 1, u = (cbase + j) >> 1;
-          sm100::mbar_wait(&p_ready[b], u & 1);
-          if (j == 0) sm100::mbar_wait(&out_empty, (i & 1) ^ 1);
+          TWAIT(1, sm100::mbar_wait(&p_ready[b], u & 1));
+          if (j == 0) TWAIT(4, sm100::mbar_wait(&out_empty, (i & 1) ^ 1));
           sm100::tc_fence_after();
-          mma_ring(acc_out, b ? aP1 : aA, FC / 64, id_D, j == 0);  // FFN-2 chunk j
-          sm100::mma_commit(&p_free[b]);
-          if (j == NJ - 2) sm100::mma_commit(&a_free);  // last read of sA this tile
+          mma_ring_ts(acc_out, tmem + D + b * FC, FC / 64, id_D, j == 0);  // FFN-2 chunk j
           if (j + 2 < NJ) ffn1(j + 2);
         }
         sm100::mma_commit(&out_full);
+#ifdef PREDTOP_TRACE
+        if (blockIdx.x == 0 && i >= 2 && i < 10) g_tail_trace3[5] += clock64() - tspan0;
+#endif
       }
     }
   } else {
-    // ------------------------------------------ epilogue warps 2..9
-    const int q = warp & 3, half = (warp - 2) >> 2;
+    // ------------------------------------------ epilogue warps 2..(1 + 4 kGroups)
+    const int q = warp & 3, grp = (warp - 2) >> 2;
     const int r = q * 32 + lane;
     const uint32_t lrow = (uint32_t)(q * 32) << 16;
     const bool leader = (warp == 2 && lane == 0);
-    constexpr int DH2 = D / 2;  // columns of the row handled by this thread
-    // One LayerNorm block of row r, this thread doing columns [half*D/2, +D/2),
+    constexpr int DG = D / kGroups;  // columns of the row handled by this thread
+    constexpr int FG = FC / kGroups;  // hidden columns of an FFN chunk per thread
+    // One LayerNorm block of row r, this thread doing columns [grp*DG, +DG),
     // register resident: z = acc (TMEM) + bias + sX (fp32 residual), mean and
-    // variance over the two halves through red_a / red_b, then
+    // variance over the column groups through red_a / red_b, then
     // y = (z - mean) * rstd * g + be  ->  sX (fp32, in place) and sH (fp16).
     auto ln_block = [&](uint32_t acc, const float* bias, const float* g, const float* be) {
-      float z[DH2];
-      sm100::tmem_ld<DH2>(acc + lrow + half * DH2, z);
+      float z[DG];
+      sm100::tmem_ld<DG>(acc + lrow + grp * DG, z);
       sm100::tc_fence_before();
       float sum = 0.f;
 #pragma unroll
-      for (int k = 0; k < DH2 / 4; ++k) {
-        const int c4 = half * DH2 / 4 + k;
+      for (int k = 0; k < DG / 4; ++k) {
+        const int c4 = grp * DG / 4 + k;
         const float4 x = *reinterpret_cast<const float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8));
         const float4 bb = reinterpret_cast<const float4*>(bias)[c4];
         z[4 * k + 0] = x.x + (z[4 * k + 0] + bb.x);
@@ -258,24 +308,30 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
         z[4 * k + 3] = x.w + (z[4 * k + 3] + bb.w);
         sum += (z[4 * k] + z[4 * k + 1]) + (z[4 * k + 2] + z[4 * k + 3]);
       }
-      red_a[half][r] = sum;
+      red_a[grp][r] = sum;
       sm100::named_bar<kEpi>(1);
-      const float mean = (red_a[0][r] + red_a[1][r]) * (1.0f / D);
+      float tot = 0.f;
+#pragma unroll
+      for (int i2 = 0; i2 < kGroups; ++i2) tot += red_a[i2][r];
+      const float mean = tot * (1.0f / D);
       float sq = 0.f;
 #pragma unroll
-      for (int k = 0; k < DH2 / 4; ++k) {
+      for (int k = 0; k < DG / 4; ++k) {
         const float a = z[4 * k] - mean, b = z[4 * k + 1] - mean, cc = z[4 * k + 2] - mean, d = z[4 * k + 3] - mean;
         sq += (a * a + b * b) + (cc * cc + d * d);
       }
-      red_b[half][r] = sq;
+      red_b[grp][r] = sq;
       sm100::named_bar<kEpi>(1);
-      const float rstd = rsqrtf((red_b[0][r] + red_b[1][r]) * (1.0f / D) + args.eps);
+      float tsq = 0.f;
 #pragma unroll
-      for (int k8 = 0; k8 < DH2 / 8; ++k8) {
+      for (int i2 = 0; i2 < kGroups; ++i2) tsq += red_b[i2][r];
+      const float rstd = rsqrtf(tsq * (1.0f / D) + args.eps);
+#pragma unroll
+      for (int k8 = 0; k8 < DG / 8; ++k8) {
         float y[8];
 #pragma unroll
         for (int h2 = 0; h2 < 2; ++h2) {
-          const int k = 2 * k8 + h2, c4 = half * DH2 / 4 + k;
+          const int k = 2 * k8 + h2, c4 = grp * DG / 4 + k;
           const float4 gm = reinterpret_cast<const float4*>(g)[c4];
           const float4 bt = reinterpret_cast<const float4*>(be)[c4];
           float4 o;
@@ -286,7 +342,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
           *reinterpret_cast<float4*>(sX + (c4 / 8) * kSub + sm100::swz<128>(r, c4 % 8)) = o;
           y[4 * h2] = o.x; y[4 * h2 + 1] = o.y; y[4 * h2 + 2] = o.z; y[4 * h2 + 3] = o.w;
         }
-        const int c = half * DH2 + 8 * k8;
+        const int c = grp * DG + 8 * k8;
         *reinterpret_cast<uint4*>(sH + (c / 64) * kSub + sm100::swz<128>(r, (c % 64) / 8)) =
             make_uint4(sm100::pack_half2(y[0], y[1]), sm100::pack_half2(y[2], y[3]),
                        sm100::pack_half2(y[4], y[5]), sm100::pack_half2(y[6], y[7]));
@@ -316,44 +372,34 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
         sm100::mbar_arrive(&h_ready);
       }
       TTRACE(i, 4);
-      // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 operand buffer
+      // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 pairs back into acc_f (the
+      // first half of this thread's column slice): the TMEM A operand of FFN-2
       for (int j = 0; j < NJ; ++j) {
         const int b = j & 1, u = (cbase + j) >> 1;
         sm100::mbar_wait(&f_full[b], u & 1);
-        sm100::mbar_wait(&p_free[b], (u & 1) ^ 1);
         TTRACE(i, 5 + 2 * (j & 3));
         TTRACEW(i, j, 0);
         sm100::tc_fence_after();
-        unsigned char* P = b ? sP1 : sA;
-        const uint32_t accf = tmem + D + b * FC + lrow;
-        const float* b1 = p_b1 + j * FC;
-        float v[FC / 2];
-        sm100::tmem_ld<FC / 2>(accf + half * FC / 2, v);
+        const uint32_t accf = tmem + D + b * FC + lrow + grp * FG;
+        const float* b1 = p_b1 + j * FC + grp * FG;
+        float v[FG];
+        sm100::tmem_ld<FG>(accf, v);
         TTRACEW(i, j, 1);
+        uint32_t pk[FG / 2];
 #pragma unroll
-        for (int g16 = 0; g16 < FC / 32; ++g16) {
-          const int c = half * FC / 2 + 16 * g16;
-          uint32_t pk[8];
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const float4 bb = reinterpret_cast<const float4*>(b1 + c)[k];
-            const float* w = v + 16 * g16 + 4 * k;
-            pk[2 * k] = sm100::pack_half2(fmaxf(w[0] + bb.x, 0.f), fmaxf(w[1] + bb.y, 0.f));
-            pk[2 * k + 1] = sm100::pack_half2(fmaxf(w[2] + bb.z, 0.f), fmaxf(w[3] + bb.w, 0.f));
-          }
-          unsigned char* sub = P + (c / 64) * kSub;
-          *reinterpret_cast<uint4*>(sub + sm100::swz<128>(r, (c % 64) / 8)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-          *reinterpret_cast<uint4*>(sub + sm100::swz<128>(r, (c % 64) / 8 + 1)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+        for (int k = 0; k < FG / 4; ++k) {
+          const float4 bb = reinterpret_cast<const float4*>(b1)[k];
+          pk[2 * k] = sm100::pack_half2(fmaxf(v[4 * k] + bb.x, 0.f), fmaxf(v[4 * k + 1] + bb.y, 0.f));
+          pk[2 * k + 1] = sm100::pack_half2(fmaxf(v[4 * k + 2] + bb.z, 0.f), fmaxf(v[4 * k + 3] + bb.w, 0.f));
         }
+#pragma unroll
+        for (int k = 0; k < FG / 32; ++k) sm100::tmem_st16(accf + 16 * k, pk + 16 * k);
+        sm100::tmem_wait_st();
         TTRACEW(i, j, 2);
         sm100::tc_fence_before();
-        sm100::fence_proxy_async();
         TTRACEW(i, j, 3);
         sm100::named_bar<kEpi>(1);
-        if (leader) {
-          sm100::mbar_arrive(&f_empty[b]);
-          sm100::mbar_arrive(&p_ready[b]);
-        }
+        if (leader) sm100::mbar_arrive(&p_ready[b]);
         TTRACE(i, 6 + 2 * (j & 3));
       }
       // ---- LN2 and stores
@@ -429,6 +475,7 @@ predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* 
 #ifdef PREDTOP_TRACE
 extern "C" PREDTOP_API int predtop_debug_tail_trace(unsigned long long* out) {
   if (cudaMemcpyFromSymbol(out, predtop::g_tail_trace, sizeof(predtop::g_tail_trace)) != cudaSuccess) return -7;
-  return cudaMemcpyFromSymbol(out + 256, predtop::g_tail_trace2, sizeof(predtop::g_tail_trace2)) == cudaSuccess ? 0 : -7;
+  if (cudaMemcpyFromSymbol(out + 256, predtop::g_tail_trace2, sizeof(predtop::g_tail_trace2)) != cudaSuccess) return -7;
+  return cudaMemcpyFromSymbol(out + 320, predtop::g_tail_trace3, sizeof(predtop::g_tail_trace3)) == cudaSuccess ? 0 : -7;
 }
 #endif

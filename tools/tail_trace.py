@@ -26,12 +26,13 @@ def main():
     for _ in range(3):
         m.forward(dag, ws, lat)
     torch.cuda.synchronize()
-    buf = (ctypes.c_ulonglong * 288)()
+    buf = (ctypes.c_ulonglong * 328)()
     pt.lib().predtop_debug_tail_trace.argtypes = [ctypes.c_void_p]
     assert pt.lib().predtop_debug_tail_trace(ctypes.cast(buf, ctypes.c_void_p)) == 0
     raw = np.frombuffer(buf, dtype=np.uint64).astype(np.int64)
     t = raw[:256].reshape(16, 16)
-    w = raw[256:].reshape(4, 8)
+    w = raw[256:320].reshape(4, 16)
+    mw = raw[320:328]
     t0 = t[0, 0]
     print("tile " + " ".join(f"{n:>9s}" for n in NAMES))
     for i in range(12):
@@ -41,6 +42,8 @@ def main():
     w0 = w[0].min()
     for k, n in enumerate(["after waits", "after tmem_ld", "after stores", "after fences"]):
         print(f"chunk1 tile4 {n:14s} (clk, per epilogue warp):", " ".join(f"{x - w0:6d}" for x in w[k]))
+    print("MMA warp, mean per tile (clk): ring_full wait %d, p_ready wait %d, h_ready wait %d, a_full wait %d, "
+          "o/out_empty wait %d, tile span %d" % tuple(mw[:6] // 8))
 
 
 if __name__ == "__main__":
