@@ -282,7 +282,7 @@ predtop_status predtop_reachability(predtop_dag dag, uint64_t* bits_out, void* c
 
 predtop_status predtop_debug_mask(predtop_dag dag, uint64_t* bits_out, void* cuda_stream) {
   if (!dag || !bits_out) { set_error("NULL argument"); return PREDTOP_ERR_INVALID_ARG; }
-  return dag_copy_bits(dag, dag->d.M, bits_out, S(cuda_stream));
+  return dag_copy_bits(dag, dag->d.M, bits_out, S(cuda_stream), /*unperm=*/true);
 }
 
 predtop_status predtop_debug_tiles(predtop_dag dag, uint8_t* tile_class_out, int64_t* pairs_out,

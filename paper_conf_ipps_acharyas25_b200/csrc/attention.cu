@@ -8,21 +8,26 @@
 // a graph are fetched from HBM once and re-read by the other heads from L2.
 //
 // Keys/values live in shared memory in 64-key chunks (one chunk = one 64-bit
-// word of every mask row).  Graphs whose K/V fit (N <= ~1000 at d_h = 16) are
-// loaded whole: one CTA barrier, then every warp runs independently.  Larger
-// graphs stream chunks through a cp.async double buffer.
+// word of every mask row), brought in by TMA ([64 keys x d_h] boxes, one
+// elected thread, one mbarrier).  Graphs whose K/V fit (N <= ~1500 at d_h =
+// 16) are loaded whole, then every warp runs independently; larger graphs
+// stream chunks through a two-buffer TMA pipeline.
 //
-// Block sparsity per warp at 16-key granularity: a 16 x 16 block with no
-// allowed pair among the warp's rows costs nothing; a block whose pairs are
-// all allowed skips the mask arithmetic; only partial blocks apply the mask
-// (compact per-thread bit masks, one select per score).  Online softmax in
-// fp32 with exp2 (MUFU ex2), P rounded once to fp16.
+// Per warp (16 query rows) and 16-key block: QK^T on the m16n8k16 tensor-core
+// MMA with the accumulator input C = -m (allowed pair) or -inf (masked), so
+// the MMA returns s - m directly; a block with no allowed pair among the
+// warp's rows is skipped (flags from k_bflags).  Online softmax in log2 units
+// (Q pre-scaled in the QKV epilogue), reference m = the row's diagonal score,
+// lazy rescaling; P = exp2(s - m) (MUFU ex2) rounded once to fp16; the row
+// sums l come from the tensor core (P x an all-ones B fragment).
 //
-// At d_h = 16/32 the kernel is bound by the exponentials (one MUFU ex2 per
-// computed score), not by the tensor pipe: QK^T and PV are 2*d_h flops per
-// score each.  The warp-level m16n8k16 MMA keeps S and P in registers (the S
-// accumulator fragment is the P operand fragment); see DESIGN.md "K6".
+// At d_h = 16/32 the kernel is bound by the exponentials and the issue slots
+// around them, not by the tensor pipe: QK^T and PV are 2*d_h flops per score
+// each.  The S accumulator fragment is the P operand fragment, so S and P
+// never leave registers; see DESIGN.md "K6".  attention_tc.cu holds an
+// opt-in tcgen05/TMEM variant.
 #include "internal.h"
+#include "sm100.cuh"
 
 namespace predtop {
 
@@ -56,16 +61,6 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t& r0, uint32_t&
                : "r"(addr));
 }
 
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool valid) {
-  const int n = valid ? 16 : 0;  // src-size 0 -> zero fill
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n));
-}
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;"); }
-template <int N>
-__device__ __forceinline__ void cp_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N));
-}
-
 __device__ __forceinline__ float dot_h2(uint32_t a, uint32_t b) {
   const float2 x = __half22float2(*reinterpret_cast<const __half2*>(&a));
   const float2 y = __half22float2(*reinterpret_cast<const __half2*>(&b));
@@ -76,14 +71,6 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
-// Zero-accumulator variant (first k-step): C = 0 without zeroing registers.
-__device__ __forceinline__ void mma16816_z(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
-  asm volatile(
-      "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
-      "{%10,%10,%10,%10};"
-      : "=f"(d[0]), "=f"(d[1]), "=f"(d[2]), "=f"(d[3])
-      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1), "f"(0.f));
-}
 // D = A*B + C with an explicit accumulator input (QK^T: C = -m or -inf).
 __device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1,
                                            const float (&c)[4]) {
@@ -94,11 +81,6 @@ __device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4]
       : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1), "f"(c[0]), "f"(c[1]), "f"(c[2]),
         "f"(c[3]));
 }
-__device__ __forceinline__ void ldsm_x2_t(uint32_t addr, uint32_t& r0, uint32_t& r1) {
-  asm volatile("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0,%1}, [%2];"
-               : "=r"(r0), "=r"(r1)
-               : "r"(addr));
-}
 
 constexpr int kChunk = 64;
 
@@ -108,33 +90,41 @@ __constant__ uint32_t c_full_bits[16] = {
     0x00000000u, 0x000F000Fu, 0x00F000F0u, 0x00FF00FFu, 0x0F000F00u, 0x0F0F0F0Fu, 0x0FF00FF0u, 0x0FFF0FFFu,
     0xF000F000u, 0xF00FF00Fu, 0xF0F0F0F0u, 0xF0FFF0FFu, 0xFF00FF00u, 0xFF0FFF0Fu, 0xFFF0FFF0u, 0xFFFFFFFFu};
 
-// Keys are permuted inside each 64-key chunk: mask bit b (key b of the chunk)
-// is stored in shared-memory row p(b) = 8*((b%16)/2) + 2*(b/16) + b%2.  Then
-// the m16n8 fragment element (n-tile nt, column 2*tq+u) of a thread holds
-// key b = 16*tq + 2*nt + u, i.e. a thread's 16 mask bits are the contiguous
-// bits [16*tq, 16*tq+16) of the word, bit 2*nt+u.  16-row block j (n-tiles
-// 2j, 2j+1) covers the mask bits 0x000F000F000F000F << 4j.  Softmax and PV
-// are invariant under a consistent permutation of K and V rows.
-__device__ __forceinline__ int key_row(int b) { return ((b & 15) >> 1) * 8 + 2 * (b >> 4) + (b & 1); }
-
+// K and V chunks sit in shared memory in natural key order, as TMA writes a
+// [64 keys x d_h] box with the swizzle of its row size (SWIZZLE_32B for d_h =
+// 16, 64B for 32): 16-byte piece p of row r is at r*RB + 16*(p ^ sw(r)),
+// sw(r) = ((r*RB) >> 7) & (RB/16 - 1).  The mask words are stored permuted
+// (internal.h mask_pos) so that the keys of a thread's accumulator fragment
+// (n-tile nt, column 2tq+u: key 8nt + 2tq + u) are the contiguous bits
+// [16tq, 16tq+16), bit 2nt+u, and 16-key block j is 0x000F000F000F000F << 4j.
 template <int DH>
 struct Attn {
-  static constexpr int PITCH = DH + 8;  // halves; 48 B / 80 B rows: conflict-free ldmatrix
+  static constexpr int RB = DH * 2;     // row bytes (TMA box row, swizzle span)
   static constexpr int KS = DH / 16;    // k-steps for QK^T
   static constexpr int DN = DH / 8;     // n-tiles of the output
-  static constexpr int CHUNK_HALVES = kChunk * PITCH;
-  static constexpr int BLK = 16 * PITCH * 2;  // bytes of a 16-key block
+  static constexpr int CHUNK_BYTES = kChunk * RB;  // one K or V chunk
+  static constexpr int BLK = 16 * RB;   // bytes of a 16-key block
 
   uint32_t qa[KS][4];
   float o[DN][4];
   float osum[4];  // P x ones (tensor-core row sums l): [0] row a, [2] row b
   float m_a, m_b;
-  uint32_t kl, vl;  // per-lane ldmatrix byte offsets
+  uint32_t kl[KS], vl[DN / 2];  // per-lane ldmatrix byte offsets (swizzled)
 
   __device__ __forceinline__ void init(int lane) {
     const int r8 = lane & 7;
-    kl = (uint32_t)(((((lane >> 4) & 1) * 8 + r8) * PITCH + ((lane >> 3) & 1) * 8) * 2);
-    vl = (uint32_t)(((((lane >> 3) & 1) * 8 + r8) * PITCH + ((lane >> 4) & 1) * 8) * 2);
+    // K (non-transposed x4): matrices (keys 0-7 | 8-15) x (cols 0-7 | 8-15) of
+    // the k-step; V (transposed x4): (keys 0-7 | 8-15) x (cols dn*8.. | +8).
+    // Block offsets (16 rows) are multiples of 128 B, so sw(r) depends on
+    // the lane only.
+    const int rk = ((lane >> 4) & 1) * 8 + r8, rv = ((lane >> 3) & 1) * 8 + r8;
+    const int swk = ((rk * RB) >> 7) & (RB / 16 - 1), swv = ((rv * RB) >> 7) & (RB / 16 - 1);
+#pragma unroll
+    for (int ks = 0; ks < KS; ++ks)
+      kl[ks] = (uint32_t)(rk * RB + 16 * ((2 * ks + ((lane >> 3) & 1)) ^ swk));
+#pragma unroll
+    for (int i = 0; i < DN / 2; ++i)
+      vl[i] = (uint32_t)(rv * RB + 16 * ((2 * i + ((lane >> 4) & 1)) ^ swv));
 #pragma unroll
     for (int i = 0; i < DN; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
     osum[0] = osum[1] = osum[2] = osum[3] = 0.f;
@@ -179,7 +169,7 @@ struct Attn {
 #pragma unroll
         for (int ks = 0; ks < KS; ++ks) {
           uint32_t b0, b1, b2, b3;
-          ldsm_x4(kbase + kl + j * BLK + ks * 32, b0, b1, b2, b3);
+          ldsm_x4(kbase + kl[ks] + j * BLK, b0, b1, b2, b3);
           if (ks == 0) {
             mma16816_c(s[2 * jj], qa[ks], b0, b1, c[0]);
             mma16816_c(s[2 * jj + 1], qa[ks], b2, b3, c[1]);
@@ -239,7 +229,7 @@ struct Attn {
 #pragma unroll
         for (int dn = 0; dn < DN; dn += 2) {
           uint32_t b0, b1, b2, b3;
-          ldsm_x4_t(vbase + vl + j * BLK + dn * 16, b0, b1, b2, b3);
+          ldsm_x4_t(vbase + vl[dn / 2] + j * BLK, b0, b1, b2, b3);
           mma16816(o[dn], pa, b0, b1);
           mma16816(o[dn + 1], pa, b2, b3);
         }
@@ -252,12 +242,12 @@ struct Attn {
 };
 
 template <int DH, bool RESIDENT>
-__global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G, int H, int dmodel,
-                                                 const __half* __restrict__ qkv,
-                                                 __half* __restrict__ out) {
+__global__ void __launch_bounds__(256, DH == 16 ? 4 : 2)
+    k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
+           const __half* __restrict__ qkv, __half* __restrict__ out) {
   using A = Attn<DH>;
   extern __shared__ __align__(16) unsigned char dsm_attn[];
-  __half* sK = reinterpret_cast<__half*>(dsm_attn);  // [nbuf][64][PITCH]
+  __shared__ __align__(8) uint64_t kv_full[2];
   const int h = blockIdx.x % H;
   const int widx = blockIdx.x / H;
   if (widx >= d.qtile_off[G]) return;
@@ -269,7 +259,8 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
   const int W = 2 * ((N + 127) / 128);
   const int nchunks = (N + kChunk - 1) / kChunk;
   const int nbuf = RESIDENT ? nchunks : 2;
-  __half* sV = sK + (size_t)nbuf * A::CHUNK_HALVES;
+  unsigned char* sK = sm100::align1024(dsm_attn);      // [nbuf][64 keys][DH], TMA swizzle
+  unsigned char* sV = sK + (size_t)nbuf * A::CHUNK_BYTES;
   const uint64_t* Mg = d.M + d.row_off[g];
   const int ld3 = 3 * dmodel;
   const __half* Qg = qkv + n0 * ld3 + h * DH;
@@ -285,40 +276,31 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
   // block flags of this warp's 16-row group, one byte per chunk (k_bflags)
   const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)(warp_live ? qt * 8 + warp : 0) * nchunks;
 
-  // Loader roles: a chunk is 2 (K, V) x 64 keys x DH/8 16-byte segments =
-  // 16*DH segments; thread t always moves the same (matrix, key, segment)
-  // slots (t, t+256, ...) of every chunk, so per chunk it only adds offsets.
-  constexpr int SEGS = kChunk * DH / 8;  // 16-byte segments per matrix per chunk
-  constexpr int PER = 2 * SEGS / 256;    // slots per thread per chunk (1 or 2)
-  static_assert(2 * SEGS % 256 == 0, "loader");
-  uint32_t ld_dst[PER];
-  int64_t ld_src[PER];
-  int ld_key[PER];
-#pragma unroll
-  for (int k = 0; k < PER; ++k) {
-    const unsigned s = threadIdx.x + 256u * k;
-    const unsigned mat = s / SEGS, r = (s % SEGS) / (DH / 8), seg = s % (DH / 8);
-    ld_key[k] = (int)r;
-    ld_src[k] = (int64_t)(mat ? 2 * dmodel : dmodel) + (int64_t)r * ld3 + seg * 8;  // from Qg
-    ld_dst[k] = static_cast<uint32_t>(__cvta_generic_to_shared((mat ? sV : sK) + key_row((int)r) * A::PITCH + seg * 8));
+  // K/V chunks by TMA (one thread): [64 keys x DH] boxes of the qkv matrix at
+  // columns d + h*DH (K) and 2d + h*DH (V); keys past N read the next graph's
+  // rows (masked) or zeros past the tensor end.
+  if (threadIdx.x == 0) {
+    sm100::mbar_init(&kv_full[0], 1);
+    sm100::mbar_init(&kv_full[1], 1);
+    sm100::fence_mbar_init();
   }
-  auto load_chunks = [&](int c0, int c1, int buf0) {
+  __syncthreads();
+  auto load_chunks = [&](int c0, int c1, int slot0, uint64_t* bar) {
+    sm100::mbar_arrive_expect_tx(bar, (uint32_t)((c1 - c0) * 2 * A::CHUNK_BYTES));
     for (int c = c0; c < c1; ++c) {
-      const uint32_t boff = (uint32_t)((buf0 + c - c0) * A::CHUNK_HALVES * 2);
-#pragma unroll
-      for (int k = 0; k < PER; ++k) {
-        const int key = c * kChunk + ld_key[k];
-        const __half* src = Qg + (key < N ? ld_src[k] + (int64_t)c * kChunk * ld3 : 0);
-        cp_async16(ld_dst[k] + boff, src, key < N);
-      }
+      const int row = (int)(n0 + c * kChunk);
+      const int slot = slot0 + c - c0;
+      sm100::tma_load_2d(sK + slot * A::CHUNK_BYTES, &tkv, bar, dmodel + h * DH, row);
+      sm100::tma_load_2d(sV + slot * A::CHUNK_BYTES, &tkv, bar, 2 * dmodel + h * DH, row);
     }
-    cp_commit();
   };
+  if (threadIdx.x == 0) {
+    if (RESIDENT) load_chunks(0, nchunks, 0, &kv_full[0]);
+    else load_chunks(0, 1, 0, &kv_full[0]);
+  }
 
   A st;
   st.init(lane);
-  // Q fragments and the K words of the rows' own keys (for the reference m)
-  // are requested before the K/V copies so their latency overlaps them
   uint32_t kw[A::KS][4];
 #pragma unroll
   for (int ks = 0; ks < A::KS; ++ks) {
@@ -334,8 +316,6 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
     kw[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel + 8) : 0u;
     kw[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel + 8) : 0u;
   }
-  if (RESIDENT) load_chunks(0, nchunks, 0);
-  else load_chunks(0, 1, 0);
   // reference m of each row: its diagonal score q.k (M includes I, so the
   // row max is >= it; with lazy rescaling m stays within 8 of the max)
   {
@@ -352,54 +332,47 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
     st.m_a = sa;
     st.m_b = sb;
   }
-  // this thread's 16 mask bits of rows a / b in chunk c: 16-bit piece tq of the word
+  // this thread's 16 mask bits of rows a / b in chunk c: 16-bit piece tq of
+  // the (stored-layout) word; raw pieces, combined only where used, so the
+  // loads for chunk c+1 are issued before chunk c and hide behind it
   const uint16_t* Ma16 = reinterpret_cast<const uint16_t*>(Ma) + tq;
   const uint16_t* Mb16 = reinterpret_cast<const uint16_t*>(Mb) + tq;
-  // raw 16-bit pieces, combined only where used: the loads of chunk c+1 are
-  // issued before chunk c and their latency hides behind it
   auto mask_lo = [&](int c) -> uint32_t { return va ? (uint32_t)Ma16[4 * c] : 0u; };
   auto mask_hi = [&](int c) -> uint32_t { return vb ? (uint32_t)Mb16[4 * c] : 0u; };
   uint32_t mlo = mask_lo(0), mhi = mask_hi(0);
-  const uint32_t kb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sK));
-  const uint32_t vb0 = static_cast<uint32_t>(__cvta_generic_to_shared(sV));
+  const uint32_t kb0 = sm100::smem_u32(sK), vb0 = sm100::smem_u32(sV);
 
   if (RESIDENT) {
-    cp_wait<0>();
-    __syncthreads();
-  }
-
-  if (RESIDENT) {
+    sm100::mbar_wait(&kv_full[0], 0);
     if (!warp_live) return;
     uint32_t fl = Fw[0];
     for (int c = 0; c < nchunks; ++c) {
       const bool more = c + 1 < nchunks;
       const uint32_t nlo = more ? mask_lo(c + 1) : 0u, nhi = more ? mask_hi(c + 1) : 0u;
       const uint32_t nfl = more ? Fw[c + 1] : 0u;
-      const uint32_t kc = kb0 + (uint32_t)(c * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(c * A::CHUNK_HALVES * 2);
-      st.chunk(kc, vc, mlo | (mhi << 16), __shfl_sync(0xffffffffu, fl, 0));
+      const uint32_t off = (uint32_t)(c * A::CHUNK_BYTES);
+      st.chunk(kb0 + off, vb0 + off, mlo | (mhi << 16), __shfl_sync(0xffffffffu, fl, 0));
       mlo = nlo;
       mhi = nhi;
       fl = nfl;
     }
   } else {
+    // two chunk buffers: chunk c+1 streams in while chunk c runs
     for (int c = 0; c < nchunks; ++c) {
       const int buf = c & 1;
       uint32_t nlo = 0u, nhi = 0u;
       if (c + 1 < nchunks) {
-        load_chunks(c + 1, c + 2, buf ^ 1);
+        if (threadIdx.x == 0) load_chunks(c + 1, c + 2, buf ^ 1, &kv_full[buf ^ 1]);
         nlo = mask_lo(c + 1);
         nhi = mask_hi(c + 1);
-        cp_wait<1>();
-      } else {
-        cp_wait<0>();
       }
-      __syncthreads();
+      sm100::mbar_wait(&kv_full[buf], (c >> 1) & 1);
       if (warp_live) {
-        const uint32_t kc = kb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2), vc = vb0 + (uint32_t)(buf * A::CHUNK_HALVES * 2);
+        const uint32_t off = (uint32_t)(buf * A::CHUNK_BYTES);
         const uint32_t fl = __shfl_sync(0xffffffffu, (uint32_t)Fw[c], 0);
-        st.chunk(kc, vc, mlo | (mhi << 16), fl);
+        st.chunk(kb0 + off, vb0 + off, mlo | (mhi << 16), fl);
       }
-      __syncthreads();
+      __syncthreads();  // every warp is done with buffer buf before it is reloaded
       mlo = nlo;
       mhi = nhi;
     }
@@ -423,10 +396,13 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2) k_attn(DagDev d, int G,
 template <int DH>
 predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
                          cudaStream_t st, unsigned blocks) {
-  constexpr int CH_BYTES = kChunk * (DH + 8) * 2;  // one K or V chunk
+  constexpr int CH_BYTES = kChunk * DH * 2;  // one K or V chunk
   const int G = dag->desc.num_graphs;
   const int maxch = (int)ceil_div(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), kChunk);
-  const int resident_bytes = 2 * maxch * CH_BYTES;
+  const int resident_bytes = 2 * maxch * CH_BYTES + 1024;
+  CUtensorMap tkv;
+  if (!encode_tma_2d(&tkv, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kChunk))
+    return PREDTOP_ERR_CUDA;
   if (resident_bytes <= 100 * 1024) {
     static bool attr_done = false;
     if (!attr_done) {
@@ -434,9 +410,9 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
                                        100 * 1024));
       attr_done = true;
     }
-    k_attn<DH, true><<<blocks, 256, resident_bytes, st>>>(dag->d, G, H, d, qkv, out);
+    k_attn<DH, true><<<blocks, 256, resident_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
   } else {
-    k_attn<DH, false><<<blocks, 256, 4 * CH_BYTES, st>>>(dag->d, G, H, d, qkv, out);
+    k_attn<DH, false><<<blocks, 256, 4 * CH_BYTES + 1024, st>>>(tkv, dag->d, G, H, d, qkv, out);
   }
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;

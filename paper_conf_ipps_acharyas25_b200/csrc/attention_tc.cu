@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(kThreads, 4)
     const uint32_t lrow = (uint32_t)(32 * q4) << 16;
     // (0) the mask word of this row and the Q/K/V tiles (TMA)
     const uint64_t* Mrow = d.M + d.row_off[g] + (int64_t)(valid ? row : 0) * W;
-    uint64_t mw = valid ? Mrow[0] : 0ull;
+    uint64_t mw_raw = valid ? Mrow[0] : 0ull, mw = 0ull;  // stored layout -> mask_unperm at use
     WAIT(&bar_ld, 0);
     // (1) reference m: the diagonal score q_row . k_row (fp32, from the SW32
     // tiles: 16-byte chunk j of row x sits at x*32 + 16*(j ^ ((x >> 2) & 1))),
@@ -282,8 +282,9 @@ __global__ void __launch_bounds__(kThreads, 4)
     // polynomial (exp2_poly2) for the last kPoly keys of each chunk.
     float mu0 = m, mu1 = m;
     auto chunk = [&](int c, int b) {
+      if (!b) mw = mask_unperm(mw_raw);
       const uint32_t bits = b ? (uint32_t)(mw >> 32) : (uint32_t)mw;
-      if (b && valid && c + 1 < nch) mw = Mrow[(c + 1) >> 1];
+      if (b && valid && c + 1 < nch) mw_raw = Mrow[(c + 1) >> 1];
       if (warp == 2 && lane == 0) ATR(2, c);
       WAIT(&s_full[b], (c >> 1) & 1);
       if (warp == 2 && lane == 0) ATR(3, c);

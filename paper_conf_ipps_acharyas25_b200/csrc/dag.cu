@@ -560,11 +560,13 @@ __global__ void __launch_bounds__(128) k_bflags(DagDev d) {
   const int W = 2 * ((N + 127) / 128), nch = (N + 63) / 64, ng = (N + 15) / 16;
   const uint64_t* Mg = d.M + d.row_off[g];
   uint8_t* out = d.bflag + d.bflag_off[g];
+  uint64_t* Mw = d.M + d.row_off[g];
   for (int it = threadIdx.x; it < ng * nch; it += blockDim.x) {
     const int rg = it / nch, c = it % nch;
     uint64_t o = 0, a = ~0ull;
     for (int r = rg * 16; r < min(N, rg * 16 + 16); ++r) {
-      const uint64_t w = Mg[(int64_t)r * W + c];
+      const uint64_t w = mask_perm(Mg[(int64_t)r * W + c]);  // natural -> stored layout
+      Mw[(int64_t)r * W + c] = w;
       o |= w;
       a &= w;
     }
@@ -579,11 +581,11 @@ __global__ void __launch_bounds__(128) k_bflags(DagDev d) {
   }
 }
 
-__global__ void k_copy_words(const int64_t* total, const uint64_t* from, uint64_t* to) {
+__global__ void k_copy_words(const int64_t* total, const uint64_t* from, uint64_t* to, bool unperm) {
   const int64_t n = *total;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
-    to[i] = from[i];
+    to[i] = unperm ? mask_unperm(from[i]) : from[i];
 }
 
 predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
@@ -669,11 +671,11 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
 }
 
 predtop_status dag_copy_bits(const predtop_dag_s* dag, const uint64_t* from, uint64_t* to,
-                             cudaStream_t st) {
+                             cudaStream_t st, bool unperm) {
   const int G = dag->desc.num_graphs;
 {
     ProfScope _p(PK_COPY, st);
-    k_copy_words<<<592, 256, 0, st>>>(dag->d.row_off + G, from, to);
+    k_copy_words<<<592, 256, 0, st>>>(dag->d.row_off + G, from, to, unperm);
     PT_LAUNCH_CHECK();
   }
   return PREDTOP_OK;

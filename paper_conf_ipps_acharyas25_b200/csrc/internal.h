@@ -37,14 +37,47 @@ struct DagDev {
   int32_t* indeg;      // [N_tot]
   // bitsets and tiles
   uint64_t* R;         // [sum N_g W_g]
-  uint64_t* M;         // [sum N_g W_g]
+  uint64_t* M;         // [sum N_g W_g]  STORED layout: mask_perm of each 64-key word
   int32_t* tile_cnt;   // [sum T_g^2]
   uint8_t* tile_cls;   // [sum T_g^2]
   int2* work;          // [qtile bound] (graph, q-tile) attention work items
   int64_t* bflag_off;  // [G+1] prefix of ceil(N/16) * ceil(N/64)
-  uint8_t* bflag;      // per (16-row group, 64-key chunk): bits 0-3 block has an allowed
-                       // pair, bits 4-7 block fully allowed (permuted 16-key blocks, attention.cu)
+  uint8_t* bflag;      // per (16-row group, 64-key chunk): bits 0-3 block (keys 16j..16j+15)
+                       // has an allowed pair, bits 4-7 block fully allowed (attention.cu)
 };
+
+// Stored layout of the attention mask words.  Key k (0..63) of a 64-key chunk
+// sits at bit mask_pos(k) = 16*((k>>1)&3) + 2*(k>>3) + (k&1): in the m16n8
+// accumulator fragment of the QK^T MMA, thread tq (= lane%4) holds for n-tile
+// nt (8 keys) the keys 8nt + 2tq + {0,1}, so its 16 keys of the chunk are the
+// contiguous bits [16tq, 16tq+16), ordered (nt, u), and 16-key block j is
+// 0x000F000F000F000F << 4j.  k_bflags converts the natural-order words the
+// mask kernels write; predtop_debug_mask converts back.
+__host__ __device__ constexpr int mask_pos(int k) { return 16 * ((k >> 1) & 3) + 2 * (k >> 3) + (k & 1); }
+__device__ __forceinline__ uint64_t mask_perm(uint64_t w) {  // natural -> stored
+  uint64_t out = 0;
+#pragma unroll
+  for (int tq = 0; tq < 4; ++tq) {  // bits (2tq, 2tq+1) of every byte -> 16-bit field tq
+    uint64_t x = (w >> (2 * tq)) & 0x0303030303030303ull;
+    x = (x | (x >> 6)) & 0x000F000F000F000Full;
+    x = (x | (x >> 12)) & 0x000000FF000000FFull;
+    x = (x | (x >> 24)) & 0xFFFFull;
+    out |= x << (16 * tq);
+  }
+  return out;
+}
+__device__ __forceinline__ uint64_t mask_unperm(uint64_t w) {  // stored -> natural
+  uint64_t out = 0;
+#pragma unroll
+  for (int tq = 0; tq < 4; ++tq) {
+    uint64_t x = (w >> (16 * tq)) & 0xFFFFull;
+    x = (x | (x << 24)) & 0x000000FF000000FFull;
+    x = (x | (x << 12)) & 0x000F000F000F000Full;
+    x = (x | (x << 6)) & 0x0303030303030303ull;
+    out |= x << (2 * tq);
+  }
+  return out;
+}
 
 }  // namespace predtop
 
@@ -100,7 +133,7 @@ namespace predtop {
 // ---- dag.cu
 predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st);
 predtop_status dag_copy_bits(const predtop_dag_s* dag, const uint64_t* from, uint64_t* to,
-                             cudaStream_t st);
+                             cudaStream_t st, bool unperm = false);
 
 // ---- tma.cu
 bool encode_tma_2d(CUtensorMap* map, const void* base, int elem_bytes, uint64_t inner,
