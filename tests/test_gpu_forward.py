@@ -74,6 +74,24 @@ def test_latency_parity_tcgen05_attention(pt, oracle_mod, name, batch_fn, monkey
     assert err.max() <= TOL
 
 
+@pytest.mark.parametrize("name, n", [("paper", 1700), ("moe", 800)])
+def test_latency_parity_streaming_attention(pt, oracle_mod, name, n):
+    """Graphs whose K/V do not fit shared memory (d_h = 16: N > 1536; d_h =
+    32: N > 768) take the two-buffer TMA streaming path of the attention
+    kernel; plus a small graph in the same batch."""
+    rng = synth.CounterRng(7, n)
+    s, d = synth.random_dag(n, 2.5 / n, rng)
+    s2, d2 = synth.random_dag(90, 0.05, rng)
+    batch = synth.pack_graphs([(n, s, d, synth._rand_feats(n, rng)), (90, s2, d2, synth._rand_feats(90, rng))])
+    cfg, blob, model = _model(pt, name)
+    y, _ = _gpu_latency(pt, model, batch)
+    want = oracle_mod.forward_batch(cfg, blob, batch)
+    err = _rel(y, want)
+    print(f"{name} N={n}: max rel err {err.max():.3e}")
+    assert np.isfinite(y).all()
+    assert err.max() <= TOL
+
+
 def test_mean_pool_and_relabelled(pt, oracle_mod):
     cfg, blob, model = _model(pt, "gpt", pool=1)
     b = synth.stage_batch("gpt", 4, first_graph=300)
