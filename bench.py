@@ -423,7 +423,18 @@ def main():
                     "peak_basis": f"MUFU ex2 {MUFU_EX2_PER_CLK_SM}/clk/SM x {NUM_SMS} SMs x {clk_mhz:.0f} MHz (median under load)",
                     "tensor_equiv_tflops": tflops,
                     "tensor_frac": tflops / peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])}
-        roof.update({"kernel": dom, "traffic": None, "peak_source": peak_src,
+        traffic = None
+        try:  # DRAM bytes per launch of the dominant kernel from a committed ncu capture
+            with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+                tr = json.load(f).get(dom)
+            if tr:
+                traffic = tr["bytes"]
+                roof["traffic_source"] = tr["source"]
+                if dom == "attention":  # algorithmic bytes: q,k,v in (3d fp16) + att out (d fp16) per node
+                    roof["traffic_algorithmic"] = float(Ntot) * 4 * d * 2
+        except (OSError, ValueError, KeyError):
+            traffic = None
+        roof.update({"kernel": dom, "traffic": traffic, "peak_source": peak_src,
                      "kernel_ms": per_launch_ms, "share_of_step": prof[dom]["share"]})
 
     cpu = None
