@@ -385,6 +385,20 @@ __device__ __forceinline__ size_t small_int_bytes(const SmallCfg& sc) {
   return align_up((size_t)4 * (4 * (size_t)sc.sn + 2 + sc.se + 24), 16);
 }
 
+#ifdef PREDTOP_TRACE
+// clock64 at the phase boundaries of k_dag_small, summed over graphs 0..63
+__device__ long long g_dag_trace[8];
+__device__ int g_dag_levels;
+#define DTR(k)                                                      \
+  do {                                                              \
+    if (lane == 0 && g < 64) atomicAdd((unsigned long long*)&g_dag_trace[k], (unsigned long long)(clock64() - dt0)); \
+  } while (0)
+#else
+#define DTR(k) \
+  do {         \
+  } while (0)
+#endif
+
 __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc) {
   extern __shared__ __align__(16) unsigned char sm_small[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -395,6 +409,9 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
   const int64_t e0 = d.edge_ptr[g];
   const int E = (int)(d.edge_ptr[g + 1] - e0);
   if (!is_small(N, E, sc)) return;
+#ifdef PREDTOP_TRACE
+  const long long dt0 = clock64();
+#endif
   unsigned char* slot = sm_small + (size_t)warp * sc.slot;
   int* indeg = reinterpret_cast<int*>(slot);
   int* soff = indeg + sc.sn;        // N+1
@@ -449,6 +466,7 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
     __syncwarp();
     for (int e = lane; e < E; e += 32) succ[atomicAdd(&lptr[src[e]], 1)] = dst[e];
     __syncwarp();
+    DTR(0);
     // Kahn, level synchronous (P:137 depth = 1 + max predecessor depth)
     int tail = 0;
     for (int base = 0; base < N; base += 32) {
@@ -461,28 +479,47 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
       }
       tail += __popc(bal);
     }
-    if (lane == 0) { *ctr = tail; lptr[0] = 0; }
+    if (lane == 0) lptr[0] = 0;
     __syncwarp();
+    // frontier topo[lb, le); the warp-uniform tail needs no atomics: the
+    // nodes a level releases are appended by ballot + prefix popcount
+    const uint32_t lt = (1u << lane) - 1u;
     int lb = 0, le = tail;
     while (lb < le) {
-      for (int i = lb + lane; i < le; i += 32) {
-        const int v = topo[i];
-        for (int k = soff[v]; k < soff[v + 1]; ++k) {
-          const int w = succ[k];
-          if (atomicSub(&indeg[w], 1) == 1) {
-            topo[atomicAdd(ctr, 1)] = w;
+      for (int i0 = lb; i0 < le; i0 += 32) {
+        int k = 0, kend = 0;
+        if (i0 + lane < le) {
+          const int v = topo[i0 + lane];
+          k = soff[v];
+          kend = soff[v + 1];
+        }
+        while (__any_sync(0xffffffffu, k < kend)) {
+          int w = 0;
+          bool ready = false;
+          if (k < kend) {
+            w = succ[k++];
+            ready = atomicSub(&indeg[w], 1) == 1;
+          }
+          const uint32_t bal = __ballot_sync(0xffffffffu, ready);
+          if (ready) {
+            topo[tail + __popc(bal & lt)] = w;
             depth[w] = level + 1;
           }
+          tail += __popc(bal);
         }
       }
       __syncwarp();
       lb = le;
-      le = *reinterpret_cast<volatile int*>(ctr);
+      le = tail;
       ++level;
       if (lane == 0) lptr[level] = lb;
-      __syncwarp();
     }
+    __syncwarp();
     if (le != N) status = PREDTOP_ERR_CYCLE;
+    DTR(1);
+#ifdef PREDTOP_TRACE
+    if (lane == 0 && g < 64) atomicAdd(&g_dag_levels, level);
+#endif
   }
   if (lane == 0) d.num_levels[g] = level;
   if (status != PREDTOP_OK) {
@@ -513,28 +550,44 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
     }
     __syncwarp();
   }
-  for (int i = lane; i < N * W; i += 32) Rg[i] = R[i];
-  // mask M = R | R^T | I (32x32 ballot transposes) and per-tile counts
+  DTR(2);
+  // mask M = R | R^T | I per 64-bit word (two 32x32 bit transposes in
+  // flight), written in the stored layout (mask_perm); R written out in the
+  // same pass; per-tile popcounts
   const uint32_t* R32 = reinterpret_cast<const uint32_t*>(R);
   const int W32 = 2 * W, NB = (N + 31) / 32;
+  uint64_t* Mw = d.M + d.row_off[g];
   for (int ur = 0; ur < NB; ++ur) {
     const int U0 = ur * 32, u = U0 + lane;
-    for (int vr = 0; vr < W32; ++vr) {
-      const int V0 = vr * 32, vrow = V0 + lane;
-      const uint32_t direct = u < N ? R32[u * W32 + vr] : 0u;
-      const uint32_t x = vrow < N ? R32[vrow * W32 + ur] : 0u;
-      const uint32_t t = transpose32(x, lane);
-      uint32_t m = direct | t;
-      if (U0 == V0 && u < N) m |= 1u << lane;
-      if (u < N) M32[(int64_t)u * W32 + vr] = m;
-      else m = 0;
-      int c = __popc(m);
+    int ctile[4] = {0, 0, 0, 0};  // this lane's popcounts per 128-key tile (W <= 8)
+    for (int vw = 0; vw < W; ++vw) {
+      const int V0 = vw * 64;
+      const uint32_t dlo = u < N ? R32[u * W32 + 2 * vw] : 0u;
+      const uint32_t dhi = u < N ? R32[u * W32 + 2 * vw + 1] : 0u;
+      const uint32_t xlo = V0 + lane < N ? R32[(V0 + lane) * W32 + ur] : 0u;
+      const uint32_t xhi = V0 + 32 + lane < N ? R32[(V0 + 32 + lane) * W32 + ur] : 0u;
+      const uint32_t tlo = transpose32(xlo, lane), thi = transpose32(xhi, lane);
+      if (u < N) Rg[(int64_t)u * W + vw] = ((uint64_t)dhi << 32) | dlo;
+      uint32_t mlo = dlo | tlo, mhi = dhi | thi;
+      if (U0 == V0) mlo |= 1u << lane;
+      if (U0 == V0 + 32) mhi |= 1u << lane;
+      if (u >= N) mlo = mhi = 0u;
+      if (u < N) Mw[(int64_t)u * W + vw] = mask_perm(((uint64_t)mhi << 32) | mlo);
+      const int c = __popc(mlo) + __popc(mhi);
+#pragma unroll
+      for (int tt = 0; tt < 4; ++tt)
+        if (tt == vw / 2) ctile[tt] += c;
+    }
+#pragma unroll
+    for (int tt = 0; tt < 4; ++tt) {
+      int c = ctile[tt];
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
-      if (lane == 0 && V0 < N) tcnt[(U0 / 128) * T + V0 / 128] += c;
+      if (lane == 0 && tt < T) tcnt[(U0 / 128) * T + tt] += c;
     }
   }
   __syncwarp();
+  DTR(3);
   long long pairs = 0;
   for (int t = lane; t < T * T; t += 32) {
     const int qt = t / T, kt = t % T;
@@ -547,16 +600,20 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
   for (int o = 16; o > 0; o >>= 1) pairs += __shfl_xor_sync(0xffffffffu, pairs, o);
   if (lane == 0) d.pairs[g] = pairs;
   for (int qt = lane; qt < T; qt += 32) d.work[d.qtile_off[g] + qt] = make_int2(g, qt);
+  DTR(4);
 }
 
 // Block flags for the attention kernel: for every 16-row group rg and 64-key
 // chunk c, bit j (j < 4) = some row of the group has an allowed key in the
 // permuted 16-key block j (mask bits 0x000F000F000F000F << 4j, attention.cu),
 // bit 4+j = every row of the group allows every key of block j.
-__global__ void __launch_bounds__(128) k_bflags(DagDev d) {
+__global__ void __launch_bounds__(128) k_bflags(DagDev d, SmallCfg sc) {
   const int g = blockIdx.x;
   if (d.status[g] == PREDTOP_ERR_TOO_LARGE || d.status[g] == PREDTOP_ERR_INVALID_ARG) return;
   const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+  // k_dag_small writes M in the stored layout already; k_mask (large graphs)
+  // in natural order, converted here
+  const bool conv = !is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc);
   const int W = 2 * ((N + 127) / 128), nch = (N + 63) / 64, ng = (N + 15) / 16;
   const uint64_t* Mg = d.M + d.row_off[g];
   uint8_t* out = d.bflag + d.bflag_off[g];
@@ -565,8 +622,11 @@ __global__ void __launch_bounds__(128) k_bflags(DagDev d) {
     const int rg = it / nch, c = it % nch;
     uint64_t o = 0, a = ~0ull;
     for (int r = rg * 16; r < min(N, rg * 16 + 16); ++r) {
-      const uint64_t w = mask_perm(Mg[(int64_t)r * W + c]);  // natural -> stored layout
-      Mw[(int64_t)r * W + c] = w;
+      uint64_t w = Mg[(int64_t)r * W + c];
+      if (conv) {
+        w = mask_perm(w);  // natural -> stored layout
+        Mw[(int64_t)r * W + c] = w;
+      }
       o |= w;
       a &= w;
     }
@@ -664,7 +724,7 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
   }
   {
     ProfScope _p(PK_DAG_FLAGS, st);
-    k_bflags<<<G, 128, 0, st>>>(d);
+    k_bflags<<<G, 128, 0, st>>>(d, sc);
     PT_LAUNCH_CHECK();
   }
   return PREDTOP_OK;
@@ -682,3 +742,10 @@ predtop_status dag_copy_bits(const predtop_dag_s* dag, const uint64_t* from, uin
 }
 
 }  // namespace predtop
+
+#ifdef PREDTOP_TRACE
+extern "C" PREDTOP_API int predtop_debug_dag_trace(long long* out) {
+  if (cudaMemcpyFromSymbol(out, predtop::g_dag_trace, sizeof(predtop::g_dag_trace)) != cudaSuccess) return -7;
+  return cudaMemcpyFromSymbol(out + 8, predtop::g_dag_levels, sizeof(int)) == cudaSuccess ? 0 : -7;
+}
+#endif
