@@ -188,6 +188,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-json", default=None)
     ap.add_argument("--eager", action="store_true", help="no CUDA-graph capture of the step")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: host-side all-gather (eager only); lets N ranks share one GPU to test the "
+                         "multi-rank flow on a 1-GPU box")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -202,10 +205,17 @@ def main():
     import torch.distributed as dist
     from paper_conf_ipps_acharyas25_b200 import build, predtop as pt, synth
 
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    gloo = args.dist_backend == "gloo"
+    if gloo:
+        args.eager = True  # a host-side collective cannot sit inside a CUDA graph
+    dev_index = local % torch.cuda.device_count() if gloo else local
+    torch.cuda.set_device(dev_index)
+    dev = torch.device("cuda", dev_index)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if gloo:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     if rank == 0:
         build.build_library()
     if world > 1:
@@ -233,7 +243,12 @@ def main():
         model.forward(dag, ws, lat)         # predtop_stage_forward
         T, _, _ = plans.latency(lat, no_sync=True)   # predtop_plan_latency
         if world > 1:
-            dist.all_gather_into_tensor(T_all, T)
+            if gloo:
+                parts = [torch.empty(P, dtype=torch.float64) for _ in range(world)]
+                dist.all_gather(parts, T.cpu())
+                T_all.copy_(torch.cat(parts))
+            else:
+                dist.all_gather_into_tensor(T_all, T)
             plans.argmin(T_all)             # global argmin by (T, global plan id)
         else:
             plans.argmin(T)
@@ -262,7 +277,7 @@ def main():
 
     def max_over_ranks(x):
         if world > 1:
-            t = torch.tensor([x], dtype=torch.float64, device=dev)
+            t = torch.tensor([x], dtype=torch.float64, device="cpu" if gloo else dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             return float(t.item())
         return x
@@ -300,7 +315,7 @@ def main():
     torch.cuda.synchronize()
 
     launches0 = L.predtop_launch_count()
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev_index) as clk:
         ms = timed(run, args.steps)
     launches = L.predtop_launch_count() - launches0
     if graph is not None:
