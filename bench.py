@@ -135,11 +135,12 @@ def run_reference(args, rank):
     from paper_conf_ipps_acharyas25_b200 import synth
     import oracle
     oracle.build()
-    cfg = synth.MODEL_CONFIGS[args.config]
+    gcfg = "gpt" if args.config == "sweep" else args.config  # sweep stages are GPT-style pool graphs
+    cfg = synth.MODEL_CONFIGS[gcfg]
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
     cores = host_cores()
     per_step = cores  # one graph per core per step
-    batch = synth.stage_batch(args.config, per_step * (args.warmup + args.steps) if args.steps * per_step <= 4096 else 4096)
+    batch = synth.tiny_batch() if gcfg == "tiny" else synth.stage_batch(gcfg, per_step * (args.warmup + args.steps) if args.steps * per_step <= 4096 else 4096)
     plans_B = 16
     done, t_total = 0, 0.0
     for s in range(args.warmup + args.steps):
@@ -165,69 +166,249 @@ def run_reference(args, rank):
     print(json.dumps(line), flush=True)
 
 
+CONFIG_TEXT = {
+    "tiny": "4 hand-made DAGs of 8-16 ops (chain, diamond, fan-out, chain with skips), 1 layer d=32 H=2 d_ff=128",
+    "gpt": "stage DAGs of 270-330 ops (fwd+bwd GPT-3 1.3B stage template), 4 layers d=128 H=8 d_ff=512",
+    "moe": "stage DAGs of 1350-1650 ops (fwd+bwd GShard-MoE 2.6B stage template, 16-expert fan-out), "
+           "4 layers d=256 H=8 d_ff=1024",
+    "16k": "stage DAGs of exactly 16384 ops (GPT-style template), 4 layers d=128 H=8 d_ff=512",
+}
+
+
+def stages_per_plan(G: int) -> int:
+    return max(1, min(4, G))
+
+
 def workload_config(args):
-    return {"workload": f"{args.config}: {args.graphs} stage DAGs/GPU x 270-330 ops (fwd+bwd GPT-3 stage "
-                        f"template), DAG-Transformer 4 layers d=128 H=8 d_ff=512, sum pool + MLP head; "
-                        f"{args.graphs // 4} plans x 4 stages x B=16 (Eqn 4)",
-            "graphs_per_gpu": args.graphs, "plans_per_gpu": args.graphs // 4, "stages_per_plan": 4,
-            "microbatches": 16, "layers": 4, "d_model": 128, "heads": 8, "d_ff": 512,
-            "parallelism": f"graph-sharded x{args.gpus} (owned plans), NCCL all-gather of plan latencies",
-            "l2": "flushed before every timed step (256 MiB memset, untimed)",
+    cfg_name = "gpt" if args.config == "sweep" else args.config
+    from paper_conf_ipps_acharyas25_b200 import synth
+    c = synth.MODEL_CONFIGS[cfg_name]
+    base = {"layers": c["num_layers"], "d_model": c["d_model"], "heads": c["num_heads"], "d_ff": c["d_ff"],
             "precision": "f16 MMA operands, f32 accumulate/softmax/LN/residual, f32 latency, f64 Eqn 4"}
+    if args.config == "sweep":
+        return dict({"workload": f"sweep: {args.plans} candidate plans (S~U{{2..8}} stages, B~U{{1,4,16,64}}), "
+                                 f"each owning its GPT-style stage graphs ({CONFIG_TEXT['gpt']}), scored in chunks "
+                                 f"of {args.chunk} graphs; Eqn 4 per plan; global argmin",
+                     "plans_total": args.plans, "chunk_graphs": args.chunk, "stage_pool": args.pool,
+                     "parallelism": f"plan-sharded x{args.gpus} (cost-balanced contiguous ranges), "
+                                    f"NCCL all-gather of plan latencies",
+                     "l2": "inputs and activations of one step (~500k graphs) far exceed the 126 MB L2"}, **base)
+    G, S = args.graphs, stages_per_plan(args.graphs)
+    return dict({"workload": f"{args.config}: {G} {CONFIG_TEXT[args.config]}, sum pool + MLP head; "
+                             f"{G // S} plans x {S} stages x B=16 (Eqn 4)",
+                 "graphs_per_gpu": G, "plans_per_gpu": G // S, "stages_per_plan": S, "microbatches": 16,
+                 "parallelism": f"graph-sharded x{args.gpus} (owned plans), NCCL all-gather of plan latencies",
+                 "l2": "flushed before every timed step (256 MiB memset, untimed)"}, **base)
 
 
 # ----------------------------------------------------------------- main leg
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=100)
-    ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="gpt")
-    ap.add_argument("--graphs", type=int, default=1024)
-    ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--profile-json", default=None)
-    ap.add_argument("--eager", action="store_true", help="no CUDA-graph capture of the step")
-    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
-                    help="gloo: host-side all-gather (eager only); lets N ranks share one GPU to test the "
-                         "multi-rank flow on a 1-GPU box")
-    args = ap.parse_args()
-    args.warmup = max(args.warmup, 3)
+DEFAULT_GRAPHS = {"tiny": 4, "gpt": 1024, "moe": 512, "16k": 1, "sweep": 0}
 
-    rank = int(os.environ.get("RANK", "0"))
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    if args.impl == "reference":
-        run_reference(args, rank)
-        return
 
-    import torch
-    import torch.distributed as dist
-    from paper_conf_ipps_acharyas25_b200 import build, predtop as pt, synth
+class Ctx:
+    """Per-rank run context: device, stream, process group, timing helpers."""
 
-    gloo = args.dist_backend == "gloo"
-    if gloo:
-        args.eager = True  # a host-side collective cannot sit inside a CUDA graph
-    dev_index = local % torch.cuda.device_count() if gloo else local
-    torch.cuda.set_device(dev_index)
-    dev = torch.device("cuda", dev_index)
-    if world > 1:
-        if gloo:
-            dist.init_process_group("gloo")
+    def __init__(self, args):
+        import torch
+        import torch.distributed as dist
+        self.torch, self.dist = torch, dist
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.world = int(os.environ.get("WORLD_SIZE", "1"))
+        local = int(os.environ.get("LOCAL_RANK", "0"))
+        self.gloo = args.dist_backend == "gloo"
+        if self.gloo:
+            args.eager = True  # a host-side collective cannot sit inside a CUDA graph
+        self.dev_index = local % torch.cuda.device_count() if self.gloo else local
+        torch.cuda.set_device(self.dev_index)
+        self.dev = torch.device("cuda", self.dev_index)
+        if self.world > 1:
+            if self.gloo:
+                dist.init_process_group("gloo")
+            else:
+                dist.init_process_group("nccl", device_id=self.dev)
+        from paper_conf_ipps_acharyas25_b200 import build
+        if self.rank == 0:
+            build.build_library()
+        if self.world > 1:
+            dist.barrier()
+        from paper_conf_ipps_acharyas25_b200 import predtop as pt
+        self.pt = pt
+        self.L = pt.lib()
+        self.stream = torch.cuda.current_stream()
+        self.flush = torch.empty(256 << 20, dtype=torch.uint8, device=self.dev)
+
+    def timed(self, fn, k, flush=True):
+        torch, dist = self.torch, self.dist
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(k)]
+        if self.world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for a, b in evs:
+            if flush:
+                self.flush.zero_()
+            a.record(self.stream)
+            fn()
+            b.record(self.stream)
+        torch.cuda.synchronize()
+        if self.world > 1:
+            dist.barrier()
+        return [a.elapsed_time(b) for a, b in evs]
+
+    def max_over_ranks(self, x):
+        if self.world > 1:
+            t = self.torch.tensor([x], dtype=self.torch.float64, device="cpu" if self.gloo else self.dev)
+            self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX)
+            return float(t.item())
+        return x
+
+    def sum_over_ranks(self, x):
+        if self.world > 1:
+            t = self.torch.tensor([x], dtype=self.torch.float64, device="cpu" if self.gloo else self.dev)
+            self.dist.all_reduce(t, op=self.dist.ReduceOp.SUM)
+            return float(t.item())
+        return x
+
+    def all_gather_T(self, T_all, T):
+        if self.gloo:
+            P = T.numel()
+            parts = [self.torch.empty(P, dtype=self.torch.float64) for _ in range(self.world)]
+            self.dist.all_gather(parts, T.cpu())
+            T_all.copy_(self.torch.cat(parts))
         else:
-            dist.init_process_group("nccl", device_id=dev)
-    if rank == 0:
-        build.build_library()
-    if world > 1:
-        dist.barrier()
-    L = pt.lib()
-    stream = torch.cuda.current_stream()
+            self.dist.all_gather_into_tensor(T_all, T)
 
-    cfg = synth.MODEL_CONFIGS[args.config]
+    def capture(self, fn):
+        """CUDA-graph capture of fn (library calls are capturable: NO_SYNC
+        build, stream-ordered kernels, NCCL all-gather); returns (replay, launches)."""
+        torch = self.torch
+        side = torch.cuda.Stream(device=self.dev)
+        side.wait_stream(self.stream)
+        with torch.cuda.stream(side):
+            fn()
+        self.stream.wait_stream(side)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        l0 = self.L.predtop_launch_count()
+        with torch.cuda.graph(g, stream=side):
+            fn()
+        n = self.L.predtop_launch_count() - l0
+        torch.cuda.synchronize()
+        self._graphs = getattr(self, "_graphs", []) + [g]
+        return g.replay, n
+
+    def profile(self, step, steps):
+        """Per-kernel CUDA-event times (predtop_profile_enable) over `steps` eager steps."""
+        import ctypes
+        L = self.L
+        L.predtop_profile_enable(1)
+        self.timed(step, steps)
+        L.predtop_profile_enable(0)
+        kinds = 32
+        kms = (ctypes.c_double * kinds)()
+        kcnt = (ctypes.c_int64 * kinds)()
+        nk = L.predtop_profile_read(kms, kcnt, kinds)
+        names = [L.predtop_profile_kind_name(i).decode() for i in range(nk)]
+        return {names[i]: {"ms_per_step": kms[i] / steps, "launches_per_step": kcnt[i] / steps}
+                for i in range(nk) if kcnt[i]}
+
+    def finish(self):
+        if self.world > 1:
+            self.dist.barrier()
+            self.dist.destroy_process_group()
+
+
+def algorithmic_work(cfg, node_total, edge_total, words, pairs):
+    """Algorithmic work per step of each kernel kind: flops for
+    tensor-bound kinds, exps for the attention (MUFU-bound), bytes for HBM-bound."""
+    d, dff, H = cfg["d_model"], cfg["d_ff"], cfg["num_heads"]
+    N, E, A = float(node_total), float(edge_total), float(pairs)
+    return {
+        "gemm_qkv": ("tensor", 2.0 * N * d * 3 * d),
+        "gemm_oproj_ln": ("tensor", 2.0 * N * d * d),
+        "gemm_ffn1": ("tensor", 2.0 * N * d * dff),
+        "gemm_ffn2_ln": ("tensor", 2.0 * N * dff * d),
+        "layer_tail": ("tensor", 2.0 * N * (d * d + 2 * d * dff)),
+        "attention": ("alu", float(H) * A),  # exps per layer (MUFU-bound, see DESIGN.md)
+        "dag_closure": ("hbm", 8.0 * words + 8.0 * E),
+        "dag_mask": ("hbm", 3 * 8.0 * words),
+        "readout": ("hbm", 4.0 * N * d),
+        "embed": ("hbm", N * (20.0 + 4 + 6 * d)),
+    }
+
+
+def roofline(prof, work, cfg, pairs, node_total, clk, step_ms):
+    """The dominant kernel's achieved rate against its peak.  `work` is per STEP;
+    per launch = per step / launches per step; time per launch from the
+    CUDA-event profile pass."""
+    for k in prof:
+        prof[k]["share"] = prof[k]["ms_per_step"] / step_ms
+    peaks, peak_src = load_peaks()
+    dom = max(prof, key=lambda k: prof[k]["ms_per_step"]) if prof else None
+    if dom not in work:
+        return None
+    bound, per_step = work[dom]
+    n_l = prof[dom]["launches_per_step"]
+    per_launch_ms = prof[dom]["ms_per_step"] / n_l
+    layer_kinds = ("gemm_qkv", "gemm_oproj_ln", "gemm_ffn1", "gemm_ffn2_ln", "layer_tail", "attention")
+    # work[] holds per-layer figures for the per-layer kernels, per-step figures otherwise
+    units = (per_step * cfg["num_layers"] if dom in layer_kinds else per_step) / n_l
+    sec = per_launch_ms / 1e3
+    d = cfg["d_model"]
+    if bound == "tensor":
+        ach = units / sec / 1e12
+        peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+        roof = {"bound": "tensor", "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
+                "peak_basis": "measured cuBLAS bf16 sustained (f16 MMA has the same nominal rate)"}
+    elif bound == "hbm":
+        ach = units / sec / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": ach / peaks["hbm_gbs"]}
+    else:
+        clk_mhz = (clk.summary()["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0))
+        peak = MUFU_EX2_PER_CLK_SM * NUM_SMS * clk_mhz * 1e6 / 1e9
+        ach = units / sec / 1e9
+        A_launch = float(pairs) * cfg["num_layers"] / n_l
+        tflops = 4.0 * d * A_launch / sec / 1e12
+        roof = {"bound": "alu", "achieved": ach, "peak": peak, "unit": "Gexp/s", "frac": ach / peak,
+                "peak_basis": f"MUFU ex2 {MUFU_EX2_PER_CLK_SM}/clk/SM x {NUM_SMS} SMs x {clk_mhz:.0f} MHz "
+                              f"(median under load)",
+                "tensor_equiv_tflops": tflops,
+                "tensor_frac": tflops / peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])}
+    traffic = None
+    try:  # DRAM bytes per launch of the dominant kernel from a committed ncu capture
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            tr = json.load(f).get(dom)
+        if tr and tr.get("config", "gpt") == cfg.get("_name", "gpt"):
+            traffic = tr["bytes"]
+            roof["traffic_source"] = tr["source"]
+            if dom == "attention":  # algorithmic bytes: q,k,v in (3d fp16) + att out (d fp16) per node
+                roof["traffic_algorithmic"] = float(node_total) * 4 * d * 2 * cfg["num_layers"] / n_l
+    except (OSError, ValueError, KeyError):
+        traffic = None
+    roof.update({"kernel": dom, "traffic": traffic, "peak_source": peak_src,
+                 "kernel_ms": per_launch_ms, "share_of_step": prof[dom]["share"]})
+    return roof
+
+
+def dag_pairs(pt, dag, sizes):
+    T_ = (np.asarray(sizes) + 127) // 128
+    _, pairs = dag.tiles(int((T_ * T_).sum()))
+    return int(pairs.sum().item())
+
+
+def run_batch(args, ctx):
+    """configs tiny/gpt/moe/16k: one step = build + forward of the rank's G graphs,
+    Eqn 4 over its owned plans, all-gather, global argmin."""
+    import torch
+    from paper_conf_ipps_acharyas25_b200 import synth
+    pt, L, dev, world, rank = ctx.pt, ctx.L, ctx.dev, ctx.world, ctx.rank
+
+    cfg = dict(synth.MODEL_CONFIGS[args.config], _name=args.config)
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
     G = args.graphs
-    host = synth.stage_batch(args.config, G, first_graph=rank * G)
-    ps = synth.owned_plans(G, 4, 16)
+    host = synth.tiny_batch() if args.config == "tiny" else synth.stage_batch(args.config, G, first_graph=rank * G)
+    S = stages_per_plan(G)
+    ps = synth.owned_plans(G, S, 16)
     model = pt.Model(cfg, blob, device=dev)
     db = pt.DeviceBatch.from_host(host, device=dev)
     dag = pt.Dag(db, no_sync=True)
@@ -236,19 +417,13 @@ def main():
     plans = pt.Plans(ps.plan_ptr, ps.plan_stage, ps.microbatches, device=dev)
     P = plans.num_plans
     T_all = torch.empty(world * P, dtype=torch.float64, device=dev)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def step():
         dag.rebuild()                       # predtop_build_dag (NO_SYNC)
         model.forward(dag, ws, lat)         # predtop_stage_forward
         T, _, _ = plans.latency(lat, no_sync=True)   # predtop_plan_latency
         if world > 1:
-            if gloo:
-                parts = [torch.empty(P, dtype=torch.float64) for _ in range(world)]
-                dist.all_gather(parts, T.cpu())
-                T_all.copy_(torch.cat(parts))
-            else:
-                dist.all_gather_into_tensor(T_all, T)
+            ctx.all_gather_T(T_all, T)
             plans.argmin(T_all)             # global argmin by (T, global plan id)
         else:
             plans.argmin(T)
@@ -260,28 +435,6 @@ def main():
     assert st == pt.OK, (st, bad)
     assert torch.isfinite(lat).all()
 
-    def timed(fn, k):
-        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(k)]
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-        for a, b in evs:
-            flush.zero_()
-            a.record(stream)
-            fn()
-            b.record(stream)
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        return [a.elapsed_time(b) for a, b in evs]
-
-    def max_over_ranks(x):
-        if world > 1:
-            t = torch.tensor([x], dtype=torch.float64, device="cpu" if gloo else dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            return float(t.item())
-        return x
-
     # eager diagnostics: host enqueue time of one step and eager device time
     torch.cuda.synchronize()
     t0 = time.perf_counter()
@@ -289,41 +442,25 @@ def main():
         step()
     host_enqueue_ms = (time.perf_counter() - t0) / 5 * 1e3
     torch.cuda.synchronize()
-    eager_ms = sum(timed(step, 5)) / 5
+    eager_ms = sum(ctx.timed(step, 5)) / 5
 
-    # The step is captured once as a CUDA graph (library calls are capturable:
-    # NO_SYNC build, stream-ordered kernels, NCCL all-gather) and replayed.
-    graph = None
     launches_per_step = None
     if not args.eager:
-        side = torch.cuda.Stream(device=dev)
-        side.wait_stream(stream)
-        with torch.cuda.stream(side):
-            step()
-        stream.wait_stream(side)
-        torch.cuda.synchronize()
-        graph = torch.cuda.CUDAGraph()
-        l0 = L.predtop_launch_count()
-        with torch.cuda.graph(graph, stream=side):
-            step()
-        launches_per_step = L.predtop_launch_count() - l0
-        torch.cuda.synchronize()
-        run = graph.replay
+        run, launches_per_step = ctx.capture(step)
     else:
         run = step
     run()
     torch.cuda.synchronize()
 
     launches0 = L.predtop_launch_count()
-    with ClockSampler(dev_index) as clk:
-        ms = timed(run, args.steps)
+    with ClockSampler(ctx.dev_index) as clk:
+        ms = ctx.timed(run, args.steps)
     launches = L.predtop_launch_count() - launches0
-    if graph is not None:
+    if launches_per_step is not None:
         launches = launches_per_step * args.steps
-    total_ms = max_over_ranks(sum(ms))
+    total_ms = ctx.max_over_ranks(sum(ms))
     value = world * G * args.steps / (total_ms / 1e3)
     plans_per_s = world * P * args.steps / (total_ms / 1e3)
-    # the replayed step computed the same results as the eager one
     assert torch.isfinite(lat).all()
 
     # ---- e2e through the C-ABI with pinned host buffers
@@ -337,10 +474,10 @@ def main():
         "plan_stage": torch.from_numpy(ps.plan_stage).pin_memory(),
         "mb": torch.from_numpy(ps.microbatches).pin_memory(),
     }
-    T_host = torch.empty(world * P, dtype=torch.float64).pin_memory()
+    T_host = torch.empty(max(world * P, 1), dtype=torch.float64).pin_memory()
     best_host = torch.empty(1, dtype=torch.int64).pin_memory()
     h2d = sum(t.numel() * t.element_size() for t in pin.values())
-    d2h = T_host.numel() * 8 + 8
+    d2h = world * P * 8 + 8
 
     def e2e_step():
         db.node_ptr.copy_(pin["node_ptr"], non_blocking=True)
@@ -352,108 +489,29 @@ def main():
         plans.plan_stage.copy_(pin["plan_stage"], non_blocking=True)
         plans.microbatches.copy_(pin["mb"], non_blocking=True)
         step()
-        T_host.copy_(T_all if world > 1 else plans.T[:P], non_blocking=True)
+        if P:
+            T_host[:world * P].copy_(T_all if world > 1 else plans.T[:P], non_blocking=True)
         best_host.copy_(plans.best, non_blocking=True)
 
-    e2e_run = e2e_step
-    if not args.eager:
-        side = torch.cuda.Stream(device=dev)
-        side.wait_stream(stream)
-        with torch.cuda.stream(side):
-            e2e_step()
-        stream.wait_stream(side)
-        torch.cuda.synchronize()
-        g2 = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(g2, stream=side):
-            e2e_step()
-        e2e_run = g2.replay
+    e2e_run = e2e_step if args.eager else ctx.capture(e2e_step)[0]
     for _ in range(2):
         e2e_run()
-    ms_e2e = timed(e2e_run, max(10, args.steps // 4))
-    tot_e2e = max_over_ranks(sum(ms_e2e))
+    ms_e2e = ctx.timed(e2e_run, max(10, args.steps // 4))
+    tot_e2e = ctx.max_over_ranks(sum(ms_e2e))
     e2e_value = world * G * len(ms_e2e) / (tot_e2e / 1e3)
-    # the host copy of the plan latencies matches the device result
     torch.cuda.synchronize()
-    assert torch.equal(T_host, (T_all if world > 1 else plans.T[:P]).cpu())
+    if P:  # the host copy of the plan latencies matches the device result
+        assert torch.equal(T_host[:world * P], (T_all if world > 1 else plans.T[:P]).cpu())
 
     # ---- per-kernel profile pass (separate from the headline timing)
-    L.predtop_profile_enable(1)
-    prof_steps = max(5, args.steps // 4)
-    ms_prof = timed(step, prof_steps)
-    L.predtop_profile_enable(0)
-    import ctypes
-    kinds = 32
-    kms = (ctypes.c_double * kinds)()
-    kcnt = (ctypes.c_int64 * kinds)()
-    nk = L.predtop_profile_read(kms, kcnt, kinds)
-    names = [L.predtop_profile_kind_name(i).decode() for i in range(nk)]
-    prof = {names[i]: {"ms_per_step": kms[i] / prof_steps, "launches_per_step": kcnt[i] / prof_steps}
-            for i in range(nk) if kcnt[i]}
-    step_ms_prof = total_ms / args.steps  # shares relative to the headline (graph) step time
-    for k in prof:
-        prof[k]["share"] = prof[k]["ms_per_step"] / step_ms_prof
-
-    # algorithmic work per launch of each kind
-    d, dff, H = cfg["d_model"], cfg["d_ff"], cfg["num_heads"]
-    Ntot = host.node_ptr[-1]
-    sizes = host.sizes
-    T_ = (sizes + 127) // 128
-    _, pairs = dag.tiles(int((T_ * T_).sum()))
-    A = int(pairs.sum().item())
-    E = int(host.edge_ptr[-1])
-    words = int(sum(n * 2 * ((n + 127) // 128) for n in sizes))
-    work = {
-        "gemm_qkv": ("tensor", 2.0 * Ntot * d * 3 * d),
-        "gemm_oproj_ln": ("tensor", 2.0 * Ntot * d * d),
-        "gemm_ffn1": ("tensor", 2.0 * Ntot * d * dff),
-        "gemm_ffn2_ln": ("tensor", 2.0 * Ntot * dff * d),
-        "layer_tail": ("tensor", 2.0 * Ntot * (d * d + 2 * d * dff)),
-        "attention": ("alu", float(H) * A),  # exps per launch (MUFU-bound)
-        "dag_closure": ("hbm", 8.0 * words + 8.0 * E),
-        "dag_mask": ("hbm", 3 * 8.0 * words),
-        "readout": ("hbm", 4.0 * Ntot * d),
-        "embed": ("hbm", Ntot * (20.0 + 4 + 6 * d)),
-    }
-    peaks, peak_src = load_peaks()
-    dom = max(prof, key=lambda k: prof[k]["ms_per_step"]) if prof else None
-    roof = None
-    if dom in work:
-        bound, units = work[dom]
-        per_launch_ms = prof[dom]["ms_per_step"] / prof[dom]["launches_per_step"]
-        sec = per_launch_ms / 1e3
-        if bound == "tensor":
-            ach = units / sec / 1e12
-            peak = peaks["bf16_tflops_sustained"] if "bf16_tflops_sustained" in peaks else peaks["bf16_tflops"]
-            roof = {"bound": "tensor", "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak}
-        elif bound == "hbm":
-            ach = units / sec / 1e9
-            roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                    "frac": ach / peaks["hbm_gbs"]}
-        else:
-            clk_mhz = (clk.summary()["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0))
-            peak = MUFU_EX2_PER_CLK_SM * NUM_SMS * clk_mhz * 1e6 / 1e9
-            ach = units / sec / 1e9
-            tflops = 4.0 * d * A / sec / 1e12
-            roof = {"bound": "alu", "achieved": ach, "peak": peak, "unit": "Gexp/s", "frac": ach / peak,
-                    "peak_basis": f"MUFU ex2 {MUFU_EX2_PER_CLK_SM}/clk/SM x {NUM_SMS} SMs x {clk_mhz:.0f} MHz (median under load)",
-                    "tensor_equiv_tflops": tflops,
-                    "tensor_frac": tflops / peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])}
-        traffic = None
-        try:  # DRAM bytes per launch of the dominant kernel from a committed ncu capture
-            with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-                tr = json.load(f).get(dom)
-            if tr:
-                traffic = tr["bytes"]
-                roof["traffic_source"] = tr["source"]
-                if dom == "attention":  # algorithmic bytes: q,k,v in (3d fp16) + att out (d fp16) per node
-                    roof["traffic_algorithmic"] = float(Ntot) * 4 * d * 2
-        except (OSError, ValueError, KeyError):
-            traffic = None
-        roof.update({"kernel": dom, "traffic": traffic, "peak_source": peak_src,
-                     "kernel_ms": per_launch_ms, "share_of_step": prof[dom]["share"]})
+    prof = ctx.profile(step, max(5, args.steps // 4))
+    words = int(sum(n * 2 * ((n + 127) // 128) for n in host.sizes))
+    A = dag_pairs(pt, dag, host.sizes)
+    work = algorithmic_work(cfg, host.node_ptr[-1], host.edge_ptr[-1], words, A)
+    roof = roofline(prof, work, cfg, A, host.node_ptr[-1], clk, total_ms / args.steps)
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config != "16k":
         v, cores, n, wall = oracle_rate(cfg, blob, host)
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": f"first {n} of {G} {args.config} stage graphs, fp64 C oracle, {cores} threads, {wall:.1f} s"}
@@ -471,13 +529,173 @@ def main():
                 "eager_ms_per_step": eager_ms, "host_enqueue_ms_per_step": host_enqueue_ms,
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
-        print(json.dumps(line), flush=True)
-        if args.profile_json:
-            with open(args.profile_json, "w") as f:
-                json.dump(line, f, indent=1)
-    if world > 1:
-        dist.barrier()
-        dist.destroy_process_group()
+        emit(line, args)
+
+
+def run_sweep(args, ctx, pool):
+    """configs[4]: an owned-mode plan sweep of args.plans plans, cost-balanced
+    over the ranks (strong scaling: the total is fixed).  One step = build +
+    forward of every stage graph of the rank's plans (chunks of args.chunk),
+    Eqn 4 over its plans, all-gather of T, global argmin."""
+    import torch
+    from paper_conf_ipps_acharyas25_b200 import synth, sweep
+    pt, L, dev, world, rank = ctx.pt, ctx.L, ctx.dev, ctx.world, ctx.rank
+
+    cfg = dict(synth.MODEL_CONFIGS["gpt"], _name="gpt")
+    blob = synth.pack_weights(cfg, synth.model_weights(cfg))
+    (p0, p1), pp, mb, s0, counts = sweep.shard_sweep(args.plans, world, rank)
+    model = pt.Model(cfg, blob, device=dev)
+    sh = sweep.SweepShard(pt, model, pool, pp, mb, s0, chunk=args.chunk, device=dev)
+    Pmax = max(counts)
+    T_pad = torch.full((Pmax,), float("inf"), dtype=torch.float64, device=dev)
+    T_all = torch.empty(world * Pmax, dtype=torch.float64, device=dev)
+    best = torch.empty(1, dtype=torch.int64, device=dev)
+    # global plan id of padded slot r*Pmax + i is (start of rank r) + i; padding is +inf, never chosen
+    # unless every T is inf; the argmin below maps the padded index back.
+    starts = np.concatenate([[0], np.cumsum(counts)])[:-1]
+
+    def step():
+        T = sh.score()
+        if world > 1:
+            T_pad[:sh.num_plans].copy_(T)
+            ctx.all_gather_T(T_all, T_pad)
+            pt.predtop_plan_argmin(T_all, best)
+        else:
+            pt.predtop_plan_argmin(T, best)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    st, bad = sh.status()
+    assert st == pt.OK, (st, bad)
+    assert torch.isfinite(sh.lat).all()
+
+    launches0 = L.predtop_launch_count()
+    with ClockSampler(ctx.dev_index) as clk:
+        ms = ctx.timed(step, args.steps, flush=False)
+    launches = L.predtop_launch_count() - launches0
+    total_ms = ctx.max_over_ranks(sum(ms))
+    graphs_total = ctx.sum_over_ranks(float(sh.num_stages))
+    value = graphs_total * args.steps / (total_ms / 1e3)
+    plans_per_s = args.plans * args.steps / (total_ms / 1e3)
+    b = int(best.item())
+    if world > 1:  # padded index -> global plan id
+        r, i = divmod(b, Pmax)
+        b = int(starts[r] + i)
+    else:
+        b += p0
+
+    # ---- e2e: every chunk's inputs copied from pinned host memory before its build
+    pins = {}
+    for key, db in sh.batches.items():
+        pins[key] = [(getattr(db, n), getattr(db, n).cpu().pin_memory())
+                     for n in ("node_ptr", "edge_ptr", "src", "dst", "feats")]
+    plan_pin = [(sh.plans.plan_ptr, sh.plans.plan_ptr.cpu().pin_memory()),
+                (sh.plans.plan_stage, sh.plans.plan_stage.cpu().pin_memory()),
+                (sh.plans.microbatches, sh.plans.microbatches.cpu().pin_memory())]
+    T_host = torch.empty(max(world * Pmax, 1), dtype=torch.float64).pin_memory()
+    h2d = sum(h.numel() * h.element_size() for _, _, k in sh.chunks for _, h in pins[k]) + \
+        sum(h.numel() * h.element_size() for _, h in plan_pin)
+    d2h = (world * Pmax if world > 1 else sh.num_plans) * 8 + 8
+
+    def e2e_step():
+        for dev_t, host_t in plan_pin:
+            dev_t.copy_(host_t, non_blocking=True)
+        for lo, hi, key in sh.chunks:
+            for dev_t, host_t in pins[key]:
+                dev_t.copy_(host_t, non_blocking=True)
+            sh.dags[key].rebuild()
+            sh.model.forward(sh.dags[key], sh.ws, sh.lat[lo:hi])
+        T, _, _ = sh.plans.latency(sh.lat, no_sync=True)
+        if world > 1:
+            T_pad[:sh.num_plans].copy_(T)
+            ctx.all_gather_T(T_all, T_pad)
+            pt.predtop_plan_argmin(T_all, best)
+            T_host.copy_(T_all, non_blocking=True)
+        else:
+            pt.predtop_plan_argmin(T, best)
+            T_host[:sh.num_plans].copy_(T, non_blocking=True)
+
+    e2e_step()
+    ms_e2e = ctx.timed(e2e_step, max(2, args.steps // 2), flush=False)
+    tot_e2e = ctx.max_over_ranks(sum(ms_e2e))
+    e2e_value = graphs_total * len(ms_e2e) / (tot_e2e / 1e3)
+
+    prof = ctx.profile(step, 2)
+    nodes = sum(sh.batches[k].total_nodes for _, _, k in sh.chunks)
+    edges = sum(sh.batches[k].total_edges for _, _, k in sh.chunks)
+    words, A = 0, 0
+    for key, dag in sh.dags.items():
+        sizes = np.diff(sh.batches[key].node_ptr.cpu().numpy())
+        uses = sum(1 for _, _, k in sh.chunks if k == key)
+        words += uses * int(sum(n * 2 * ((n + 127) // 128) for n in sizes))
+        A += uses * dag_pairs(pt, dag, sizes)
+    work = algorithmic_work(cfg, nodes, edges, words, A)
+    roof = roofline(prof, work, cfg, A, nodes, clk, total_ms / args.steps)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        host = synth.pack_graphs(list(pool[:1024]))
+        v, cores, n, wall = oracle_rate(cfg, blob, host)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"first {n} pool stage graphs, fp64 C oracle, {cores} threads, {wall:.1f} s"}
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f16", "data": "synthetic",
+                "config": workload_config(args),
+                "plans_per_s": plans_per_s, "graphs_per_step": graphs_total, "best_plan": b,
+                "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+                        "d2h_bytes_per_step": int(d2h)},
+                "gpu_launches": int(launches), "launch_mode": "eager",
+                "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
+        emit(line, args)
+
+
+def emit(line, args):
+    print(json.dumps(line), flush=True)
+    if args.profile_json:
+        with open(args.profile_json, "w") as f:
+            json.dump(line, f, indent=1)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="gpt", choices=["tiny", "gpt", "moe", "16k", "sweep"])
+    ap.add_argument("--graphs", type=int, default=None, help="stage graphs per GPU (default per config)")
+    ap.add_argument("--plans", type=int, default=100000, help="sweep: total candidate plans")
+    ap.add_argument("--chunk", type=int, default=4096, help="sweep: stage graphs per build+forward launch")
+    ap.add_argument("--pool", type=int, default=8192, help="sweep: distinct synthetic stage graphs")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile-json", default=None)
+    ap.add_argument("--eager", action="store_true", help="no CUDA-graph capture of the step")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: host-side all-gather (eager only); lets N ranks share one GPU to test the "
+                         "multi-rank flow on a 1-GPU box")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.graphs is None:
+        args.graphs = DEFAULT_GRAPHS[args.config]
+
+    rank = int(os.environ.get("RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+    pool = None
+    if args.config == "sweep":  # host generation before any CUDA context (forked pool)
+        from paper_conf_ipps_acharyas25_b200 import synth
+        pool = synth.stage_graphs_parallel("gpt", args.pool)
+    ctx = Ctx(args)
+    if args.config == "sweep":
+        run_sweep(args, ctx, pool)
+    else:
+        run_batch(args, ctx)
+    ctx.finish()
 
 
 if __name__ == "__main__":

@@ -641,6 +641,32 @@ def stage_batch(config: str, num_graphs: int, first_graph: int = 0,
     return pack_graphs(gs)
 
 
+def _stage_graphs_worker(args):
+    config, lo, hi, seed = args
+    b = stage_batch(config, hi - lo, first_graph=lo, seed=seed)
+    return [tuple(np.array(a) if isinstance(a, np.ndarray) else a for a in b.graph(g))
+            for g in range(b.num_graphs)]
+
+
+def stage_graphs_parallel(config: str, num_graphs: int, first_graph: int = 0,
+                          seed: Optional[int] = None, procs: Optional[int] = None) -> List[Tuple]:
+    """Graph tuples (N, src, dst, feats) of graphs [first_graph, first_graph +
+    num_graphs), generated by a process pool.  Identical to stage_batch (each
+    graph depends only on (seed, global id)); only faster for large pools."""
+    import multiprocessing as mproc
+    import os
+    procs = procs or max(1, min(32, len(os.sched_getaffinity(0))))
+    if procs == 1 or num_graphs < 64:
+        b = stage_batch(config, num_graphs, first_graph, seed)
+        return [b.graph(g) for g in range(b.num_graphs)]
+    step = (num_graphs + procs - 1) // procs
+    jobs = [(config, first_graph + s, first_graph + min(num_graphs, s + step), seed)
+            for s in range(0, num_graphs, step)]
+    with mproc.get_context("fork").Pool(len(jobs)) as pool:
+        parts = pool.map(_stage_graphs_worker, jobs)
+    return [g for p in parts for g in p]
+
+
 # --------------------------------------------------------------------------
 # Model configuration and weights (reading R14 in DESIGN.md)
 # --------------------------------------------------------------------------
