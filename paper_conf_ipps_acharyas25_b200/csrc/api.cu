@@ -417,6 +417,13 @@ static bool use_fused_tail(int d, int dff) {
   return !unfused && layer_tail_supported(d, dff);
 }
 
+// d = 128: the two-CTA-per-SM tail (layer2.cu); PREDTOP_TAIL_V1=1 selects the
+// one-CTA kernel of layer.cu instead (tests compare the two).
+static bool use_tail_v2(int d, int dff) {
+  const char* e = getenv("PREDTOP_TAIL_V1");
+  return !(e && e[0] == '1') && layer_tail2_supported(d, dff);
+}
+
 static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, size_t ws_bytes,
                                    int last_layer, float* latency_out, float* x_out,
                                    cudaStream_t st) {
@@ -453,7 +460,9 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     if ((s = attention_launch(dag, d, H, w.qkv, w.att, st)) != PREDTOP_OK) return s;
     if (use_fused_tail(d, f)) {
       ProfScope _p(PK_LAYER_TAIL, st);
-      if ((s = layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st)) != PREDTOP_OK) return s;
+      s = use_tail_v2(d, f) ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
+                            : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
+      if (s != PREDTOP_OK) return s;
       continue;
     }
     a = GemmArgs{};

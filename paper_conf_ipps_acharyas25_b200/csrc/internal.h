@@ -177,6 +177,9 @@ predtop_status argmin_launch(int64_t n, const double* T, int64_t* best, cudaStre
 
 // ---- layer.cu (fused O-proj + LN1 + FFN + LN2)
 bool layer_tail_supported(int d, int dff);
+bool layer_tail2_supported(int d, int dff);
+predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
+                                  __half* x16, int M, cudaStream_t st);
 predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
                                  __half* x16, int M, cudaStream_t st);
 

@@ -74,6 +74,24 @@ def test_latency_parity_tcgen05_attention(pt, oracle_mod, name, batch_fn, monkey
     assert err.max() <= TOL
 
 
+@pytest.mark.parametrize("name, batch_fn", [
+    ("gpt", lambda: synth.stage_batch("gpt", 24)),
+    ("gpt", lambda: synth.stage_batch("gpt", 5, seed=7)),
+])
+def test_latency_parity_tail_v1(pt, oracle_mod, name, batch_fn, monkeypatch):
+    """The one-CTA-per-SM fused layer tail (layer.cu, PREDTOP_TAIL_V1=1) that
+    the default two-CTA kernel (layer2.cu) replaced at d = 128."""
+    monkeypatch.setenv("PREDTOP_TAIL_V1", "1")
+    cfg, blob, model = _model(pt, name)
+    batch = batch_fn()
+    y, _ = _gpu_latency(pt, model, batch)
+    want = oracle_mod.forward_batch(cfg, blob, batch)
+    err = _rel(y, want)
+    print(f"{name} (tail v1): max rel err {err.max():.3e}")
+    assert np.isfinite(y).all()
+    assert err.max() <= TOL
+
+
 @pytest.mark.parametrize("name, n", [("paper", 1700), ("moe", 800)])
 def test_latency_parity_streaming_attention(pt, oracle_mod, name, n):
     """Graphs whose K/V do not fit shared memory (d_h = 16: N > 1536; d_h =
