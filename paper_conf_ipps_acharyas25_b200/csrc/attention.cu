@@ -241,21 +241,26 @@ struct Attn {
 
 };
 
-template <int DH, bool RESIDENT>
-__global__ void __launch_bounds__(256, DH == 16 ? 4 : 2)
+// NW warps per CTA: 8 (a whole 128-row q-tile) or 4 (half of one: two CTAs
+// per work item, so a short last q-tile idles at most 3 warps, not 7).
+template <int DH, bool RESIDENT, int NW = 8>
+__global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
     k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
            const __half* __restrict__ qkv, __half* __restrict__ out) {
   using A = Attn<DH>;
   extern __shared__ __align__(16) unsigned char dsm_attn[];
   __shared__ __align__(8) uint64_t kv_full[2];
   const int h = blockIdx.x % H;
-  const int widx = blockIdx.x / H;
+  const int widx = (blockIdx.x / H) / (8 / NW);
+  const int part = (blockIdx.x / H) % (8 / NW);
   if (widx >= d.qtile_off[G]) return;
   const int2 wk = d.work[widx];
   const int g = wk.x, qt = wk.y;
   if (d.status[g] != PREDTOP_OK) return;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
+  const int rbase = qt * 128 + part * NW * 16;  // first query row of this CTA
+  if (rbase >= N) return;
   const int W = 2 * ((N + 127) / 128);
   const int nchunks = (N + kChunk - 1) / kChunk;
   const int nbuf = RESIDENT ? nchunks : 2;
@@ -267,14 +272,14 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int gq = lane >> 2, tq = lane & 3;
-  const int ra = qt * 128 + warp * 16 + gq;  // graph-local query rows of this thread
+  const int ra = rbase + warp * 16 + gq;  // graph-local query rows of this thread
   const int rb = ra + 8;
   const bool va = ra < N, vb = rb < N;
-  const bool warp_live = qt * 128 + warp * 16 < N;
+  const bool warp_live = rbase + warp * 16 < N;
   const uint64_t* Ma = Mg + (int64_t)(va ? ra : 0) * W;
   const uint64_t* Mb = Mg + (int64_t)(vb ? rb : 0) * W;
   // block flags of this warp's 16-row group, one byte per chunk (k_bflags)
-  const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)(warp_live ? qt * 8 + warp : 0) * nchunks;
+  const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)(warp_live ? rbase / 16 + warp : 0) * nchunks;
 
   // K/V chunks by TMA (one thread): [64 keys x DH] boxes of the qkv matrix at
   // columns d + h*DH (K) and 2d + h*DH (V); keys past N read the next graph's
@@ -393,6 +398,207 @@ __global__ void __launch_bounds__(256, DH == 16 ? 4 : 2)
   }
 }
 
+// Persistent variant for graphs whose K/V fit twice in shared memory (the
+// GPT stage graphs): a CTA walks a static list of (graph, head) items,
+// item it = blockIdx.x + it * gridDim.x, with the K/V of items it and it+1 in
+// two TMA buffers.  Warps take the 16-row groups of the CTA's item sequence
+// round-robin ACROSS item boundaries (warp w: groups w, w+8, w+16, ... of the
+// concatenated list), so no warp idles on a partial 128-row tile and the
+// per-item start-up (status, node_ptr, K/V TMA) overlaps the previous item.
+// The last warp to leave an item issues the TMA for the item two ahead into
+// the buffer it frees.  Same per-group arithmetic as k_attn (Attn::chunk).
+#ifndef PREDTOP_ATTN_P_CTAS
+#define PREDTOP_ATTN_P_CTAS 3
+#endif
+template <int DH>
+__global__ void __launch_bounds__(256, DH == 16 ? PREDTOP_ATTN_P_CTAS : 2)
+    k_attn_p(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
+             const __half* __restrict__ qkv, __half* __restrict__ out, int maxch) {
+  using A = Attn<DH>;
+  extern __shared__ __align__(16) unsigned char dsm_attn[];
+  __shared__ __align__(8) uint64_t kv_full[2];
+  __shared__ int done_cnt[2];
+  // per-warp walk state, parked in shared memory while a group is processed
+  // (keeps the chunk loop at the register count of k_attn: no spills)
+  __shared__ int w_state[8][4];  // it, grp, g (or -1 past the end), ng
+  unsigned char* buf0 = sm100::align1024(dsm_attn);
+  const int bufb = 2 * maxch * A::CHUNK_BYTES;  // K chunks, then V chunks, of one item
+  const int total = G * H;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int gq = lane >> 2, tq = lane & 3;
+  const int ld3 = 3 * dmodel;
+
+  auto issue = [&](int it) {  // one thread: K/V of CTA-local item `it` -> buffer it & 1
+    const int id = blockIdx.x + it * gridDim.x;
+    if (id >= total) return;
+    const int g = id / H, h = id % H;
+    uint64_t* bar = &kv_full[it & 1];
+    if (d.status[g] != PREDTOP_OK) {  // no K/V: complete the phase without data
+      sm100::mbar_arrive(bar);
+      return;
+    }
+    const int64_t n0 = d.node_ptr[g];
+    const int N = (int)(d.node_ptr[g + 1] - n0);
+    const int nch = (N + kChunk - 1) / kChunk;
+    unsigned char* sK = buf0 + (it & 1) * bufb;
+    unsigned char* sV = sK + maxch * A::CHUNK_BYTES;
+    sm100::mbar_arrive_expect_tx(bar, (uint32_t)(nch * 2 * A::CHUNK_BYTES));
+    for (int c = 0; c < nch; ++c) {
+      const int row = (int)(n0 + c * kChunk);
+      sm100::tma_load_2d(sK + c * A::CHUNK_BYTES, &tkv, bar, dmodel + h * DH, row);
+      sm100::tma_load_2d(sV + c * A::CHUNK_BYTES, &tkv, bar, 2 * dmodel + h * DH, row);
+    }
+  };
+  if (threadIdx.x == 0) {
+    sm100::mbar_init(&kv_full[0], 1);
+    sm100::mbar_init(&kv_full[1], 1);
+    done_cnt[0] = done_cnt[1] = 0;
+    sm100::fence_mbar_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    issue(0);
+    issue(1);
+  }
+
+  // this warp leaves item `it`; the last of the 8 warps refills its buffer
+  auto warp_done = [&](int it) {
+    __syncwarp();
+    if (lane == 0) {
+      sm100::fence_proxy_async();  // our ldmatrix reads of the buffer before the TMA rewrite
+      if (atomicAdd(&done_cnt[it & 1], 1) == 7) {
+        done_cnt[it & 1] = 0;
+        issue(it + 2);
+      }
+    }
+    __syncwarp();
+  };
+
+  // walk: this warp's next group (grp of CTA-local item it)
+  volatile int* ws = w_state[warp];
+  if (lane == 0) {
+    ws[0] = 0;
+    ws[1] = warp;
+    ws[2] = -2;  // item info not loaded
+  }
+  __syncwarp();
+  A st;
+  for (;;) {
+    int it = ws[0], grp = ws[1];
+    int g = ws[2], ng = ws[3];
+    const auto load_item = [&](int it_) {
+      const int id = blockIdx.x + it_ * gridDim.x;
+      if (id >= total) {
+        g = -1;
+        ng = -1;
+        return;
+      }
+      g = id / H;
+      const int n = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
+      ng = d.status[g] == PREDTOP_OK ? (n + 15) / 16 : 0;
+    };
+    if (g == -2) load_item(it);
+    while (ng >= 0 && grp >= ng) {  // past this item: leave it (after its K/V arrived)
+      sm100::mbar_wait(&kv_full[it & 1], (it >> 1) & 1);
+      warp_done(it);
+      grp -= ng;
+      ++it;
+      load_item(it);
+    }
+    if (ng < 0) break;
+    __syncwarp();
+    if (lane == 0) {
+      ws[0] = it;
+      ws[1] = grp + 8;
+      ws[2] = g;
+      ws[3] = ng;
+    }
+    __syncwarp();
+    const int h = (blockIdx.x + it * gridDim.x) % H;
+    const int64_t n0 = d.node_ptr[g];
+    const int N = (int)(d.node_ptr[g + 1] - n0);
+    // ---- 16-row group `grp` of item (g, h)
+    const int W = 2 * ((N + 127) / 128);
+    const int nchunks = (N + kChunk - 1) / kChunk;
+    const uint64_t* Mg = d.M + d.row_off[g];
+    const __half* Qg = qkv + n0 * ld3 + h * DH;
+    const int ra = grp * 16 + gq, rb = ra + 8;
+    const bool va = ra < N, vb = rb < N;
+    const uint64_t* Ma = Mg + (int64_t)(va ? ra : 0) * W;
+    const uint64_t* Mb = Mg + (int64_t)(vb ? rb : 0) * W;
+    const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)grp * nchunks;
+    st.init(lane);
+    uint32_t kw[A::KS][4];
+#pragma unroll
+    for (int ks = 0; ks < A::KS; ++ks) {
+      const int k0 = ks * 16 + 2 * tq;
+      const __half* qa_p = Qg + (int64_t)ra * ld3 + k0;
+      const __half* qb_p = Qg + (int64_t)rb * ld3 + k0;
+      st.qa[ks][0] = va ? *reinterpret_cast<const uint32_t*>(qa_p) : 0u;
+      st.qa[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(qb_p) : 0u;
+      st.qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + 8) : 0u;
+      st.qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + 8) : 0u;
+      kw[ks][0] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel) : 0u;
+      kw[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel) : 0u;
+      kw[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel + 8) : 0u;
+      kw[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel + 8) : 0u;
+    }
+    const uint16_t* Ma16 = reinterpret_cast<const uint16_t*>(Ma) + tq;
+    const uint16_t* Mb16 = reinterpret_cast<const uint16_t*>(Mb) + tq;
+    auto mask_lo = [&](int c) -> uint32_t { return va ? (uint32_t)Ma16[4 * c] : 0u; };
+    auto mask_hi = [&](int c) -> uint32_t { return vb ? (uint32_t)Mb16[4 * c] : 0u; };
+    uint32_t mlo = mask_lo(0), mhi = mask_hi(0);
+    uint32_t fl = Fw[0];
+    {
+      float sa = 0.f, sb = 0.f;
+#pragma unroll
+      for (int ks = 0; ks < A::KS; ++ks) {
+        sa += dot_h2(st.qa[ks][0], kw[ks][0]) + dot_h2(st.qa[ks][2], kw[ks][2]);
+        sb += dot_h2(st.qa[ks][1], kw[ks][1]) + dot_h2(st.qa[ks][3], kw[ks][3]);
+      }
+      sa += __shfl_xor_sync(0xffffffffu, sa, 1);
+      sa += __shfl_xor_sync(0xffffffffu, sa, 2);
+      sb += __shfl_xor_sync(0xffffffffu, sb, 1);
+      sb += __shfl_xor_sync(0xffffffffu, sb, 2);
+      st.m_a = sa;
+      st.m_b = sb;
+    }
+    sm100::mbar_wait(&kv_full[it & 1], (it >> 1) & 1);
+    const uint32_t kb0 = sm100::smem_u32(buf0 + (it & 1) * bufb);
+    const uint32_t vb0 = kb0 + (uint32_t)(maxch * A::CHUNK_BYTES);
+    for (int c = 0; c < nchunks; ++c) {
+      const bool more = c + 1 < nchunks;
+      const uint32_t nlo = more ? mask_lo(c + 1) : 0u, nhi = more ? mask_hi(c + 1) : 0u;
+      const uint32_t nfl = more ? Fw[c + 1] : 0u;
+      const uint32_t off = (uint32_t)(c * A::CHUNK_BYTES);
+      st.chunk(kb0 + off, vb0 + off, mlo | (mhi << 16), __shfl_sync(0xffffffffu, fl, 0));
+      mlo = nlo;
+      mhi = nhi;
+      fl = nfl;
+    }
+    {
+      // output rows: re-derive the item from the parked state (nothing of
+      // the set-up above stays live across the chunk loop)
+      const int it2 = ws[0], g2 = ws[2], grp2 = ws[1] - 8;
+      const int h2 = (blockIdx.x + it2 * gridDim.x) % H;
+      const int64_t m0 = d.node_ptr[g2];
+      const int N2 = (int)(d.node_ptr[g2 + 1] - m0);
+      const int ra2 = grp2 * 16 + gq, rb2 = ra2 + 8;
+      const float l_a = st.osum[0], l_b = st.osum[2];
+      const float ia = l_a > 0.f ? 1.f / l_a : 0.f, ib = l_b > 0.f ? 1.f / l_b : 0.f;
+      __half* Og = out + m0 * dmodel + h2 * DH;
+#pragma unroll
+      for (int dn = 0; dn < A::DN; ++dn) {
+        const int col = dn * 8 + 2 * tq;
+        if (ra2 < N2)
+          *reinterpret_cast<uint32_t*>(Og + (int64_t)ra2 * dmodel + col) = pack_h2(st.o[dn][0] * ia, st.o[dn][1] * ia);
+        if (rb2 < N2)
+          *reinterpret_cast<uint32_t*>(Og + (int64_t)rb2 * dmodel + col) = pack_h2(st.o[dn][2] * ib, st.o[dn][3] * ib);
+      }
+    }
+  }
+}
+
 template <int DH>
 predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
                          cudaStream_t st, unsigned blocks) {
@@ -403,7 +609,37 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
   CUtensorMap tkv;
   if (!encode_tma_2d(&tkv, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kChunk))
     return PREDTOP_ERR_CUDA;
-  if (resident_bytes <= 100 * 1024) {
+  const int per_sm = DH == 16 ? PREDTOP_ATTN_P_CTAS : 2;
+  const int pers_bytes = 2 * resident_bytes;  // two item buffers (+ alignment slack)
+  const char* ap = getenv("PREDTOP_ATTN_MODE");  // "p": persistent, "8": 8-warp CTAs, default 4-warp
+  const bool persistent = ap && ap[0] == 'p';
+  const bool half_tiles = !(ap && ap[0] == '8');
+  if (persistent && pers_bytes * per_sm <= 220 * 1024) {
+    static bool attr_p = false;
+    if (!attr_p) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn_p<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       220 * 1024 / per_sm));
+      attr_p = true;
+    }
+    static int sms = 0;
+    if (!sms) {
+      int dev = 0;
+      PT_CUDA_TRY(cudaGetDevice(&dev));
+      PT_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    }
+    const int64_t items = (int64_t)G * H;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(items, (int64_t)sms * per_sm));
+    k_attn_p<DH><<<grid, 256, pers_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, maxch);
+  } else if (half_tiles && resident_bytes * 8 <= 200 * 1024) {
+    // 4-warp CTAs (half q-tiles), up to 8 per SM
+    static bool attr_h = false;
+    if (!attr_h) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       25 * 1024));
+      attr_h = true;
+    }
+    k_attn<DH, true, 4><<<2 * blocks, 128, resident_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+  } else if (resident_bytes <= 100 * 1024) {
     static bool attr_done = false;
     if (!attr_done) {
       PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
