@@ -570,10 +570,21 @@ def run_sweep(args, ctx, pool):
     assert st == pt.OK, (st, bad)
     assert torch.isfinite(sh.lat).all()
 
+    # CUDA-graph capture of the whole sweep step (~125 chunk builds + forwards):
+    # eager, the step is bound by host enqueue, not by the kernels
+    capture = not (args.eager or ctx.gloo)
+    launches_per_step = None
+    run = step
+    if capture:
+        run, launches_per_step = ctx.capture(step)
+        run()
+        torch.cuda.synchronize()
     launches0 = L.predtop_launch_count()
     with ClockSampler(ctx.dev_index) as clk:
-        ms = ctx.timed(step, args.steps, flush=False)
+        ms = ctx.timed(run, args.steps, flush=False)
     launches = L.predtop_launch_count() - launches0
+    if launches_per_step is not None:
+        launches = launches_per_step * args.steps
     total_ms = ctx.max_over_ranks(sum(ms))
     graphs_total = ctx.sum_over_ranks(float(sh.num_stages))
     value = graphs_total * args.steps / (total_ms / 1e3)
@@ -616,8 +627,9 @@ def run_sweep(args, ctx, pool):
             pt.predtop_plan_argmin(T, best)
             T_host[:sh.num_plans].copy_(T, non_blocking=True)
 
-    e2e_step()
-    ms_e2e = ctx.timed(e2e_step, max(2, args.steps // 2), flush=False)
+    e2e_run = ctx.capture(e2e_step)[0] if capture else e2e_step
+    e2e_run()
+    ms_e2e = ctx.timed(e2e_run, max(2, args.steps // 2), flush=False)
     tot_e2e = ctx.max_over_ranks(sum(ms_e2e))
     e2e_value = graphs_total * len(ms_e2e) / (tot_e2e / 1e3)
 
@@ -647,7 +659,7 @@ def run_sweep(args, ctx, pool):
                 "plans_per_s": plans_per_s, "graphs_per_step": graphs_total, "best_plan": b,
                 "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                         "d2h_bytes_per_step": int(d2h)},
-                "gpu_launches": int(launches), "launch_mode": "eager",
+                "gpu_launches": int(launches), "launch_mode": "cuda_graph" if capture else "eager",
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
         emit(line, args)

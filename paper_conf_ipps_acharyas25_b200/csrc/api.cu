@@ -166,12 +166,18 @@ static bool device_ok() {
     set_error("no CUDA device");
     return false;
   }
-  cudaDeviceProp p;
-  if (cudaGetDeviceProperties(&p, dev) != cudaSuccess || p.major < 10) {
+  // cached per device: cudaGetDeviceProperties costs milliseconds of host
+  // time, and this runs on every build (the eager sweep builds ~100 chunks)
+  static int ok_dev[64] = {0};  // 0 unknown, 1 ok, -1 not sm_100
+  if (dev >= 0 && dev < 64 && ok_dev[dev] == 1) return true;
+  int major = 0;
+  if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess || major < 10) {
     set_error("libpredtop needs an sm_100 (Blackwell) device");
     cudaGetLastError();
+    if (dev >= 0 && dev < 64) ok_dev[dev] = -1;
     return false;
   }
+  if (dev >= 0 && dev < 64) ok_dev[dev] = 1;
   return true;
 }
 

@@ -618,7 +618,10 @@ __global__ void __launch_bounds__(128) k_bflags(DagDev d, SmallCfg sc) {
   const uint64_t* Mg = d.M + d.row_off[g];
   uint8_t* out = d.bflag + d.bflag_off[g];
   uint64_t* Mw = d.M + d.row_off[g];
-  for (int it = threadIdx.x; it < ng * nch; it += blockDim.x) {
+  // grid (G, Y): the (16-row group, chunk) items of a graph are spread over
+  // gridDim.y CTAs, so one large graph (16k nodes: 262k items) is not a
+  // single-CTA loop
+  for (int it = blockIdx.y * blockDim.x + threadIdx.x; it < ng * nch; it += gridDim.y * blockDim.x) {
     const int rg = it / nch, c = it % nch;
     uint64_t o = 0, a = ~0ull;
     for (int r = rg * 16; r < min(N, rg * 16 + 16); ++r) {
@@ -724,7 +727,9 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
   }
   {
     ProfScope _p(PK_DAG_FLAGS, st);
-    k_bflags<<<G, 128, 0, st>>>(d, sc);
+    const int64_t items = ceil_div(b.max_nodes, 16) * ceil_div(b.max_nodes, 64);
+    dim3 gb(G, (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(items, 128), 1024)));
+    k_bflags<<<gb, 128, 0, st>>>(d, sc);
     PT_LAUNCH_CHECK();
   }
   return PREDTOP_OK;
