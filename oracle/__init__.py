@@ -60,6 +60,7 @@ def lib():
             L.orc_row_words.argtypes = [i32]
             L.orc_row_words.restype = i32
             L.orc_reach.argtypes = [i32, i32, P, P, P]
+            L.orc_reach_k.argtypes = [i32, i32, P, P, i32, P]
             L.orc_mask.argtypes = [i32, P, P]
             L.orc_tiles.argtypes = [i32, P, P]
             L.orc_tiles.restype = i64
@@ -73,6 +74,8 @@ def lib():
             L.orc_readout.restype = dbl
             L.orc_forward.argtypes = [P, P, i32, i32, P, P, P, P, P]
             L.orc_forward.restype = i32
+            L.orc_forward_k.argtypes = [P, P, i32, i32, P, P, P, i32, P, P]
+            L.orc_forward_k.restype = i32
             L.orc_plan_T.argtypes = [i64, P, P, P, P, i64, P]
             L.orc_argmin.argtypes = [i64, P]
             L.orc_argmin.restype = i64
@@ -114,11 +117,15 @@ def row_words(n: int) -> int:
     return 2 * ((n + 127) // 128)
 
 
-def reach(n, src, dst) -> np.ndarray:
-    """Closure bitsets [n, W] uint64 (layout of include/predtop.h)."""
+def reach(n, src, dst, hops: int = 0) -> np.ndarray:
+    """Closure bitsets [n, W] uint64 (layout of include/predtop.h).  hops > 0:
+    the k-hop relation R_k (finite-k DAGRA, reading R19)."""
     s, d = _i32(src), _i32(dst)
     out = np.zeros((n, row_words(n)), np.uint64)
-    lib().orc_reach(n, len(s), _p(s), _p(d), _p(out))
+    if hops > 0:
+        lib().orc_reach_k(n, len(s), _p(s), _p(d), int(hops), _p(out))
+    else:
+        lib().orc_reach(n, len(s), _p(s), _p(d), _p(out))
     return out
 
 
@@ -190,20 +197,20 @@ def readout(model_cfg, blob, n, x) -> float:
     return float(lib().orc_readout(ctypes.byref(c), _p(b), n, _p(np.ascontiguousarray(x, np.float64))))
 
 
-def forward(model_cfg, blob, n, src, dst, feats, taps: bool = False):
-    """One stage graph -> (status, latency, taps or None)."""
+def forward(model_cfg, blob, n, src, dst, feats, taps: bool = False, hops: int = 0):
+    """One stage graph -> (status, latency, taps or None).  hops > 0: k-hop mask."""
     c = cfg(model_cfg)
     b = np.ascontiguousarray(blob, np.float32)
     s, d = _i32(src), _i32(dst)
     y = np.zeros(1, np.float64)
     t = np.zeros((model_cfg["num_layers"] + 1, n, model_cfg["d_model"]), np.float64) if taps else None
-    st = lib().orc_forward(ctypes.byref(c), _p(b), n, len(s), _p(s), _p(d), _p(_feats(feats)),
-                           _p(y), _p(t))
+    st = lib().orc_forward_k(ctypes.byref(c), _p(b), n, len(s), _p(s), _p(d), _p(_feats(feats)),
+                             int(hops), _p(y), _p(t))
     return st, float(y[0]), t
 
 
 def forward_batch(model_cfg, blob, batch, graphs: Optional[Sequence[int]] = None,
-                  threads: Optional[int] = None) -> np.ndarray:
+                  threads: Optional[int] = None, hops: int = 0) -> np.ndarray:
     """Latency of every graph (or the listed ones) of a synth.StageBatch, one
     graph per worker thread (ctypes releases the GIL)."""
     gs = list(range(batch.num_graphs)) if graphs is None else list(graphs)
@@ -212,7 +219,7 @@ def forward_batch(model_cfg, blob, batch, graphs: Optional[Sequence[int]] = None
 
     def one(g):
         n, s, d, f = batch.graph(g)
-        return forward(model_cfg, blob, n, s, d, f)[1]
+        return forward(model_cfg, blob, n, s, d, f, hops=hops)[1]
 
     if threads <= 1 or len(gs) <= 1:
         return np.asarray([one(g) for g in gs], np.float64)

@@ -134,6 +134,42 @@ void orc_reach(int n, int e, const int32_t* src, const int32_t* dst, uint64_t* R
   free(seen); free(stack); free_csr(&succ);
 }
 
+/* ------------------------------------------------------------------------ */
+/* Finite-k DAGRA ("u in N_k(v)"; "the constant k ... specifies  */
+/* the neighborhood range for attention calculation").       */
+/* Reading R19: N_k(v) = the nodes joined to v by a directed path of at most */
+/* k edges in either direction (the DAG Transformer's k-hop receptive field).*/
+/* R_k[v] = { u != v : the shortest directed path v ~> u has 1..k edges },   */
+/* by one breadth-first search along successors per v, stopped at depth k.   */
+/* k <= 0 means k = infinity, i.e. orc_reach.                        */
+/* ------------------------------------------------------------------------ */
+void orc_reach_k(int n, int e, const int32_t* src, const int32_t* dst, int k, uint64_t* R) {
+  if (k <= 0) { orc_reach(n, e, src, dst, R); return; }
+  int W = orc_row_words(n);
+  memset(R, 0, sizeof(uint64_t) * (size_t)n * (size_t)W);
+  orc_csr succ = build_csr(n, e, src, dst);
+  int* dist = (int*)malloc(sizeof(int) * ((size_t)n + 1));
+  int* queue = (int*)malloc(sizeof(int) * ((size_t)n + 1));
+  for (int v = 0; v < n; ++v) {
+    for (int u = 0; u < n; ++u) dist[u] = -1;
+    int head = 0, tail = 0;
+    dist[v] = 0;
+    queue[tail++] = v;
+    while (head < tail) {
+      int u = queue[head++];
+      if (dist[u] == k) continue; /* do not expand past k edges */
+      for (int i = succ.off[u]; i < succ.off[u + 1]; ++i) {
+        int w = succ.adj[i];
+        if (dist[w] < 0) { dist[w] = dist[u] + 1; queue[tail++] = w; }
+      }
+    }
+    for (int u = 0; u < n; ++u)
+      if (u != v && dist[u] >= 1 && dist[u] <= k)
+        R[(size_t)v * W + (size_t)(u / 64)] |= (uint64_t)1 << (u % 64);
+  }
+  free(dist); free(queue); free_csr(&succ);
+}
+
 static int bit(const uint64_t* B, int W, int row, int col) {
   return (int)((B[(size_t)row * W + (size_t)(col / 64)] >> (col % 64)) & 1u);
 }
@@ -383,6 +419,13 @@ double orc_readout(const orc_cfg* c, const float* blob, int n, const double* x) 
 /* Returns the validation status; y = NaN for an invalid graph.              */
 int orc_forward(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
                 const int32_t* dst, const orc_feat* feats, double* y, double* taps) {
+  return orc_forward_k(c, blob, n, e, src, dst, feats, 0, y, taps);
+}
+
+/* The same forward pass with the k-hop mask M = R_k | R_k^T | I (P:142,     */
+/* P:145; R19).  k <= 0 is k = infinity.                                     */
+int orc_forward_k(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
+                  const int32_t* dst, const orc_feat* feats, int k, double* y, double* taps) {
   int st = orc_validate(n, e, src, dst);
   if (st != ORC_OK) { *y = NAN; return st; }
   int d = c->d, W = orc_row_words(n);
@@ -392,7 +435,7 @@ int orc_forward(const orc_cfg* c, const float* blob, int n, int e, const int32_t
   double* x = (double*)malloc(sizeof(double) * (size_t)n * d);
   double* x2 = (double*)malloc(sizeof(double) * (size_t)n * d);
   orc_depth(n, e, src, dst, depth);
-  orc_reach(n, e, src, dst, R);
+  orc_reach_k(n, e, src, dst, k, R);
   orc_mask(n, R, M);
   orc_embed(c, blob, n, feats, depth, x);
   if (taps) memcpy(taps, x, sizeof(double) * (size_t)n * d);

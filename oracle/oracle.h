@@ -58,6 +58,7 @@ int orc_validate(int n, int e, const int32_t* src, const int32_t* dst);
 void orc_depth(int n, int e, const int32_t* src, const int32_t* dst, int32_t* depth);
 int orc_row_words(int n);
 void orc_reach(int n, int e, const int32_t* src, const int32_t* dst, uint64_t* R);
+void orc_reach_k(int n, int e, const int32_t* src, const int32_t* dst, int k, uint64_t* R);
 void orc_mask(int n, const uint64_t* R, uint64_t* M);
 int64_t orc_tiles(int n, const uint64_t* M, uint8_t* cls);
 
@@ -72,6 +73,8 @@ void orc_layer(const orc_cfg* c, const float* blob, int layer, int n, const uint
 double orc_readout(const orc_cfg* c, const float* blob, int n, const double* x);
 int orc_forward(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
                 const int32_t* dst, const orc_feat* feats, double* y, double* taps);
+int orc_forward_k(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
+                  const int32_t* dst, const orc_feat* feats, int k, double* y, double* taps);
 
 void orc_plan_T(int64_t P, const int64_t* plan_ptr, const int32_t* plan_stage,
                 const int32_t* B, const float* t, int64_t num_stages, double* T);
