@@ -113,18 +113,18 @@ def host_cores() -> int:
         return os.cpu_count() or 1
 
 
-def oracle_rate(cfg, blob, batch, target_s: float = 15.0, max_graphs: int = 1024):
+def oracle_rate(cfg, blob, batch, target_s: float = 15.0, max_graphs: int = 1024, hops: int = 0):
     """Oracle graphs/s on a bounded sample with all host cores."""
     import oracle
     oracle.build()
     cores = host_cores()
     t0 = time.perf_counter()
-    oracle.forward_batch(cfg, blob, batch, graphs=[0], threads=1)
+    oracle.forward_batch(cfg, blob, batch, graphs=[0], threads=1, hops=hops)
     t1 = time.perf_counter() - t0
     n = int(max(cores, min(max_graphs, batch.num_graphs, round(target_s * cores / max(t1, 1e-6)))))
     n = min(n, batch.num_graphs)
     t0 = time.perf_counter()
-    oracle.forward_batch(cfg, blob, batch, graphs=list(range(n)), threads=cores)
+    oracle.forward_batch(cfg, blob, batch, graphs=list(range(n)), threads=cores, hops=hops)
     wall = time.perf_counter() - t0
     return n / wall, cores, n, wall
 
@@ -198,7 +198,8 @@ def workload_config(args):
                              f"{G // S} plans x {S} stages x B=16 (Eqn 4)",
                  "graphs_per_gpu": G, "plans_per_gpu": G // S, "stages_per_plan": S, "microbatches": 16,
                  "parallelism": f"graph-sharded x{args.gpus} (owned plans), NCCL all-gather of plan latencies",
-                 "l2": "flushed before every timed step (256 MiB memset, untimed)"}, **base)
+                 "l2": "flushed before every timed step (256 MiB memset, untimed)",
+                 "dagra_k": args.hops if args.hops > 0 else "inf"}, **base)
 
 
 # ----------------------------------------------------------------- main leg
@@ -411,7 +412,7 @@ def run_batch(args, ctx):
     ps = synth.owned_plans(G, S, 16)
     model = pt.Model(cfg, blob, device=dev)
     db = pt.DeviceBatch.from_host(host, device=dev)
-    dag = pt.Dag(db, no_sync=True)
+    dag = pt.Dag(db, no_sync=True, hops=args.hops)
     ws = model.forward_workspace(dag)
     lat = torch.empty(G, dtype=torch.float32, device=dev)
     plans = pt.Plans(ps.plan_ptr, ps.plan_stage, ps.microbatches, device=dev)
@@ -512,7 +513,7 @@ def run_batch(args, ctx):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config != "16k":
-        v, cores, n, wall = oracle_rate(cfg, blob, host)
+        v, cores, n, wall = oracle_rate(cfg, blob, host, hops=getattr(args, "hops", 0))
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": f"first {n} of {G} {args.config} stage graphs, fp64 C oracle, {cores} threads, {wall:.1f} s"}
 
@@ -683,6 +684,8 @@ def main():
     ap.add_argument("--plans", type=int, default=100000, help="sweep: total candidate plans")
     ap.add_argument("--chunk", type=int, default=4096, help="sweep: stage graphs per build+forward launch")
     ap.add_argument("--pool", type=int, default=8192, help="sweep: distinct synthetic stage graphs")
+    ap.add_argument("--hops", type=int, default=0,
+                    help="DAGRA range k (P:145): 0 = infinity (the paper's setting); k >= 1 = k-hop mask")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-json", default=None)
     ap.add_argument("--eager", action="store_true", help="no CUDA-graph capture of the step")

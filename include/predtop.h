@@ -57,7 +57,7 @@
 extern "C" {
 #endif
 
-#define PREDTOP_ABI_VERSION 1
+#define PREDTOP_ABI_VERSION 2 /* 2: predtop_batch_desc.hops */
 
 typedef enum {
   PREDTOP_OK = 0,
@@ -119,6 +119,11 @@ typedef struct {
   int64_t total_nodes;  /* = node_ptr[G] */
   int64_t total_edges;  /* = edge_ptr[G] */
   uint32_t flags;       /* PREDTOP_NO_SYNC or 0 */
+  int32_t hops;         /* DAGRA range k (Eqn 1 "u in N_k(v)" P:142; "the constant k ...
+                           specifies the neighborhood range" P:145): 0 = k = infinity
+                           (the paper's setting, full closure); k >= 1 = the k-hop
+                           relation R_k below.  < 0 -> INVALID_ARG.  Occupies what was
+                           tail padding: a zero-initialised ABI-v1 descriptor means k = inf. */
 } predtop_batch_desc;
 
 typedef struct predtop_dag_s* predtop_dag;
@@ -136,6 +141,10 @@ PREDTOP_API size_t predtop_build_dag_workspace(const predtop_batch_desc* desc);
  *    1 + max over predecessors p of depth(p)  (longest path from a source).
  *  - reachability (DAGRA, P:135, P:145 with k = infinity): R[v] = the set of
  *    nodes u != v reachable from v by a directed path of >= 1 edge.
+ *    With desc->hops = k >= 1 (finite-k DAGRA; R19):
+ *    R_k[v] = the nodes u != v whose shortest directed path from v has at
+ *    most k edges; predtop_reachability, the mask and stage_forward then use
+ *    R_k (M = R_k | R_k^T | I).  k >= the longest path gives R exactly.
  *    The attention mask used by stage_forward is M = R | R^T | I
  *    ("a path from m to n or vice versa"; reflexive).
  * Arguments:

@@ -222,6 +222,7 @@ predtop_status predtop_build_dag(const predtop_batch_desc* desc, const int64_t* 
   *out = nullptr;
   DagBounds bd;
   if (!dag_bounds(desc, &bd)) { set_error("invalid batch descriptor"); return PREDTOP_ERR_INVALID_ARG; }
+  if (desc->hops < 0) { set_error("hops %d < 0", desc->hops); return PREDTOP_ERR_INVALID_ARG; }
   if (desc->max_nodes > PREDTOP_MAX_NODES) {
     set_error("max_nodes %d > PREDTOP_MAX_NODES", desc->max_nodes);
     return PREDTOP_ERR_TOO_LARGE;
@@ -246,6 +247,7 @@ predtop_status predtop_build_dag(const predtop_batch_desc* desc, const int64_t* 
   dag->d.src = edge_src;
   dag->d.dst = edge_dst;
   dag->d.feats = feats;
+  dag->d.hops = desc->hops;
   if (depth_out) dag->d.depth = depth_out;
   dag->words_bound = bd.words;
   dag->tiles_bound = bd.tiles;

@@ -264,6 +264,35 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
     Rs = (uint64_t*)(sm + (csr_in_smem ? csr_bytes : 0));
     rs = CW;
   }
+  const int K = d.hops;
+  if (K > 0 && K < L - 1) {
+    __syncthreads();  // the staged CSR above
+    // finite-k DAGRA: K synchronous rounds over all rows,
+    // R_j[v] = OR_{w in succ(v)} ({w} | R_{j-1}[w]), R_0 = 0, ping-ponging
+    // between Rs and a second buffer of the same column slice (the global R
+    // rows when Rs is shared memory, else the M rows, which k_mask rewrites
+    // later); round j writes Rs iff K - j is even, so R_K ends in Rs.
+    uint64_t* Xs = global_mode ? d.M + d.row_off[g] + word0 : Rg + word0;
+    const int64_t xs = W;
+    for (int j = 1; j <= K; ++j) {
+      const bool to_rs = ((K - j) & 1) == 0;
+      for (int64_t it = tid; it < (int64_t)N * nw; it += nt) {
+        const int v = (int)(it / nw), c = (int)(it % nw);
+        const int word = word0 + c;
+        uint64_t acc = 0;
+        for (int k = soff[v]; k < soff[v + 1]; ++k) {
+          const int w = succ[k];
+          if (j > 1) acc |= to_rs ? __ldcg(Xs + (int64_t)w * xs + c)
+                                  : (global_mode ? __ldcg(Rs + (int64_t)w * rs + c) : Rs[(int64_t)w * rs + c]);
+          if ((w >> 6) == word) acc |= 1ull << (w & 63);
+        }
+        if (to_rs) Rs[(int64_t)v * rs + c] = acc;
+        else Xs[(int64_t)v * xs + c] = acc;
+      }
+      __threadfence();
+      __syncthreads();
+    }
+  } else {
   for (int64_t it = tid; it < (int64_t)N * nw; it += nt) Rs[(it / nw) * rs + it % nw] = 0;
   __syncthreads();
   for (int level = L - 1; level >= 0; --level) {
@@ -282,6 +311,7 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
       Rs[(int64_t)v * rs + j] = acc;
     }
     __syncthreads();
+  }
   }
   if (!global_mode)
     for (int64_t it = tid; it < (int64_t)N * nw; it += nt)
@@ -533,6 +563,31 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
     for (int t = lane; t < T * T; t += 32) cls[t] = 0;
     return;
   }
+  const int K = d.hops;
+  if (K > 0 && K < level - 1) {
+    // finite-k DAGRA: K synchronous rounds R_j[v] = OR_{w in
+    // succ(v)} ({w} | R_{j-1}[w]), R_0 = 0, ping-ponging between the shared
+    // slot and the graph's global R rows (rewritten from the slot below);
+    // round j writes the slot iff K - j is even, so R_K ends in the slot.
+    // (K >= longest path = level - 1 gives the full closure: path below.)
+    for (int j = 1; j <= K; ++j) {
+      const bool to_smem = ((K - j) & 1) == 0;
+      uint64_t* dstb = to_smem ? R : Rg;
+      const uint64_t* srcb = to_smem ? Rg : R;
+      for (int it = lane; it < N * W; it += 32) {
+        const int v = it / W, c = it % W;
+        uint64_t acc = 0;
+        for (int k = soff[v]; k < soff[v + 1]; ++k) {
+          const int w = succ[k];
+          if (j > 1) acc |= to_smem ? __ldcg(srcb + w * W + c) : srcb[w * W + c];
+          if ((w >> 6) == c) acc |= 1ull << (w & 63);
+        }
+        dstb[it] = acc;
+      }
+      __threadfence();
+      __syncwarp();
+    }
+  } else {
   // closure R[v] = OR_{w in succ(v)} (R[w] | {w}), deepest level first
   for (int i = lane; i < N * W; i += 32) R[i] = 0;
   __syncwarp();
@@ -549,6 +604,7 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
       R[v * W + j] = acc;
     }
     __syncwarp();
+  }
   }
   DTR(2);
   // mask M = R | R^T | I per 64-bit word (two 32x32 bit transposes in

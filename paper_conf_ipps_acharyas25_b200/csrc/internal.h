@@ -44,6 +44,7 @@ struct DagDev {
   int64_t* bflag_off;  // [G+1] prefix of ceil(N/16) * ceil(N/64)
   uint8_t* bflag;      // per (16-row group, 64-key chunk): bits 0-3 block (keys 16j..16j+15)
                        // has an allowed pair, bits 4-7 block fully allowed (attention.cu)
+  int32_t hops;        // DAGRA range k (0 = infinity): R is then the k-hop relation R_k
 };
 
 // Stored layout of the attention mask words.  Key k (0..63) of a 64-key chunk

@@ -40,7 +40,7 @@ class PredtopError(RuntimeError):
 class BatchDesc(ctypes.Structure):
     _fields_ = [("num_graphs", ctypes.c_int32), ("max_nodes", ctypes.c_int32),
                 ("total_nodes", ctypes.c_int64), ("total_edges", ctypes.c_int64),
-                ("flags", ctypes.c_uint32)]
+                ("flags", ctypes.c_uint32), ("hops", ctypes.c_int32)]
 
 
 class ModelConfig(ctypes.Structure):
@@ -181,18 +181,20 @@ class DeviceBatch:
                            t(batch.src, torch.int32), t(batch.dst, torch.int32),
                            torch.from_numpy(fb.copy()).to(device), int(sizes.max()) if len(sizes) else 1)
 
-    def desc(self, flags=0) -> BatchDesc:
-        return BatchDesc(self.num_graphs, self.max_nodes, self.total_nodes, self.total_edges, flags)
+    def desc(self, flags=0, hops: int = 0) -> BatchDesc:
+        """hops: DAGRA range k (0 = infinity); k >= 1 builds the k-hop mask."""
+        return BatchDesc(self.num_graphs, self.max_nodes, self.total_nodes, self.total_edges, flags, hops)
 
 
 class Dag:
     """predtop_build_dag over a DeviceBatch; owns the workspace and depth."""
 
     def __init__(self, batch: DeviceBatch, no_sync: bool = False, stream=None, check: bool = True,
-                 workspace: Optional[torch.Tensor] = None, depth: Optional[torch.Tensor] = None):
+                 workspace: Optional[torch.Tensor] = None, depth: Optional[torch.Tensor] = None,
+                 hops: int = 0):
         self.batch = batch
         dev = batch.node_ptr.device
-        self.desc = batch.desc(NO_SYNC if no_sync else 0)
+        self.desc = batch.desc(NO_SYNC if no_sync else 0, hops)
         need = lib().predtop_build_dag_workspace(ctypes.byref(self.desc))
         if need == 0:
             raise PredtopError(INVALID_ARG, "invalid batch descriptor")

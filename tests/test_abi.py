@@ -48,7 +48,8 @@ def test_sass_is_blackwell_native(libpath):
 def test_host_validation_without_gpu(libpath):
     from paper_conf_ipps_acharyas25_b200 import predtop as pt
     L = pt.lib()
-    assert L.predtop_abi_version() == 1
+    assert L.predtop_abi_version() == 2
+    assert ctypes.sizeof(pt.BatchDesc) == 32  # hops sits in the v1 tail padding
     assert L.predtop_status_string(-4) == b"graph has a cycle"
     d = pt.BatchDesc(0, 1, 0, 0, 0)
     assert L.predtop_build_dag_workspace(ctypes.byref(d)) == 0          # G < 1

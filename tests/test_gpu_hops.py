@@ -1,0 +1,120 @@
+"""GPU parity of finite-k DAGRA ("u in N_k(v)", P:145 k
+a hyperparameter; reading R19): predtop_build_dag with desc.hops = k writes
+the k-hop relation R_k, bit-exact against the oracle's k-limited BFS, on both
+build paths (the fused one-warp-per-graph path for N <= 512 and the
+multi-kernel column-slice path for larger graphs), and the forward pass under
+M_k = R_k | R_k^T | I matches the oracle's forward_k within 2e-3."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_ipps_acharyas25_b200 import synth
+
+pytestmark = pytest.mark.gpu
+TOL = 2e-3
+
+
+@pytest.fixture(scope="module")
+def pt():
+    from paper_conf_ipps_acharyas25_b200 import build, predtop
+    build.build_library()
+    assert torch.cuda.is_available()
+    return predtop
+
+
+def _check(pt, oracle_mod, batch, k):
+    dag = pt.Dag(pt.DeviceBatch.from_host(batch), hops=k)
+    assert dag.status == pt.OK
+    R = dag.reachability().cpu().numpy().view(np.uint64)
+    M = dag.mask().cpu().numpy().view(np.uint64)
+    depth = dag.depth.cpu().numpy()
+    sizes = batch.sizes
+    T = (sizes + 127) // 128
+    cls, pairs = dag.tiles(int((T * T).sum()))
+    cls, pairs = cls.cpu().numpy(), pairs.cpu().numpy()
+    woff = toff = 0
+    for g in range(batch.num_graphs):
+        n, s, d, _ = batch.graph(g)
+        Ro = oracle_mod.reach(n, s, d, hops=k)
+        Mo = oracle_mod.mask(n, Ro)
+        co, po = oracle_mod.tiles(n, Mo)
+        W = oracle_mod.row_words(n)
+        n0 = batch.node_ptr[g]
+        np.testing.assert_array_equal(depth[n0:n0 + n], oracle_mod.depth(n, s, d))
+        np.testing.assert_array_equal(R[woff:woff + n * W], Ro.ravel(), err_msg=f"R_k g={g} k={k}")
+        np.testing.assert_array_equal(M[woff:woff + n * W], Mo.ravel(), err_msg=f"M_k g={g} k={k}")
+        np.testing.assert_array_equal(cls[toff:toff + len(co)], co)
+        assert pairs[g] == po
+        woff += n * W
+        toff += len(co)
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 8, 1000])
+def test_small_path_gpt_graphs(pt, oracle_mod, k):
+    _check(pt, oracle_mod, synth.stage_batch("gpt", 12, first_graph=3), k)
+
+
+@pytest.mark.parametrize("k", [1, 2, 5, 64])
+def test_large_path_moe_graphs(pt, oracle_mod, k):
+    _check(pt, oracle_mod, synth.stage_batch("moe", 2), k)
+
+
+def test_random_relabelled_mixed_sizes(pt, oracle_mod):
+    rng = synth.CounterRng(77, 3)
+    gs = []
+    for n, p in [(1, 0.0), (2, 1.0), (65, 0.05), (129, 0.03), (300, 0.02), (700, 0.004)]:
+        s, d = synth.random_dag(n, p, rng)
+        gs.append((n, s, d, synth._rand_feats(n, rng)))
+    s, d = synth.chain(513)  # deep chain on the large path
+    gs.append((513, s, d, synth._rand_feats(513, rng)))
+    b = synth.pack_graphs(gs)
+    for k in (1, 2, 4, 7):
+        _check(pt, oracle_mod, b, k)
+
+
+def test_16k_graph_k4(pt, oracle_mod):
+    b = synth.stage_batch("16k", 1)
+    n, s, d, _ = b.graph(0)
+    dag = pt.Dag(pt.DeviceBatch.from_host(b), hops=4)
+    R = dag.reachability().cpu().numpy().view(np.uint64)
+    W = oracle_mod.row_words(n)
+    # sampled rows against the oracle's k-limited BFS on the whole graph
+    Ro = oracle_mod.reach(n, s, d, hops=4)
+    rows = synth.CounterRng(5, 5).permutation(n)[:512]
+    np.testing.assert_array_equal(R.reshape(n, W)[rows], Ro[rows])
+
+
+def test_large_k_equals_closure(pt):
+    b = synth.stage_batch("gpt", 8, first_graph=40)
+    db = pt.DeviceBatch.from_host(b)
+    R_inf = pt.Dag(db).reachability().cpu()
+    R_big = pt.Dag(db, hops=100000).reachability().cpu()
+    assert torch.equal(R_inf, R_big)
+
+
+def test_negative_hops_rejected(pt):
+    b = synth.tiny_batch()
+    with pytest.raises(pt.PredtopError):
+        pt.Dag(pt.DeviceBatch.from_host(b), hops=-1)
+
+
+@pytest.mark.parametrize("name, batch_fn, k", [
+    ("gpt", lambda: synth.stage_batch("gpt", 16), 2),
+    ("gpt", lambda: synth.stage_batch("gpt", 16, first_graph=16), 6),
+    ("moe", lambda: synth.stage_batch("moe", 2), 3),
+])
+def test_forward_parity(pt, oracle_mod, name, batch_fn, k):
+    cfg = dict(synth.MODEL_CONFIGS[name])
+    blob = synth.pack_weights(cfg, synth.model_weights(cfg))
+    model = pt.Model(cfg, blob)
+    batch = batch_fn()
+    dag = pt.Dag(pt.DeviceBatch.from_host(batch), hops=k)
+    y = model.forward(dag)
+    torch.cuda.synchronize()
+    y = y.cpu().numpy().astype(np.float64)
+    want = oracle_mod.forward_batch(cfg, blob, batch, hops=k)
+    inf = oracle_mod.forward_batch(cfg, blob, batch)
+    assert not np.array_equal(want, inf)  # the k-hop mask changes the prediction
+    err = np.abs(y - want) / np.abs(want)
+    print(f"{name} k={k}: max rel err {err.max():.3e}")
+    assert err.max() <= TOL
