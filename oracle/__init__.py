@@ -79,6 +79,8 @@ def lib():
             L.orc_plan_T.argtypes = [i64, P, P, P, P, i64, P]
             L.orc_argmin.argtypes = [i64, P]
             L.orc_argmin.restype = i64
+            L.orc_plan_search.argtypes = [i32, i32, P, i32, P, i32, P, P, P]
+            L.orc_plan_search.restype = dbl
             _lib = L
     return _lib
 
@@ -241,3 +243,23 @@ def plan_T(plan_ptr, plan_stage, microbatches, stage_latency) -> np.ndarray:
 def argmin(T) -> int:
     T = np.ascontiguousarray(T, np.float64)
     return int(lib().orc_argmin(len(T), _p(T)))
+
+
+def plan_search(stage_latency, choice_devices, num_devices: int, microbatches: int):
+    """Optimal pipeline plan over a stage table t[L][L][K] (fp32; entries with
+    i > j unused; non-finite or negative = infeasible) by exhaustive
+    enumeration (reading R20) -> (T*, [(first, last, choice), ...])."""
+    t = np.ascontiguousarray(stage_latency, np.float32)
+    L, L2, K = t.shape
+    assert L == L2
+    dev = np.ascontiguousarray(choice_devices, np.int32)
+    S = ctypes.c_int32(0)
+    ends = np.zeros(64, np.int32)
+    ch = np.zeros(64, np.int32)
+    T = lib().orc_plan_search(L, K, _p(dev), int(num_devices), _p(t), int(microbatches),
+                              ctypes.byref(S), _p(ends), _p(ch))
+    stages, a = [], 0
+    for i in range(S.value):
+        stages.append((a, int(ends[i]), int(ch[i])))
+        a = int(ends[i]) + 1
+    return float(T), stages

@@ -491,3 +491,77 @@ int64_t orc_argmin(int64_t n, const double* T) {
   }
   return best;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Inter-stage plan search over a shared stage table.       */
+/* Alpa's inter-operator optimizer picks the pipeline plan with the   */
+/* 1F1B model; it iterates through all possible stages and        */
+/* submeshes; PredTOP predicts every stage on every mesh and applies  */
+/* the pipeline model (Eqn 4).  Plain definition (reading R20): a plan       */
+/* slices the L layers into S >= 1 contiguous stages [a_s, b_s] and gives    */
+/* each a choice c_s (a mesh / intra-op configuration, Tables II-III) using  */
+/* dev[c_s] devices, with sum_s dev[c_s] == D (the whole cluster) and every  */
+/* t[a_s][b_s][c_s] feasible (finite, >= 0).  T(plan) = Eqn 4 over its S     */
+/* stage latencies (orc_plan_T, R13).  The optimum is the minimum over ALL   */
+/* plans, found here by exhaustive enumeration (no DP); ties keep the first  */
+/* plan in the enumeration order (stage ends ascending, then choices         */
+/* ascending).  Table layout: t[(i*L + j)*K + c], entries with i > j unused. */
+/* Returns T* (+inf when no plan is feasible, S_out = 0).                    */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  int L, K, D, B;
+  const int32_t* dev;
+  const float* t;
+  int S;
+  int32_t end[64], choice[64];
+  double best;
+  int best_S;
+  int32_t best_end[64], best_choice[64];
+} orc_search;
+
+static void search_rec(orc_search* s, int k, int d) {
+  if (k == s->L) {
+    if (d != 0 || s->S == 0) return;
+    int64_t ptr[2] = {0, s->S};
+    int32_t idx[64];
+    int a = 0;
+    for (int i = 0; i < s->S; ++i) {
+      idx[i] = (int32_t)(((int64_t)a * s->L + s->end[i]) * s->K + s->choice[i]);
+      a = s->end[i] + 1;
+    }
+    int32_t B = s->B;
+    double T;
+    orc_plan_T(1, ptr, idx, &B, s->t, (int64_t)s->L * s->L * s->K, &T);
+    if (T < s->best) {
+      s->best = T;
+      s->best_S = s->S;
+      for (int i = 0; i < s->S; ++i) { s->best_end[i] = s->end[i]; s->best_choice[i] = s->choice[i]; }
+    }
+    return;
+  }
+  if (d <= 0 || s->S >= 64) return;
+  for (int j = k; j < s->L; ++j)
+    for (int c = 0; c < s->K; ++c) {
+      float v = s->t[((int64_t)k * s->L + j) * s->K + c];
+      if (!(isfinite(v) && v >= 0.0f) || s->dev[c] > d) continue;
+      s->end[s->S] = j;
+      s->choice[s->S] = c;
+      s->S++;
+      search_rec(s, j + 1, d - s->dev[c]);
+      s->S--;
+    }
+}
+
+double orc_plan_search(int L, int K, const int32_t* dev, int D, const float* t, int B,
+                       int32_t* S_out, int32_t* stage_end, int32_t* stage_choice) {
+  orc_search s;
+  memset(&s, 0, sizeof(s));
+  s.L = L; s.K = K; s.D = D; s.B = B; s.dev = dev; s.t = t;
+  s.best = INFINITY;
+  for (int c = 0; c < K; ++c)
+    if (dev[c] < 1) { *S_out = 0; return NAN; }
+  if (L >= 1 && L <= 64 && B >= 1) search_rec(&s, 0, D);
+  *S_out = s.best_S;
+  for (int i = 0; i < s.best_S; ++i) { stage_end[i] = s.best_end[i]; stage_choice[i] = s.best_choice[i]; }
+  return s.best;
+}

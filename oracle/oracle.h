@@ -79,6 +79,8 @@ int orc_forward_k(const orc_cfg* c, const float* blob, int n, int e, const int32
 void orc_plan_T(int64_t P, const int64_t* plan_ptr, const int32_t* plan_stage,
                 const int32_t* B, const float* t, int64_t num_stages, double* T);
 int64_t orc_argmin(int64_t n, const double* T);
+double orc_plan_search(int L, int K, const int32_t* dev, int D, const float* t, int B,
+                       int32_t* S_out, int32_t* stage_end, int32_t* stage_choice);
 
 #ifdef __cplusplus
 }
