@@ -296,6 +296,52 @@ PREDTOP_API predtop_status predtop_plan_argmin(int64_t num_plans, const double* 
                                    void* workspace, size_t ws_bytes, void* cuda_stream);
 
 /* Misc. */
+/* ---------------------------------------------------------------------------
+ * Inter-stage plan search over a shared stage table.
+ * Alpa's inter-operator optimizer picks the pipeline plan under the
+ * 1F1B model; it enumerates all stages on all submeshes; P:222:
+ * PredTOP predicts every stage's latency on every mesh, then applies the
+ * pipeline model (Eqn 4).  A plan slices layers 0..L-1 into S >= 1
+ * contiguous stages [a_s, b_s], gives stage s a choice c_s (a mesh and
+ * intra-op configuration, Tables II-III) that uses
+ * choice_devices[c_s] devices, uses every device (sum = num_devices), and
+ * costs T = sum_s t_s + (B-1) max_s t_s with t_s = table[a_s][b_s][c_s].
+ * The call returns, per problem, the minimum T over all plans and one plan
+ * attaining it (reading R20 in DESIGN.md; Alpa's t_max-enumeration DP).
+ *  num_problems P >= 1; num_layers L in [1, 64]; num_choices K in [1, 32];
+ *  choice_devices[K]   [host] int32, each >= 1
+ *  num_devices D       [1, 64]
+ *  stage_latency       device fp32 [num_tables][L][L][K]: entry (i, j, c) is
+ *                      the latency of layers i..j on choice c; an entry is
+ *                      feasible iff finite and >= 0 (use +inf for a stage that
+ *                      does not fit a mesh); entries with i > j are ignored
+ *  problem_table[P]    device int32, nullable (then problem p uses table p)
+ *  microbatches[P]     device int32, B >= 1
+ *  T_out[P]            device fp64: T*; +inf if no plan exists; NaN for an
+ *                      invalid problem (table index out of range or B < 1)
+ *  num_stages_out[P]   device int32: S of the returned plan (0 if none)
+ *  stage_end_out[P][L], stage_choice_out[P][L]  device int32: b_s and c_s for
+ *                      s < S (a_0 = 0, a_{s+1} = b_s + 1); the rest untouched
+ *  workspace           device, >= predtop_plan_search_workspace(P, L, K) bytes,
+ *                      256-byte aligned
+ * Exactness: T* is the exact minimum of Eqn 4 over all plans whenever the
+ * fp64 sums of fp32 latencies are exact (every feasible latency within a
+ * factor 2^24 of the largest), e.g. bit-identical to exhaustive enumeration;
+ * among plans with equal T the one returned is the first in (t_max, j, c)
+ * order (deterministic).  Host-checkable argument errors -> INVALID_ARG;
+ * otherwise stream-ordered, no synchronisation. */
+#define PREDTOP_SEARCH_MAX_LAYERS 64
+#define PREDTOP_SEARCH_MAX_CHOICES 32
+#define PREDTOP_SEARCH_MAX_DEVICES 64
+PREDTOP_API size_t predtop_plan_search_workspace(int64_t num_problems, int32_t num_layers, int32_t num_choices);
+PREDTOP_API predtop_status predtop_plan_search(int64_t num_problems, int32_t num_layers, int32_t num_choices,
+                                               const int32_t* choice_devices, int32_t num_devices,
+                                               const float* stage_latency, int64_t num_tables,
+                                               const int32_t* problem_table, const int32_t* microbatches,
+                                               double* T_out, int32_t* num_stages_out,
+                                               int32_t* stage_end_out, int32_t* stage_choice_out,
+                                               void* workspace, size_t ws_bytes, void* cuda_stream);
+
 PREDTOP_API const char* predtop_status_string(predtop_status s);
 PREDTOP_API const char* predtop_last_error(void); /* thread-local */
 PREDTOP_API int predtop_abi_version(void);

@@ -558,6 +558,46 @@ predtop_status predtop_plan_latency(int64_t num_plans, const int64_t* plan_ptr,
 
 size_t predtop_plan_argmin_workspace(int64_t) { return 256; }
 
+size_t predtop_plan_search_workspace(int64_t num_problems, int32_t num_layers, int32_t num_choices) {
+  if (num_problems < 1 || num_layers < 1 || num_layers > PREDTOP_SEARCH_MAX_LAYERS || num_choices < 1 ||
+      num_choices > PREDTOP_SEARCH_MAX_CHOICES)
+    return 0;
+  return search_workspace_bytes(num_problems, num_layers, num_choices);
+}
+
+predtop_status predtop_plan_search(int64_t num_problems, int32_t num_layers, int32_t num_choices,
+                                   const int32_t* choice_devices, int32_t num_devices,
+                                   const float* stage_latency, int64_t num_tables,
+                                   const int32_t* problem_table, const int32_t* microbatches,
+                                   double* T_out, int32_t* num_stages_out, int32_t* stage_end_out,
+                                   int32_t* stage_choice_out, void* workspace, size_t ws_bytes,
+                                   void* cuda_stream) {
+  const size_t need = predtop_plan_search_workspace(num_problems, num_layers, num_choices);
+  if (need == 0) {
+    set_error("plan_search: bad sizes (P=%lld L=%d K=%d)", (long long)num_problems, num_layers, num_choices);
+    return PREDTOP_ERR_INVALID_ARG;
+  }
+  if (num_devices < 1 || num_devices > PREDTOP_SEARCH_MAX_DEVICES || num_tables < 1) {
+    set_error("plan_search: num_devices %d / num_tables %lld out of range", num_devices, (long long)num_tables);
+    return PREDTOP_ERR_INVALID_ARG;
+  }
+  if (!choice_devices || !stage_latency || !microbatches || !T_out || !num_stages_out || !stage_end_out ||
+      !stage_choice_out || !workspace) {
+    set_error("plan_search: NULL argument");
+    return PREDTOP_ERR_INVALID_ARG;
+  }
+  for (int c = 0; c < num_choices; ++c)
+    if (choice_devices[c] < 1) { set_error("plan_search: choice_devices[%d] < 1", c); return PREDTOP_ERR_INVALID_ARG; }
+  if (((uintptr_t)workspace & 255) || ws_bytes < need) {
+    set_error("plan_search: workspace too small or misaligned (%zu < %zu)", ws_bytes, need);
+    return PREDTOP_ERR_WORKSPACE;
+  }
+  if (!device_ok()) return PREDTOP_ERR_CUDA;
+  return search_launch(num_problems, num_layers, num_choices, choice_devices, num_devices, stage_latency,
+                       num_tables, problem_table, microbatches, T_out, num_stages_out, stage_end_out,
+                       stage_choice_out, workspace, S(cuda_stream));
+}
+
 predtop_status predtop_plan_argmin(int64_t num_plans, const double* T, int64_t* best_out,
                                    void* workspace, size_t ws_bytes, void* cuda_stream) {
   (void)workspace;

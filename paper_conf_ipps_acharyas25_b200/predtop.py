@@ -29,6 +29,7 @@ NO_SYNC = 1
 POOL_SUM, POOL_MEAN = 0, 1
 MAX_NODES = 65536
 MAX_PLAN_STAGES = 64
+SEARCH_MAX_LAYERS, SEARCH_MAX_CHOICES, SEARCH_MAX_DEVICES = 64, 32, 64
 
 
 class PredtopError(RuntimeError):
@@ -73,6 +74,8 @@ _SIGS = {
     "predtop_plan_latency": (_I32, [_I64, _P, _P, _P, _P, _I64, _P, _P, _SZ, _U32, _P, _P]),
     "predtop_plan_argmin_workspace": (_SZ, [_I64]),
     "predtop_plan_argmin": (_I32, [_I64, _P, _P, _P, _SZ, _P]),
+    "predtop_plan_search_workspace": (_SZ, [_I64, _I32, _I32]),
+    "predtop_plan_search": (_I32, [_I64, _I32, _I32, _P, _I32, _P, _I64, _P, _P, _P, _P, _P, _P, _P, _SZ, _P]),
     "predtop_status_string": (ctypes.c_char_p, [_I32]),
     "predtop_last_error": (ctypes.c_char_p, []),
     "predtop_abi_version": (ctypes.c_int, []),
@@ -326,3 +329,55 @@ class Plans:
         T = self.T[:self.num_plans] if T is None else T
         predtop_plan_argmin(T, self.best, stream)
         return self.best
+
+
+def predtop_plan_search(stage_latency: torch.Tensor, choice_devices, num_devices: int,
+                        microbatches: torch.Tensor, problem_table: Optional[torch.Tensor], T_out, S_out,
+                        end_out, choice_out, workspace: torch.Tensor, stream=None):
+    """Raw call: stage_latency [num_tables, L, L, K] fp32 (device)."""
+    nt, L, L2, K = stage_latency.shape
+    assert L == L2
+    dev = (ctypes.c_int32 * K)(*[int(x) for x in choice_devices])
+    _check(lib().predtop_plan_search(microbatches.numel(), L, K, dev, int(num_devices), _ptr(stage_latency), nt,
+                                     _ptr(problem_table), _ptr(microbatches), _ptr(T_out), _ptr(S_out),
+                                     _ptr(end_out), _ptr(choice_out), _ptr(workspace), workspace.numel(),
+                                     _stream(stream)))
+
+
+class PlanSearch:
+    """Inter-stage plan search for P problems over shared
+    stage tables: buffers for predtop_plan_search plus host-side decoding."""
+
+    def __init__(self, num_problems: int, num_layers: int, choice_devices, num_devices: int, device="cuda"):
+        self.P, self.L = int(num_problems), int(num_layers)
+        self.choice_devices = [int(x) for x in choice_devices]
+        self.K, self.D = len(self.choice_devices), int(num_devices)
+        need = lib().predtop_plan_search_workspace(self.P, self.L, self.K)
+        if need == 0:
+            raise PredtopError(INVALID_ARG, "plan search sizes out of range")
+        self.workspace = torch.empty(need, dtype=torch.uint8, device=device)
+        self.T = torch.empty(self.P, dtype=torch.float64, device=device)
+        self.S = torch.empty(self.P, dtype=torch.int32, device=device)
+        self.ends = torch.zeros((self.P, self.L), dtype=torch.int32, device=device)
+        self.choices = torch.zeros((self.P, self.L), dtype=torch.int32, device=device)
+
+    def run(self, stage_latency: torch.Tensor, microbatches: torch.Tensor,
+            problem_table: Optional[torch.Tensor] = None, stream=None):
+        predtop_plan_search(stage_latency, self.choice_devices, self.D, microbatches, problem_table,
+                            self.T, self.S, self.ends, self.choices, self.workspace, stream)
+        return self.T
+
+    def plans(self):
+        """Host decode: per problem (T*, [(first, last, choice), ...])."""
+        T = self.T.cpu().numpy()
+        S = self.S.cpu().numpy()
+        E = self.ends.cpu().numpy()
+        C = self.choices.cpu().numpy()
+        out = []
+        for p in range(self.P):
+            st, a = [], 0
+            for s in range(int(S[p])):
+                st.append((a, int(E[p, s]), int(C[p, s])))
+                a = int(E[p, s]) + 1
+            out.append((float(T[p]), st))
+        return out
