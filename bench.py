@@ -135,7 +135,7 @@ def run_reference(args, rank):
     from paper_conf_ipps_acharyas25_b200 import synth
     import oracle
     oracle.build()
-    gcfg = "gpt" if args.config == "sweep" else args.config  # sweep stages are GPT-style pool graphs
+    gcfg = "gpt" if args.config in ("sweep", "search") else args.config  # sweep stages are GPT-style pool graphs
     cfg = synth.MODEL_CONFIGS[gcfg]
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
     cores = host_cores()
@@ -180,7 +180,7 @@ def stages_per_plan(G: int) -> int:
 
 
 def workload_config(args):
-    cfg_name = "gpt" if args.config == "sweep" else args.config
+    cfg_name = "gpt" if args.config in ("sweep", "search") else args.config
     from paper_conf_ipps_acharyas25_b200 import synth
     c = synth.MODEL_CONFIGS[cfg_name]
     base = {"layers": c["num_layers"], "d_model": c["d_model"], "heads": c["num_heads"], "d_ff": c["d_ff"],
@@ -203,7 +203,7 @@ def workload_config(args):
 
 
 # ----------------------------------------------------------------- main leg
-DEFAULT_GRAPHS = {"tiny": 4, "gpt": 1024, "moe": 512, "16k": 1, "sweep": 0}
+DEFAULT_GRAPHS = {"tiny": 4, "gpt": 1024, "moe": 512, "16k": 1, "sweep": 0, "search": 0}
 
 
 class Ctx:
@@ -533,6 +533,113 @@ def run_batch(args, ctx):
         emit(line, args)
 
 
+def run_search(args, ctx):
+    """the shared stage table + plan search.  All L(L+1)/2
+    layer-range stages of GPT-3 1.3B (24 layers, Table IV) scored by one
+    model per Table III mesh choice (6), stage DAGs cost-balanced over the
+    ranks, one exact sum-all-reduce of the stage table, then the plan search
+    on Platform 2's 4 GPUs for B in {1..64} (7 problems)."""
+    import torch
+    from paper_conf_ipps_acharyas25_b200 import synth, stage_table
+    pt, L, dev, world, rank = ctx.pt, ctx.L, ctx.dev, ctx.world, ctx.rank
+    nl = args.layers
+    host = synth.layer_range_stages("gpt", nl)
+    cfgs = synth.mesh_model_configs("search", len(synth.MESH_CHOICES))
+    blobs = [synth.pack_weights(c, synth.model_weights(c)) for c in cfgs]
+    devs = [d for _, d in synth.MESH_CHOICES]
+    Bs = [1, 2, 4, 8, 16, 32, 64]
+    sts = stage_table.StageTableSearch(pt, cfgs, blobs, host, nl, devs, 4, Bs, rank=rank, world=world,
+                                       device=dev, hops=args.hops)
+    K, NT = len(cfgs), sts.NT
+    step = sts.step
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    tab = sts.table.cpu().numpy()
+    assert np.isfinite(tab).all() and (tab > 0).all(), "stage latencies must be positive (R17)"
+    run, launches_per_step = (step, None) if args.eager else ctx.capture(step)
+    run()
+    torch.cuda.synchronize()
+    with ClockSampler(ctx.dev_index) as clk:
+        ms = ctx.timed(run, args.steps)
+    total_ms = ctx.max_over_ranks(sum(ms))
+    value = K * NT * args.steps / (total_ms / 1e3)          # stage-DAG scorings, all ranks
+    searches = len(Bs) * args.steps / (total_ms / 1e3)
+    plans = sts.search.plans()
+    # e2e: the stage DAGs' inputs from pinned host memory every step, T* and plans back
+    db = sts.db
+    pin = None
+    if db is not None:
+        loc = sts.local
+        pin = {"node_ptr": torch.from_numpy(loc.node_ptr).pin_memory(),
+               "edge_ptr": torch.from_numpy(loc.edge_ptr).pin_memory(),
+               "src": torch.from_numpy(loc.src).pin_memory(), "dst": torch.from_numpy(loc.dst).pin_memory(),
+               "feats": torch.from_numpy(np.ascontiguousarray(loc.feats).view(np.uint8).reshape(-1).copy()).pin_memory()}
+    outs = [torch.empty(len(Bs), dtype=torch.float64).pin_memory(),
+            torch.empty((len(Bs), nl), dtype=torch.int32).pin_memory(),
+            torch.empty((len(Bs), nl), dtype=torch.int32).pin_memory(),
+            torch.empty(len(Bs), dtype=torch.int32).pin_memory()]
+
+    def e2e_step():
+        if pin is not None:
+            for k_, t_ in pin.items():
+                getattr(db, k_ if k_ != "feats" else "feats").copy_(t_, non_blocking=True)
+        step()
+        outs[0].copy_(sts.search.T, non_blocking=True)
+        outs[1].copy_(sts.search.ends, non_blocking=True)
+        outs[2].copy_(sts.search.choices, non_blocking=True)
+        outs[3].copy_(sts.search.S, non_blocking=True)
+
+    e2e_run = e2e_step if args.eager else ctx.capture(e2e_step)[0]
+    e2e_run()
+    ms_e2e = ctx.timed(e2e_run, max(5, args.steps // 2))
+    tot_e2e = ctx.max_over_ranks(sum(ms_e2e))
+    e2e_value = K * NT * len(ms_e2e) / (tot_e2e / 1e3)
+    h2d = ctx.sum_over_ranks(sum(t.numel() * t.element_size() for t in pin.values()) if pin else 0) / max(world, 1)
+    d2h = sum(t.numel() * t.element_size() for t in outs)
+    prof = ctx.profile(step, max(3, args.steps // 4))
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        cores = host_cores()
+        gs = list(range(0, NT, max(1, NT // (2 * cores))))[:2 * cores]
+        t0 = time.perf_counter()
+        oracle.forward_batch(cfgs[0], blobs[0], host, graphs=gs, threads=cores)
+        wall = time.perf_counter() - t0
+        # one oracle forward per (stage, choice); rate in stage-DAG scorings/s
+        cpu = {"value": len(gs) / wall, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{len(gs)} of the {NT} layer-range stages (every {max(1, NT // (2 * cores))}th, "
+                         f"{min(host.sizes[gs])}-{max(host.sizes[gs])} nodes) on one mesh model, fp64 C "
+                         f"oracle, {cores} threads, {wall:.1f} s; the plan search itself is not timed"}
+    if rank == 0:
+        for k in prof:
+            prof[k]["share"] = prof[k]["ms_per_step"] / (total_ms / args.steps)
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f16", "data": "synthetic",
+                "config": {"workload": f"search: all {NT} layer-range stages of GPT-3 1.3B ({nl} layers, Table IV; "
+                                       f"{int(host.sizes.min())}-{int(host.sizes.max())} nodes) x {K} mesh models "
+                                       f"(Table III), stage table all-reduce, plan search on 4 GPUs (Platform 2) "
+                                       f"for B in {Bs}",
+                           "stages": NT, "mesh_choices": K, "choice_devices": devs, "cluster_devices": 4,
+                           "microbatches": Bs,
+                           "parallelism": f"stage-sharded x{world} (cost-balanced), sum-all-reduce of the stage table",
+                           "l2": "not flushed: one step's inputs and activations (~0.4 GB) exceed the 126 MB L2",
+                           "dagra_k": args.hops if args.hops > 0 else "inf",
+                           "layers": cfgs[0]["num_layers"], "d_model": cfgs[0]["d_model"],
+                           "heads": cfgs[0]["num_heads"], "d_ff": cfgs[0]["d_ff"]},
+                "searches_per_s": searches,
+                "best_plans": {str(B): {"T": T, "stages": st} for B, (T, st) in zip(Bs, plans)},
+                "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+                        "d2h_bytes_per_step": int(d2h)},
+                "gpu_launches": int((launches_per_step or 0) * args.steps),
+                "launch_mode": "eager" if args.eager else "cuda_graph",
+                "roofline": None, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
+        emit(line, args)
+
+
 def run_sweep(args, ctx, pool):
     """configs[4]: an owned-mode plan sweep of args.plans plans, cost-balanced
     over the ranks (strong scaling: the total is fixed).  One step = build +
@@ -679,7 +786,8 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="gpt", choices=["tiny", "gpt", "moe", "16k", "sweep"])
+    ap.add_argument("--config", default="gpt", choices=["tiny", "gpt", "moe", "16k", "sweep", "search"])
+    ap.add_argument("--layers", type=int, default=24, help="search: model layers (GPT-3 1.3B: 24)")
     ap.add_argument("--graphs", type=int, default=None, help="stage graphs per GPU (default per config)")
     ap.add_argument("--plans", type=int, default=100000, help="sweep: total candidate plans")
     ap.add_argument("--chunk", type=int, default=4096, help="sweep: stage graphs per build+forward launch")
@@ -708,6 +816,8 @@ def main():
     ctx = Ctx(args)
     if args.config == "sweep":
         run_sweep(args, ctx, pool)
+    elif args.config == "search":
+        run_search(args, ctx)
     else:
         run_batch(args, ctx)
     ctx.finish()

@@ -311,10 +311,14 @@ PREDTOP_API predtop_status predtop_plan_argmin(int64_t num_plans, const double* 
  *  num_problems P >= 1; num_layers L in [1, 64]; num_choices K in [1, 32];
  *  choice_devices[K]   [host] int32, each >= 1
  *  num_devices D       [1, 64]
- *  stage_latency       device fp32 [num_tables][L][L][K]: entry (i, j, c) is
- *                      the latency of layers i..j on choice c; an entry is
- *                      feasible iff finite and >= 0 (use +inf for a stage that
- *                      does not fit a mesh); entries with i > j are ignored
+ *  stage_latency       device fp32 [num_tables][K][table_stride]: the latency
+ *                      of layers i..j (i <= j) on choice c is element
+ *                      tri(i, j) = i*L - i*(i-1)/2 + (j - i) of row c (the
+ *                      packed upper triangle, so a stage_forward over the
+ *                      L(L+1)/2 stage DAGs in that order writes row c
+ *                      directly); an entry is feasible iff finite and >= 0
+ *                      (use +inf for a stage that does not fit a mesh)
+ *  table_stride        >= L(L+1)/2 (lets row c be an all-gather output)
  *  problem_table[P]    device int32, nullable (then problem p uses table p)
  *  microbatches[P]     device int32, B >= 1
  *  T_out[P]            device fp64: T*; +inf if no plan exists; NaN for an
@@ -336,7 +340,8 @@ PREDTOP_API predtop_status predtop_plan_argmin(int64_t num_plans, const double* 
 PREDTOP_API size_t predtop_plan_search_workspace(int64_t num_problems, int32_t num_layers, int32_t num_choices);
 PREDTOP_API predtop_status predtop_plan_search(int64_t num_problems, int32_t num_layers, int32_t num_choices,
                                                const int32_t* choice_devices, int32_t num_devices,
-                                               const float* stage_latency, int64_t num_tables,
+                                               const float* stage_latency, int64_t table_stride,
+                                               int64_t num_tables,
                                                const int32_t* problem_table, const int32_t* microbatches,
                                                double* T_out, int32_t* num_stages_out,
                                                int32_t* stage_end_out, int32_t* stage_choice_out,

@@ -567,7 +567,7 @@ size_t predtop_plan_search_workspace(int64_t num_problems, int32_t num_layers, i
 
 predtop_status predtop_plan_search(int64_t num_problems, int32_t num_layers, int32_t num_choices,
                                    const int32_t* choice_devices, int32_t num_devices,
-                                   const float* stage_latency, int64_t num_tables,
+                                   const float* stage_latency, int64_t table_stride, int64_t num_tables,
                                    const int32_t* problem_table, const int32_t* microbatches,
                                    double* T_out, int32_t* num_stages_out, int32_t* stage_end_out,
                                    int32_t* stage_choice_out, void* workspace, size_t ws_bytes,
@@ -575,6 +575,10 @@ predtop_status predtop_plan_search(int64_t num_problems, int32_t num_layers, int
   const size_t need = predtop_plan_search_workspace(num_problems, num_layers, num_choices);
   if (need == 0) {
     set_error("plan_search: bad sizes (P=%lld L=%d K=%d)", (long long)num_problems, num_layers, num_choices);
+    return PREDTOP_ERR_INVALID_ARG;
+  }
+  if (table_stride < (int64_t)num_layers * (num_layers + 1) / 2) {
+    set_error("plan_search: table_stride %lld < L(L+1)/2", (long long)table_stride);
     return PREDTOP_ERR_INVALID_ARG;
   }
   if (num_devices < 1 || num_devices > PREDTOP_SEARCH_MAX_DEVICES || num_tables < 1) {
@@ -594,7 +598,7 @@ predtop_status predtop_plan_search(int64_t num_problems, int32_t num_layers, int
   }
   if (!device_ok()) return PREDTOP_ERR_CUDA;
   return search_launch(num_problems, num_layers, num_choices, choice_devices, num_devices, stage_latency,
-                       num_tables, problem_table, microbatches, T_out, num_stages_out, stage_end_out,
+                       table_stride, num_tables, problem_table, microbatches, T_out, num_stages_out, stage_end_out,
                        stage_choice_out, workspace, S(cuda_stream));
 }
 

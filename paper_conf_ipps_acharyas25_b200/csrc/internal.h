@@ -177,9 +177,9 @@ predtop_status plan_launch(int64_t P, const int64_t* plan_ptr, const int32_t* pl
 predtop_status argmin_launch(int64_t n, const double* T, int64_t* best, cudaStream_t st);
 
 // ---- search.cu (inter-stage plan search)
-size_t search_workspace_bytes(int64_t P, int L, int K);
+size_t search_workspace_bytes(int64_t P, int L, int K);  // [P][K * L(L+1)/2] candidate T
 predtop_status search_launch(int64_t P, int L, int K, const int32_t* dev, int D, const float* t,
-                             int64_t num_tables, const int32_t* table_of, const int32_t* B,
+                             int64_t stride, int64_t num_tables, const int32_t* table_of, const int32_t* B,
                              double* T_out, int32_t* S_out, int32_t* end_out, int32_t* choice_out,
                              void* ws, cudaStream_t st);
 

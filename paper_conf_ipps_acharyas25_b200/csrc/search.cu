@@ -15,6 +15,9 @@
 // the optimal plan p* is admissible at t_max = max(p*), and every candidate
 // value bounds the true Eqn 4 of the plan it stands for from above.
 //
+// Table layout: [num_tables][K][stride], stage (i, j) of choice c at
+// c * stride + tri(i, j), tri(i, j) = i L - i (i-1)/2 + (j - i).
+//
 //   k_search_cand   one warp per (problem, candidate): the DP in shared memory,
 //                   lanes over the (j, c) transitions, warp min-reductions
 //   k_search_pick   one CTA per problem: argmin over candidates by
@@ -37,12 +40,14 @@ constexpr double kInf = __builtin_huge_val();
 struct SearchArgs {
   int L, K, D;
   int32_t dev[PREDTOP_SEARCH_MAX_CHOICES];
-  const float* t;           // [num_tables][L][L][K]
+  const float* t;           // [num_tables][K][stride], stage (i, j) at tri(i, j) of row c
+  int64_t stride;           // >= NT
   int64_t num_tables;
   const int32_t* table_of;  // [P] or nullptr (problem p uses table p)
   const int32_t* B;         // [P]
   int64_t P;
-  int64_t C;                // candidates per problem = L*L*K (entries with i > j are never feasible)
+  int NT;                   // L(L+1)/2 stages
+  int64_t C;                // candidates per problem = K * NT (every table entry)
   double* Tc;               // [P][C]
 };
 
@@ -50,7 +55,7 @@ __device__ __forceinline__ bool problem_ok(const SearchArgs& a, int64_t p, const
   const int64_t tb = a.table_of ? (int64_t)a.table_of[p] : p;
   *B = a.B[p];
   if (tb < 0 || tb >= a.num_tables || *B < 1) return false;
-  *tp = a.t + tb * (int64_t)a.L * a.L * a.K;
+  *tp = a.t + tb * (int64_t)a.K * a.stride;
   return true;
 }
 
@@ -65,7 +70,7 @@ __device__ double warp_dp(const SearchArgs& a, const int32_t* dev, const float* 
   __syncwarp();
   for (int k = L - 1; k >= 0; --k) {
     const int nitems = (L - k) * K;
-    const float* row = tp + (size_t)k * L * K;  // t[k][*][*]
+    const int tk = k * L - k * (k - 1) / 2;  // tri(k, k): stages (k, j) are tk + (j - k)
     if (lane == 0) {
       F[k * D1] = kInf;
       if (arg) arg[k * D1] = -1;
@@ -77,7 +82,7 @@ __device__ double warp_dp(const SearchArgs& a, const int32_t* dev, const float* 
         const int j = k + it / K, c = it - (it / K) * K;
         const int dv = dev[c];
         if (dv > d) continue;
-        const float v = __ldg(row + (size_t)j * K + c);
+        const float v = __ldg(tp + (size_t)c * a.stride + tk + (j - k));
         if (!(v >= 0.f && v <= tmax)) continue;  // infeasible (NaN, < 0, inf) or above the bound
         const double f = F[(j + 1) * D1 + d - dv];
         if (f == kInf) continue;
@@ -116,10 +121,10 @@ __global__ void __launch_bounds__(128) k_search_cand(SearchArgs a) {
     if (!problem_ok(a, p, &tp, &B)) {
       T = __longlong_as_double(0x7ff8000000000000ll);  // NaN: invalid problem
     } else {
-      const int c = (int)(ci % a.K), j = (int)((ci / a.K) % a.L), i = (int)(ci / ((int64_t)a.K * a.L));
-      const float tmax = tp[ci];
+      const int c = (int)(ci / a.NT), s = (int)(ci - (int64_t)c * a.NT);
+      const float tmax = tp[(size_t)c * a.stride + s];
       T = kInf;
-      if (i <= j && tmax >= 0.f && tmax < __int_as_float(0x7f800000)) {
+      if (tmax >= 0.f && tmax < __int_as_float(0x7f800000)) {
         const double f = warp_dp(a, s_dev, tp, tmax, F, nullptr);
         if (f != kInf) T = __dadd_rn(f, __dmul_rn((double)(B - 1), (double)tmax));
       }
@@ -160,7 +165,8 @@ __global__ void __launch_bounds__(256) k_search_pick(SearchArgs a, double* T_out
   for (int64_t ci = threadIdx.x; ci < a.C; ci += blockDim.x) {
     const double T = Tc[ci];
     if (!(T < kInf)) continue;
-    const float tm = tp[ci];
+    const int c = (int)(ci / a.NT);
+    const float tm = tp[(size_t)c * a.stride + (ci - (int64_t)c * a.NT)];
     if (cand_better(T, tm, ci, bT, btm, bci)) { bT = T; btm = tm; bci = ci; }
   }
 #pragma unroll
@@ -214,19 +220,20 @@ __global__ void __launch_bounds__(256) k_search_pick(SearchArgs a, double* T_out
 }  // namespace
 
 size_t search_workspace_bytes(int64_t P, int L, int K) {
-  return align_up((size_t)P * (size_t)L * L * K * sizeof(double), 256);
+  return align_up((size_t)P * (size_t)K * ((size_t)L * (L + 1) / 2) * sizeof(double), 256);
 }
 
 predtop_status search_launch(int64_t P, int L, int K, const int32_t* dev, int D, const float* t,
-                             int64_t num_tables, const int32_t* table_of, const int32_t* B,
+                             int64_t stride, int64_t num_tables, const int32_t* table_of, const int32_t* B,
                              double* T_out, int32_t* S_out, int32_t* end_out, int32_t* choice_out,
                              void* ws, cudaStream_t st) {
   if (P <= 0) return PREDTOP_OK;
   SearchArgs a{};
   a.L = L; a.K = K; a.D = D;
   for (int c = 0; c < PREDTOP_SEARCH_MAX_CHOICES; ++c) a.dev[c] = c < K ? dev[c] : 1 << 20;
-  a.t = t; a.num_tables = num_tables; a.table_of = table_of; a.B = B; a.P = P;
-  a.C = (int64_t)L * L * K;
+  a.t = t; a.stride = stride; a.num_tables = num_tables;
+  a.NT = L * (L + 1) / 2; a.table_of = table_of; a.B = B; a.P = P;
+  a.C = (int64_t)K * a.NT;
   a.Tc = reinterpret_cast<double*>(ws);
   const size_t fbytes = (size_t)(L + 1) * (D + 1) * sizeof(double);
   static size_t attr_cand = 0, attr_pick = 0;

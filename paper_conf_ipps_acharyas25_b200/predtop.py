@@ -75,7 +75,7 @@ _SIGS = {
     "predtop_plan_argmin_workspace": (_SZ, [_I64]),
     "predtop_plan_argmin": (_I32, [_I64, _P, _P, _P, _SZ, _P]),
     "predtop_plan_search_workspace": (_SZ, [_I64, _I32, _I32]),
-    "predtop_plan_search": (_I32, [_I64, _I32, _I32, _P, _I32, _P, _I64, _P, _P, _P, _P, _P, _P, _P, _SZ, _P]),
+    "predtop_plan_search": (_I32, [_I64, _I32, _I32, _P, _I32, _P, _I64, _I64, _P, _P, _P, _P, _P, _P, _P, _SZ, _P]),
     "predtop_status_string": (ctypes.c_char_p, [_I32]),
     "predtop_last_error": (ctypes.c_char_p, []),
     "predtop_abi_version": (ctypes.c_int, []),
@@ -331,17 +331,25 @@ class Plans:
         return self.best
 
 
-def predtop_plan_search(stage_latency: torch.Tensor, choice_devices, num_devices: int,
+def predtop_plan_search(stage_latency: torch.Tensor, num_layers: int, choice_devices, num_devices: int,
                         microbatches: torch.Tensor, problem_table: Optional[torch.Tensor], T_out, S_out,
                         end_out, choice_out, workspace: torch.Tensor, stream=None):
-    """Raw call: stage_latency [num_tables, L, L, K] fp32 (device)."""
-    nt, L, L2, K = stage_latency.shape
-    assert L == L2
+    """Raw call: stage_latency [num_tables, K, stride] fp32 (device), stage
+    (i, j) of choice c at [.., c, tri(i, j)] (include/predtop.h)."""
+    nt, K, stride = stage_latency.shape
+    assert stage_latency.is_contiguous()
     dev = (ctypes.c_int32 * K)(*[int(x) for x in choice_devices])
-    _check(lib().predtop_plan_search(microbatches.numel(), L, K, dev, int(num_devices), _ptr(stage_latency), nt,
-                                     _ptr(problem_table), _ptr(microbatches), _ptr(T_out), _ptr(S_out),
-                                     _ptr(end_out), _ptr(choice_out), _ptr(workspace), workspace.numel(),
-                                     _stream(stream)))
+    _check(lib().predtop_plan_search(microbatches.numel(), int(num_layers), K, dev, int(num_devices),
+                                     _ptr(stage_latency), stride, nt, _ptr(problem_table), _ptr(microbatches),
+                                     _ptr(T_out), _ptr(S_out), _ptr(end_out), _ptr(choice_out), _ptr(workspace),
+                                     workspace.numel(), _stream(stream)))
+
+
+def pack_stage_table(dense: np.ndarray) -> np.ndarray:
+    """Host helper: dense [L, L, K] (entry (i, j, c), i <= j) -> packed [K, L(L+1)/2]."""
+    L, _, K = dense.shape
+    iu, ju = np.triu_indices(L)  # row-major upper triangle = tri(i, j) order
+    return np.ascontiguousarray(dense[iu, ju, :].T, dtype=np.float32)
 
 
 class PlanSearch:
@@ -363,7 +371,8 @@ class PlanSearch:
 
     def run(self, stage_latency: torch.Tensor, microbatches: torch.Tensor,
             problem_table: Optional[torch.Tensor] = None, stream=None):
-        predtop_plan_search(stage_latency, self.choice_devices, self.D, microbatches, problem_table,
+        """stage_latency: [num_tables, K, stride] (pack_stage_table layout)."""
+        predtop_plan_search(stage_latency, self.L, self.choice_devices, self.D, microbatches, problem_table,
                             self.T, self.S, self.ends, self.choices, self.workspace, stream)
         return self.T
 

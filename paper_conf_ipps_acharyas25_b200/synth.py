@@ -244,15 +244,18 @@ def _tape(style: str, mb: int, split: int, n_layers: int) -> _Tape:
         return _TAPE_CACHE[key]
     t = _Tape()
     S = 1024
+    t.layer_start = []  # first record of each transformer layer (layer 0 also owns the embedding)
     if style == "gpt":   # GPT-3 1.3B (Table IV): hidden 2048, 32 heads
         Hd, nh = 2048 // split, 32 // split
         x = t.rec("gather", "f16", [mb, S, Hd], [_P([51200 // split, Hd]), _L("i32")])
         for _ in range(n_layers):
+            t.layer_start.append(len(t.recs))
             x = _gpt_layer(t, x, mb, S, Hd, nh)
     elif style == "moe":  # GShard MoE 2.6B (Table IV): hidden 768, 16 heads, 16 experts
         Hd, nh = 768 // split, 16 // split
         x = t.rec("gather", "f16", [mb, S, Hd], [_P([32000 // split, Hd]), _L("i32")])
         for li in range(n_layers):
+            t.layer_start.append(len(t.recs))
             if li % 2 == 1:
                 x = _moe_layer(t, x, mb, S, Hd, nh, 16, 2048 // split)
             else:
@@ -535,6 +538,35 @@ def stage_graph(style: str, n_target: int, seed: int, gid: int):
     return n_target, np.asarray(gb.src, np.int32), np.asarray(gb.dst, np.int32), _feats_of(gb)
 
 
+def layer_range_stages(style: str, num_layers: int, mb: int = 1, split: int = 1):
+    """Every candidate pipeline stage of a num_layers-layer model (P:212-214:
+    Alpa enumerates all stages = contiguous layer ranges): one fwd+bwd stage
+    DAG per (first, last) layer pair, in the packed upper-triangle order the
+    plan-search ABI uses (stage (i, j) at i*L - i*(i-1)/2 + (j - i)).  GPT-3
+    1.3B has 24 layers, GShard MoE 2.6B 32 (Table IV).  Nodes stay in
+    construction (topological) order; no padding."""
+    tape = _tape(style, mb, split, num_layers)
+    ls = list(tape.layer_start) + [len(tape.recs)]
+    ls[0] = 0  # layer 0 includes the embedding gather
+    graphs = []
+    for i in range(num_layers):
+        for j in range(i, num_layers):
+            gb = _build_stage(tape, ls[i], ls[j + 1] - ls[i])
+            graphs.append((len(gb), np.asarray(gb.src, np.int32), np.asarray(gb.dst, np.int32), _feats_of(gb)))
+    return pack_graphs(graphs)
+
+
+def tri_index(i: int, j: int, L: int) -> int:
+    """Packed upper-triangle index of stage (i, j), i <= j < L."""
+    return i * L - i * (i - 1) // 2 + (j - i)
+
+
+# Table III (P:253-262): (mesh, configuration) pairs on Platform 2's 2 nodes x
+# 2 GPUs (P:235); PredTOP trains one model per pair (P:219).  Devices per pair:
+MESH_CHOICES = [("mesh1 single GPU", 1), ("mesh2 2-way DP", 2), ("mesh2 2-way MP", 2),
+                ("mesh3 4-way DP", 4), ("mesh3 2-way DP x 2-way MP", 4), ("mesh3 4-way MP", 4)]
+
+
 # --------------------------------------------------------------------------
 # Hand-made tiny graphs (config 0) and structured test graphs
 # --------------------------------------------------------------------------
@@ -690,7 +722,37 @@ MODEL_CONFIGS = {
                 head_scale=0.007, out_bias=0.0, seed=103),
     "16k": dict(num_layers=4, d_model=128, num_heads=8, d_ff=512, pool=0, ln_eps=1e-5,
                 head_scale=0.25, out_bias=1.0, seed=104),
+    # layer-range stages of the plan search: 191..4495 nodes,
+    # so a smaller head scale keeps the sum-pooled outputs positive (R17);
+    # mesh choice c uses seed 110 + c (one model per mesh)
+    "search": dict(num_layers=4, d_model=128, num_heads=8, d_ff=512, pool=0, ln_eps=1e-5,
+                   head_scale=0.02, out_bias=6.0, seed=110),
 }
+
+
+# R17 for the layer-range stages: the raw (scale 1, bias 0) head output of the
+# untrained search models is close to proportional to the stage size N, with
+# a seed-dependent sign (raw/N in [-0.85, -0.67], [-0.90, -0.64], [0.29, 0.62],
+# [-0.005, 0.17], [-1.43, -1.00], [0.93, 1.33] for seeds 110..115 over the 300
+# GPT-3 stages, tools/head_dist.py on 1xB200); these scales map it to
+# latency-like values ~ f_c N / 100 + 1 (positive on every stage) with
+# f = (1, 0.55, 0.6, 0.3, 0.32, 0.35): more devices, shorter stages, so the
+# best plan depends on B as in Alpa's search (one stage on 4 GPUs for small
+# B, a 2-stage pipeline for large B).
+SEARCH_HEAD_SCALES = [-0.01316, -0.00714, 0.01333, 0.0375, -0.00267, 0.0031]
+
+
+def mesh_model_configs(base: str = "search", num_choices: int = 6) -> List[dict]:
+    """One DAG-Transformer per (mesh, configuration) pair (Table III)."""
+    out = []
+    for c in range(num_choices):
+        cfg = dict(MODEL_CONFIGS[base])
+        cfg["seed"] = cfg["seed"] + c
+        if base == "search":
+            cfg["head_scale"] = SEARCH_HEAD_SCALES[c % len(SEARCH_HEAD_SCALES)]
+            cfg["out_bias"] = 1.0
+        out.append(cfg)
+    return out
 
 
 def weight_shapes(cfg: dict) -> List[Tuple[str, Tuple[int, ...]]]:

@@ -88,3 +88,54 @@ def test_gloo_world2_gather_matches_single_process(oracle_mod, uneven):
     for rank, tb, best in res:
         assert tb == T_ref.tobytes()      # every rank holds the global T, bit-exact
         assert best == best_ref           # same global argmin (ties -> lower id)
+
+
+def _table_worker(rank, world, port, result_q, dense_rows, ranges, dev, D, Bs):
+    """One rank of the shared-stage-table flow (stage_table.py steps 3-4):
+    write its own range of the [K][NT] table, sum-all-reduce, then run the
+    plan search (oracle here) on the gathered table."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    K, NT = dense_rows.shape
+    g0, g1 = ranges[rank]
+    mine = torch.zeros((1, K, NT), dtype=torch.float32)
+    mine[0, :, g0:g1] = torch.from_numpy(dense_rows[:, g0:g1])
+    dist.all_reduce(mine)
+    table = mine[0].numpy()
+    L = int((np.sqrt(8 * NT + 1) - 1) / 2)
+    dense = np.full((L, L, K), np.inf, np.float32)
+    for i in range(L):
+        for j in range(i, L):
+            dense[i, j] = table[:, synth.tri_index(i, j, L)]
+    res = [oracle.plan_search(dense, dev, D, B)[0] for B in Bs]
+    result_q.put((rank, table.tobytes(), res))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_stage_table_allreduce(oracle_mod):
+    from paper_conf_ipps_acharyas25_b200 import stage_table
+    L, K = 7, 3
+    NT = L * (L + 1) // 2
+    r = synth.CounterRng(12, 12)
+    rows = np.asarray([[r.randint(1, 200) / 32.0 for _ in range(NT)] for _ in range(K)], np.float32)
+    sizes = [100 + 50 * i for i in range(NT)]
+    ranges = shard.balanced_ranges(stage_table.stage_costs(sizes, 128), 2)
+    want_table = stage_table.assemble_table_host([(a, b, rows[:, a:b]) for a, b in ranges], K, NT)
+    np.testing.assert_array_equal(want_table, rows)
+    dev, D, Bs = [1, 2, 4], 4, [1, 4, 16]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_table_worker, args=(rk, 2, port, q, rows, ranges, dev, D, Bs)) for rk in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(2)]
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    (_, t0, r0), (_, t1, r1) = res
+    assert t0 == t1 == rows.tobytes()  # the sum of disjoint ranges is exact
+    assert r0 == r1                    # replicated search: identical optima on every rank

@@ -24,12 +24,16 @@ def pt():
     return predtop
 
 
-def _run(pt, tables, dev, D, Bs, table_of=None):
+def _run(pt, tables, dev, D, Bs, table_of=None, pad=0):
     tables = np.ascontiguousarray(tables, np.float32)
     if tables.ndim == 3:
         tables = tables[None]
-    ps = pt.PlanSearch(len(Bs), tables.shape[1], dev, D)
-    t = torch.from_numpy(tables).cuda()
+    L = tables.shape[1]
+    packed = np.stack([pt.pack_stage_table(t) for t in tables])
+    if pad:  # rows with a stride beyond L(L+1)/2 (all-gather layouts)
+        packed = np.concatenate([packed, np.full(packed.shape[:2] + (pad,), -1.0, np.float32)], axis=2)
+    ps = pt.PlanSearch(len(Bs), L, dev, D)
+    t = torch.from_numpy(np.ascontiguousarray(packed)).cuda()
     B = torch.tensor(Bs, dtype=torch.int32, device="cuda")
     to = None if table_of is None else torch.tensor(table_of, dtype=torch.int32, device="cuda")
     ps.run(t, B, to)
@@ -97,7 +101,7 @@ def test_random_vs_exhaustive(pt, oracle_mod, seed):
     probs = [(tb, D, B) for tb in range(3) for D in (1, 2, 4) for B in (1, 2, 16, 64)]
     for D in (1, 2, 4):
         sub = [(tb, B) for tb, d, B in probs if d == D]
-        got = _run(pt, tables, dev, D, [B for _, B in sub], [tb for tb, _ in sub])
+        got = _run(pt, tables, dev, D, [B for _, B in sub], [tb for tb, _ in sub], pad=seed % 3 * 5)
         for (tb, B), (T, st) in zip(sub, got):
             Tw, _ = oracle_mod.plan_search(tables[tb], dev, D, B)
             assert T == Tw, (seed, tb, D, B)
@@ -139,3 +143,32 @@ def test_invalid_problems(pt):
     assert math.isnan(got[2][0]) and got[2][1] == []
     with pytest.raises(pt.PredtopError):
         _run(pt, t, [0], 1, [4])
+
+
+def test_stage_table_end_to_end(pt, oracle_mod):
+    """The f1 flow on one GPU: every layer-range stage of a 6-layer GPT model
+    scored by 2 mesh models straight into the stage table (<= 2e-3 against
+    the oracle forward), then the plan search on that table == the oracle's
+    exhaustive search over the same table, bit for bit."""
+    from paper_conf_ipps_acharyas25_b200 import stage_table
+    L = 6
+    host = synth.layer_range_stages("gpt", L)
+    cfgs = synth.mesh_model_configs("search", 2)
+    blobs = [synth.pack_weights(c, synth.model_weights(c)) for c in cfgs]
+    dev, Bs = [1, 2], [1, 4, 16]
+    sts = stage_table.StageTableSearch(pt, cfgs, blobs, host, L, dev, 2, Bs)
+    sts.step()
+    torch.cuda.synchronize()
+    table = sts.table[0].cpu().numpy()
+    for c in range(2):
+        want = oracle_mod.forward_batch(cfgs[c], blobs[c], host)
+        err = np.abs(table[c] - want) / np.abs(want)
+        assert (want > 0).all() and err.max() <= 2e-3, err.max()
+    dense = np.full((L, L, 2), np.inf, np.float32)
+    for i in range(L):
+        for j in range(i, L):
+            dense[i, j] = table[:, synth.tri_index(i, j, L)]
+    for B, (T, st) in zip(Bs, sts.search.plans()):
+        Tw, _ = oracle_mod.plan_search(dense, dev, 2, B)
+        assert T == Tw
+        _valid(oracle_mod, dense, dev, 2, B, T, st)
