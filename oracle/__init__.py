@@ -79,6 +79,8 @@ def lib():
             L.orc_plan_T.argtypes = [i64, P, P, P, P, i64, P]
             L.orc_argmin.argtypes = [i64, P]
             L.orc_argmin.restype = i64
+            L.orc_prune.argtypes = [i32, i32, P, P, P, P, i32, P, P, P, P, P]
+            L.orc_prune.restype = i32
             L.orc_plan_search.argtypes = [i32, i32, P, i32, P, i32, P, P, P]
             L.orc_plan_search.restype = dbl
             _lib = L
@@ -263,3 +265,20 @@ def plan_search(stage_latency, choice_devices, num_devices: int, microbatches: i
         stages.append((a, int(ends[i]), int(ch[i])))
         a = int(ends[i]) + 1
     return float(T), stages
+
+
+def prune(n, src, dst, feats, ops=(64, 65)):
+    """Graph pruning (SIV-B4; reading R21) -> (status, nk, src', dst', feats')."""
+    s, d, f = _i32(src), _i32(dst), _feats(feats)
+    o = np.ascontiguousarray(ops, np.uint16)
+    nk = ctypes.c_int32(0)
+    ne = ctypes.c_int64(0)
+    cap = max(1, n * n)
+    os_ = np.zeros(cap, np.int32)
+    od = np.zeros(cap, np.int32)
+    of = np.zeros(max(n, 1), FEAT_DTYPE)
+    st = lib().orc_prune(n, len(s), _p(s), _p(d), _p(f), _p(o), len(o), ctypes.byref(nk), _p(os_), _p(od),
+                         ctypes.byref(ne), _p(of))
+    if st != OK:
+        return st, 0, None, None, None
+    return st, nk.value, os_[:ne.value].copy(), od[:ne.value].copy(), of[:nk.value].copy()

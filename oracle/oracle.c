@@ -565,3 +565,58 @@ double orc_plan_search(int L, int K, const int32_t* dev, int D, const float* t, 
   for (int i = 0; i < s.best_S; ++i) { stage_end[i] = s.best_end[i]; stage_choice[i] = s.best_choice[i]; }
   return s.best;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Graph pruning (SIV-B4): "operations whose effects can be      */
+/* stored in the graph even after removing them ... such as reshape and     */
+/* convert_element_type ... We remove these redundant operators".  Reading  */
+/* R21: an OPERATOR node whose op id is in `ops` is removed; every other    */
+/* node is kept, renumbered in its original order with its record unchanged;*/
+/* kept u gets an edge to kept w iff the raw graph has a path u -> ... -> w */
+/* of >= 1 edge whose interior nodes are all removed (the removed node's    */
+/* inputs are spliced to its consumers).  Output edges are unique and       */
+/* sorted by (src, dst).  Plain per-node DFS through removed nodes.         */
+/* Returns ORC_OK or the validation status of the raw graph (outputs then   */
+/* untouched).  out_src/out_dst must hold the result (at most nk*nk).       */
+/* ------------------------------------------------------------------------ */
+int orc_prune(int n, int e, const int32_t* src, const int32_t* dst, const orc_feat* feats,
+              const uint16_t* ops, int n_ops, int32_t* nk_out, int32_t* out_src, int32_t* out_dst,
+              int64_t* ne_out, orc_feat* out_feats) {
+  int st = orc_validate(n, e, src, dst);
+  if (st != ORC_OK) return st;
+  char* removed = (char*)calloc((size_t)n + 1, 1);
+  int* newid = (int*)malloc(sizeof(int) * ((size_t)n + 1));
+  int nk = 0;
+  for (int v = 0; v < n; ++v) {
+    int hit = 0;
+    for (int i = 0; i < n_ops; ++i) hit |= feats[v].op == ops[i];
+    removed[v] = (char)(hit && feats[v].kind == 2 /* operator */);
+    newid[v] = removed[v] ? -1 : nk;
+    if (!removed[v]) out_feats[nk++] = feats[v];
+  }
+  orc_csr succ = build_csr(n, e, src, dst);
+  char* seen = (char*)malloc((size_t)n + 1);
+  char* target = (char*)malloc((size_t)n + 1);
+  int* stack = (int*)malloc(sizeof(int) * ((size_t)e + (size_t)n + 1));
+  int64_t ne = 0;
+  for (int u = 0; u < n; ++u) {
+    if (removed[u]) continue;
+    memset(seen, 0, (size_t)n);
+    memset(target, 0, (size_t)n);
+    int sp = 0;
+    for (int i = succ.off[u]; i < succ.off[u + 1]; ++i) stack[sp++] = succ.adj[i];
+    while (sp > 0) {
+      int w = stack[--sp];
+      if (!removed[w]) { target[w] = 1; continue; } /* a kept node ends the path */
+      if (seen[w]) continue;
+      seen[w] = 1;
+      for (int i = succ.off[w]; i < succ.off[w + 1]; ++i) stack[sp++] = succ.adj[i];
+    }
+    for (int w = 0; w < n; ++w) /* ascending kept ids = ascending new ids */
+      if (target[w]) { out_src[ne] = newid[u]; out_dst[ne] = newid[w]; ++ne; }
+  }
+  *nk_out = nk;
+  *ne_out = ne;
+  free(removed); free(newid); free(seen); free(target); free(stack); free_csr(&succ);
+  return ORC_OK;
+}

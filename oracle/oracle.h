@@ -79,6 +79,9 @@ int orc_forward_k(const orc_cfg* c, const float* blob, int n, int e, const int32
 void orc_plan_T(int64_t P, const int64_t* plan_ptr, const int32_t* plan_stage,
                 const int32_t* B, const float* t, int64_t num_stages, double* T);
 int64_t orc_argmin(int64_t n, const double* T);
+int orc_prune(int n, int e, const int32_t* src, const int32_t* dst, const orc_feat* feats,
+              const uint16_t* ops, int n_ops, int32_t* nk_out, int32_t* out_src, int32_t* out_dst,
+              int64_t* ne_out, orc_feat* out_feats);
 double orc_plan_search(int L, int K, const int32_t* dev, int D, const float* t, int B,
                        int32_t* S_out, int32_t* stage_end, int32_t* stage_choice);
 

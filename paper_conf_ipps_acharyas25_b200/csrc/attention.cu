@@ -11,7 +11,7 @@
 // word of every mask row), brought in by TMA ([64 keys x d_h] boxes, one
 // elected thread, one mbarrier).  Graphs whose K/V fit (N <= ~1500 at d_h =
 // 16) are loaded whole, then every warp runs independently; larger graphs
-// stream chunks through a two-buffer TMA pipeline.
+// stream through a 3-stage ring of 256-key stages (two stages in flight).
 //
 // Per warp (16 query rows) and 16-key block: QK^T on the m16n8k16 tensor-core
 // MMA with the accumulator input C = -m (allowed pair) or -inf (masked), so
@@ -83,6 +83,8 @@ __device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4]
 }
 
 constexpr int kChunk = 64;
+constexpr int kStages = 3;       // streaming path: ring of stages ...
+constexpr int kStageChunks = 4;  // ... of 4 chunks (256 keys) each
 
 // flag nibble f (bit j = block j fully allowed) -> the thread's mask bits of
 // those blocks in rows a (bits 0-15) and b (bits 16-31): nibble j of each half
@@ -249,7 +251,7 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
            const __half* __restrict__ qkv, __half* __restrict__ out) {
   using A = Attn<DH>;
   extern __shared__ __align__(16) unsigned char dsm_attn[];
-  __shared__ __align__(8) uint64_t kv_full[2];
+  __shared__ __align__(8) uint64_t kv_full[kStages];
   const int h = blockIdx.x % H;
   const int widx = (blockIdx.x / H) / (8 / NW);
   const int part = (blockIdx.x / H) % (8 / NW);
@@ -263,7 +265,7 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
   if (rbase >= N) return;
   const int W = 2 * ((N + 127) / 128);
   const int nchunks = (N + kChunk - 1) / kChunk;
-  const int nbuf = RESIDENT ? nchunks : 2;
+  const int nbuf = RESIDENT ? nchunks : kStages * kStageChunks;
   unsigned char* sK = sm100::align1024(dsm_attn);      // [nbuf][64 keys][DH], TMA swizzle
   unsigned char* sV = sK + (size_t)nbuf * A::CHUNK_BYTES;
   const uint64_t* Mg = d.M + d.row_off[g];
@@ -285,8 +287,7 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
   // columns d + h*DH (K) and 2d + h*DH (V); keys past N read the next graph's
   // rows (masked) or zeros past the tensor end.
   if (threadIdx.x == 0) {
-    sm100::mbar_init(&kv_full[0], 1);
-    sm100::mbar_init(&kv_full[1], 1);
+    for (int i = 0; i < kStages; ++i) sm100::mbar_init(&kv_full[i], 1);
     sm100::fence_mbar_init();
   }
   __syncthreads();
@@ -300,8 +301,12 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
     }
   };
   if (threadIdx.x == 0) {
-    if (RESIDENT) load_chunks(0, nchunks, 0, &kv_full[0]);
-    else load_chunks(0, 1, 0, &kv_full[0]);
+    if (RESIDENT) {
+      load_chunks(0, nchunks, 0, &kv_full[0]);
+    } else {
+      for (int s = 0; s < kStages && s * kStageChunks < nchunks; ++s)
+        load_chunks(s * kStageChunks, min(nchunks, (s + 1) * kStageChunks), s * kStageChunks, &kv_full[s]);
+    }
   }
 
   A st;
@@ -362,24 +367,31 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
       fl = nfl;
     }
   } else {
-    // two chunk buffers: chunk c+1 streams in while chunk c runs
-    for (int c = 0; c < nchunks; ++c) {
-      const int buf = c & 1;
-      uint32_t nlo = 0u, nhi = 0u;
-      if (c + 1 < nchunks) {
-        if (threadIdx.x == 0) load_chunks(c + 1, c + 2, buf ^ 1, &kv_full[buf ^ 1]);
-        nlo = mask_lo(c + 1);
-        nhi = mask_hi(c + 1);
-      }
-      sm100::mbar_wait(&kv_full[buf], (c >> 1) & 1);
-      if (warp_live) {
-        const uint32_t off = (uint32_t)(buf * A::CHUNK_BYTES);
-        const uint32_t fl = __shfl_sync(0xffffffffu, (uint32_t)Fw[c], 0);
-        st.chunk(kb0 + off, vb0 + off, mlo | (mhi << 16), fl);
+    // streaming: a ring of kStages stages of kStageChunks chunks each; stage
+    // s+kStages is loaded into the buffer of stage s once every warp is done
+    // with it (one CTA barrier per stage), so kStages-1 stages (>= 512 keys)
+    // are in flight ahead of the compute and the TMA latency stays hidden
+    const int nst = (nchunks + kStageChunks - 1) / kStageChunks;
+    for (int s = 0; s < nst; ++s) {
+      const int buf = s % kStages;
+      const int c0 = s * kStageChunks, c1 = min(nchunks, c0 + kStageChunks);
+      sm100::mbar_wait(&kv_full[buf], (s / kStages) & 1);
+      for (int c = c0; c < c1; ++c) {
+        const bool more = c + 1 < nchunks;
+        const uint32_t nlo = more ? mask_lo(c + 1) : 0u, nhi = more ? mask_hi(c + 1) : 0u;
+        if (warp_live) {
+          const uint32_t off = (uint32_t)((buf * kStageChunks + c - c0) * A::CHUNK_BYTES);
+          const uint32_t fl = __shfl_sync(0xffffffffu, (uint32_t)Fw[c], 0);
+          st.chunk(kb0 + off, vb0 + off, mlo | (mhi << 16), fl);
+        }
+        mlo = nlo;
+        mhi = nhi;
       }
       __syncthreads();  // every warp is done with buffer buf before it is reloaded
-      mlo = nlo;
-      mhi = nhi;
+      if (threadIdx.x == 0 && s + kStages < nst) {
+        const int n0c = (s + kStages) * kStageChunks;
+        load_chunks(n0c, min(nchunks, n0c + kStageChunks), buf * kStageChunks, &kv_full[buf]);
+      }
     }
     if (!warp_live) return;
   }
@@ -648,7 +660,14 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
     }
     k_attn<DH, true><<<blocks, 256, resident_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
   } else {
-    k_attn<DH, false><<<blocks, 256, 4 * CH_BYTES + 1024, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    constexpr int stream_bytes = 2 * kStages * kStageChunks * CH_BYTES + 1024;
+    static bool attr_s = false;
+    if (!attr_s) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       stream_bytes));
+      attr_s = true;
+    }
+    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
   }
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;

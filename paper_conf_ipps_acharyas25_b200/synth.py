@@ -567,6 +567,74 @@ MESH_CHOICES = [("mesh1 single GPU", 1), ("mesh2 2-way DP", 2), ("mesh2 2-way MP
                 ("mesh3 4-way DP", 4), ("mesh3 2-way DP x 2-way MP", 4), ("mesh3 4-way MP", 4)]
 
 
+# Raw Jaxpr primitives that the paper prunes (SIV-B4).  They are
+# outside the 64-slot Table I vocabulary (a pruned graph never contains them;
+# include/predtop.h: op ids >= 64 encode an all-zero one-hot).
+RAW_OP_RESHAPE, RAW_OP_CONVERT = 64, 65
+PRUNED_OPS = (RAW_OP_RESHAPE, RAW_OP_CONVERT)
+
+
+def insert_pruned_ops(n: int, src, dst, feats, rng: CounterRng, frac: float = 0.3):
+    """A raw (pre-pruning) version of a stage graph: reshape / convert nodes
+    spliced onto about `frac` of the edges (u -> r -> v, sometimes a chain of
+    two), some shared by several consumers of u (u -> r -> {v1, v2, ..}), and
+    a few dangling ones (u -> r with no consumer).  Original nodes keep ids
+    0..n-1; inserted nodes are appended.  Returns (n', src', dst', feats')."""
+    src = [int(x) for x in src]
+    dst = [int(x) for x in dst]
+    f = list(np.asarray(feats, FEAT_DTYPE))
+    out_s, out_d = [], []
+    extra = []
+
+    def new_node(like: int) -> int:
+        rec = np.zeros((), FEAT_DTYPE)
+        rec["op"] = RAW_OP_RESHAPE if rng.uniform() < 0.5 else RAW_OP_CONVERT
+        rec["kind"] = KIND_OPERATOR
+        rec["dtype"] = (int(f[like]["dtype"]) + (1 if rec["op"] == RAW_OP_CONVERT else 0)) % NUM_DTYPES
+        rec["dims"] = f[like]["dims"]
+        extra.append(rec)
+        return n + len(extra) - 1
+
+    by_src: Dict[int, List[int]] = {}
+    for e in range(len(src)):
+        by_src.setdefault(src[e], []).append(e)
+    done = set()
+    for u, es in by_src.items():
+        if len(es) >= 2 and rng.uniform() < frac:  # shared: two or more consumers through one r
+            k = rng.randint(2, len(es) + 1)
+            r = new_node(u)
+            out_s.append(u)
+            out_d.append(r)
+            for e in es[:k]:
+                out_s.append(r)
+                out_d.append(dst[e])
+                done.add(e)
+    for e in range(len(src)):
+        if e in done:
+            continue
+        u, v = src[e], dst[e]
+        x = rng.uniform()
+        if x < frac:
+            r = new_node(u)
+            out_s += [u, r]
+            out_d += [r, v]
+        elif x < frac * 1.3:
+            r1 = new_node(u)
+            r2 = new_node(u)
+            out_s += [u, r1, r2]
+            out_d += [r1, r2, v]
+        else:
+            out_s.append(u)
+            out_d.append(v)
+    for _ in range(max(1, n // 50)):  # dangling pruned nodes
+        u = rng.randint(0, n)
+        r = new_node(u)
+        out_s.append(u)
+        out_d.append(r)
+    allf = np.asarray(f + extra, FEAT_DTYPE)
+    return n + len(extra), np.asarray(out_s, np.int32), np.asarray(out_d, np.int32), allf
+
+
 # --------------------------------------------------------------------------
 # Hand-made tiny graphs (config 0) and structured test graphs
 # --------------------------------------------------------------------------
