@@ -297,6 +297,46 @@ PREDTOP_API predtop_status predtop_plan_argmin(int64_t num_plans, const double* 
 
 /* Misc. */
 /* ---------------------------------------------------------------------------
+ * Graph pruning (SIV-B4 "Graph Pruning"): "There
+ * are several operations whose effects can be stored in the graph even after
+ * removing them ... such as reshape and convert_element_type ... We remove
+ * these redundant operators from our graphs".  Reading R21: an
+ * OPERATOR node (kind 2) whose op id is in pruned_ops is removed; every other
+ * node is kept, renumbered in its original order with its record unchanged;
+ * kept u gets an edge to kept w iff the raw graph has a path u -> ... -> w of
+ * >= 1 edge whose interior nodes are all removed (the removed node's inputs
+ * are spliced to its consumers).  Output edges are unique and sorted by
+ * (src, dst) within each graph; the output is a batch in the input layout,
+ * ready for predtop_build_dag.  Raw primitives outside the Table I vocabulary
+ * use op ids >= PREDTOP_NUM_OPS (e.g. the two named by the paper below).
+ *  desc, node_ptr, edge_ptr, edge_src, edge_dst, feats: the RAW batch, as for
+ *                      predtop_build_dag (device)
+ *  pruned_ops[n]       [host] op ids to remove, 1 <= n <= PREDTOP_PRUNE_MAX_OPS
+ *  workspace           device, >= predtop_prune_workspace(desc), 256-B aligned
+ *  out_node_ptr[G+1], out_edge_ptr[G+1]  device int64
+ *  out_src/out_dst     device int32 [edge_capacity], graph-local new ids
+ *  out_feats           device [desc->total_nodes] (kept records)
+ *  totals              [host] int64[2], nullable: kept nodes, output edges
+ *  first_bad_graph     [host] nullable
+ * Synchronises `cuda_stream` once (the output sizes).  A raw graph that
+ * fails validation (RANGE / SELF_LOOP / CYCLE, TOO_LARGE) -> that status,
+ * nothing emitted.  More output edges than edge_capacity -> WORKSPACE (totals
+ * still set; call again with a larger buffer).  A graph whose nodes are all
+ * removed becomes an empty graph (0 nodes), which predtop_build_dag rejects. */
+#define PREDTOP_OP_RESHAPE 64
+#define PREDTOP_OP_CONVERT_ELEMENT_TYPE 65
+#define PREDTOP_PRUNE_MAX_OPS 16
+PREDTOP_API size_t predtop_prune_workspace(const predtop_batch_desc* desc);
+PREDTOP_API predtop_status predtop_prune_graphs(const predtop_batch_desc* desc, const int64_t* node_ptr,
+                                                const int64_t* edge_ptr, const int32_t* edge_src,
+                                                const int32_t* edge_dst, const predtop_node_feat* feats,
+                                                const uint16_t* pruned_ops, int32_t num_pruned_ops,
+                                                void* workspace, size_t ws_bytes, int64_t* out_node_ptr,
+                                                int64_t* out_edge_ptr, int32_t* out_src, int32_t* out_dst,
+                                                int64_t edge_capacity, predtop_node_feat* out_feats,
+                                                int64_t* totals, int32_t* first_bad_graph, void* cuda_stream);
+
+/* ---------------------------------------------------------------------------
  * Inter-stage plan search over a shared stage table.
  * Alpa's inter-operator optimizer picks the pipeline plan under the
  * 1F1B model; it enumerates all stages on all submeshes; P:222:

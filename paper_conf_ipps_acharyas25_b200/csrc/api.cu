@@ -558,6 +558,40 @@ predtop_status predtop_plan_latency(int64_t num_plans, const int64_t* plan_ptr,
 
 size_t predtop_plan_argmin_workspace(int64_t) { return 256; }
 
+size_t predtop_prune_workspace(const predtop_batch_desc* desc) {
+  DagBounds bd;
+  if (!dag_bounds(desc, &bd)) return 0;
+  return prune_workspace_bytes(desc);
+}
+
+predtop_status predtop_prune_graphs(const predtop_batch_desc* desc, const int64_t* node_ptr,
+                                    const int64_t* edge_ptr, const int32_t* edge_src, const int32_t* edge_dst,
+                                    const predtop_node_feat* feats, const uint16_t* pruned_ops,
+                                    int32_t num_pruned_ops, void* workspace, size_t ws_bytes,
+                                    int64_t* out_node_ptr, int64_t* out_edge_ptr, int32_t* out_src,
+                                    int32_t* out_dst, int64_t edge_capacity, predtop_node_feat* out_feats,
+                                    int64_t* totals, int32_t* first_bad_graph, void* cuda_stream) {
+  if (first_bad_graph) *first_bad_graph = -1;
+  DagBounds bd;
+  if (!dag_bounds(desc, &bd)) { set_error("prune: invalid batch descriptor"); return PREDTOP_ERR_INVALID_ARG; }
+  if (desc->max_nodes > PREDTOP_MAX_NODES) { set_error("prune: max_nodes too large"); return PREDTOP_ERR_TOO_LARGE; }
+  if (!node_ptr || !edge_ptr || !feats || (desc->total_edges > 0 && (!edge_src || !edge_dst)) || !workspace ||
+      !out_node_ptr || !out_edge_ptr || !out_feats || (edge_capacity > 0 && (!out_src || !out_dst)) ||
+      !pruned_ops || num_pruned_ops < 1 || num_pruned_ops > PREDTOP_PRUNE_MAX_OPS || edge_capacity < 0) {
+    set_error("prune: NULL or out-of-range argument");
+    return PREDTOP_ERR_INVALID_ARG;
+  }
+  const size_t need = predtop_prune_workspace(desc);
+  if (((uintptr_t)workspace & 255) || ws_bytes < need) {
+    set_error("prune: workspace too small or misaligned (%zu < %zu)", ws_bytes, need);
+    return PREDTOP_ERR_WORKSPACE;
+  }
+  if (!device_ok()) return PREDTOP_ERR_CUDA;
+  return prune_launch(desc, node_ptr, edge_ptr, edge_src, edge_dst, feats, pruned_ops, num_pruned_ops, workspace,
+                      out_node_ptr, out_edge_ptr, out_src, out_dst, edge_capacity, out_feats, totals,
+                      first_bad_graph, S(cuda_stream));
+}
+
 size_t predtop_plan_search_workspace(int64_t num_problems, int32_t num_layers, int32_t num_choices) {
   if (num_problems < 1 || num_layers < 1 || num_layers > PREDTOP_SEARCH_MAX_LAYERS || num_choices < 1 ||
       num_choices > PREDTOP_SEARCH_MAX_CHOICES)

@@ -19,7 +19,7 @@ enum ProfKind {
   PK_DAG_META, PK_DAG_DEPTH, PK_DAG_CLOSURE, PK_DAG_MASK, PK_DAG_CLASSIFY, PK_DAG_WORK,
   PK_PE, PK_EMBED, PK_GEMM_QKV, PK_ATTN, PK_GEMM_O_LN, PK_GEMM_FF1, PK_GEMM_FF2_LN,
   PK_READOUT, PK_PLAN, PK_ARGMIN, PK_COPY, PK_LAYER_TAIL, PK_DAG_SMALL, PK_DAG_FLAGS,
-  PK_SEARCH_CAND, PK_SEARCH_PICK, PK_COUNT
+  PK_SEARCH_CAND, PK_SEARCH_PICK, PK_PRUNE, PK_COUNT
 };
 struct ProfScope {
   int kind;

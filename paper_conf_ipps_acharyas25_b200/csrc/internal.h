@@ -176,6 +176,15 @@ predtop_status plan_launch(int64_t P, const int64_t* plan_ptr, const int32_t* pl
                            int64_t* first_bad, cudaStream_t st);
 predtop_status argmin_launch(int64_t n, const double* T, int64_t* best, cudaStream_t st);
 
+// ---- prune.cu (graph pruning)
+size_t prune_workspace_bytes(const predtop_batch_desc* b);
+predtop_status prune_launch(const predtop_batch_desc* b, const int64_t* node_ptr, const int64_t* edge_ptr,
+                            const int32_t* src, const int32_t* dst, const predtop_node_feat* feats,
+                            const uint16_t* ops, int n_ops, void* ws, int64_t* out_node_ptr,
+                            int64_t* out_edge_ptr, int32_t* out_src, int32_t* out_dst,
+                            int64_t edge_capacity, predtop_node_feat* out_feats, int64_t* totals_host,
+                            int32_t* first_bad_host, cudaStream_t st);
+
 // ---- search.cu (inter-stage plan search)
 size_t search_workspace_bytes(int64_t P, int L, int K);  // [P][K * L(L+1)/2] candidate T
 predtop_status search_launch(int64_t P, int L, int K, const int32_t* dev, int D, const float* t,

@@ -35,7 +35,7 @@ const char* kNames[PK_COUNT] = {
     "dag_meta", "dag_depth", "dag_closure", "dag_mask", "dag_classify", "dag_work",
     "pe_table", "embed", "gemm_qkv", "attention", "gemm_oproj_ln", "gemm_ffn1",
     "gemm_ffn2_ln", "readout", "plan_latency", "plan_argmin", "copy", "layer_tail", "dag_small", "dag_flags",
-    "search_cand", "search_pick"};
+    "search_cand", "search_pick", "prune"};
 }  // namespace
 
 ProfScope::ProfScope(int k, cudaStream_t s) : kind(k), st(s) {

@@ -30,6 +30,7 @@ POOL_SUM, POOL_MEAN = 0, 1
 MAX_NODES = 65536
 MAX_PLAN_STAGES = 64
 SEARCH_MAX_LAYERS, SEARCH_MAX_CHOICES, SEARCH_MAX_DEVICES = 64, 32, 64
+OP_RESHAPE, OP_CONVERT_ELEMENT_TYPE = 64, 65
 
 
 class PredtopError(RuntimeError):
@@ -74,6 +75,8 @@ _SIGS = {
     "predtop_plan_latency": (_I32, [_I64, _P, _P, _P, _P, _I64, _P, _P, _SZ, _U32, _P, _P]),
     "predtop_plan_argmin_workspace": (_SZ, [_I64]),
     "predtop_plan_argmin": (_I32, [_I64, _P, _P, _P, _SZ, _P]),
+    "predtop_prune_workspace": (_SZ, [_P]),
+    "predtop_prune_graphs": (_I32, [_P, _P, _P, _P, _P, _P, _P, _I32, _P, _SZ, _P, _P, _P, _P, _I64, _P, _P, _P, _P]),
     "predtop_plan_search_workspace": (_SZ, [_I64, _I32, _I32]),
     "predtop_plan_search": (_I32, [_I64, _I32, _I32, _P, _I32, _P, _I64, _I64, _P, _P, _P, _P, _P, _P, _P, _SZ, _P]),
     "predtop_status_string": (ctypes.c_char_p, [_I32]),
@@ -390,3 +393,40 @@ class PlanSearch:
                 a = int(E[p, s]) + 1
             out.append((float(T[p]), st))
         return out
+
+
+def prune_graphs(batch: "DeviceBatch", pruned_ops=(OP_RESHAPE, OP_CONVERT_ELEMENT_TYPE), edge_capacity=None,
+                 stream=None):
+    """predtop_prune_graphs (SIV-B4): raw DeviceBatch -> pruned
+    DeviceBatch (device tensors).  Retries once with the exact edge count if
+    the first capacity guess (the raw edge count) is too small."""
+    dev = batch.node_ptr.device
+    desc = batch.desc()
+    need = lib().predtop_prune_workspace(ctypes.byref(desc))
+    if need == 0:
+        raise PredtopError(INVALID_ARG, "invalid batch descriptor")
+    ws = torch.empty(need, dtype=torch.uint8, device=dev)
+    G = batch.num_graphs
+    ops = (ctypes.c_uint16 * len(pruned_ops))(*[int(o) for o in pruned_ops])
+    onp = torch.empty(G + 1, dtype=torch.int64, device=dev)
+    oep = torch.empty(G + 1, dtype=torch.int64, device=dev)
+    ofe = torch.empty(max(batch.total_nodes, 1) * FEAT_BYTES, dtype=torch.uint8, device=dev)
+    cap = int(edge_capacity if edge_capacity is not None else max(batch.total_edges, 1))
+    tot = (ctypes.c_int64 * 2)()
+    bad = ctypes.c_int32(-1)
+    for _ in range(2):
+        osrc = torch.empty(max(cap, 1), dtype=torch.int32, device=dev)
+        odst = torch.empty(max(cap, 1), dtype=torch.int32, device=dev)
+        st = lib().predtop_prune_graphs(ctypes.byref(desc), _ptr(batch.node_ptr), _ptr(batch.edge_ptr),
+                                        _ptr(batch.src), _ptr(batch.dst), _ptr(batch.feats), ops, len(pruned_ops),
+                                        _ptr(ws), ws.numel(), _ptr(onp), _ptr(oep), _ptr(osrc), _ptr(odst), cap,
+                                        _ptr(ofe), tot, ctypes.byref(bad), _stream(stream))
+        if st == WORKSPACE and tot[1] > cap:
+            cap = int(tot[1])
+            continue
+        _check(st)
+        break
+    nn, ne = int(tot[0]), int(tot[1])
+    sizes = torch.diff(onp).cpu()
+    return DeviceBatch(onp, oep, osrc[:ne], odst[:ne], ofe[:nn * FEAT_BYTES],
+                       int(sizes.max()) if G else 1)
