@@ -499,10 +499,78 @@ def run_batch(args, ctx):
         e2e_run()
     ms_e2e = ctx.timed(e2e_run, max(10, args.steps // 4))
     tot_e2e = ctx.max_over_ranks(sum(ms_e2e))
-    e2e_value = world * G * len(ms_e2e) / (tot_e2e / 1e3)
+    e2e_serial = world * G * len(ms_e2e) / (tot_e2e / 1e3)
     torch.cuda.synchronize()
     if P:  # the host copy of the plan latencies matches the device result
         assert torch.equal(T_host[:world * P], (T_all if world > 1 else plans.T[:P]).cpu())
+
+    # ---- e2e pipelined: two input buffer sets; the host->device copy of step
+    # i+1 runs on a copy stream while step i computes (each step still copies
+    # its own inputs inside the timed region and reads its result back)
+    e2e_value, e2e_mode = e2e_serial, "serial"
+    if not args.eager and world == 1:
+        db2 = pt.DeviceBatch(db.node_ptr.clone(), db.edge_ptr.clone(), db.src.clone(), db.dst.clone(),
+                             db.feats.clone(), db.max_nodes)
+        dag2 = pt.Dag(db2, no_sync=True, hops=args.hops)
+        plans2 = pt.Plans(ps.plan_ptr, ps.plan_stage, ps.microbatches, device=dev)
+        sets = [(db, dag, plans), (db2, dag2, plans2)]
+
+        def make_step(k):
+            dbk, dagk, plk = sets[k]
+
+            def f():
+                dagk.rebuild()
+                model.forward(dagk, ws, lat)
+                T, _, _ = plk.latency(lat, no_sync=True)
+                plk.argmin(T)
+                if P:
+                    T_host[:P].copy_(plk.T[:P], non_blocking=True)
+                best_host.copy_(plk.best, non_blocking=True)
+            return f
+
+        graphs = [ctx.capture(make_step(k))[0] for k in range(2)]
+        cs = torch.cuda.Stream(device=dev)
+        ev_in = [torch.cuda.Event(), torch.cuda.Event()]
+        ev_done = [torch.cuda.Event(), torch.cuda.Event()]
+
+        def copy_in(k):
+            dbk, _, plk = sets[k]
+            with torch.cuda.stream(cs):
+                cs.wait_event(ev_done[k])  # step k-2 finished with buffer set k
+                dbk.node_ptr.copy_(pin["node_ptr"], non_blocking=True)
+                dbk.edge_ptr.copy_(pin["edge_ptr"], non_blocking=True)
+                dbk.src.copy_(pin["src"], non_blocking=True)
+                dbk.dst.copy_(pin["dst"], non_blocking=True)
+                dbk.feats.copy_(pin["feats"], non_blocking=True)
+                plk.plan_ptr.copy_(pin["plan_ptr"], non_blocking=True)
+                plk.plan_stage.copy_(pin["plan_stage"], non_blocking=True)
+                plk.microbatches.copy_(pin["mb"], non_blocking=True)
+                ev_in[k].record(cs)
+
+        def pipelined(n):
+            copy_in(0)
+            for i in range(n):
+                k = i & 1
+                if i + 1 < n:
+                    copy_in(k ^ 1)
+                ctx.stream.wait_event(ev_in[k])
+                graphs[k]()
+                ev_done[k].record(ctx.stream)
+
+        pipelined(4)
+        torch.cuda.synchronize()
+        n_e2e = max(10, args.steps)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        a.record(ctx.stream)
+        pipelined(n_e2e)
+        b.record(ctx.stream)
+        torch.cuda.synchronize()
+        e2e_value = G * n_e2e / (a.elapsed_time(b) / 1e3)
+        e2e_mode = (f"pipelined: {n_e2e} steps back to back, the H2D copy of step i+1 (copy stream) "
+                    f"overlaps step i; every step copies its inputs and reads T* back; no L2 flush")
+        if P:
+            assert torch.equal(T_host[:P], plans.T[:P].cpu())
 
     # ---- per-kernel profile pass (separate from the headline timing)
     prof = ctx.profile(step, max(5, args.steps // 4))
@@ -524,7 +592,7 @@ def run_batch(args, ctx):
                 "config": workload_config(args),
                 "plans_per_s": plans_per_s,
                 "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-                        "d2h_bytes_per_step": int(d2h)},
+                        "d2h_bytes_per_step": int(d2h), "mode": e2e_mode, "serial_value": e2e_serial},
                 "gpu_launches": int(launches),
                 "launch_mode": "eager" if args.eager else "cuda_graph",
                 "eager_ms_per_step": eager_ms, "host_enqueue_ms_per_step": host_enqueue_ms,
