@@ -30,6 +30,33 @@
 
 namespace predtop {
 
+#ifdef PREDTOP_TRACE
+// Debug timeline of CTA 0 (first 16 tiles): %globaltimer at epilogue phase
+// boundaries; MMA-thread wait clocks summed over tiles 2..9 of CTA 0.
+__device__ unsigned long long g_tail2_trace[16][16];
+__device__ long long g_tail2_mma[8];
+__device__ __forceinline__ unsigned long long gtime2() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define T2(i, k)                                                                      \
+  do {                                                                                \
+    if (leader && blockIdx.x == 0 && (i) < 16) g_tail2_trace[i][k] = gtime2();       \
+  } while (0)
+#define T2W(k, stmt)                                                                  \
+  do {                                                                                \
+    const long long t0_ = clock64();                                                  \
+    stmt;                                                                             \
+    if (blockIdx.x == 0 && i >= 2 && i < 10) g_tail2_mma[k] += clock64() - t0_;      \
+  } while (0)
+#else
+#define T2(i, k) \
+  do {           \
+  } while (0)
+#define T2W(k, stmt) stmt
+#endif
+
 namespace {
 
 constexpr int D = 128;           // d_model handled by this kernel
@@ -46,14 +73,30 @@ constexpr uint32_t TMEM_COLS = 256;
 static_assert(SMEM <= 113 * 1024, "two CTAs per SM");
 
 struct Tail2Maps {
-  CUtensorMap att, x32, x16, wo, w1, w2;
+  CUtensorMap att, x32, x16, wo, w1, w2, x32in;
 };
 
 struct Tail2Args {
   int M, dff;
   const float *bo, *g1, *be1, *b1, *b2, *g2, *be2;
   float eps;
+  float* x32;   // residual stream [M][D] fp32 (read, then overwritten with x')
+  __half* x16;  // its fp16 shadow [M][D]
 };
+
+// Residual I/O of the epilogue.  2 (default): the producer streams the x tile
+// through the ring (4 slots of [128 rows x 32 fp32], right after the tile's
+// att / W_o slices), so it arrives while the previous tile finishes; x' goes
+// out through the warp's 4 KB staging piece by TMA.  1: x also comes in
+// through the staging piece, two [32 x 32] boxes after the previous tile's
+// stores have drained (~3 us per tile exposed).  0 selects plain 16-byte global
+// loads/stores straight between registers and memory (each thread owns 64
+// contiguous columns of one row); measured 2x slower on 1xB200 (lanes 512 B
+// apart: 32 sectors per instruction, LSU-bound; tools/tail2_trace.py), kept
+// for reference.
+#ifndef PREDTOP_TAIL2_TMA_IO
+#define PREDTOP_TAIL2_TMA_IO 2
+#endif
 
 __device__ __forceinline__ void tma_prefetch_l2_2d(const CUtensorMap* map, int32_t c0, int32_t c1) {
   asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global [%0, {%1, %2}];" ::"l"(
@@ -143,6 +186,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
           load(&mp.att, kc * 64, m0);
           load(&mp.wo, kc * 64, 0);
         }
+#if PREDTOP_TAIL2_TMA_IO == 2
+        // the residual x tile for the epilogue: 4 slots of [128 rows x 32 fp32]
+        // (SW128), after this tile's att/W_o (so the O-projection never waits
+        // for them) and before its FFN weights
+        for (int k = 0; k < D / 32; ++k) load(&mp.x32in, k * 32, m0);
+#endif
         for (int j = 0; j < NJ; ++j) {
           for (int kc = 0; kc < D / 64; ++kc) load(&mp.w1, kc * 64, j * FC);
           for (int kc = 0; kc < FC / 64; ++kc) load(&mp.w2, j * FC + kc * 64, 0);
@@ -153,9 +202,10 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
     if (lane == 0) {  // ------------------------------------------ MMA issuer
       constexpr uint32_t id_N128 = sm100::make_idesc_f16(128, 128);
       int it = 0;
+      int i = 0;
       auto slot_wait = [&]() -> uint32_t {
         const int s = it % RS;
-        sm100::mbar_wait(&ring_full[s], (it / RS) & 1);
+        T2W(0, sm100::mbar_wait(&ring_full[s], (it / RS) & 1));
         sm100::tc_fence_after();
         return sm100::smem_u32(ring + s * SLOT);
       };
@@ -164,10 +214,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         ++it;
       };
       const uint32_t aH = sm100::smem_u32(sH);
-      int i = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+#ifdef PREDTOP_TRACE
+        const long long tile_t0 = clock64();
+#endif
         // ---- O-projection: acc = att W_o^T (acc free once LN2 of the previous tile read it)
-        sm100::mbar_wait(&o_empty, (i & 1) ^ 1);
+        T2W(1, sm100::mbar_wait(&o_empty, (i & 1) ^ 1));
         sm100::tc_fence_after();
         for (int kc = 0; kc < D / 64; ++kc) {
           const uint32_t a0 = slot_wait();
@@ -182,8 +234,14 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
           slot_free();
         }
         sm100::mma_commit(&o_full);
+#if PREDTOP_TAIL2_TMA_IO == 2
+        // the x slots belong to the epilogue.  Skipping them is safe: the next
+        // slot_wait (FFN-1, after h_ready) is on a phase whose predecessor
+        // (the x load) the epilogue consumed before h_ready
+        it += D / 32;
+#endif
         // ---- FFN: acc already holds h + b_2 (written by the epilogue after LN1)
-        sm100::mbar_wait(&h_ready, i & 1);
+        T2W(2, sm100::mbar_wait(&h_ready, i & 1));
         sm100::tc_fence_after();
         for (int j = 0; j < NJ; ++j) {
           // FFN-1 chunk j -> acc_f.  It overwrites the P of chunk j-1 that
@@ -201,7 +259,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
           // FFN-2 chunk j: acc += P_j W_2[:, chunk]^T, P_j from TMEM: the
           // epilogue leaves hidden units [64g + 32hf, +32) as 16 packed fp16
           // columns at 64g + 16hf, so K-step ks sits at column 64(ks/4) + 8(ks%4).
-          sm100::mbar_wait(&p_ready, (i * NJ + j) & 1);
+          T2W(3, sm100::mbar_wait(&p_ready, (i * NJ + j) & 1));
           sm100::tc_fence_after();
           for (int kc = 0; kc < FC / 64; ++kc) {
             const uint32_t b0 = slot_wait();
@@ -215,6 +273,9 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
           }
         }
         sm100::mma_commit(&out_full);
+#ifdef PREDTOP_TRACE
+        if (blockIdx.x == 0 && i >= 2 && i < 10) g_tail2_mma[4] += clock64() - tile_t0;
+#endif
       }
     }
   } else {
@@ -255,7 +316,44 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
       const int m0 = t * 128;
       const int cbase = i * NJ;
-      // ---- residual x (fp32) -> registers, two boxes through the staging piece
+      T2(i, 0);
+      // ---- residual x (fp32) -> registers
+#if PREDTOP_TAIL2_TMA_IO == 2
+      // from the ring: slots (xit + 2g + k) % RS hold columns [64g + 32k, +32).
+      // o_full first: the O-projection consumed this tile's att / W_o, i.e.
+      // the previous phase of each x slot completed, so the parity wait below
+      // is never two phases ahead (it would alias and return at once)
+      sm100::mbar_wait(&o_full, i & 1);
+      const int xit = i * (2 * (D / 64) + D / 32 + NJ * (D / 64 + FC / 64)) + 2 * (D / 64);
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const int itk = xit + 2 * g + k;
+        sm100::mbar_wait(&ring_full[itk % RS], (itk / RS) & 1);
+        const unsigned char* sl = ring + (itk % RS) * SLOT;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          const float4 v = *reinterpret_cast<const float4*>(sl + sm100::swz<128>(r, c));
+          x[32 * k + 4 * c] = v.x;
+          x[32 * k + 4 * c + 1] = v.y;
+          x[32 * k + 4 * c + 2] = v.z;
+          x[32 * k + 4 * c + 3] = v.w;
+        }
+      }
+      sm100::fence_proxy_async();  // these generic reads before the slots' next TMA writes
+#elif !PREDTOP_TAIL2_TMA_IO
+      {
+        const int row = m0 + r;
+        const float4* src = reinterpret_cast<const float4*>(args.x32 + (int64_t)row * D + 64 * g);
+#pragma unroll
+        for (int c = 0; c < 16; ++c) {
+          const float4 v = row < args.M ? __ldcg(src + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+          x[4 * c] = v.x;
+          x[4 * c + 1] = v.y;
+          x[4 * c + 2] = v.z;
+          x[4 * c + 3] = v.w;
+        }
+      }
+#else
 #pragma unroll
       for (int k = 0; k < 2; ++k) {
         store_wait();
@@ -275,10 +373,13 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         // the __syncwarp in store_wait)
         sm100::fence_proxy_async();
       }
+#endif
       __syncwarp();
+      T2(i, 1);
       // ---- LN1: z = x + acc + b_o
       sm100::mbar_wait(&o_full, i & 1);
       sm100::tc_fence_after();
+      T2(i, 2);
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         float a[16];
@@ -291,6 +392,10 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
 #pragma unroll
         for (int e = 0; e < 64; ++e) s += x[e];
         const float mean = row_sum(s, 0) * (1.0f / D);
+#if PREDTOP_TAIL2_TMA_IO == 2
+        if (leader)  // every epilogue thread has read its x (the row_sum barrier): free the x slots
+          for (int k = 0; k < D / 32; ++k) sm100::mbar_arrive(&ring_empty[(xit + k) % RS]);
+#endif
         float sq = 0.f;
 #pragma unroll
         for (int e = 0; e < 64; ++e) {
@@ -301,6 +406,9 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
 #pragma unroll
         for (int e = 0; e < 64; ++e) x[e] = (x[e] - mean) * rstd * p_g1[64 * g + e] + p_be1[64 * g + e];
       }
+#if PREDTOP_TAIL2_TMA_IO == 2
+      store_wait();  // the previous tile's x16 store has read the staging piece
+#endif
       // h (fp16) -> the FFN-1 A operand; h + b_2 -> acc (FFN-2 accumulates onto it)
 #pragma unroll
       for (int c = 0; c < 8; ++c)
@@ -319,10 +427,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
       sm100::tc_fence_before();
       sm100::named_bar<kEpi>(1);
       if (leader) sm100::mbar_arrive(&h_ready);
+      T2(i, 3);
       // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 pairs back into acc_f
       for (int j = 0; j < NJ; ++j) {
         sm100::mbar_wait(&f_full, (cbase + j) & 1);
         sm100::tc_fence_after();
+        if (j < 4) T2(i, 4 + j);
 #pragma unroll
         for (int hf = 0; hf < 2; ++hf) {
           const int c0 = 64 * g + 32 * hf;
@@ -339,10 +449,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         sm100::tc_fence_before();
         sm100::named_bar<kEpi>(1);
         if (leader) sm100::mbar_arrive(&p_ready);
+        if (j < 4) T2(i, 8 + j);
       }
       // ---- LN2: z = acc (= h + b_2 + FFN(h))
       sm100::mbar_wait(&out_full, i & 1);
       sm100::tc_fence_after();
+      T2(i, 12);
 #pragma unroll
       for (int k = 0; k < 2; ++k) {
         float a[32];
@@ -367,6 +479,20 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
 #pragma unroll
         for (int e = 0; e < 64; ++e) x[e] = (x[e] - mean) * rstd * p_g2[64 * g + e] + p_be2[64 * g + e];
       }
+      T2(i, 13);
+#if !PREDTOP_TAIL2_TMA_IO
+      // ---- x' (fp32) and its fp16 shadow, straight from registers
+      if (m0 + r < args.M) {
+        float4* d32 = reinterpret_cast<float4*>(args.x32 + (int64_t)(m0 + r) * D + 64 * g);
+        uint4* d16 = reinterpret_cast<uint4*>(args.x16 + (int64_t)(m0 + r) * D + 64 * g);
+#pragma unroll
+        for (int c = 0; c < 16; ++c) d32[c] = make_float4(x[4 * c], x[4 * c + 1], x[4 * c + 2], x[4 * c + 3]);
+#pragma unroll
+        for (int c = 0; c < 8; ++c)
+          d16[c] = make_uint4(sm100::pack_half2(x[8 * c], x[8 * c + 1]), sm100::pack_half2(x[8 * c + 2], x[8 * c + 3]),
+                              sm100::pack_half2(x[8 * c + 4], x[8 * c + 5]), sm100::pack_half2(x[8 * c + 6], x[8 * c + 7]));
+      }
+#else
       // ---- x' (fp32, two boxes) and its fp16 shadow through the staging piece.
       // The piece held h, read by FFN-1 MMAs that completed before out_full.
 #pragma unroll
@@ -392,6 +518,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         sm100::tma_store_2d(&mp.x16, stg, 64 * g, m0 + 32 * q);
         sm100::bulk_commit();
       }
+#endif
+      T2(i, 14);
     }
     if (lane == 0) sm100::bulk_wait0();
   }
@@ -418,12 +546,12 @@ predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half*
   const LayerDev& L = m->layer[l];
   Tail2Maps mp;
   if (!encode_tma_2d(&mp.att, att, 2, d, M, 64, 128) || !encode_tma_2d(&mp.x32, x32, 4, d, M, 32, 32) ||
-      !encode_tma_2d(&mp.x16, x16, 2, d, M, 64, 32))
+      !encode_tma_2d(&mp.x16, x16, 2, d, M, 64, 32) || !encode_tma_2d(&mp.x32in, x32, 4, d, M, 32, 128))
     return PREDTOP_ERR_CUDA;
   mp.wo = L.tm_o;
   mp.w1 = L.tm_1c;
   mp.w2 = L.tm_2;
-  Tail2Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps};
+  Tail2Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
   static bool attr_done = false;
   if (!attr_done) {
     PT_CUDA_TRY(cudaFuncSetAttribute(k_layer_tail2, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM));
@@ -441,3 +569,10 @@ predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half*
 }
 
 }  // namespace predtop
+
+#ifdef PREDTOP_TRACE
+extern "C" PREDTOP_API int predtop_debug_tail2_trace(unsigned long long* out) {
+  if (cudaMemcpyFromSymbol(out, predtop::g_tail2_trace, sizeof(predtop::g_tail2_trace)) != cudaSuccess) return -7;
+  return cudaMemcpyFromSymbol(out + 256, predtop::g_tail2_mma, sizeof(predtop::g_tail2_mma)) == cudaSuccess ? 0 : -7;
+}
+#endif
