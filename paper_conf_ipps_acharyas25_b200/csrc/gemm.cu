@@ -46,7 +46,14 @@ struct Cfg {
   // to the fp32 one and a 2-stage ring; the fp16 copy is then stored directly.
   static constexpr bool F16_DIRECT =
       EPI == EPI_BIAS_RESID_LN && 128 * BN * 6 + 2 * STAGE_BYTES + 1024 > kSmemBudget;
-  static constexpr int OUT16_BYTES = F16_DIRECT ? 0 : 128 * BN * 2;
+  // bias epilogues with 32-column-aligned halves: every epilogue warp stores
+  // its own [32 rows x 32 cols] boxes from a double-buffered staging tile (no
+  // CTA-wide barrier, the stores of tile i drain while tile i+1 is staged)
+  static constexpr bool PER_WARP = EPI != EPI_BIAS_RESID_LN && (BN / 2) % 32 == 0;
+  // double-buffered only if the operand ring keeps >= 3 stages (BN = 256
+  // would drop to one stage; it keeps a single staging tile)
+  static constexpr bool DBUF = PER_WARP && (kSmemBudget - 2 * 128 * BN * 2 - 1024) / STAGE_BYTES >= 3;
+  static constexpr int OUT16_BYTES = F16_DIRECT ? 0 : (DBUF ? 2 : 1) * 128 * BN * 2;
   static constexpr int STAGING = OUT16_BYTES + OUT32_BYTES;
   static constexpr int STAGES_FIT = (kSmemBudget - STAGING - 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 4 ? 4 : STAGES_FIT;
@@ -85,12 +92,16 @@ __device__ __forceinline__ void bulk_wait_read0() {
   asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read1() {
+  asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sm100::smem_u32(bar)) : "memory");
 }
 
 struct Maps {
   CUtensorMap a, b, out16, x32;  // x32: residual load + fp32 store (LN epilogue)
+  CUtensorMap out16w;            // [32 cols x 32 rows] per-warp store boxes (SW64)
 };
 
 template <int BN, int KCH, int EPI>
@@ -184,6 +195,60 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int cbeg = half * (BN / 2), cend = cbeg + BN / 2;
     const bool leader = (warp == 2 && lane == 0);
     int local = 0;
+    if constexpr (C::PER_WARP) {
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++local) {
+        const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
+        const int acc = local & 1;
+        unsigned char* stage = st16 + (C::DBUF ? (local & 1) * (128 * BN * 2) : 0);
+        // this warp's stores of the tile that last used this staging buffer
+        // (local-2 double-buffered, local-1 otherwise) have read it
+        if (lane == 0) {
+          if (C::DBUF) bulk_wait_read1();
+          else bulk_wait_read0();
+        }
+        __syncwarp();
+        sm100::mbar_wait(&tfull[acc], (local >> 1) & 1);
+        sm100::tc_fence_after();
+        const uint32_t t_row = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * BN);
+        float v[16];
+#pragma unroll 1
+        for (int c = cbeg; c < cend; c += 16) {
+          sm100::tmem_ld16(t_row + c, v);
+          const float4* b4 = reinterpret_cast<const float4*>(args.bias + n0 + c);
+          float bb[16];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const float4 t4 = __ldg(b4 + k);
+            bb[4 * k] = t4.x; bb[4 * k + 1] = t4.y; bb[4 * k + 2] = t4.z; bb[4 * k + 3] = t4.w;
+          }
+          uint32_t p[8];
+          const float qs = (n0 + c < args.qcols) ? args.qscale : 1.f;
+#pragma unroll
+          for (int j = 0; j < 16; j += 2) {
+            float x0 = (v[j] + bb[j]) * qs;
+            float x1 = (v[j + 1] + bb[j + 1]) * qs;
+            if (EPI == EPI_BIAS_RELU_F16) { x0 = fmaxf(x0, 0.f); x1 = fmaxf(x1, 0.f); }
+            p[j / 2] = pack_half2(x0, x1);
+          }
+          // box c/32: [128 rows x 32 cols] fp16, 64-byte rows, SWIZZLE_64B
+          unsigned char* box = stage + (c / 32) * (128 * 64);
+          const int ch = (c % 32) / 8;
+          *reinterpret_cast<uint4*>(box + swz<64>(r, ch)) = make_uint4(p[0], p[1], p[2], p[3]);
+          *reinterpret_cast<uint4*>(box + swz<64>(r, ch + 1)) = make_uint4(p[4], p[5], p[6], p[7]);
+        }
+        sm100::tc_fence_before();
+        mbar_arrive(&tempty[acc]);  // accumulator may be overwritten now
+        fence_proxy_async();         // staging writes -> visible to the TMA (async proxy)
+        __syncwarp();
+        if (lane == 0) {
+          // rows 32q.. of each of this warp's boxes: 32 rows x 64 B, contiguous
+          for (int c = cbeg; c < cend; c += 32)
+            tma_store_2d(&maps.out16w, stage + (c / 32) * (128 * 64) + q * 32 * 64, n0 + c, m0 + 32 * q);
+          bulk_commit();
+        }
+      }
+      if (lane == 0) bulk_wait0();
+    } else
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++local) {
       const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
       const int acc = local & 1;
@@ -402,6 +467,11 @@ predtop_status gemm_launch(const CUtensorMap* tmA, const CUtensorMap* tmB, int b
     if (!encode_tma_2d(&m.x32, a.out32, 4, a.N, a.M, 32, 128)) return PREDTOP_ERR_CUDA;
   } else {
     m.x32 = m.out16;
+  }
+  if (epi != EPI_BIAS_RESID_LN && (bn / 2) % 32 == 0) {
+    if (!encode_tma_2d(&m.out16w, a.out16, 2, a.N, a.M, 32, 32)) return PREDTOP_ERR_CUDA;
+  } else {
+    m.out16w = m.out16;
   }
   if (a.K % 64 == 0) return launch_bn<64>(bn, epi, m, a, st);
   if (a.K == 32) return launch_bn<32>(bn, epi, m, a, st);
