@@ -398,7 +398,8 @@ predtop_status predtop_model_create(const predtop_model_config* cfg, const float
               encode_tma_2d_f16(&L.tm_o, L.Wo, d, d, kch_for(d), d) &&
               encode_tma_2d_f16(&L.tm_1, L.W1, d, f, kch_for(d), m->bn_ff1) &&
               encode_tma_2d_f16(&L.tm_2, L.W2, f, d, kch_for(f), d) &&
-              (f < 128 || encode_tma_2d_f16(&L.tm_1c, L.W1, d, f, kch_for(d), 128));
+              (f < 128 || encode_tma_2d_f16(&L.tm_1c, L.W1, d, f, kch_for(d), 128)) &&
+              (f < 64 || encode_tma_2d_f16(&L.tm_1h, L.W1, d, f, kch_for(d), 64));
     if (!ok) {
       delete m;
       return PREDTOP_ERR_CUDA;

@@ -110,7 +110,8 @@ struct LayerDev {
   float* g2;
   float* be2;
   CUtensorMap tm_qkv, tm_o, tm_1, tm_2;  // B-operand TMA maps (unfused GEMMs)
-  CUtensorMap tm_1c;                     // W_1 in 128-row chunks (fused layer tail)
+  CUtensorMap tm_1c;                     // W_1 in 128-row chunks (fused layer tail v1)
+  CUtensorMap tm_1h;                     // W_1 in 64-row chunks (layer tail v2)
 };
 
 }  // namespace predtop

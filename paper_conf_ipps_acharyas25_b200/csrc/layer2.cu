@@ -60,7 +60,7 @@ __device__ __forceinline__ unsigned long long gtime2() {
 namespace {
 
 constexpr int D = 128;           // d_model handled by this kernel
-constexpr int FC = 128;          // FFN chunk (hidden units per chunk)
+constexpr int FC = 64;           // FFN chunk (hidden units per chunk), two TMEM buffers
 constexpr int RS = 4;            // ring slots
 constexpr int SLOT = 128 * 128;  // bytes of one [128 rows x 64 fp16] slice
 constexpr int SH = 128 * D * 2;  // fp16 h tile (two K-slices)
@@ -136,7 +136,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
   }
   for (int i = threadIdx.x; i < args.dff; i += blockDim.x) p_b1[i] = args.b1[i];
   __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
-  __shared__ __align__(8) uint64_t o_full, o_empty, h_ready, f_full, p_ready, out_full;
+  __shared__ __align__(8) uint64_t o_full, o_empty, h_ready, out_full;
+  __shared__ __align__(8) uint64_t f_full[2], p_ready[2];  // per acc_f buffer
   __shared__ __align__(8) uint64_t xbar[kEpiWarps];
   __shared__ uint32_t tmem_slot;
   __shared__ float red[2][2][128];
@@ -150,8 +151,10 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
       sm100::mbar_init(&ring_full[s], 1);
       sm100::mbar_init(&ring_empty[s], 1);
     }
-    uint64_t* singles[] = {&o_full, &o_empty, &h_ready, &f_full, &p_ready, &out_full};
+    uint64_t* singles[] = {&o_full, &o_empty, &h_ready, &out_full, &f_full[0], &f_full[1]};
     for (uint64_t* b : singles) sm100::mbar_init(b, 1);
+    sm100::mbar_init(&p_ready[0], kEpiWarps);  // one arrival per epilogue warp
+    sm100::mbar_init(&p_ready[1], kEpiWarps);
     for (int w = 0; w < kEpiWarps; ++w) sm100::mbar_init(&xbar[w], 1);
     sm100::fence_mbar_init();
   }
@@ -160,6 +163,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
   __syncthreads();
   sm100::tc_fence_after();
   const uint32_t tmem = tmem_slot;
+  // TMEM: acc [0, 128) O-projection, then h + b_2 + FFN(h); acc_f buffers
+  // [128, 192) and [192, 256): FFN-1 chunk j in buffer j & 1
   const uint32_t acc = tmem, acc_f = tmem + D;
 
   if (warp == 0) {
@@ -192,9 +197,20 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         // for them) and before its FFN weights
         for (int k = 0; k < D / 32; ++k) load(&mp.x32in, k * 32, m0);
 #endif
+        // W_1 chunk j: one slot, two [64 x 64] K-slices; W_2 chunk j: one
+        // [128 x 64] slot.  Order = MMA order: F1_0 F1_1 F2_0 F1_2 F2_1 ...
+        auto load_w1 = [&](int j) {
+          const int s = it % RS;
+          sm100::mbar_wait(&ring_empty[s], ((it / RS) & 1) ^ 1);
+          sm100::mbar_arrive_expect_tx(&ring_full[s], SLOT);
+          for (int kc = 0; kc < D / 64; ++kc)
+            sm100::tma_load_2d(ring + s * SLOT + kc * (FC * 128), &mp.w1, &ring_full[s], kc * 64, j * FC);
+          ++it;
+        };
+        load_w1(0);
         for (int j = 0; j < NJ; ++j) {
-          for (int kc = 0; kc < D / 64; ++kc) load(&mp.w1, kc * 64, j * FC);
-          for (int kc = 0; kc < FC / 64; ++kc) load(&mp.w2, j * FC + kc * 64, 0);
+          if (j + 1 < NJ) load_w1(j + 1);
+          load(&mp.w2, j * FC, 0);
         }
       }
     }
@@ -243,34 +259,37 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         // ---- FFN: acc already holds h + b_2 (written by the epilogue after LN1)
         T2W(2, sm100::mbar_wait(&h_ready, i & 1));
         sm100::tc_fence_after();
-        for (int j = 0; j < NJ; ++j) {
-          // FFN-1 chunk j -> acc_f.  It overwrites the P of chunk j-1 that
-          // FFN-2 (issued just before by this thread) reads: tcgen05.mma of
-          // one thread executes in issue order.
-          for (int kc = 0; kc < D / 64; ++kc) {
-            const uint32_t b0 = slot_wait();
+        constexpr uint32_t id_N64 = sm100::make_idesc_f16(128, FC);
+        // FFN-1 chunk j -> acc_f buffer j & 1.  Chunk j+2 reuses the buffer
+        // whose P FFN-2 chunk j (issued just before by this thread) reads:
+        // tcgen05.mma of one thread executes in issue order.
+        auto ffn1 = [&](int j) {
+          const uint32_t b0 = slot_wait();
+          const uint32_t dst = acc_f + (uint32_t)((j & 1) * FC);
+#pragma unroll
+          for (int kc = 0; kc < D / 64; ++kc)
 #pragma unroll
             for (int kk = 0; kk < 4; ++kk)
-              sm100::mma_f16_ss(acc_f, sm100::make_sdesc<128>(aH + kc * SLOT + kk * 32),
-                                sm100::make_sdesc<128>(b0 + kk * 32), id_N128, (kc | kk) != 0);
-            slot_free();
-          }
-          sm100::mma_commit(&f_full);
-          // FFN-2 chunk j: acc += P_j W_2[:, chunk]^T, P_j from TMEM: the
-          // epilogue leaves hidden units [64g + 32hf, +32) as 16 packed fp16
-          // columns at 64g + 16hf, so K-step ks sits at column 64(ks/4) + 8(ks%4).
-          T2W(3, sm100::mbar_wait(&p_ready, (i * NJ + j) & 1));
+              sm100::mma_f16_ss(dst, sm100::make_sdesc<128>(aH + kc * SLOT + kk * 32),
+                                sm100::make_sdesc<128>(b0 + kc * (FC * 128) + kk * 32), id_N64, (kc | kk) != 0);
+          slot_free();
+          sm100::mma_commit(&f_full[j & 1]);
+        };
+        ffn1(0);
+        for (int j = 0; j < NJ; ++j) {
+          if (j + 1 < NJ) ffn1(j + 1);  // keeps the tensor pipe busy during ReLU_j
+          // FFN-2 chunk j: acc += P_j W_2[:, chunk]^T, P_j from TMEM: epilogue
+          // warp g leaves hidden units [32g, 32g + 32) as 16 packed fp16
+          // columns at 32g of the buffer, so K-step ks sits at 32(ks/2) + 8(ks%2).
+          T2W(3, sm100::mbar_wait(&p_ready[j & 1], ((i * NJ + j) >> 1) & 1));
           sm100::tc_fence_after();
-          for (int kc = 0; kc < FC / 64; ++kc) {
-            const uint32_t b0 = slot_wait();
+          const uint32_t b0 = slot_wait();
+          const uint32_t src = acc_f + (uint32_t)((j & 1) * FC);
 #pragma unroll
-            for (int kk = 0; kk < 4; ++kk) {
-              const int ks = 4 * kc + kk;
-              sm100::mma_f16_ts(acc, acc_f + (uint32_t)(64 * (ks / 4) + 8 * (ks % 4)),
-                                sm100::make_sdesc<128>(b0 + kk * 32), id_N128, 1u);
-            }
-            slot_free();
-          }
+          for (int ks = 0; ks < FC / 16; ++ks)
+            sm100::mma_f16_ts(acc, src + (uint32_t)(32 * (ks / 2) + 8 * (ks % 2)),
+                              sm100::make_sdesc<128>(b0 + ks * 32), id_N128, 1u);
+          slot_free();
         }
         sm100::mma_commit(&out_full);
 #ifdef PREDTOP_TRACE
@@ -324,7 +343,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
       // the previous phase of each x slot completed, so the parity wait below
       // is never two phases ahead (it would alias and return at once)
       sm100::mbar_wait(&o_full, i & 1);
-      const int xit = i * (2 * (D / 64) + D / 32 + NJ * (D / 64 + FC / 64)) + 2 * (D / 64);
+      const int xit = i * (2 * (D / 64) + D / 32 + 2 * NJ) + 2 * (D / 64);
 #pragma unroll
       for (int k = 0; k < 2; ++k) {
         const int itk = xit + 2 * g + k;
@@ -430,25 +449,25 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
       T2(i, 3);
       // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 pairs back into acc_f
       for (int j = 0; j < NJ; ++j) {
-        sm100::mbar_wait(&f_full, (cbase + j) & 1);
+        const int cj = cbase + j;
+        sm100::mbar_wait(&f_full[j & 1], (cj >> 1) & 1);
         sm100::tc_fence_after();
         if (j < 4) T2(i, 4 + j);
-#pragma unroll
-        for (int hf = 0; hf < 2; ++hf) {
-          const int c0 = 64 * g + 32 * hf;
+        {
+          const uint32_t buf = acc_f + (uint32_t)((j & 1) * FC);
           float v[32];
-          sm100::tmem_ld<32>(acc_f + lrow + c0, v);
-          const float* b1 = p_b1 + j * FC + c0;
+          sm100::tmem_ld<32>(buf + lrow + 32 * g, v);
+          const float* b1 = p_b1 + j * FC + 32 * g;
           uint32_t pk[16];
 #pragma unroll
           for (int k = 0; k < 16; ++k)
             pk[k] = sm100::pack_half2(fmaxf(v[2 * k] + b1[2 * k], 0.f), fmaxf(v[2 * k + 1] + b1[2 * k + 1], 0.f));
-          sm100::tmem_st16(acc_f + lrow + 64 * g + 16 * hf, pk);
+          sm100::tmem_st16(buf + lrow + 32 * g, pk);
         }
         sm100::tmem_wait_st();
         sm100::tc_fence_before();
-        sm100::named_bar<kEpi>(1);
-        if (leader) sm100::mbar_arrive(&p_ready);
+        __syncwarp();
+        if (lane == 0) sm100::mbar_arrive(&p_ready[j & 1]);  // this warp's part of P_j is in TMEM
         if (j < 4) T2(i, 8 + j);
       }
       // ---- LN2: z = acc (= h + b_2 + FFN(h))
@@ -533,7 +552,7 @@ int g_sms2 = 0;
 
 }  // namespace
 
-bool layer_tail2_supported(int d, int dff) { return d == D && dff % FC == 0 && dff <= 1024; }
+bool layer_tail2_supported(int d, int dff) { return d == D && dff % (2 * FC) == 0 && dff <= 1024; }  // even chunk count (buffer phases)
 
 predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
                                   __half* x16, int M, cudaStream_t st) {
@@ -549,7 +568,7 @@ predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half*
       !encode_tma_2d(&mp.x16, x16, 2, d, M, 64, 32) || !encode_tma_2d(&mp.x32in, x32, 4, d, M, 32, 128))
     return PREDTOP_ERR_CUDA;
   mp.wo = L.tm_o;
-  mp.w1 = L.tm_1c;
+  mp.w1 = L.tm_1h;
   mp.w2 = L.tm_2;
   Tail2Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
   static bool attr_done = false;
