@@ -245,8 +245,11 @@ struct Attn {
 
 // NW warps per CTA: 8 (a whole 128-row q-tile) or 4 (half of one: two CTAs
 // per work item, so a short last q-tile idles at most 3 warps, not 7).
+#ifndef PREDTOP_ATTN_MINB16
+#define PREDTOP_ATTN_MINB16 8  // CTAs per SM of the 4-warp d_h = 16 kernel (register target)
+#endif
 template <int DH, bool RESIDENT, int NW = 8>
-__global__ void __launch_bounds__(NW * 32, (DH == 16 ? 4 : 2) * (8 / NW))
+__global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_MINB16 : (DH == 16 ? 4 : 2) * (8 / NW))
     k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
            const __half* __restrict__ qkv, __half* __restrict__ out) {
   using A = Attn<DH>;
