@@ -433,6 +433,12 @@ static bool use_tail_v2(int d, int dff) {
   return !(e && e[0] == '1') && layer_tail2_supported(d, dff);
 }
 
+// PREDTOP_TAIL_V3=1: two tiles per CTA sharing the weight ring (layer3.cu)
+static bool use_tail_v3(int d, int dff) {
+  const char* e = getenv("PREDTOP_TAIL_V3");
+  return e && e[0] == '1' && layer_tail3_supported(d, dff);
+}
+
 static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, size_t ws_bytes,
                                    int last_layer, float* latency_out, float* x_out,
                                    cudaStream_t st) {
@@ -469,8 +475,9 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     if ((s = attention_launch(dag, d, H, w.qkv, w.att, st)) != PREDTOP_OK) return s;
     if (use_fused_tail(d, f)) {
       ProfScope _p(PK_LAYER_TAIL, st);
-      s = use_tail_v2(d, f) ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
-                            : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
+      s = use_tail_v3(d, f)   ? layer_tail3_launch(m, l, w.att, w.x32, w.x16, M, st)
+          : use_tail_v2(d, f) ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
+                              : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
       if (s != PREDTOP_OK) return s;
       continue;
     }

@@ -92,6 +92,24 @@ def test_latency_parity_tail_v1(pt, oracle_mod, name, batch_fn, monkeypatch):
     assert err.max() <= TOL
 
 
+@pytest.mark.parametrize("name, batch_fn", [
+    ("gpt", lambda: synth.stage_batch("gpt", 24)),
+    ("gpt", lambda: synth.stage_batch("gpt", 7, first_graph=50)),
+])
+def test_latency_parity_tail_v3(pt, oracle_mod, name, batch_fn, monkeypatch):
+    """The two-tiles-per-CTA fused layer tail (layer3.cu, PREDTOP_TAIL_V3=1);
+    the second batch has an odd number of 128-row tiles (a half-empty pair)."""
+    monkeypatch.setenv("PREDTOP_TAIL_V3", "1")
+    cfg, blob, model = _model(pt, name)
+    batch = batch_fn()
+    y, _ = _gpu_latency(pt, model, batch)
+    want = oracle_mod.forward_batch(cfg, blob, batch)
+    err = _rel(y, want)
+    print(f"{name} (tail v3): max rel err {err.max():.3e}")
+    assert np.isfinite(y).all()
+    assert err.max() <= TOL
+
+
 @pytest.mark.parametrize("name, n", [("paper", 1700), ("moe", 800)])
 def test_latency_parity_streaming_attention(pt, oracle_mod, name, n):
     """Graphs whose K/V do not fit shared memory (d_h = 16: N > 1536; d_h =
