@@ -269,8 +269,15 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   const int W = 2 * ((N + 127) / 128);
   const int nchunks = (N + kChunk - 1) / kChunk;
   const int nbuf = RESIDENT ? nchunks : kStages * kStageChunks;
-  unsigned char* sK = sm100::align1024(dsm_attn);      // [nbuf][64 keys][DH], TMA swizzle
+  // K/V chunks (swizzle period <= 512 B: 256-byte alignment suffices for SW32/SW64
+  // relative addressing... the resident kernel keeps 1 KB alignment only when
+  // the mask staging does not need the room)
+  unsigned char* sK = RESIDENT ? sm100::align256(dsm_attn) : sm100::align1024(dsm_attn);
   unsigned char* sV = sK + (size_t)nbuf * A::CHUNK_BYTES;
+  // resident path: this CTA's mask rows (NW*16 rows x W words) staged in shared
+  // memory by one bulk copy with the K/V, so the per-chunk mask reads in the
+  // inner loop are shared-memory loads, not L2 round trips
+  unsigned char* sM = sV + (size_t)nbuf * A::CHUNK_BYTES;
   const uint64_t* Mg = d.M + d.row_off[g];
   const int ld3 = 3 * dmodel;
   const __half* Qg = qkv + n0 * ld3 + h * DH;
@@ -305,6 +312,10 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   };
   if (threadIdx.x == 0) {
     if (RESIDENT) {
+      const int rows = min(NW * 16, N - rbase);
+      const uint32_t mbytes = (uint32_t)(rows * W * 8);
+      sm100::mbar_expect_tx(&kv_full[0], mbytes);
+      sm100::bulk_load_1d(sM, Mg + (int64_t)rbase * W, mbytes, &kv_full[0]);
       load_chunks(0, nchunks, 0, &kv_full[0]);
     } else {
       for (int s = 0; s < kStages && s * kStageChunks < nchunks; ++s)
@@ -348,16 +359,19 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   // this thread's 16 mask bits of rows a / b in chunk c: 16-bit piece tq of
   // the (stored-layout) word; raw pieces, combined only where used, so the
   // loads for chunk c+1 are issued before chunk c and hide behind it
-  const uint16_t* Ma16 = reinterpret_cast<const uint16_t*>(Ma) + tq;
-  const uint16_t* Mb16 = reinterpret_cast<const uint16_t*>(Mb) + tq;
+  const uint16_t* Ma16 = RESIDENT ? reinterpret_cast<const uint16_t*>(sM + (size_t)(warp * 16 + gq) * W * 8) + tq
+                                  : reinterpret_cast<const uint16_t*>(Ma) + tq;
+  const uint16_t* Mb16 = RESIDENT ? Ma16 + 8 * W * 4 : reinterpret_cast<const uint16_t*>(Mb) + tq;
   auto mask_lo = [&](int c) -> uint32_t { return va ? (uint32_t)Ma16[4 * c] : 0u; };
   auto mask_hi = [&](int c) -> uint32_t { return vb ? (uint32_t)Mb16[4 * c] : 0u; };
-  uint32_t mlo = mask_lo(0), mhi = mask_hi(0);
+  uint32_t mlo = RESIDENT ? 0u : mask_lo(0), mhi = RESIDENT ? 0u : mask_hi(0);
   const uint32_t kb0 = sm100::smem_u32(sK), vb0 = sm100::smem_u32(sV);
 
   if (RESIDENT) {
     sm100::mbar_wait(&kv_full[0], 0);
     if (!warp_live) return;
+    mlo = mask_lo(0);
+    mhi = mask_hi(0);
     uint32_t fl = Fw[0];
     for (int c = 0; c < nchunks; ++c) {
       const bool more = c + 1 < nchunks;
@@ -621,6 +635,9 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
   const int G = dag->desc.num_graphs;
   const int maxch = (int)ceil_div(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), kChunk);
   const int resident_bytes = 2 * maxch * CH_BYTES + 1024;
+  // the 4-warp resident kernel also stages its 64 mask rows (W words each)
+  const int wmax = 2 * (int)ceil_div(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), 128);
+  const int resident4_bytes = 2 * maxch * CH_BYTES + 64 * wmax * 8 + 256;
   CUtensorMap tkv;
   if (!encode_tma_2d(&tkv, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kChunk))
     return PREDTOP_ERR_CUDA;
@@ -645,23 +662,23 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
     const int64_t items = (int64_t)G * H;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(items, (int64_t)sms * per_sm));
     k_attn_p<DH><<<grid, 256, pers_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, maxch);
-  } else if (half_tiles && resident_bytes * 8 <= 200 * 1024) {
-    // 4-warp CTAs (half q-tiles), up to 8 per SM
+  } else if (half_tiles && resident4_bytes <= 28 * 1024) {
+    // 4-warp CTAs (half q-tiles), up to 8 per SM (28 KB + 1 KB static each)
     static bool attr_h = false;
     if (!attr_h) {
       PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       25 * 1024));
+                                       28 * 1024));
       attr_h = true;
     }
-    k_attn<DH, true, 4><<<2 * blocks, 128, resident_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
-  } else if (resident_bytes <= 100 * 1024) {
+    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+  } else if (resident_bytes + 128 * wmax * 8 <= 100 * 1024) {
     static bool attr_done = false;
     if (!attr_done) {
       PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        100 * 1024));
       attr_done = true;
     }
-    k_attn<DH, true><<<blocks, 256, resident_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out);
   } else {
     constexpr int stream_bytes = 2 * kStages * kStageChunks * CH_BYTES + 1024;
     static bool attr_s = false;
