@@ -109,7 +109,12 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
 }
 
 // K1: validation + successor CSR + Kahn levels / depth.  One CTA per graph.
-__global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc) {
+// With `smem_nodes` >= N the in-degree counters and the Kahn queue live in
+// shared memory (the per-level atomicSub and the frontier reads are then
+// shared-memory round trips, not L2 ones: a deep graph runs ~11k levels)
+// and the queue is copied to global (topo) at the end.
+__global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_nodes) {
+  extern __shared__ __align__(16) int32_t sm_depth[];
   const int g = blockIdx.x;
   if (d.status[g] != PREDTOP_OK) return;
   if (is_small((int)(d.node_ptr[g + 1] - d.node_ptr[g]), (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
@@ -119,11 +124,13 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc) {
   const int N = (int)(d.node_ptr[g + 1] - n0);
   const int64_t e0 = d.edge_ptr[g];
   const int E = (int)(d.edge_ptr[g + 1] - e0);
-  int32_t* indeg = d.indeg + n0;
+  const bool in_smem = N <= smem_nodes;
+  int32_t* indeg = in_smem ? sm_depth : d.indeg + n0;
   int32_t* soff = d.succ_off + n0 + g;   // N+1
   int32_t* lptr = d.level_ptr + n0 + g;  // N+1 (first used as fill cursor)
   int32_t* succ = d.succ + e0;
-  int32_t* topo = d.topo + n0;
+  int32_t* const topo_g = d.topo + n0;
+  int32_t* topo = in_smem ? sm_depth + smem_nodes : topo_g;
   int32_t* depth = d.depth + n0;
   const int32_t* src = d.src + e0;
   const int32_t* dst = d.dst + e0;
@@ -199,6 +206,8 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc) {
     __syncthreads();
   }
   if (tid == 0) d.num_levels[g] = level;
+  if (in_smem)
+    for (int i = tid; i < le; i += nt) topo_g[i] = topo[i];
   if (le != N) {
     if (tid == 0) {
       d.status[g] = PREDTOP_ERR_CYCLE;
@@ -738,8 +747,16 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
     PT_LAUNCH_CHECK();
   }
 {
+    // in-degrees and the Kahn queue in shared memory when the largest graph fits
+    const int smem_nodes = b.max_nodes <= 26 * 1024 ? b.max_nodes : 0;
+    const int dsm = 2 * 4 * smem_nodes;
+    static int attr_depth = 0;
+    if (dsm > 48 * 1024 && dsm > attr_depth) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_depth, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm));
+      attr_depth = dsm;
+    }
     ProfScope _p(PK_DAG_DEPTH, st);
-    k_depth<<<G, 256, 0, st>>>(d, sc);
+    k_depth<<<G, 256, dsm, st>>>(d, sc, smem_nodes);
     PT_LAUNCH_CHECK();
   }
   // closure: shared memory for a column slice of all rows of the largest graph
