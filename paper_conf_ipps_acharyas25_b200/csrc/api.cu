@@ -67,6 +67,7 @@ static size_t carve_dag(const predtop_batch_desc* b, const DagBounds& bd, void* 
   t.succ_off = c.take<int32_t>(N + G);
   t.succ = c.take<int32_t>(E);
   t.indeg = c.take<int32_t>(N);
+  t.rec = c.take<int4>(N);
   t.R = c.take<uint64_t>(bd.words);
   t.M = c.take<uint64_t>(bd.words);
   t.tile_cnt = c.take<int32_t>(bd.tiles);

@@ -208,6 +208,16 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_n
   if (tid == 0) d.num_levels[g] = level;
   if (in_smem)
     for (int i = tid; i < le; i += nt) topo_g[i] = topo[i];
+  if (le == N) {  // closure records in topo order: node, degree, first four successors inline
+    int4* rec = d.rec + n0;
+    for (int i = tid; i < N; i += nt) {
+      const int v = topo[i];
+      const int b = soff[v], deg = soff[v + 1] - b;
+      int s4[4] = {0, 0, 0, 0};
+      for (int k = 0; k < 4 && k < deg; ++k) s4[k] = succ[b + k];
+      rec[i] = make_int4(v | (min(deg, 0xFFFF) << 16), s4[0] | (s4[1] << 16), s4[2] | (s4[3] << 16), b);
+    }
+  }
   if (le != N) {
     if (tid == 0) {
       d.status[g] = PREDTOP_ERR_CYCLE;
@@ -253,6 +263,100 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   const int32_t* soff = d.succ_off + n0 + g;
   const int32_t* succ = d.succ + d.edge_ptr[g];
   const int32_t* lptr = d.level_ptr + n0 + g;
+  const int K = d.hops;
+  if (!csr_in_smem && !global_mode && !(K > 0 && K < L - 1)) {
+    // Deep graphs whose CSR does not fit next to the slice (e.g. 16k nodes,
+    // ~11k levels): the level loop is latency-bound, so it reads per-node
+    // records (node, degree, first four successors; built by k_depth in topo
+    // order) prefetched four levels ahead into registers, and the level
+    // bounds from a shared-memory copy: no dependent L2 round trip per level.
+    uint64_t* Rsm = reinterpret_cast<uint64_t*>(sm);
+    const int rs2 = CW;
+    const size_t slice_bytes = align_up((size_t)N * CW * 8, 16);
+    const bool lptr_smem = slice_bytes + (size_t)4 * (L + 1) <= (size_t)smem_bytes;
+    int32_t* s_lp = reinterpret_cast<int32_t*>(sm + slice_bytes);
+    if (lptr_smem)
+      for (int i = tid; i <= L; i += nt) s_lp[i] = lptr[i];
+    const int32_t* lp = lptr_smem ? s_lp : lptr;
+    const int4* rec = d.rec + n0;
+    for (int64_t it = tid; it < (int64_t)N * nw; it += nt) Rsm[(it / nw) * rs2 + it % nw] = 0;
+    __syncthreads();
+    // the level loop runs on warp 0 alone (levels hold ~1-2 nodes): warp
+    // barriers instead of CTA barriers between levels
+    if (tid >= 32) return;
+    auto first_rec = [&](int l) -> int4 {  // this thread's first item of level l
+      if (l < 0) return make_int4(0, 0, 0, 0);
+      const int b = lp[l], e = lp[l + 1];
+      return tid < (e - b) * nw ? __ldg(rec + b + tid / nw) : make_int4(0, 0, 0, 0);
+    };
+    // level `level` with its prefetched first record r; then r <- the record of
+    // level - 4 (four fixed registers, unrolled by four: no register moves, so
+    // a load is only waited for when its level comes up)
+    auto do_level = [&](int level, int4& r0) {
+      const int lb = lp[level], items = (lp[level + 1] - lb) * nw;
+      if (nw == 1) {  // one word column (the deep-graph case): no index division
+        const uint32_t w0 = (uint32_t)word0;
+        for (int i = tid; i < items; i += 32) {
+          const int4 r = i == tid ? r0 : __ldg(rec + lb + i);
+          const uint32_t v = (uint32_t)r.x & 0xFFFFu, deg = (uint32_t)r.x >> 16;
+          const uint32_t s4[4] = {(uint32_t)r.y & 0xFFFFu, (uint32_t)r.y >> 16, (uint32_t)r.z & 0xFFFFu,
+                                  (uint32_t)r.z >> 16};
+          uint64_t acc = 0;
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            if ((uint32_t)k < deg) {
+              const uint32_t w = s4[k];
+              acc |= Rsm[w] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
+            }
+          if (deg > 4) {
+            const uint32_t dg = deg == 0xFFFFu ? (uint32_t)(soff[v + 1] - r.w) : deg;
+            for (uint32_t k = 4; k < dg; ++k) {
+              const uint32_t w = (uint32_t)succ[r.w + k];
+              acc |= Rsm[w] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
+            }
+          }
+          Rsm[v] = acc;
+        }
+        r0 = first_rec(level - 4);
+        __syncwarp();
+        return;
+      }
+      for (int it = tid; it < items; it += 32) {
+        const int4 r = it == tid ? r0 : __ldg(rec + lb + it / nw);
+        const int v = r.x & 0xFFFF;
+        int deg = (int)((unsigned)r.x >> 16);
+        if (deg == 0xFFFF) deg = soff[v + 1] - r.w;  // capped in the record
+        const int j = it % nw, word = word0 + j;
+        uint64_t acc = 0;
+        const int s4[4] = {r.y & 0xFFFF, (int)((unsigned)r.y >> 16), r.z & 0xFFFF, (int)((unsigned)r.z >> 16)};
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          if (k < deg) {
+            const int w = s4[k];
+            acc |= Rsm[(int64_t)w * rs2 + j];
+            if ((w >> 6) == word) acc |= 1ull << (w & 63);
+          }
+        for (int k = 4; k < deg; ++k) {
+          const int w = succ[r.w + k];
+          acc |= Rsm[(int64_t)w * rs2 + j];
+          if ((w >> 6) == word) acc |= 1ull << (w & 63);
+        }
+        Rsm[(int64_t)v * rs2 + j] = acc;
+      }
+      r0 = first_rec(level - 4);
+      __syncwarp();
+    };
+    int4 r0 = first_rec(L - 1), r1 = first_rec(L - 2), r2 = first_rec(L - 3), r3 = first_rec(L - 4);
+    for (int level = L - 1; level >= 0; level -= 4) {
+      do_level(level, r0);
+      if (level >= 1) do_level(level - 1, r1);
+      if (level >= 2) do_level(level - 2, r2);
+      if (level >= 3) do_level(level - 3, r3);
+    }
+    for (int64_t it = tid; it < (int64_t)N * nw; it += 32)
+      Rg[(it / nw) * W + word0 + it % nw] = Rsm[(it / nw) * rs2 + it % nw];
+    return;
+  }
   uint64_t* Rs;
   int64_t rs;  // row stride of Rs in words
   if (csr_in_smem) {
@@ -273,7 +377,6 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
     Rs = (uint64_t*)(sm + (csr_in_smem ? csr_bytes : 0));
     rs = CW;
   }
-  const int K = d.hops;
   if (K > 0 && K < L - 1) {
     __syncthreads();  // the staged CSR above
     // finite-k DAGRA: K synchronous rounds over all rows,

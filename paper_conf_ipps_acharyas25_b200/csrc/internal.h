@@ -35,6 +35,8 @@ struct DagDev {
   int32_t* succ_off;   // [N_tot + G] graph g at node_ptr[g] + g
   int32_t* succ;       // [E]  graph-local successor lists
   int32_t* indeg;      // [N_tot]
+  int4* rec;           // [N_tot] per topo position: {v | deg << 16, s0 | s1 << 16, s2 | s3 << 16, soff[v]}
+                       // (the first four successors inline; large-graph closure)
   // bitsets and tiles
   uint64_t* R;         // [sum N_g W_g]
   uint64_t* M;         // [sum N_g W_g]  STORED layout: mask_perm of each 64-key word
