@@ -68,11 +68,17 @@ class StageTableSearch:
             m.forward(self.dag, workspace=self.ws, out=self.mine[0, c, self.g0:self.g1])
 
     def gather(self):
-        """Step 3 (multi-GPU): the exact sum-all-reduce of disjoint ranges."""
+        """Step 3 (multi-GPU): the exact sum-all-reduce of disjoint ranges
+        (NCCL on the device tensor; a host round trip for gloo)."""
         if self.world > 1:
             import torch.distributed as dist
-            self.table.copy_(self.mine)
-            dist.all_reduce(self.table, group=self.group)
+            if dist.get_backend(self.group) == "gloo":
+                t = self.mine.cpu()
+                dist.all_reduce(t, group=self.group)
+                self.table.copy_(t)
+            else:
+                self.table.copy_(self.mine)
+                dist.all_reduce(self.table, group=self.group)
 
     def step(self):
         self.score()
