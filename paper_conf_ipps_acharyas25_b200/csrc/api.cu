@@ -400,7 +400,9 @@ predtop_status predtop_model_create(const predtop_model_config* cfg, const float
               encode_tma_2d_f16(&L.tm_1, L.W1, d, f, kch_for(d), m->bn_ff1) &&
               encode_tma_2d_f16(&L.tm_2, L.W2, f, d, kch_for(f), d) &&
               (f < 128 || encode_tma_2d_f16(&L.tm_1c, L.W1, d, f, kch_for(d), 128)) &&
-              (f < 64 || encode_tma_2d_f16(&L.tm_1h, L.W1, d, f, kch_for(d), 64));
+              (f < 64 || encode_tma_2d_f16(&L.tm_1h, L.W1, d, f, kch_for(d), 64)) &&
+              (d != 256 || (encode_tma_2d_f16(&L.tm_o32, L.Wo, d, d, 32, d) &&
+                            encode_tma_2d_f16(&L.tm_2_32, L.W2, f, d, 32, d)));
     if (!ok) {
       delete m;
       return PREDTOP_ERR_CUDA;
@@ -459,6 +461,13 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
       !encode_tma_2d_f16(&tm_att, w.att, d, Ntot, kch_for(d), 128) ||
       !encode_tma_2d_f16(&tm_hid, w.hid, f, Ntot, kch_for(f), 128))
     return PREDTOP_ERR_CUDA;
+  // d = 256 LayerNorm GEMMs: the fp32 residual tile takes 128 KB of staging,
+  // so 64-wide K-slices leave a one-stage operand ring; 32-wide slices give 3
+  const bool ln32 = d == 256;
+  CUtensorMap tm_att32, tm_hid32;
+  if (ln32 && (!encode_tma_2d_f16(&tm_att32, w.att, d, Ntot, 32, 128) ||
+               !encode_tma_2d_f16(&tm_hid32, w.hid, f, Ntot, 32, 128)))
+    return PREDTOP_ERR_CUDA;
   predtop_status s;
   const int pe_rows = std::min<int>(dag->desc.max_nodes, PREDTOP_MAX_NODES);
   if ((s = pe_table_launch(w.pe, pe_rows, d, st)) != PREDTOP_OK) return s;
@@ -487,7 +496,10 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     a.gamma = L.g1; a.beta = L.be1; a.eps = m->cfg.ln_eps;
     {
       ProfScope _p(PK_GEMM_O_LN, st);
-      if ((s = gemm_launch(&tm_att, &L.tm_o, d, EPI_BIAS_RESID_LN, a, st)) != PREDTOP_OK) return s;
+      a.kch = ln32 ? 32 : 0;
+      if ((s = gemm_launch(ln32 ? &tm_att32 : &tm_att, ln32 ? &L.tm_o32 : &L.tm_o, d, EPI_BIAS_RESID_LN, a, st)) !=
+          PREDTOP_OK)
+        return s;
     }
     a = GemmArgs{};
     a.M = M; a.K = d; a.N = f; a.bias = L.b1; a.out16 = w.hid;
@@ -500,7 +512,10 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     a.gamma = L.g2; a.beta = L.be2; a.eps = m->cfg.ln_eps;
     {
       ProfScope _p(PK_GEMM_FF2_LN, st);
-      if ((s = gemm_launch(&tm_hid, &L.tm_2, d, EPI_BIAS_RESID_LN, a, st)) != PREDTOP_OK) return s;
+      a.kch = ln32 ? 32 : 0;
+      if ((s = gemm_launch(ln32 ? &tm_hid32 : &tm_hid, ln32 ? &L.tm_2_32 : &L.tm_2, d, EPI_BIAS_RESID_LN, a, st)) !=
+          PREDTOP_OK)
+        return s;
     }
   }
   if (latency_out)

@@ -473,6 +473,7 @@ predtop_status gemm_launch(const CUtensorMap* tmA, const CUtensorMap* tmB, int b
   } else {
     m.out16w = m.out16;
   }
+  if (a.kch == 32 && a.K % 32 == 0) return launch_bn<32>(bn, epi, m, a, st);
   if (a.K % 64 == 0) return launch_bn<64>(bn, epi, m, a, st);
   if (a.K == 32) return launch_bn<32>(bn, epi, m, a, st);
   set_error("unsupported GEMM K=%d", a.K);

@@ -114,6 +114,7 @@ struct LayerDev {
   CUtensorMap tm_qkv, tm_o, tm_1, tm_2;  // B-operand TMA maps (unfused GEMMs)
   CUtensorMap tm_1c;                     // W_1 in 128-row chunks (fused layer tail v1)
   CUtensorMap tm_1h;                     // W_1 in 64-row chunks (layer tail v2)
+  CUtensorMap tm_o32, tm_2_32;           // W_o, W_2 in 32-wide K-slices (LN GEMMs at d = 256)
 };
 
 }  // namespace predtop
@@ -158,6 +159,7 @@ struct GemmArgs {
   float eps;
   int qcols;      // bias epilogue: output columns [0, qcols) are multiplied by qscale
   float qscale;   // (QKV: Q pre-scaled by log2(e)/sqrt(d_h) for the attention kernel)
+  int kch;        // K-slice of the operand maps (0: 64 if K % 64 == 0, else 32)
 };
 predtop_status gemm_launch(const CUtensorMap* tmA, const CUtensorMap* tmB, int bn, int epi,
                            const GemmArgs& a, cudaStream_t st);
