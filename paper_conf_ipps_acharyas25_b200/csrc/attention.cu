@@ -83,8 +83,15 @@ __device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4]
 }
 
 constexpr int kChunk = 64;
-constexpr int kStages = 3;       // streaming path: ring of stages ...
-constexpr int kStageChunks = 4;  // ... of 4 chunks (256 keys) each
+#ifndef PREDTOP_ATTN_MINB32
+#define PREDTOP_ATTN_MINB32 3  // CTAs per SM of the 8-warp d_h = 32 kernels (78 registers)
+#endif
+constexpr int kStages = 3;  // streaming path: a ring of 3 stages of stage_chunks<DH>() 64-key chunks
+// d_h = 16: 4 chunks (256 keys, 48 KB of ring, 4 CTAs/SM); d_h = 32: 2 chunks
+// (128 keys, 48 KB, so 3 CTAs/SM fit -- 1xB200 MoE attention 20.9 -> 18.3 ms/step
+// against 4 chunks at 2 CTAs/SM)
+template <int DH>
+constexpr int stage_chunks() { return DH == 32 ? 2 : 4; }
 
 // flag nibble f (bit j = block j fully allowed) -> the thread's mask bits of
 // those blocks in rows a (bits 0-15) and b (bits 16-31): nibble j of each half
@@ -249,10 +256,12 @@ struct Attn {
 #define PREDTOP_ATTN_MINB16 8  // CTAs per SM of the 4-warp d_h = 16 kernel (register target)
 #endif
 template <int DH, bool RESIDENT, int NW = 8>
-__global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_MINB16 : (DH == 16 ? 4 : 2) * (8 / NW))
+__global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_MINB16
+                                           : (DH == 16 ? 4 : PREDTOP_ATTN_MINB32) * (8 / NW))
     k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
            const __half* __restrict__ qkv, __half* __restrict__ out) {
   using A = Attn<DH>;
+  constexpr int kStageChunks = stage_chunks<DH>();
   extern __shared__ __align__(16) unsigned char dsm_attn[];
   __shared__ __align__(8) uint64_t kv_full[kStages];
   const int h = blockIdx.x % H;
@@ -680,7 +689,7 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
     }
     k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out);
   } else {
-    constexpr int stream_bytes = 2 * kStages * kStageChunks * CH_BYTES + 1024;
+    constexpr int stream_bytes = 2 * kStages * stage_chunks<DH>() * CH_BYTES + 1024;
     static bool attr_s = false;
     if (!attr_s) {
       PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
