@@ -93,3 +93,38 @@ def test_no_gpu_fails_loudly(libpath):
                              None, None)
     assert st == pt.CUDA
     assert b"device" in L.predtop_last_error()
+
+
+def test_next_rows_host_validation(libpath):
+    """Host-checkable argument errors of the NEXT-row entry points (finite-k
+    DAGRA, graph pruning, plan search) are reported without touching a GPU."""
+    from paper_conf_ipps_acharyas25_b200 import predtop as pt
+    L = pt.lib()
+    # hops < 0 -> INVALID_ARG (before any device work)
+    d = pt.BatchDesc(1, 4, 4, 3, 0, -1)
+    h = ctypes.c_void_p()
+    dummy = ctypes.c_void_p(256)
+    st = L.predtop_build_dag(ctypes.byref(d), dummy, dummy, dummy, dummy, dummy, dummy, 1 << 20, None,
+                             ctypes.byref(h), None, None)
+    assert st == pt.INVALID_ARG and b"hops" in L.predtop_last_error()
+    # plan search: sizes and workspace
+    assert L.predtop_plan_search_workspace(0, 4, 1) == 0
+    assert L.predtop_plan_search_workspace(1, 65, 1) == 0          # L > 64
+    assert L.predtop_plan_search_workspace(1, 4, 33) == 0          # K > 32
+    assert L.predtop_plan_search_workspace(7, 24, 6) == (7 * 6 * 300 * 8 + 255) // 256 * 256  # fp64 per candidate
+    dev = (ctypes.c_int32 * 1)(0)                                   # a choice with 0 devices
+    st = L.predtop_plan_search(1, 4, 1, dev, 1, dummy, 10, 1, None, dummy, dummy, dummy, dummy, dummy,
+                               dummy, 1 << 20, None)
+    assert st == pt.INVALID_ARG
+    dev = (ctypes.c_int32 * 1)(1)
+    st = L.predtop_plan_search(1, 4, 1, dev, 1, dummy, 9, 1, None, dummy, dummy, dummy, dummy, dummy,
+                               dummy, 1 << 20, None)                # stride < L(L+1)/2
+    assert st == pt.INVALID_ARG
+    # pruning: no ops / too many ops
+    d = pt.BatchDesc(1, 4, 4, 3, 0)
+    assert L.predtop_prune_workspace(ctypes.byref(d)) > 0
+    ops = (ctypes.c_uint16 * 1)(64)
+    tot = (ctypes.c_int64 * 2)()
+    st = L.predtop_prune_graphs(ctypes.byref(d), dummy, dummy, dummy, dummy, dummy, ops, 0, dummy, 1 << 20,
+                                dummy, dummy, dummy, dummy, 10, dummy, tot, None, None)
+    assert st == pt.INVALID_ARG
