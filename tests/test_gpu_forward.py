@@ -194,3 +194,19 @@ def test_full_gpt_config_sampled(pt, oracle_mod):
     err = _rel(y[sample], want)
     print(f"gpt full: max rel err {err.max():.3e} median {np.median(err):.3e}")
     assert err.max() <= TOL
+
+
+@pytest.mark.slow
+def test_full_moe_config_sampled(pt, oracle_mod):
+    """configs[2] at full size (512 MoE-style graphs of ~1500 ops in one
+    batch: the bench launch configuration, streaming d_h = 32 attention and
+    the d = 256 GEMM path); oracle on a sample of graphs."""
+    cfg, blob, model = _model(pt, "moe")
+    batch = synth.stage_batch("moe", 512)
+    y, _ = _gpu_latency(pt, model, batch)
+    assert np.isfinite(y).all()
+    sample = [0, 171, 342, 511]
+    want = oracle_mod.forward_batch(cfg, blob, batch, graphs=sample)
+    err = _rel(y[sample], want)
+    print(f"moe full: max rel err {err.max():.3e}")
+    assert err.max() <= TOL

@@ -172,3 +172,37 @@ def test_stage_table_end_to_end(pt, oracle_mod):
         Tw, _ = oracle_mod.plan_search(dense, dev, 2, B)
         assert T == Tw
         _valid(oracle_mod, dense, dev, 2, B, T, st)
+
+
+@pytest.mark.slow
+def test_search_config_full_size_sampled(pt, oracle_mod):
+    """The --config search workload at full size (300 layer-range stages of
+    GPT-3's 24 layers x 6 mesh models): sampled table entries against the
+    oracle forward, and the plan search on the GPU table == exhaustive
+    enumeration on the same table."""
+    from paper_conf_ipps_acharyas25_b200 import stage_table
+    L = 24
+    host = synth.layer_range_stages("gpt", L)
+    cfgs = synth.mesh_model_configs("search", 6)
+    blobs = [synth.pack_weights(c, synth.model_weights(c)) for c in cfgs]
+    dev, Bs = [d for _, d in synth.MESH_CHOICES], [1, 16, 64]
+    sts = stage_table.StageTableSearch(pt, cfgs, blobs, host, L, dev, 4, Bs)
+    sts.step()
+    torch.cuda.synchronize()
+    table = sts.table[0].cpu().numpy()
+    assert np.isfinite(table).all() and (table > 0).all()
+    # stages of 1, 3, 6 and 4 layers (~190 to ~1100 ops) on four of the mesh models
+    picks = [(0, [synth.tri_index(0, 0, L), synth.tri_index(0, 2, L)]), (2, [synth.tri_index(3, 8, L)]),
+             (3, [synth.tri_index(10, 13, L)]), (5, [synth.tri_index(23, 23, L)])]
+    for c, gs in picks:
+        want = oracle_mod.forward_batch(cfgs[c], blobs[c], host, graphs=gs)
+        err = np.abs(table[c, gs] - want) / np.abs(want)
+        assert err.max() <= 2e-3, (c, err)
+    dense = np.full((L, L, 6), np.inf, np.float32)
+    for i in range(L):
+        for j in range(i, L):
+            dense[i, j] = table[:, synth.tri_index(i, j, L)]
+    for B, (T, st) in zip(Bs, sts.search.plans()):
+        Tw, _ = oracle_mod.plan_search(dense, dev, 4, B)
+        assert T == Tw
+        _valid(oracle_mod, dense, dev, 4, B, T, st)
