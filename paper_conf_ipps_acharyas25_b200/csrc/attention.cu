@@ -83,6 +83,12 @@ __device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4]
 }
 
 constexpr int kChunk = 64;
+// graphs whose mask allows at most this fraction of the N^2 pairs go to the
+// gather kernel k_attn_sparse when the DAG was built with a finite k (hops)
+constexpr int kSparseDensityInv = 5;  // density <= 1/5
+__device__ __forceinline__ bool is_sparse(const DagDev& d, int g, int N) {
+  return d.pairs[g] * kSparseDensityInv <= (int64_t)N * N;
+}
 #ifndef PREDTOP_ATTN_MINB32
 #define PREDTOP_ATTN_MINB32 3  // CTAs per SM of the 8-warp d_h = 32 kernels (78 registers)
 #endif
@@ -259,7 +265,7 @@ template <int DH, bool RESIDENT, int NW = 8>
 __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_MINB16
                                            : (DH == 16 ? 4 : PREDTOP_ATTN_MINB32) * (8 / NW))
     k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
-           const __half* __restrict__ qkv, __half* __restrict__ out) {
+           const __half* __restrict__ qkv, __half* __restrict__ out, int sparse_split) {
   using A = Attn<DH>;
   constexpr int kStageChunks = stage_chunks<DH>();
   extern __shared__ __align__(16) unsigned char dsm_attn[];
@@ -275,6 +281,7 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   const int N = (int)(d.node_ptr[g + 1] - n0);
   const int rbase = qt * 128 + part * NW * 16;  // first query row of this CTA
   if (rbase >= N) return;
+  if (sparse_split && is_sparse(d, g, N)) return;  // k_attn_sparse takes this graph
   const int W = 2 * ((N + 127) / 128);
   const int nchunks = (N + kChunk - 1) / kChunk;
   const int nbuf = RESIDENT ? nchunks : kStages * kStageChunks;
@@ -637,6 +644,130 @@ __global__ void __launch_bounds__(256, DH == 16 ? PREDTOP_ATTN_P_CTAS : 2)
   }
 }
 
+// Sparse masks (finite-k DAGRA: at k = 4 ~6 % of the N^2 pairs
+// are allowed and the 16-key blocks above compute ~9 scores per useful one).
+// Opt-in experiment (slower, see launch_dh): one thread per query row walks the set bits of its mask row and
+// gathers the allowed keys one by one from the resident K/V chunks -- scores
+// and the online softmax in fp32 on the CUDA cores, work proportional to |A|.
+// One CTA = (graph, 128-row q-tile, head); graphs of density > kSparseDensity
+// stay on k_attn (which skips the sparse ones when both are launched).
+template <int DH>
+__global__ void __launch_bounds__(128) k_attn_sparse(const __grid_constant__ CUtensorMap tkv, DagDev d, int G,
+                                                     int H, int dmodel, const __half* __restrict__ qkv,
+                                                     __half* __restrict__ out) {
+  constexpr int RB = DH * 2, CHB = kChunk * RB;
+  extern __shared__ __align__(16) unsigned char dsm_sp[];
+  __shared__ __align__(8) uint64_t kv_full;
+  const int h = blockIdx.x % H;
+  const int widx = blockIdx.x / H;
+  if (widx >= d.qtile_off[G]) return;
+  const int2 wk = d.work[widx];
+  const int g = wk.x, qt = wk.y;
+  if (d.status[g] != PREDTOP_OK) return;
+  const int64_t n0 = d.node_ptr[g];
+  const int N = (int)(d.node_ptr[g + 1] - n0);
+  if (!is_sparse(d, g, N)) return;
+  const int W = 2 * ((N + 127) / 128);
+  const int nchunks = (N + kChunk - 1) / kChunk;
+  unsigned char* sK = sm100::align256(dsm_sp);
+  unsigned char* sV = sK + (size_t)nchunks * CHB;
+  if (threadIdx.x == 0) {
+    sm100::mbar_init(&kv_full, 1);
+    sm100::fence_mbar_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    sm100::mbar_arrive_expect_tx(&kv_full, (uint32_t)(nchunks * 2 * CHB));
+    for (int c = 0; c < nchunks; ++c) {
+      sm100::tma_load_2d(sK + c * CHB, &tkv, &kv_full, dmodel + h * DH, (int)(n0 + c * kChunk));
+      sm100::tma_load_2d(sV + c * CHB, &tkv, &kv_full, 2 * dmodel + h * DH, (int)(n0 + c * kChunk));
+    }
+  }
+  const int r = qt * 128 + threadIdx.x;
+  const bool valid = r < N;
+  float q[DH];
+  if (valid) {
+    const uint4* qp = reinterpret_cast<const uint4*>(qkv + (n0 + r) * 3 * dmodel + h * DH);
+#pragma unroll
+    for (int p = 0; p < DH / 8; ++p) {
+      const uint4 u = qp[p];
+      const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w4[e]));
+        q[8 * p + 2 * e] = f.x;
+        q[8 * p + 2 * e + 1] = f.y;
+      }
+    }
+  }
+  sm100::mbar_wait(&kv_full, 0);
+  if (!valid) return;
+  // row k of a swizzled [64 x DH] chunk: 16-byte piece p at rr*RB + 16*(p ^ sw(rr))
+  auto row_dot = [&](const unsigned char* base, int k) -> float {
+    const int rr = k & 63;
+    const unsigned char* rowp = base + (k >> 6) * CHB + rr * RB;
+    const int sw = ((rr * RB) >> 7) & (RB / 16 - 1);
+    float acc = 0.f;
+#pragma unroll
+    for (int p = 0; p < DH / 8; ++p) {
+      const uint4 u = *reinterpret_cast<const uint4*>(rowp + 16 * (p ^ sw));
+      const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w4[e]));
+        acc = fmaf(q[8 * p + 2 * e], f.x, acc);
+        acc = fmaf(q[8 * p + 2 * e + 1], f.y, acc);
+      }
+    }
+    return acc;
+  };
+  float o[DH];
+#pragma unroll
+  for (int e = 0; e < DH; ++e) o[e] = 0.f;
+  float m = row_dot(sK, r), l = 0.f;  // reference: the diagonal score (M includes I)
+  const uint64_t* Mr = d.M + d.row_off[g] + (int64_t)r * W;
+  for (int c = 0; c < nchunks; ++c) {
+    uint64_t w = Mr[c];
+    while (w) {
+      const int b = __ffsll((long long)w) - 1;
+      w &= w - 1;
+      // stored bit b -> key: b = 16*((k>>1)&3) + 2*(k>>3) + (k&1) (internal.h mask_pos)
+      const int rem = b & 15;
+      const int k = c * 64 + ((rem >> 1) << 3) + ((b >> 4) << 1) + (rem & 1);
+      const float sc = row_dot(sK, k);
+      if (sc > m) {  // online softmax in log2 units (Q pre-scaled by log2 e / sqrt(d_h))
+        const float a = ex2(m - sc);
+        l *= a;
+#pragma unroll
+        for (int e = 0; e < DH; ++e) o[e] *= a;
+        m = sc;
+      }
+      const float pw = ex2(sc - m);
+      l += pw;
+      const int rr = k & 63;
+      const unsigned char* vrow = sV + (k >> 6) * CHB + rr * RB;
+      const int sw = ((rr * RB) >> 7) & (RB / 16 - 1);
+#pragma unroll
+      for (int p = 0; p < DH / 8; ++p) {
+        const uint4 u = *reinterpret_cast<const uint4*>(vrow + 16 * (p ^ sw));
+        const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w4[e]));
+          o[8 * p + 2 * e] = fmaf(pw, f.x, o[8 * p + 2 * e]);
+          o[8 * p + 2 * e + 1] = fmaf(pw, f.y, o[8 * p + 2 * e + 1]);
+        }
+      }
+    }
+  }
+  const float il = l > 0.f ? 1.f / l : 0.f;
+  uint4* op = reinterpret_cast<uint4*>(out + (n0 + r) * dmodel + h * DH);
+#pragma unroll
+  for (int p = 0; p < DH / 8; ++p)
+    op[p] = make_uint4(pack_h2(o[8 * p] * il, o[8 * p + 1] * il), pack_h2(o[8 * p + 2] * il, o[8 * p + 3] * il),
+                       pack_h2(o[8 * p + 4] * il, o[8 * p + 5] * il), pack_h2(o[8 * p + 6] * il, o[8 * p + 7] * il));
+}
+
 template <int DH>
 predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
                          cudaStream_t st, unsigned blocks) {
@@ -650,6 +781,26 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
   CUtensorMap tkv;
   if (!encode_tma_2d(&tkv, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kChunk))
     return PREDTOP_ERR_CUDA;
+  // finite-k masks: graphs of low density go to the gather kernel (K/V resident:
+  // only when the batch's largest graph fits 2 x 24 KB... up to ~96 KB)
+  const int sparse_bytes = 2 * maxch * CH_BYTES + 256;
+  // opt-in (PREDTOP_ATTN_SPARSE=1): measured 2.5x slower than the block-sparse
+  // MMA kernel at k = 4 on the GPT config (2.75 vs 1.08 ms/step: one thread
+  // per row diverges on the per-row key counts and gathers 32-byte rows one
+  // at a time), kept parity-tested for reference
+  const char* sp = getenv("PREDTOP_ATTN_SPARSE");
+  const char* ap0 = getenv("PREDTOP_ATTN_MODE");
+  const int split = dag->desc.hops > 0 && sp && sp[0] == '1' && sparse_bytes <= 96 * 1024 &&
+                    !(ap0 && ap0[0] == 'p');  // the persistent variant has no split
+  if (split) {
+    static int attr_sp = 0;
+    if (sparse_bytes > 48 * 1024 && sparse_bytes > attr_sp) {
+      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn_sparse<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024));
+      attr_sp = 96 * 1024;
+    }
+    k_attn_sparse<DH><<<blocks, 128, sparse_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    PT_LAUNCH_CHECK();
+  }
   const int per_sm = DH == 16 ? PREDTOP_ATTN_P_CTAS : 2;
   const int pers_bytes = 2 * resident_bytes;  // two item buffers (+ alignment slack)
   const char* ap = getenv("PREDTOP_ATTN_MODE");  // "p": persistent, "8": 8-warp CTAs, default 4-warp
@@ -679,7 +830,7 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
                                        28 * 1024));
       attr_h = true;
     }
-    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, split);
   } else if (resident_bytes + 128 * wmax * 8 <= 100 * 1024) {
     static bool attr_done = false;
     if (!attr_done) {
@@ -687,7 +838,7 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
                                        100 * 1024));
       attr_done = true;
     }
-    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out, split);
   } else {
     constexpr int stream_bytes = 2 * kStages * stage_chunks<DH>() * CH_BYTES + 1024;
     static bool attr_s = false;
@@ -696,7 +847,7 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
                                        stream_bytes));
       attr_s = true;
     }
-    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, split);
   }
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;
