@@ -391,6 +391,45 @@ def roofline(prof, work, cfg, pairs, node_total, clk, step_ms):
     return roof
 
 
+def kernel_rooflines(prof, cfg, node_total, edge_total, words, pairs, clk):
+    """Every kernel's algorithmic work / its measured time against its own
+    bound, plus the layer stack (projections + attention + FFN)
+    as one tensor-roofline fraction.  Per step; per-layer kinds x num_layers."""
+    peaks, _ = load_peaks()
+    tpk = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    hbm = peaks["hbm_gbs"]
+    d, dff, H, Lm = cfg["d_model"], cfg["d_ff"], cfg["num_heads"], cfg["num_layers"]
+    N, E, A = float(node_total), float(edge_total), float(pairs)
+    clk_mhz = clk.summary()["sm_mhz"] or peaks.get("sm_max_mhz", 1965.0)
+    mufu = MUFU_EX2_PER_CLK_SM * NUM_SMS * clk_mhz * 1e6
+    out = {}
+
+    def sec(k):
+        return prof[k]["ms_per_step"] / 1e3 if k in prof else None
+
+    def put(k, bound, work, peak, unit):
+        t = sec(k)
+        if t:
+            ach = work / t
+            out[k] = {"bound": bound, "achieved": ach / (1e12 if unit == "TFLOP/s" else 1e9),
+                      "peak": peak, "unit": unit, "frac": ach / (peak * (1e12 if unit == "TFLOP/s" else 1e9))}
+
+    put("gemm_qkv", "hbm", Lm * N * (2 * d + 6 * d), hbm, "GB/s")
+    put("attention", "alu", Lm * H * A, mufu / 1e9, "Gexp/s")
+    put("layer_tail", "tensor", Lm * 2 * N * (d * d + 2 * d * dff), tpk, "TFLOP/s")
+    put("embed", "hbm", N * (20.0 + 4 + 6 * d), hbm, "GB/s")
+    put("readout", "hbm", 4.0 * N * d, hbm, "GB/s")
+    put("dag_small", "hbm", 8.0 * E + 4.0 * N + 2 * 8.0 * words, hbm, "GB/s")
+    t_layers = sum(sec(k) or 0.0 for k in ("gemm_qkv", "attention", "layer_tail", "gemm_oproj_ln", "gemm_ffn1",
+                                             "gemm_ffn2_ln"))
+    if t_layers:
+        fl = Lm * (2 * N * (3 * d * d + d * d + 2 * d * dff) + 4.0 * d * A)
+        out["layer_stack"] = {"bound": "tensor", "achieved": fl / t_layers / 1e12, "peak": tpk, "unit": "TFLOP/s",
+                              "frac": fl / t_layers / 1e12 / tpk,
+                              "note": "QKV + attention (4 d |A|) + O-proj + FFN flops over the time of those kernels"}
+    return out
+
+
 def dag_pairs(pt, dag, sizes):
     T_ = (np.asarray(sizes) + 127) // 128
     _, pairs = dag.tiles(int((T_ * T_).sum()))
@@ -578,6 +617,7 @@ def run_batch(args, ctx):
     A = dag_pairs(pt, dag, host.sizes)
     work = algorithmic_work(cfg, host.node_ptr[-1], host.edge_ptr[-1], words, A)
     roof = roofline(prof, work, cfg, A, host.node_ptr[-1], clk, total_ms / args.steps)
+    kroof = kernel_rooflines(prof, cfg, host.node_ptr[-1], host.edge_ptr[-1], words, A, clk)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config != "16k":
@@ -596,7 +636,7 @@ def run_batch(args, ctx):
                 "gpu_launches": int(launches),
                 "launch_mode": "eager" if args.eager else "cuda_graph",
                 "eager_ms_per_step": eager_ms, "host_enqueue_ms_per_step": host_enqueue_ms,
-                "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "roofline": roof, "kernel_rooflines": kroof, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
         emit(line, args)
 
