@@ -56,15 +56,6 @@ __device__ long long g_tail_trace3[8];
     if (lane == 0 && blockIdx.x == 0 && (i) == 4 && (j) == 1) g_tail_trace2[k][warp - 2] = clock64(); \
   } while (0)
 #else
-// MMA warp, tiles 2..9 of CTA 0: total clocks spent waiting on [0] ring_full,
-// [1] p_ready, [2] h_ready, [3] a_full, [4] o_empty / out_empty; [5] tile span
-__device__ long long g_tail_trace3[8];
-#define TWAIT(k, stmt)                                                   \
-  do {                                                                   \
-    const long long t0_ = clock64();                                     \
-    stmt;                                                                \
-    if (blockIdx.x == 0 && tile_i >= 2 && tile_i < 10) g_tail_trace3[k] += clock64() - t0_; \
-  } while (0)
 #define TTRACEW(i, j, k) \
   do {                   \
   } while (0)

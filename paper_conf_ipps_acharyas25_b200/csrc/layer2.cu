@@ -306,6 +306,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
     const bool leader = (ew == 0 && lane == 0);
     // this warp's 4 KB piece of the h tile: rows 32q.. of K-slice g (SW128)
     unsigned char* stg = sH + g * SLOT + q * 4096;
+#if PREDTOP_TAIL2_TMA_IO == 1
     uint64_t* xb = &xbar[ew];
     uint32_t xphase = 0;
     auto x_load = [&](int m0, int k) {  // [32 rows x 32 fp32] box of the residual
@@ -314,6 +315,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
         sm100::tma_load_2d(stg, &mp.x32, xb, 64 * g + 32 * k, m0 + 32 * q);
       }
     };
+#endif
     auto stage_f32 = [&](const float* v) {  // 32 fp32 of row `lane` -> staging (SW128)
 #pragma unroll
       for (int c = 0; c < 8; ++c)
