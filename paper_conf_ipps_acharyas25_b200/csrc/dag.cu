@@ -700,18 +700,50 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
       __syncwarp();
     }
   } else {
-  // closure R[v] = OR_{w in succ(v)} (R[w] | {w}), deepest level first
+  // closure R[v] = OR_{w in succ(v)} (R[w] | {w}), deepest level first.
+  // Per topo position a packed record replaces the topo -> soff -> succ load
+  // chain of the latency-bound level loop: lo = v | deg << 9 | s0 << 12 |
+  // s1 << 21 (in topo[]), hi = s2 | s3 << 9 | s4 << 18 (in indeg[], dead
+  // after Kahn); node ids < 512 fit 9 bits; deg > 5 is marked 7 and read
+  // from the CSR.
+  for (int i = lane; i < N; i += 32) {
+    const int v = topo[i], b = soff[v], deg = soff[v + 1] - b;
+    int sv[5] = {0, 0, 0, 0, 0};
+#pragma unroll
+    for (int k = 0; k < 5; ++k)
+      if (k < deg) sv[k] = succ[b + k];
+    topo[i] = v | (min(deg, 6) == 6 ? 7 << 9 : deg << 9) | (sv[0] << 12) | (sv[1] << 21);
+    indeg[i] = sv[2] | (sv[3] << 9) | (sv[4] << 18);
+  }
   for (int i = lane; i < N * W; i += 32) R[i] = 0;
   __syncwarp();
+  const int ln = lane / W, lw = lane - (lane / W) * W;  // this lane's first item of a level
   for (int l = level - 1; l >= 0; --l) {
-    const int lb = lptr[l], le = lptr[l + 1];
-    for (int it = lane; it < (le - lb) * W; it += 32) {
-      const int v = topo[lb + it / W], j = it % W;
+    const int lb = lptr[l], items = (lptr[l + 1] - lb) * W;
+    for (int it = lane; it < items; it += 32) {
+      int ni = ln, j = lw;
+      if (it != lane) {
+        ni = it / W;
+        j = it - ni * W;
+      }
+      const uint32_t lo = (uint32_t)topo[lb + ni], hi = (uint32_t)indeg[lb + ni];
+      const int v = (int)(lo & 511u), degc = (int)((lo >> 9) & 7u);
       uint64_t acc = 0;
-      for (int k = soff[v]; k < soff[v + 1]; ++k) {
-        const int w = succ[k];
-        acc |= R[w * W + j];
-        if ((w >> 6) == j) acc |= 1ull << (w & 63);
+      if (degc <= 5) {
+        const int sv[5] = {(int)((lo >> 12) & 511u), (int)((lo >> 21) & 511u), (int)(hi & 511u),
+                           (int)((hi >> 9) & 511u), (int)((hi >> 18) & 511u)};
+#pragma unroll
+        for (int k = 0; k < 5; ++k)
+          if (k < degc) {
+            const int w = sv[k];
+            acc |= R[w * W + j] | ((w >> 6) == j ? 1ull << (w & 63) : 0ull);
+          }
+      } else {
+        for (int k = soff[v]; k < soff[v + 1]; ++k) {
+          const int w = succ[k];
+          acc |= R[w * W + j];
+          if ((w >> 6) == j) acc |= 1ull << (w & 63);
+        }
       }
       R[v * W + j] = acc;
     }
