@@ -306,16 +306,16 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
           for (int k = 0; k < 4; ++k)
             if ((uint32_t)k < deg) {
               const uint32_t w = s4[k];
-              acc |= Rsm[w] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
+              acc |= Rsm[(size_t)w * rs2] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
             }
           if (deg > 4) {
             const uint32_t dg = deg == 0xFFFFu ? (uint32_t)(soff[v + 1] - r.w) : deg;
             for (uint32_t k = 4; k < dg; ++k) {
               const uint32_t w = (uint32_t)succ[r.w + k];
-              acc |= Rsm[w] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
+              acc |= Rsm[(size_t)w * rs2] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
             }
           }
-          Rsm[v] = acc;
+          Rsm[(size_t)v * rs2] = acc;  // rs2 = CW > 1 when only the last slice is one word wide
         }
         r0 = first_rec(level - 4);
         __syncwarp();

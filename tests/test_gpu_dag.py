@@ -125,3 +125,19 @@ def test_rebuild_deterministic(pt):
     assert dag.rebuild() == pt.OK
     assert torch.equal(R1, dag.reachability().cpu())
     assert torch.equal(d1, dag.depth)
+
+
+@pytest.mark.parametrize("n", [6780, 9000])
+def test_large_graph_column_slicing(pt, oracle_mod, n):
+    """Graphs between the fused path and the 16k stress case on the deep-graph
+    record path: n = 6780 gives W = 106 words in three-word shared-memory
+    slices, the last slice one word wide (its row stride is still 3) and
+    holding real columns 6720..6779."""
+    rng = synth.CounterRng(n, 17)
+    s, d = synth.random_dag(n, 1.6 / n, rng)
+    b = synth.pack_graphs([(n, s, d, synth._rand_feats(n, rng))])
+    dag = pt.Dag(pt.DeviceBatch.from_host(b))
+    assert dag.status == pt.OK
+    R = dag.reachability().cpu().numpy().view(np.uint64)
+    np.testing.assert_array_equal(R, oracle_mod.reach(n, s, d).ravel())
+    np.testing.assert_array_equal(dag.depth.cpu().numpy(), oracle_mod.depth(n, s, d))
