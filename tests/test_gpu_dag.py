@@ -141,3 +141,30 @@ def test_large_graph_column_slicing(pt, oracle_mod, n):
     R = dag.reachability().cpu().numpy().view(np.uint64)
     np.testing.assert_array_equal(R, oracle_mod.reach(n, s, d).ravel())
     np.testing.assert_array_equal(dag.depth.cpu().numpy(), oracle_mod.depth(n, s, d))
+
+
+@pytest.mark.parametrize("n, kind", [(520, "random"), (3000, "random"), (4100, "chain"), (7000, "chain"),
+                                     (12000, "random")])
+def test_large_path_modes(pt, oracle_mod, n, kind):
+    """Multi-kernel build path across the column-slice modes (CSR staged in
+    shared memory or not, 1-4 word columns per CTA, deep chains with one
+    node per level): depth, R and the mask tiles bit-exact."""
+    rng = synth.CounterRng(n, 23)
+    if kind == "chain":
+        s, d = synth.chain(n)
+        perm = rng.permutation(n)
+        s, d = perm[s].astype(np.int32), perm[d].astype(np.int32)
+    else:
+        s, d = synth.random_dag(n, 2.0 / n, rng)
+    b = synth.pack_graphs([(n, s, d, synth._rand_feats(n, rng))])
+    dag = pt.Dag(pt.DeviceBatch.from_host(b))
+    assert dag.status == pt.OK
+    R = dag.reachability().cpu().numpy().view(np.uint64)
+    Ro = oracle_mod.reach(n, s, d)
+    np.testing.assert_array_equal(R, Ro.ravel())
+    np.testing.assert_array_equal(dag.depth.cpu().numpy(), oracle_mod.depth(n, s, d))
+    T = (n + 127) // 128
+    cls, pairs = dag.tiles(T * T)
+    co, po = oracle_mod.tiles(n, oracle_mod.mask(n, Ro))
+    np.testing.assert_array_equal(cls.cpu().numpy(), co)
+    assert int(pairs.cpu()[0]) == po
