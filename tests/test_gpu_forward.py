@@ -210,3 +210,23 @@ def test_full_moe_config_sampled(pt, oracle_mod):
     err = _rel(y[sample], want)
     print(f"moe full: max rel err {err.max():.3e}")
     assert err.max() <= TOL
+
+
+@pytest.mark.parametrize("name", ["gpt", "paper"])
+def test_mixed_odd_sizes(pt, oracle_mod, name):
+    """One batch mixing 1-node, tile-boundary (127/128/129) and multi-kernel-
+    path (513, 700) graphs: every graph within 2e-3 of the oracle."""
+    cfg, blob, model = _model(pt, name)
+    rng = synth.CounterRng(31, 7)
+    gs = []
+    for n, p in [(1, 0.0), (2, 1.0), (17, 0.2), (127, 0.03), (128, 0.03), (129, 0.03), (513, 0.006),
+                 (700, 0.004)]:
+        s, d = synth.random_dag(n, p, rng)
+        gs.append((n, s, d, synth._rand_feats(n, rng)))
+    batch = synth.pack_graphs(gs)
+    y, _ = _gpu_latency(pt, model, batch)
+    want = oracle_mod.forward_batch(cfg, blob, batch)
+    err = _rel(y, want)
+    print(f"{name} mixed sizes: max rel err {err.max():.3e}")
+    assert np.isfinite(y).all()
+    assert err.max() <= TOL
