@@ -290,8 +290,14 @@ class Ctx:
         torch.cuda.synchronize()
         g = torch.cuda.CUDAGraph()
         l0 = self.L.predtop_launch_count()
-        with torch.cuda.graph(g, stream=side):
-            fn()
+        try:
+            with torch.cuda.graph(g, stream=side):
+                fn()
+        except RuntimeError as e:  # e.g. a collective backend that cannot be captured: run eagerly
+            print(f"bench: CUDA-graph capture failed ({e}); timing eager steps", file=sys.stderr)
+            torch.cuda.synchronize()
+            self.capture_failed = True
+            return fn, None
         n = self.L.predtop_launch_count() - l0
         torch.cuda.synchronize()
         self._graphs = getattr(self, "_graphs", []) + [g]
@@ -634,7 +640,7 @@ def run_batch(args, ctx):
                 "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                         "d2h_bytes_per_step": int(d2h), "mode": e2e_mode, "serial_value": e2e_serial},
                 "gpu_launches": int(launches),
-                "launch_mode": "eager" if args.eager else "cuda_graph",
+                "launch_mode": "eager" if args.eager or getattr(ctx, "capture_failed", False) else "cuda_graph",
                 "eager_ms_per_step": eager_ms, "host_enqueue_ms_per_step": host_enqueue_ms,
                 "roofline": roof, "kernel_rooflines": kroof, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
@@ -742,7 +748,7 @@ def run_search(args, ctx):
                 "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                         "d2h_bytes_per_step": int(d2h)},
                 "gpu_launches": int((launches_per_step or 0) * args.steps),
-                "launch_mode": "eager" if args.eager else "cuda_graph",
+                "launch_mode": "eager" if args.eager or getattr(ctx, "capture_failed", False) else "cuda_graph",
                 "roofline": None, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
         emit(line, args)
