@@ -831,14 +831,32 @@ def run_sweep(args, ctx, pool):
         sum(h.numel() * h.element_size() for _, h in plan_pin)
     d2h = (world * Pmax if world > 1 else sh.num_plans) * 8 + 8
 
+    # the H2D copy of chunk c+1 runs on a copy stream while chunk c is scored
+    # (every chunk has its own device buffers); the copies stay inside the step
+    cs = torch.cuda.Stream(device=dev)
+    evs = [torch.cuda.Event() for _ in sh.chunks]
+
     def e2e_step():
-        for dev_t, host_t in plan_pin:
-            dev_t.copy_(host_t, non_blocking=True)
-        for lo, hi, key in sh.chunks:
-            for dev_t, host_t in pins[key]:
+        cur = torch.cuda.current_stream()
+        cs.wait_stream(cur)
+
+        def copy_chunk(c):
+            with torch.cuda.stream(cs):
+                for dev_t, host_t in pins[sh.chunks[c][2]]:
+                    dev_t.copy_(host_t, non_blocking=True)
+                evs[c].record(cs)
+
+        with torch.cuda.stream(cs):
+            for dev_t, host_t in plan_pin:
                 dev_t.copy_(host_t, non_blocking=True)
+        copy_chunk(0)
+        for c, (lo, hi, key) in enumerate(sh.chunks):
+            if c + 1 < len(sh.chunks):
+                copy_chunk(c + 1)
+            cur.wait_event(evs[c])
             sh.dags[key].rebuild()
             sh.model.forward(sh.dags[key], sh.ws, sh.lat[lo:hi])
+        cur.wait_stream(cs)
         T, _, _ = sh.plans.latency(sh.lat, no_sync=True)
         if world > 1:
             T_pad[:sh.num_plans].copy_(T)
