@@ -1,13 +1,16 @@
 #!/usr/bin/env python
-"""bench.py -- PredTOP prediction path on B200 (BASELINE.json configs[1]).
+"""bench.py -- PredTOP prediction path on B200.
 
 One step = the whole hot path over one batch: predtop_build_dag (validate,
 depth, closure, mask) + predtop_stage_forward (DAG-Transformer, 4 layers) +
 predtop_plan_latency (Eqn 4) + [N>1: NCCL all-gather of plan latencies] +
-predtop_plan_argmin.  Workload per GPU: 1024 GPT-style stage DAGs of 270-330
-ops (seeded, synthetic), d=128, 8 heads, d_ff=512; 256 plans of 4 stages x 16
-microbatches (owned mode).  Weak scaling: rank r scores graphs
-[1024 r, 1024 (r+1)).
+predtop_plan_argmin.  Default workload per GPU (the largest single-GPU config,
+BASELINE.json configs[2]): 512 MoE-style stage DAGs of 1350-1650 ops (seeded,
+synthetic), d=256, 8 heads, d_ff=1024; 128 plans of 4 stages x 16 microbatches
+(owned mode); configs[1] (1024 GPT-style DAGs, d=128) is measured in the same
+run and reported under "also".  Weak scaling: rank r scores graphs
+[G r, G (r+1)).  `--gpus N` without a torchrun environment re-launches itself
+under torch.distributed.run with N ranks.
 
 Timing: W warm-up steps, then K steps, each preceded by an untimed L2 flush
 (256 MiB memset > 126 MB L2) and bracketed by CUDA events on the compute
@@ -114,7 +117,8 @@ def host_cores() -> int:
 
 
 def oracle_rate(cfg, blob, batch, target_s: float = 15.0, max_graphs: int = 1024, hops: int = 0):
-    """Oracle graphs/s on a bounded sample with all host cores."""
+    """Oracle graphs/s on a bounded sample (the first n graphs) with all host
+    cores; also returns the oracle latencies of the sample (parity)."""
     import oracle
     oracle.build()
     cores = host_cores()
@@ -124,14 +128,28 @@ def oracle_rate(cfg, blob, batch, target_s: float = 15.0, max_graphs: int = 1024
     n = int(max(cores, min(max_graphs, batch.num_graphs, round(target_s * cores / max(t1, 1e-6)))))
     n = min(n, batch.num_graphs)
     t0 = time.perf_counter()
-    oracle.forward_batch(cfg, blob, batch, graphs=list(range(n)), threads=cores, hops=hops)
+    y = oracle.forward_batch(cfg, blob, batch, graphs=list(range(n)), threads=cores, hops=hops)
     wall = time.perf_counter() - t0
-    return n / wall, cores, n, wall
+    return n / wall, cores, n, wall, y
+
+
+def parity_stats(y_gpu, y_oracle, bias):
+    """GPU-vs-oracle relative error per graph (north star: <= 2e-3), also of
+    the bias-free part y - c_o (R17)."""
+    y = np.asarray(y_gpu, np.float64)
+    w = np.asarray(y_oracle, np.float64)
+    r = np.abs(y - w) / np.abs(w)
+    rb = np.abs(y - w) / np.abs(w - bias)
+    return {"max_rel": float(r.max()), "median_rel": float(np.median(r)), "max_rel_nobias": float(rb.max()),
+            "median_rel_nobias": float(np.median(rb)), "graphs": int(len(y)), "tolerance": 2e-3,
+            "pass": bool(r.max() <= 2e-3 and rb.max() <= 2e-3)}
 
 
 def run_reference(args, rank):
     if rank != 0:
         return
+    if args.config == "16k":
+        return run_reference_16k(args)
     from paper_conf_ipps_acharyas25_b200 import synth
     import oracle
     oracle.build()
@@ -140,19 +158,24 @@ def run_reference(args, rank):
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
     cores = host_cores()
     per_step = cores  # one graph per core per step
-    batch = synth.tiny_batch() if gcfg == "tiny" else synth.stage_batch(gcfg, per_step * (args.warmup + args.steps) if args.steps * per_step <= 4096 else 4096)
-    plans_B = 16
+    nb = min(per_step * (min(args.warmup, 1) + args.steps), 4096 if gcfg == "gpt" else 512)
+    batch = synth.tiny_batch() if gcfg == "tiny" else synth.stage_batch(gcfg, nb)
+    plans_B = plan_microbatches(args.config)
     done, t_total = 0, 0.0
-    for s in range(args.warmup + args.steps):
+    # a CPU program has nothing to warm beyond its first step: one untimed
+    # warm-up step whatever W is (an MoE step is ~5-10 s of oracle work)
+    nwarm = min(args.warmup, 1)
+    for s in range(nwarm + args.steps):
         gs = [(s * per_step + i) % batch.num_graphs for i in range(per_step)]
         t0 = time.perf_counter()
         y = oracle.forward_batch(cfg, blob, batch, graphs=gs, threads=cores)
         # plan formula over the sampled stages (owned mode, 4 stages x B = 16)
-        P = len(gs) // 4
+        S = stages_per_plan(args.config, len(gs))
+        P = len(gs) // S
         if P:
-            oracle.plan_T(np.arange(P + 1) * 4, np.arange(4 * P), np.full(P, plans_B), y[:4 * P].astype(np.float32))
+            oracle.plan_T(np.arange(P + 1) * S, np.arange(S * P), np.full(P, plans_B), y[:S * P].astype(np.float32))
         dt = time.perf_counter() - t0
-        if s >= args.warmup:
+        if s >= nwarm:
             done += len(gs)
             t_total += dt
     value = done / t_total
@@ -175,8 +198,39 @@ CONFIG_TEXT = {
 }
 
 
-def stages_per_plan(G: int) -> int:
-    return max(1, min(4, G))
+def stages_per_plan(config: str, G: int) -> int:
+    """tiny: 1-stage plans (BASELINE configs[0]); else 4-stage plans."""
+    return 1 if config == "tiny" else max(1, min(4, G))
+
+
+def plan_microbatches(config: str) -> int:
+    return 4 if config == "tiny" else 16
+
+
+def run_reference_16k(args):
+    """--impl reference for configs[3]: the oracle on the 16 384-op DAG, its
+    layers evaluated row block by row block on all host cores
+    (oracle.forward_rows); one step = one whole forward (~30-60 s), so the
+    run times min(steps, 1) step after no warm-up."""
+    from paper_conf_ipps_acharyas25_b200 import synth
+    import oracle
+    oracle.build()
+    cfg = synth.MODEL_CONFIGS["16k"]
+    blob = synth.pack_weights(cfg, synth.model_weights(cfg))
+    cores = host_cores()
+    b = synth.stage_batch("16k", 1)
+    tm = {}
+    oracle.forward_rows(cfg, blob, *b.graph(0), threads=cores, timings=tm)
+    value = 1.0 / tm["total_s"]
+    sample = (f"1 whole 16k stage graph (depth, closure, mask single-threaded {tm['graph_steps_s']:.1f} s; "
+              f"4 layers row-parallel on {cores} threads {sum(tm['layers_s']):.1f} s), fp64 oracle")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": 1, "warmup": 0, "ms_per_step": 1000 * tm["total_s"], "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": workload_config(args),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
 
 
 def workload_config(args):
@@ -193,10 +247,10 @@ def workload_config(args):
                      "parallelism": f"plan-sharded x{args.gpus} (cost-balanced contiguous ranges), "
                                     f"NCCL all-gather of plan latencies",
                      "l2": "inputs and activations of one step (~500k graphs) far exceed the 126 MB L2"}, **base)
-    G, S = args.graphs, stages_per_plan(args.graphs)
+    G, S, B = args.graphs, stages_per_plan(args.config, args.graphs), plan_microbatches(args.config)
     return dict({"workload": f"{args.config}: {G} {CONFIG_TEXT[args.config]}, sum pool + MLP head; "
-                             f"{G // S} plans x {S} stages x B=16 (Eqn 4)",
-                 "graphs_per_gpu": G, "plans_per_gpu": G // S, "stages_per_plan": S, "microbatches": 16,
+                             f"{G // S} plans x {S} stages x B={B} (Eqn 4)",
+                 "graphs_per_gpu": G, "plans_per_gpu": G // S, "stages_per_plan": S, "microbatches": B,
                  "parallelism": f"graph-sharded x{args.gpus} (owned plans), NCCL all-gather of plan latencies",
                  "l2": "flushed before every timed step (256 MiB memset, untimed)",
                  "dagra_k": args.hops if args.hops > 0 else "inf"}, **base)
@@ -204,6 +258,8 @@ def workload_config(args):
 
 # ----------------------------------------------------------------- main leg
 DEFAULT_GRAPHS = {"tiny": 4, "gpt": 1024, "moe": 512, "16k": 1, "sweep": 0, "search": 0}
+ALSO_KEYS = ("metric", "value", "unit", "ms_per_step", "steps", "config", "e2e", "gpu_launches", "roofline",
+             "cpu_baseline", "parity", "result", "clocks")
 
 
 class Ctx:
@@ -453,8 +509,8 @@ def run_batch(args, ctx):
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
     G = args.graphs
     host = synth.tiny_batch() if args.config == "tiny" else synth.stage_batch(args.config, G, first_graph=rank * G)
-    S = stages_per_plan(G)
-    ps = synth.owned_plans(G, S, 16)
+    S = stages_per_plan(args.config, G)
+    ps = synth.owned_plans(G, S, plan_microbatches(args.config))
     model = pt.Model(cfg, blob, device=dev)
     db = pt.DeviceBatch.from_host(host, device=dev)
     dag = pt.Dag(db, no_sync=True, hops=args.hops)
@@ -508,6 +564,21 @@ def run_batch(args, ctx):
     value = world * G * args.steps / (total_ms / 1e3)
     plans_per_s = world * P * args.steps / (total_ms / 1e3)
     assert torch.isfinite(lat).all()
+    # the plan latencies of ALL ranks (gathered) and the global best plan: a
+    # 1-rank run over world*G graphs gives bitwise the same (tests/test_bench_ranks.py)
+    import hashlib
+    T_fin = (T_all if world > 1 else plans.T[:P]).cpu().numpy()
+    result = {"T_sha256": hashlib.sha256(T_fin.tobytes()).hexdigest(), "plans": int(T_fin.size),
+              "best_plan": int(plans.best.item()) if P else None}
+    if args.no_extras:
+        if rank == 0:
+            emit({"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                  "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+                  "scaling": "weak", "vs_baseline": None, "dtype": "f16", "data": "synthetic",
+                  "config": workload_config(args), "plans_per_s": plans_per_s, "result": result,
+                  "launch_mode": "eager" if args.eager or getattr(ctx, "capture_failed", False) else "cuda_graph",
+                  "clocks": clk.summary(), "note": "--no-extras: e2e, profile, cpu_baseline skipped"}, args)
+        return
 
     # ---- e2e through the C-ABI with pinned host buffers
     pin = {
@@ -625,11 +696,26 @@ def run_batch(args, ctx):
     roof = roofline(prof, work, cfg, A, host.node_ptr[-1], clk, total_ms / args.steps)
     kroof = kernel_rooflines(prof, cfg, host.node_ptr[-1], host.edge_ptr[-1], words, A, clk)
 
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config != "16k":
-        v, cores, n, wall = oracle_rate(cfg, blob, host, hops=getattr(args, "hops", 0))
+    cpu, parity = None, None
+    c_o = float(synth.model_weights(cfg)["c_o"][0])
+    y_gpu = lat.cpu().numpy().astype(np.float64)
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config == "16k":
+        import oracle
+        oracle.build()
+        cores = host_cores()
+        tm = {}
+        _, y16, _ = oracle.forward_rows(cfg, blob, *host.graph(0), threads=cores, timings=tm)
+        cpu = {"value": 1.0 / tm["total_s"], "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"the whole 16k stage graph: depth, closure, mask {tm['graph_steps_s']:.1f} s "
+                         f"(single-threaded) + 4 layers {sum(tm['layers_s']):.1f} s (row blocks on {cores} threads), "
+                         f"fp64 C oracle"}
+        parity = parity_stats(y_gpu[:1], [y16], c_o)
+    elif rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, cores, n, wall, y_or = oracle_rate(cfg, blob, host, hops=getattr(args, "hops", 0))
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": f"first {n} of {G} {args.config} stage graphs, fp64 C oracle, {cores} threads, {wall:.1f} s"}
+        parity = parity_stats(y_gpu[:n], y_or, c_o)
+        parity["sample"] = f"the {n} cpu_baseline graphs"
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -642,9 +728,11 @@ def run_batch(args, ctx):
                 "gpu_launches": int(launches),
                 "launch_mode": "eager" if args.eager or getattr(ctx, "capture_failed", False) else "cuda_graph",
                 "eager_ms_per_step": eager_ms, "host_enqueue_ms_per_step": host_enqueue_ms,
-                "roofline": roof, "kernel_rooflines": kroof, "cpu_baseline": cpu, "clocks": clk.summary(),
+                "roofline": roof, "kernel_rooflines": kroof, "cpu_baseline": cpu, "parity": parity,
+                "result": result, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
-        emit(line, args)
+        return line
+    return None
 
 
 def run_search(args, ctx):
@@ -831,18 +919,26 @@ def run_sweep(args, ctx, pool):
         sum(h.numel() * h.element_size() for _, h in plan_pin)
     d2h = (world * Pmax if world > 1 else sh.num_plans) * 8 + 8
 
-    # the H2D copy of chunk c+1 runs on a copy stream while chunk c is scored
-    # (every chunk has its own device buffers); the copies stay inside the step
+    # the H2D copy of chunk c+1 runs on a copy stream while chunk c is scored;
+    # chunks share device buffer sets (SweepShard keys them by pool offset and
+    # size), so a copy into set `key` first waits for the forward of the last
+    # chunk that read that set (write-after-read); when chunk c+1 reuses chunk
+    # c's own set, its copy is issued only after chunk c's forward
     cs = torch.cuda.Stream(device=dev)
     evs = [torch.cuda.Event() for _ in sh.chunks]
+    done = [torch.cuda.Event() for _ in sh.chunks]
 
     def e2e_step():
         cur = torch.cuda.current_stream()
         cs.wait_stream(cur)
+        last_user = {}
 
         def copy_chunk(c):
+            key = sh.chunks[c][2]
             with torch.cuda.stream(cs):
-                for dev_t, host_t in pins[sh.chunks[c][2]]:
+                if key in last_user:
+                    cs.wait_event(done[last_user[key]])
+                for dev_t, host_t in pins[key]:
                     dev_t.copy_(host_t, non_blocking=True)
                 evs[c].record(cs)
 
@@ -850,12 +946,18 @@ def run_sweep(args, ctx, pool):
             for dev_t, host_t in plan_pin:
                 dev_t.copy_(host_t, non_blocking=True)
         copy_chunk(0)
+        n = len(sh.chunks)
         for c, (lo, hi, key) in enumerate(sh.chunks):
-            if c + 1 < len(sh.chunks):
+            early = c + 1 < n and sh.chunks[c + 1][2] != key
+            if early:
                 copy_chunk(c + 1)
             cur.wait_event(evs[c])
             sh.dags[key].rebuild()
             sh.model.forward(sh.dags[key], sh.ws, sh.lat[lo:hi])
+            done[c].record(cur)
+            last_user[key] = c
+            if c + 1 < n and not early:
+                copy_chunk(c + 1)
         cur.wait_stream(cs)
         T, _, _ = sh.plans.latency(sh.lat, no_sync=True)
         if world > 1:
@@ -899,7 +1001,8 @@ def run_sweep(args, ctx, pool):
                 "plans_per_s": plans_per_s, "graphs_per_step": graphs_total, "best_plan": b,
                 "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                         "d2h_bytes_per_step": int(d2h)},
-                "gpu_launches": int(launches), "launch_mode": "cuda_graph" if capture else "eager",
+                "gpu_launches": int(launches),
+                "launch_mode": "eager" if not capture or getattr(ctx, "capture_failed", False) else "cuda_graph",
                 "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(),
                 "kernels": {k: {kk: round(vv, 5) for kk, vv in v.items()} for k, v in prof.items()}}
         emit(line, args)
@@ -918,7 +1021,11 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="gpt", choices=["tiny", "gpt", "moe", "16k", "sweep", "search"])
+    ap.add_argument("--config", default="moe", choices=["tiny", "gpt", "moe", "16k", "sweep", "search"])
+    ap.add_argument("--no-also", action="store_true",
+                    help="moe: skip the configs[1] (GPT) measurement reported under 'also'")
+    ap.add_argument("--no-extras", action="store_true",
+                    help="time the step only (no e2e, profile, cpu_baseline); the line carries the T hash")
     ap.add_argument("--layers", type=int, default=24, help="search: model layers (GPT-3 1.3B: 24)")
     ap.add_argument("--graphs", type=int, default=None, help="stage graphs per GPU (default per config)")
     ap.add_argument("--plans", type=int, default=100000, help="sweep: total candidate plans")
@@ -937,6 +1044,16 @@ def main():
     if args.graphs is None:
         args.graphs = DEFAULT_GRAPHS[args.config]
 
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: re-launch under torch.distributed.run
+        import socket
+        import subprocess
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+        sys.exit(subprocess.call(cmd))
     rank = int(os.environ.get("RANK", "0"))
     if args.impl == "reference":
         run_reference(args, rank)
@@ -951,7 +1068,17 @@ def main():
     elif args.config == "search":
         run_search(args, ctx)
     else:
-        run_batch(args, ctx)
+        line = run_batch(args, ctx)
+        if args.config == "moe" and not args.no_also and not args.no_extras:
+            import copy
+            a2 = copy.copy(args)
+            a2.config, a2.graphs, a2.steps = "gpt", DEFAULT_GRAPHS["gpt"], max(10, args.steps // 2)
+            a2.profile_json = None
+            l2 = run_batch(a2, ctx)
+            if line is not None and l2 is not None:
+                line["also"] = {"gpt": {k: l2[k] for k in ALSO_KEYS if k in l2}}
+        if line is not None:
+            emit(line, args)
     ctx.finish()
 
 

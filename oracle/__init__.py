@@ -70,6 +70,9 @@ def lib():
             L.orc_embed.argtypes = [P, P, i32, P, P, P]
             L.orc_attention.argtypes = [P, P, i32, i32, P, P, P]
             L.orc_layer.argtypes = [P, P, i32, i32, P, P, P]
+            L.orc_qkv_rows.argtypes = [P, P, i32, i32, i32, P, P]
+            L.orc_attention_rows.argtypes = [P, i32, P, P, i32, i32, P]
+            L.orc_layer_post_rows.argtypes = [P, P, i32, i32, i32, P, P, P]
             L.orc_readout.argtypes = [P, P, i32, P]
             L.orc_readout.restype = dbl
             L.orc_forward.argtypes = [P, P, i32, i32, P, P, P, P, P]
@@ -229,6 +232,80 @@ def forward_batch(model_cfg, blob, batch, graphs: Optional[Sequence[int]] = None
         return np.asarray([one(g) for g in gs], np.float64)
     with ThreadPoolExecutor(threads) as ex:
         return np.asarray(list(ex.map(one, gs)), np.float64)
+
+
+# ---- one large graph, row block by row block --------------------------------
+def _ranges(rows, threads):
+    """Split a sorted row list into <= ~4*threads contiguous runs."""
+    rows = np.asarray(rows, np.int64)
+    runs, a = [], 0
+    for i in range(1, len(rows) + 1):
+        if i == len(rows) or rows[i] != rows[i - 1] + 1:
+            runs.append((int(rows[a]), int(rows[i - 1]) + 1))
+            a = i
+    out = []
+    target = max(1, len(rows) // max(1, 4 * threads))
+    for r0, r1 in runs:
+        for b in range(r0, r1, target):
+            out.append((b, min(r1, b + target)))
+    return out
+
+
+def layer_rows(model_cfg, blob, li, n, M, x, rows=None, threads=None) -> np.ndarray:
+    """orc_layer for one graph evaluated row block by row block on `threads`
+    workers, from the same pieces orc_layer composes (orc_qkv_rows for every
+    row, orc_attention_rows and orc_layer_post_rows for the requested rows).
+    rows: None = all rows (returns [n, d]); else a sorted subset (returns
+    [len(rows), d])."""
+    L = lib()
+    c = cfg(model_cfg)
+    d = model_cfg["d_model"]
+    threads = threads or (os.cpu_count() or 1)
+    b = np.ascontiguousarray(blob, np.float32)
+    x = np.ascontiguousarray(x, np.float64)
+    M = np.ascontiguousarray(M, np.uint64)
+    qkv = np.zeros((n, 3 * d), np.float64)
+    a = np.zeros((n, d), np.float64)
+    out = np.zeros((n, d), np.float64)
+    sel = np.arange(n) if rows is None else np.asarray(sorted(rows), np.int64)
+    with ThreadPoolExecutor(threads) as ex:
+        list(ex.map(lambda r: L.orc_qkv_rows(ctypes.byref(c), _p(b), li, r[0], r[1], _p(x), _p(qkv)),
+                    _ranges(np.arange(n), threads)))
+        blocks = _ranges(sel, threads)
+        list(ex.map(lambda r: L.orc_attention_rows(ctypes.byref(c), n, _p(M), _p(qkv), r[0], r[1], _p(a)), blocks))
+        list(ex.map(lambda r: L.orc_layer_post_rows(ctypes.byref(c), _p(b), li, r[0], r[1], _p(a), _p(x), _p(out)),
+                    blocks))
+    return out if rows is None else out[sel]
+
+
+def forward_rows(model_cfg, blob, n, src, dst, feats, threads=None, taps: bool = False, timings=None):
+    """orc_forward for ONE (large) graph with every layer evaluated row block
+    by row block in parallel (layer_rows); the graph steps (validate, depth,
+    reach, mask), embedding and readout are the single-threaded oracle calls.
+    Returns (status, latency, taps or None); `timings` (dict) gets the wall
+    seconds of the graph steps and of each layer."""
+    import time
+    t0 = time.perf_counter()
+    st = validate(n, src, dst)
+    if st != OK:
+        return st, float("nan"), None
+    dep = depth(n, src, dst)
+    R = reach(n, src, dst)
+    M = mask(n, R)
+    t1 = time.perf_counter()
+    x = embed(model_cfg, blob, n, feats, dep)
+    tp = [x] if taps else None
+    lt = []
+    for li in range(model_cfg["num_layers"]):
+        a = time.perf_counter()
+        x = layer_rows(model_cfg, blob, li, n, M, x, threads=threads)
+        lt.append(time.perf_counter() - a)
+        if taps:
+            tp.append(x)
+    y = readout(model_cfg, blob, n, x)
+    if timings is not None:
+        timings.update({"graph_steps_s": t1 - t0, "layers_s": lt, "total_s": time.perf_counter() - t0})
+    return OK, y, (np.stack(tp) if taps else None)
 
 
 # ---- pipeline formula ------------------------------------------------------

@@ -331,17 +331,23 @@ void orc_embed(const orc_cfg* c, const float* blob, int n, const orc_feat* feats
 /* Softmax is the plain two-pass form over the allowed set (max, exp, sum).  */
 /* Output: concat_h O_h, [n][d].                                             */
 /* ------------------------------------------------------------------------ */
-void orc_attention(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
-                   const double* x, double* concat_out) {
+/* q|k|v rows [r0, r1) of layer `layer`: qkv[u] = W_qkv x[u] + b_qkv.       */
+void orc_qkv_rows(const orc_cfg* c, const float* blob, int layer, int r0, int r1, const double* x,
+                  double* qkv) {
+  int d = c->d;
+  orc_lw w = layer_weights(c, blob, layer);
+  linear(r1 - r0, d, 3 * d, x + (size_t)r0 * d, w.Wqkv, w.bqkv, qkv + (size_t)r0 * 3 * d);
+}
+
+/* Attention output rows u in [r0, r1) from the full q|k|v matrix [n][3d].   */
+void orc_attention_rows(const orc_cfg* c, int n, const uint64_t* M, const double* qkv, int r0, int r1,
+                        double* concat_out) {
   int d = c->d, H = c->H, dh = c->d / c->H;
   int W = orc_row_words(n);
-  orc_lw w = layer_weights(c, blob, layer);
-  double* qkv = (double*)malloc(sizeof(double) * (size_t)n * 3 * d);
-  linear(n, d, 3 * d, x, w.Wqkv, w.bqkv, qkv);
   double* s = (double*)malloc(sizeof(double) * (size_t)n);
   double scale = 1.0 / sqrt((double)dh);
   for (int h = 0; h < H; ++h)
-    for (int u = 0; u < n; ++u) {
+    for (int u = r0; u < r1; ++u) {
       const double* q = qkv + (size_t)u * 3 * d + h * dh;
       double mx = -INFINITY;
       for (int v = 0; v < n; ++v) {
@@ -364,21 +370,32 @@ void orc_attention(const orc_cfg* c, const float* blob, int layer, int n, const 
         for (int j = 0; j < dh; ++j) o[j] += p * vv[j];
       }
     }
-  free(qkv); free(s);
+  free(s);
+}
+
+void orc_attention(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
+                   const double* x, double* concat_out) {
+  double* qkv = (double*)malloc(sizeof(double) * (size_t)n * 3 * c->d);
+  orc_qkv_rows(c, blob, layer, 0, n, x, qkv);
+  orc_attention_rows(c, n, M, qkv, 0, n, concat_out);
+  free(qkv);
 }
 
 /* DAG Transformer layer (Fig. 4; reading R6, post-LN encoder  */
 /* layer of [34] with ReLU FFN):                                             */
 /*   h = LN1(x + W_o a + b_o),  x' = LN2(h + W_2 ReLU(W_1 h + b_1) + b_2).   */
-void orc_layer(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
-               const double* x_in, double* x_out) {
-  int d = c->d, f = c->d_ff;
+/* orc_layer_post_rows: everything after the attention, rows [r0, r1) of the */
+/* full [n][d] arrays a (attention output), x_in and x_out (row-wise ops).   */
+void orc_layer_post_rows(const orc_cfg* c, const float* blob, int layer, int r0, int r1, const double* a_full,
+                         const double* x_in_full, double* x_out_full) {
+  int d = c->d, f = c->d_ff, n = r1 - r0;
   orc_lw w = layer_weights(c, blob, layer);
-  double* a = (double*)malloc(sizeof(double) * (size_t)n * d);
+  const double* a = a_full + (size_t)r0 * d;
+  const double* x_in = x_in_full + (size_t)r0 * d;
+  double* x_out = x_out_full + (size_t)r0 * d;
   double* z = (double*)malloc(sizeof(double) * (size_t)n * d);
   double* h = (double*)malloc(sizeof(double) * (size_t)n * d);
   double* u = (double*)malloc(sizeof(double) * (size_t)n * f);
-  orc_attention(c, blob, layer, n, M, x_in, a);
   linear(n, d, d, a, w.Wo, w.bo, z);
   for (long i = 0; i < (long)n * d; ++i) z[i] += x_in[i];
   layer_norm(n, d, z, w.g1, w.be1, c->ln_eps, h);
@@ -387,7 +404,15 @@ void orc_layer(const orc_cfg* c, const float* blob, int layer, int n, const uint
   linear(n, f, d, u, w.W2, w.b2, z);
   for (long i = 0; i < (long)n * d; ++i) z[i] += h[i];
   layer_norm(n, d, z, w.g2, w.be2, c->ln_eps, x_out);
-  free(a); free(z); free(h); free(u);
+  free(z); free(h); free(u);
+}
+
+void orc_layer(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
+               const double* x_in, double* x_out) {
+  double* a = (double*)malloc(sizeof(double) * (size_t)n * c->d);
+  orc_attention(c, blob, layer, n, M, x_in, a);
+  orc_layer_post_rows(c, blob, layer, 0, n, a, x_in, x_out);
+  free(a);
 }
 
 /* Readout: global add pool, Eqn 2: x_i = sum_n x_n^i (mean if the   */

@@ -70,6 +70,14 @@ void orc_attention(const orc_cfg* c, const float* blob, int layer, int n, const 
                    const double* x, double* concat_out);
 void orc_layer(const orc_cfg* c, const float* blob, int layer, int n, const uint64_t* M,
                const double* x_in, double* x_out);
+/* The same layer split into row-wise pieces (orc_layer is their composition), */
+/* so one large graph can be evaluated row block by row block (16k config).    */
+void orc_qkv_rows(const orc_cfg* c, const float* blob, int layer, int r0, int r1, const double* x,
+                  double* qkv);
+void orc_attention_rows(const orc_cfg* c, int n, const uint64_t* M, const double* qkv, int r0, int r1,
+                        double* concat_out);
+void orc_layer_post_rows(const orc_cfg* c, const float* blob, int layer, int r0, int r1, const double* a,
+                         const double* x_in, double* x_out);
 double orc_readout(const orc_cfg* c, const float* blob, int n, const double* x);
 int orc_forward(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
                 const int32_t* dst, const orc_feat* feats, double* y, double* taps);

@@ -8,7 +8,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <new>
+#include <utility>
 #include <vector>
 
 #include "internal.h"
@@ -25,6 +28,32 @@ void set_error(const char* fmt, ...) {
   va_start(ap, fmt);
   vsnprintf(g_err, sizeof(g_err), fmt, ap);
   va_end(ap);
+}
+
+cudaError_t smem_attr(const void* func, int bytes) {
+  if (bytes <= 48 * 1024) return cudaSuccess;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  static std::mutex mu;
+  static std::map<std::pair<int, const void*>, int> done;
+  std::lock_guard<std::mutex> lock(mu);
+  int& have = done[{dev, func}];
+  if (have >= bytes) return cudaSuccess;
+  e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) have = bytes;
+  return e;
+}
+
+int num_sms() {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  static std::atomic<int> cache[64] = {};
+  if (dev >= 0 && dev < 64 && cache[dev].load()) return cache[dev].load();
+  int n = 0;
+  if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
+  if (dev >= 0 && dev < 64) cache[dev] = n;
+  return n;
 }
 
 static inline cudaStream_t S(void* s) { return reinterpret_cast<cudaStream_t>(s); }
@@ -169,11 +198,14 @@ static bool device_ok() {
   }
   // cached per device: cudaGetDeviceProperties costs milliseconds of host
   // time, and this runs on every build (the eager sweep builds ~100 chunks)
-  static int ok_dev[64] = {0};  // 0 unknown, 1 ok, -1 not sm_100
-  if (dev >= 0 && dev < 64 && ok_dev[dev] == 1) return true;
-  int major = 0;
-  if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess || major < 10) {
-    set_error("libpredtop needs an sm_100 (Blackwell) device");
+  static std::atomic<int> ok_dev[64] = {};  // 0 unknown, 1 ok, -1 not sm_100
+  if (dev >= 0 && dev < 64 && ok_dev[dev].load() == 1) return true;
+  // only sm_100a SASS is built: compute capability exactly 10.0 (sm_103 / sm_12x would fail at launch)
+  int major = 0, minor = 0;
+  if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess || major != 10 ||
+      minor != 0) {
+    set_error("libpredtop is built for sm_100a only and needs a compute capability 10.0 (B200) device");
     cudaGetLastError();
     if (dev >= 0 && dev < 64) ok_dev[dev] = -1;
     return false;
@@ -436,11 +468,6 @@ static bool use_tail_v2(int d, int dff) {
   return !(e && e[0] == '1') && layer_tail2_supported(d, dff);
 }
 
-// PREDTOP_TAIL_V3=1: two tiles per CTA sharing the weight ring (layer3.cu)
-static bool use_tail_v3(int d, int dff) {
-  const char* e = getenv("PREDTOP_TAIL_V3");
-  return e && e[0] == '1' && layer_tail3_supported(d, dff);
-}
 
 static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, size_t ws_bytes,
                                    int last_layer, float* latency_out, float* x_out,
@@ -485,9 +512,8 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     if ((s = attention_launch(dag, d, H, w.qkv, w.att, st)) != PREDTOP_OK) return s;
     if (use_fused_tail(d, f)) {
       ProfScope _p(PK_LAYER_TAIL, st);
-      s = use_tail_v3(d, f)   ? layer_tail3_launch(m, l, w.att, w.x32, w.x16, M, st)
-          : use_tail_v2(d, f) ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
-                              : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
+      s = use_tail_v2(d, f) ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
+                            : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
       if (s != PREDTOP_OK) return s;
       continue;
     }

@@ -83,12 +83,6 @@ __device__ __forceinline__ void mma16816_c(float (&d)[4], const uint32_t (&a)[4]
 }
 
 constexpr int kChunk = 64;
-// graphs whose mask allows at most this fraction of the N^2 pairs go to the
-// gather kernel k_attn_sparse when the DAG was built with a finite k (hops)
-constexpr int kSparseDensityInv = 5;  // density <= 1/5
-__device__ __forceinline__ bool is_sparse(const DagDev& d, int g, int N) {
-  return d.pairs[g] * kSparseDensityInv <= (int64_t)N * N;
-}
 #ifndef PREDTOP_ATTN_MINB32
 #define PREDTOP_ATTN_MINB32 3  // CTAs per SM of the 8-warp d_h = 32 kernels (78 registers)
 #endif
@@ -265,7 +259,7 @@ template <int DH, bool RESIDENT, int NW = 8>
 __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_MINB16
                                            : (DH == 16 ? 4 : PREDTOP_ATTN_MINB32) * (8 / NW))
     k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
-           const __half* __restrict__ qkv, __half* __restrict__ out, int sparse_split) {
+           const __half* __restrict__ qkv, __half* __restrict__ out) {
   using A = Attn<DH>;
   constexpr int kStageChunks = stage_chunks<DH>();
   extern __shared__ __align__(16) unsigned char dsm_attn[];
@@ -276,12 +270,11 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   if (widx >= d.qtile_off[G]) return;
   const int2 wk = d.work[widx];
   const int g = wk.x, qt = wk.y;
-  if (d.status[g] != PREDTOP_OK) return;
+  if ((unsigned)g >= (unsigned)G || d.status[g] != PREDTOP_OK) return;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
   const int rbase = qt * 128 + part * NW * 16;  // first query row of this CTA
   if (rbase >= N) return;
-  if (sparse_split && is_sparse(d, g, N)) return;  // k_attn_sparse takes this graph
   const int W = 2 * ((N + 127) / 128);
   const int nchunks = (N + kChunk - 1) / kChunk;
   const int nbuf = RESIDENT ? nchunks : kStages * kStageChunks;
@@ -443,331 +436,6 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   }
 }
 
-// Persistent variant for graphs whose K/V fit twice in shared memory (the
-// GPT stage graphs): a CTA walks a static list of (graph, head) items,
-// item it = blockIdx.x + it * gridDim.x, with the K/V of items it and it+1 in
-// two TMA buffers.  Warps take the 16-row groups of the CTA's item sequence
-// round-robin ACROSS item boundaries (warp w: groups w, w+8, w+16, ... of the
-// concatenated list), so no warp idles on a partial 128-row tile and the
-// per-item start-up (status, node_ptr, K/V TMA) overlaps the previous item.
-// The last warp to leave an item issues the TMA for the item two ahead into
-// the buffer it frees.  Same per-group arithmetic as k_attn (Attn::chunk).
-#ifndef PREDTOP_ATTN_P_CTAS
-#define PREDTOP_ATTN_P_CTAS 3
-#endif
-template <int DH>
-__global__ void __launch_bounds__(256, DH == 16 ? PREDTOP_ATTN_P_CTAS : 2)
-    k_attn_p(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
-             const __half* __restrict__ qkv, __half* __restrict__ out, int maxch) {
-  using A = Attn<DH>;
-  extern __shared__ __align__(16) unsigned char dsm_attn[];
-  __shared__ __align__(8) uint64_t kv_full[2];
-  __shared__ int done_cnt[2];
-  // per-warp walk state, parked in shared memory while a group is processed
-  // (keeps the chunk loop at the register count of k_attn: no spills)
-  __shared__ int w_state[8][4];  // it, grp, g (or -1 past the end), ng
-  unsigned char* buf0 = sm100::align1024(dsm_attn);
-  const int bufb = 2 * maxch * A::CHUNK_BYTES;  // K chunks, then V chunks, of one item
-  const int total = G * H;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int gq = lane >> 2, tq = lane & 3;
-  const int ld3 = 3 * dmodel;
-
-  auto issue = [&](int it) {  // one thread: K/V of CTA-local item `it` -> buffer it & 1
-    const int id = blockIdx.x + it * gridDim.x;
-    if (id >= total) return;
-    const int g = id / H, h = id % H;
-    uint64_t* bar = &kv_full[it & 1];
-    if (d.status[g] != PREDTOP_OK) {  // no K/V: complete the phase without data
-      sm100::mbar_arrive(bar);
-      return;
-    }
-    const int64_t n0 = d.node_ptr[g];
-    const int N = (int)(d.node_ptr[g + 1] - n0);
-    const int nch = (N + kChunk - 1) / kChunk;
-    unsigned char* sK = buf0 + (it & 1) * bufb;
-    unsigned char* sV = sK + maxch * A::CHUNK_BYTES;
-    sm100::mbar_arrive_expect_tx(bar, (uint32_t)(nch * 2 * A::CHUNK_BYTES));
-    for (int c = 0; c < nch; ++c) {
-      const int row = (int)(n0 + c * kChunk);
-      sm100::tma_load_2d(sK + c * A::CHUNK_BYTES, &tkv, bar, dmodel + h * DH, row);
-      sm100::tma_load_2d(sV + c * A::CHUNK_BYTES, &tkv, bar, 2 * dmodel + h * DH, row);
-    }
-  };
-  if (threadIdx.x == 0) {
-    sm100::mbar_init(&kv_full[0], 1);
-    sm100::mbar_init(&kv_full[1], 1);
-    done_cnt[0] = done_cnt[1] = 0;
-    sm100::fence_mbar_init();
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    issue(0);
-    issue(1);
-  }
-
-  // this warp leaves item `it`; the last of the 8 warps refills its buffer
-  auto warp_done = [&](int it) {
-    __syncwarp();
-    if (lane == 0) {
-      sm100::fence_proxy_async();  // our ldmatrix reads of the buffer before the TMA rewrite
-      if (atomicAdd(&done_cnt[it & 1], 1) == 7) {
-        done_cnt[it & 1] = 0;
-        issue(it + 2);
-      }
-    }
-    __syncwarp();
-  };
-
-  // walk: this warp's next group (grp of CTA-local item it)
-  volatile int* ws = w_state[warp];
-  if (lane == 0) {
-    ws[0] = 0;
-    ws[1] = warp;
-    ws[2] = -2;  // item info not loaded
-  }
-  __syncwarp();
-  A st;
-  for (;;) {
-    int it = ws[0], grp = ws[1];
-    int g = ws[2], ng = ws[3];
-    const auto load_item = [&](int it_) {
-      const int id = blockIdx.x + it_ * gridDim.x;
-      if (id >= total) {
-        g = -1;
-        ng = -1;
-        return;
-      }
-      g = id / H;
-      const int n = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
-      ng = d.status[g] == PREDTOP_OK ? (n + 15) / 16 : 0;
-    };
-    if (g == -2) load_item(it);
-    while (ng >= 0 && grp >= ng) {  // past this item: leave it (after its K/V arrived)
-      sm100::mbar_wait(&kv_full[it & 1], (it >> 1) & 1);
-      warp_done(it);
-      grp -= ng;
-      ++it;
-      load_item(it);
-    }
-    if (ng < 0) break;
-    __syncwarp();
-    if (lane == 0) {
-      ws[0] = it;
-      ws[1] = grp + 8;
-      ws[2] = g;
-      ws[3] = ng;
-    }
-    __syncwarp();
-    const int h = (blockIdx.x + it * gridDim.x) % H;
-    const int64_t n0 = d.node_ptr[g];
-    const int N = (int)(d.node_ptr[g + 1] - n0);
-    // ---- 16-row group `grp` of item (g, h)
-    const int W = 2 * ((N + 127) / 128);
-    const int nchunks = (N + kChunk - 1) / kChunk;
-    const uint64_t* Mg = d.M + d.row_off[g];
-    const __half* Qg = qkv + n0 * ld3 + h * DH;
-    const int ra = grp * 16 + gq, rb = ra + 8;
-    const bool va = ra < N, vb = rb < N;
-    const uint64_t* Ma = Mg + (int64_t)(va ? ra : 0) * W;
-    const uint64_t* Mb = Mg + (int64_t)(vb ? rb : 0) * W;
-    const uint8_t* Fw = d.bflag + d.bflag_off[g] + (int64_t)grp * nchunks;
-    st.init(lane);
-    uint32_t kw[A::KS][4];
-#pragma unroll
-    for (int ks = 0; ks < A::KS; ++ks) {
-      const int k0 = ks * 16 + 2 * tq;
-      const __half* qa_p = Qg + (int64_t)ra * ld3 + k0;
-      const __half* qb_p = Qg + (int64_t)rb * ld3 + k0;
-      st.qa[ks][0] = va ? *reinterpret_cast<const uint32_t*>(qa_p) : 0u;
-      st.qa[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(qb_p) : 0u;
-      st.qa[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + 8) : 0u;
-      st.qa[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + 8) : 0u;
-      kw[ks][0] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel) : 0u;
-      kw[ks][1] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel) : 0u;
-      kw[ks][2] = va ? *reinterpret_cast<const uint32_t*>(qa_p + dmodel + 8) : 0u;
-      kw[ks][3] = vb ? *reinterpret_cast<const uint32_t*>(qb_p + dmodel + 8) : 0u;
-    }
-    const uint16_t* Ma16 = reinterpret_cast<const uint16_t*>(Ma) + tq;
-    const uint16_t* Mb16 = reinterpret_cast<const uint16_t*>(Mb) + tq;
-    auto mask_lo = [&](int c) -> uint32_t { return va ? (uint32_t)Ma16[4 * c] : 0u; };
-    auto mask_hi = [&](int c) -> uint32_t { return vb ? (uint32_t)Mb16[4 * c] : 0u; };
-    uint32_t mlo = mask_lo(0), mhi = mask_hi(0);
-    uint32_t fl = Fw[0];
-    {
-      float sa = 0.f, sb = 0.f;
-#pragma unroll
-      for (int ks = 0; ks < A::KS; ++ks) {
-        sa += dot_h2(st.qa[ks][0], kw[ks][0]) + dot_h2(st.qa[ks][2], kw[ks][2]);
-        sb += dot_h2(st.qa[ks][1], kw[ks][1]) + dot_h2(st.qa[ks][3], kw[ks][3]);
-      }
-      sa += __shfl_xor_sync(0xffffffffu, sa, 1);
-      sa += __shfl_xor_sync(0xffffffffu, sa, 2);
-      sb += __shfl_xor_sync(0xffffffffu, sb, 1);
-      sb += __shfl_xor_sync(0xffffffffu, sb, 2);
-      st.m_a = sa;
-      st.m_b = sb;
-    }
-    sm100::mbar_wait(&kv_full[it & 1], (it >> 1) & 1);
-    const uint32_t kb0 = sm100::smem_u32(buf0 + (it & 1) * bufb);
-    const uint32_t vb0 = kb0 + (uint32_t)(maxch * A::CHUNK_BYTES);
-    for (int c = 0; c < nchunks; ++c) {
-      const bool more = c + 1 < nchunks;
-      const uint32_t nlo = more ? mask_lo(c + 1) : 0u, nhi = more ? mask_hi(c + 1) : 0u;
-      const uint32_t nfl = more ? Fw[c + 1] : 0u;
-      const uint32_t off = (uint32_t)(c * A::CHUNK_BYTES);
-      st.chunk(kb0 + off, vb0 + off, mlo | (mhi << 16), __shfl_sync(0xffffffffu, fl, 0));
-      mlo = nlo;
-      mhi = nhi;
-      fl = nfl;
-    }
-    {
-      // output rows: re-derive the item from the parked state (nothing of
-      // the set-up above stays live across the chunk loop)
-      const int it2 = ws[0], g2 = ws[2], grp2 = ws[1] - 8;
-      const int h2 = (blockIdx.x + it2 * gridDim.x) % H;
-      const int64_t m0 = d.node_ptr[g2];
-      const int N2 = (int)(d.node_ptr[g2 + 1] - m0);
-      const int ra2 = grp2 * 16 + gq, rb2 = ra2 + 8;
-      const float l_a = st.osum[0], l_b = st.osum[2];
-      const float ia = l_a > 0.f ? 1.f / l_a : 0.f, ib = l_b > 0.f ? 1.f / l_b : 0.f;
-      __half* Og = out + m0 * dmodel + h2 * DH;
-#pragma unroll
-      for (int dn = 0; dn < A::DN; ++dn) {
-        const int col = dn * 8 + 2 * tq;
-        if (ra2 < N2)
-          *reinterpret_cast<uint32_t*>(Og + (int64_t)ra2 * dmodel + col) = pack_h2(st.o[dn][0] * ia, st.o[dn][1] * ia);
-        if (rb2 < N2)
-          *reinterpret_cast<uint32_t*>(Og + (int64_t)rb2 * dmodel + col) = pack_h2(st.o[dn][2] * ib, st.o[dn][3] * ib);
-      }
-    }
-  }
-}
-
-// Sparse masks (finite-k DAGRA: at k = 4 ~6 % of the N^2 pairs
-// are allowed and the 16-key blocks above compute ~9 scores per useful one).
-// Opt-in experiment (slower, see launch_dh): one thread per query row walks the set bits of its mask row and
-// gathers the allowed keys one by one from the resident K/V chunks -- scores
-// and the online softmax in fp32 on the CUDA cores, work proportional to |A|.
-// One CTA = (graph, 128-row q-tile, head); graphs of density > kSparseDensity
-// stay on k_attn (which skips the sparse ones when both are launched).
-template <int DH>
-__global__ void __launch_bounds__(128) k_attn_sparse(const __grid_constant__ CUtensorMap tkv, DagDev d, int G,
-                                                     int H, int dmodel, const __half* __restrict__ qkv,
-                                                     __half* __restrict__ out) {
-  constexpr int RB = DH * 2, CHB = kChunk * RB;
-  extern __shared__ __align__(16) unsigned char dsm_sp[];
-  __shared__ __align__(8) uint64_t kv_full;
-  const int h = blockIdx.x % H;
-  const int widx = blockIdx.x / H;
-  if (widx >= d.qtile_off[G]) return;
-  const int2 wk = d.work[widx];
-  const int g = wk.x, qt = wk.y;
-  if (d.status[g] != PREDTOP_OK) return;
-  const int64_t n0 = d.node_ptr[g];
-  const int N = (int)(d.node_ptr[g + 1] - n0);
-  if (!is_sparse(d, g, N)) return;
-  const int W = 2 * ((N + 127) / 128);
-  const int nchunks = (N + kChunk - 1) / kChunk;
-  unsigned char* sK = sm100::align256(dsm_sp);
-  unsigned char* sV = sK + (size_t)nchunks * CHB;
-  if (threadIdx.x == 0) {
-    sm100::mbar_init(&kv_full, 1);
-    sm100::fence_mbar_init();
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    sm100::mbar_arrive_expect_tx(&kv_full, (uint32_t)(nchunks * 2 * CHB));
-    for (int c = 0; c < nchunks; ++c) {
-      sm100::tma_load_2d(sK + c * CHB, &tkv, &kv_full, dmodel + h * DH, (int)(n0 + c * kChunk));
-      sm100::tma_load_2d(sV + c * CHB, &tkv, &kv_full, 2 * dmodel + h * DH, (int)(n0 + c * kChunk));
-    }
-  }
-  const int r = qt * 128 + threadIdx.x;
-  const bool valid = r < N;
-  float q[DH];
-  if (valid) {
-    const uint4* qp = reinterpret_cast<const uint4*>(qkv + (n0 + r) * 3 * dmodel + h * DH);
-#pragma unroll
-    for (int p = 0; p < DH / 8; ++p) {
-      const uint4 u = qp[p];
-      const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w4[e]));
-        q[8 * p + 2 * e] = f.x;
-        q[8 * p + 2 * e + 1] = f.y;
-      }
-    }
-  }
-  sm100::mbar_wait(&kv_full, 0);
-  if (!valid) return;
-  // row k of a swizzled [64 x DH] chunk: 16-byte piece p at rr*RB + 16*(p ^ sw(rr))
-  auto row_dot = [&](const unsigned char* base, int k) -> float {
-    const int rr = k & 63;
-    const unsigned char* rowp = base + (k >> 6) * CHB + rr * RB;
-    const int sw = ((rr * RB) >> 7) & (RB / 16 - 1);
-    float acc = 0.f;
-#pragma unroll
-    for (int p = 0; p < DH / 8; ++p) {
-      const uint4 u = *reinterpret_cast<const uint4*>(rowp + 16 * (p ^ sw));
-      const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w4[e]));
-        acc = fmaf(q[8 * p + 2 * e], f.x, acc);
-        acc = fmaf(q[8 * p + 2 * e + 1], f.y, acc);
-      }
-    }
-    return acc;
-  };
-  float o[DH];
-#pragma unroll
-  for (int e = 0; e < DH; ++e) o[e] = 0.f;
-  float m = row_dot(sK, r), l = 0.f;  // reference: the diagonal score (M includes I)
-  const uint64_t* Mr = d.M + d.row_off[g] + (int64_t)r * W;
-  for (int c = 0; c < nchunks; ++c) {
-    uint64_t w = Mr[c];
-    while (w) {
-      const int b = __ffsll((long long)w) - 1;
-      w &= w - 1;
-      // stored bit b -> key: b = 16*((k>>1)&3) + 2*(k>>3) + (k&1) (internal.h mask_pos)
-      const int rem = b & 15;
-      const int k = c * 64 + ((rem >> 1) << 3) + ((b >> 4) << 1) + (rem & 1);
-      const float sc = row_dot(sK, k);
-      if (sc > m) {  // online softmax in log2 units (Q pre-scaled by log2 e / sqrt(d_h))
-        const float a = ex2(m - sc);
-        l *= a;
-#pragma unroll
-        for (int e = 0; e < DH; ++e) o[e] *= a;
-        m = sc;
-      }
-      const float pw = ex2(sc - m);
-      l += pw;
-      const int rr = k & 63;
-      const unsigned char* vrow = sV + (k >> 6) * CHB + rr * RB;
-      const int sw = ((rr * RB) >> 7) & (RB / 16 - 1);
-#pragma unroll
-      for (int p = 0; p < DH / 8; ++p) {
-        const uint4 u = *reinterpret_cast<const uint4*>(vrow + 16 * (p ^ sw));
-        const uint32_t w4[4] = {u.x, u.y, u.z, u.w};
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const float2 f = __half22float2(*reinterpret_cast<const __half2*>(&w4[e]));
-          o[8 * p + 2 * e] = fmaf(pw, f.x, o[8 * p + 2 * e]);
-          o[8 * p + 2 * e + 1] = fmaf(pw, f.y, o[8 * p + 2 * e + 1]);
-        }
-      }
-    }
-  }
-  const float il = l > 0.f ? 1.f / l : 0.f;
-  uint4* op = reinterpret_cast<uint4*>(out + (n0 + r) * dmodel + h * DH);
-#pragma unroll
-  for (int p = 0; p < DH / 8; ++p)
-    op[p] = make_uint4(pack_h2(o[8 * p] * il, o[8 * p + 1] * il), pack_h2(o[8 * p + 2] * il, o[8 * p + 3] * il),
-                       pack_h2(o[8 * p + 4] * il, o[8 * p + 5] * il), pack_h2(o[8 * p + 6] * il, o[8 * p + 7] * il));
-}
-
 template <int DH>
 predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
                          cudaStream_t st, unsigned blocks) {
@@ -781,73 +449,19 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
   CUtensorMap tkv;
   if (!encode_tma_2d(&tkv, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kChunk))
     return PREDTOP_ERR_CUDA;
-  // finite-k masks: graphs of low density go to the gather kernel (K/V resident:
-  // only when the batch's largest graph fits 2 x 24 KB... up to ~96 KB)
-  const int sparse_bytes = 2 * maxch * CH_BYTES + 256;
-  // opt-in (PREDTOP_ATTN_SPARSE=1): measured 2.5x slower than the block-sparse
-  // MMA kernel at k = 4 on the GPT config (2.75 vs 1.08 ms/step: one thread
-  // per row diverges on the per-row key counts and gathers 32-byte rows one
-  // at a time), kept parity-tested for reference
-  const char* sp = getenv("PREDTOP_ATTN_SPARSE");
-  const char* ap0 = getenv("PREDTOP_ATTN_MODE");
-  const int split = dag->desc.hops > 0 && sp && sp[0] == '1' && sparse_bytes <= 96 * 1024 &&
-                    !(ap0 && ap0[0] == 'p');  // the persistent variant has no split
-  if (split) {
-    static int attr_sp = 0;
-    if (sparse_bytes > 48 * 1024 && sparse_bytes > attr_sp) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn_sparse<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024));
-      attr_sp = 96 * 1024;
-    }
-    k_attn_sparse<DH><<<blocks, 128, sparse_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
-    PT_LAUNCH_CHECK();
-  }
-  const int per_sm = DH == 16 ? PREDTOP_ATTN_P_CTAS : 2;
-  const int pers_bytes = 2 * resident_bytes;  // two item buffers (+ alignment slack)
-  const char* ap = getenv("PREDTOP_ATTN_MODE");  // "p": persistent, "8": 8-warp CTAs, default 4-warp
-  const bool persistent = ap && ap[0] == 'p';
+  const char* ap = getenv("PREDTOP_ATTN_MODE");  // "8": 8-warp CTAs, default 4-warp
   const bool half_tiles = !(ap && ap[0] == '8');
-  if (persistent && pers_bytes * per_sm <= 220 * 1024) {
-    static bool attr_p = false;
-    if (!attr_p) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn_p<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       220 * 1024 / per_sm));
-      attr_p = true;
-    }
-    static int sms = 0;
-    if (!sms) {
-      int dev = 0;
-      PT_CUDA_TRY(cudaGetDevice(&dev));
-      PT_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    }
-    const int64_t items = (int64_t)G * H;
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(items, (int64_t)sms * per_sm));
-    k_attn_p<DH><<<grid, 256, pers_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, maxch);
-  } else if (half_tiles && resident4_bytes <= 28 * 1024) {
+  if (half_tiles && resident4_bytes <= 28 * 1024) {
     // 4-warp CTAs (half q-tiles), up to 8 per SM (28 KB + 1 KB static each)
-    static bool attr_h = false;
-    if (!attr_h) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       28 * 1024));
-      attr_h = true;
-    }
-    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, split);
+    PT_SMEM_ATTR((k_attn<DH, true, 4>), 28 * 1024);
+    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
   } else if (resident_bytes + 128 * wmax * 8 <= 100 * 1024) {
-    static bool attr_done = false;
-    if (!attr_done) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       100 * 1024));
-      attr_done = true;
-    }
-    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out, split);
+    PT_SMEM_ATTR((k_attn<DH, true>), 100 * 1024);
+    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out);
   } else {
     constexpr int stream_bytes = 2 * kStages * stage_chunks<DH>() * CH_BYTES + 1024;
-    static bool attr_s = false;
-    if (!attr_s) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_attn<DH, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       stream_bytes));
-      attr_s = true;
-    }
-    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, split);
+    PT_SMEM_ATTR((k_attn<DH, false>), stream_bytes);
+    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
   }
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;

@@ -126,7 +126,7 @@ __global__ void __launch_bounds__(kThreads, 4)
   if (widx >= d.qtile_off[G]) return;
   const int2 wk = d.work[widx];
   const int g = wk.x, qt = wk.y;
-  if (d.status[g] != PREDTOP_OK) return;
+  if ((unsigned)g >= (unsigned)G || d.status[g] != PREDTOP_OK) return;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
   const int W = 2 * ((N + 127) / 128);
@@ -402,11 +402,7 @@ predtop_status attention_tc_launch(const predtop_dag_s* dag, int d, int H, const
   // never wait for each other
   const size_t smem = std::max<size_t>(1024 + 3 * kQBytes + 1024 + (size_t)krows_cap * 64 + (size_t)nch_cap * kVtBytes,
                                        46 * 1024);
-  static size_t attr = 0;
-  if (smem > attr) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_attn_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    attr = smem;
-  }
+  PT_SMEM_ATTR(k_attn_tc, smem);
   CUtensorMap tq;
   if (!encode_tma_2d(&tq, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, kDh, 128))
     return PREDTOP_ERR_CUDA;

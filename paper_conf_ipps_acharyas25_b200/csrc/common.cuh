@@ -32,6 +32,14 @@ struct ProfScope {
 // Thread-local last-error message.
 void set_error(const char* fmt, ...);
 
+// Raise `func`'s dynamic shared-memory limit to at least `bytes` on the
+// current device.  The attribute is per device, so the cache is keyed by
+// (device, kernel); thread-safe (api.cu).
+cudaError_t smem_attr(const void* func, int bytes);
+// SM count of the current device (cached per device); 0 on error.
+int num_sms();
+#define PT_SMEM_ATTR(func, bytes) PT_CUDA_TRY(::predtop::smem_attr((const void*)(func), (int)(bytes)))
+
 #define PT_CUDA_TRY(expr)                                                        \
   do {                                                                           \
     cudaError_t _e = (expr);                                                     \

@@ -11,7 +11,9 @@
 //  k_mask      K3: M = R | R^T | I with warp-ballot 32x32 bit transposes and
 //              popcounts per 128x128 tile
 //  k_classify  tile classes (empty / partial / full) and |A| per graph
-//  k_work      attention work list (graph, 128-row q-tile)
+//  k_dag_small all of the above fused, one warp per graph (N <= 512)
+//  k_bflags    16x64 attention block flags, mask words to the stored layout
+// The attention work list (graph, 128-row q-tile) is written by k_meta.
 #include <algorithm>
 #include <climits>
 
@@ -46,13 +48,14 @@ __device__ T block_excl_scan(T v, T* total, T* sh /*[32]*/) {
   return base + x - v;
 }
 
-// Graphs with N <= sc.sn nodes and E <= sc.se edges take the fused one-warp-
-// per-graph path (k_dag_small); the multi-kernel path below skips them.
+// Graphs with N <= sc.sn nodes take the fused one-warp-per-graph path
+// (k_dag_small; its successor lists sit in shared memory when E <= sc.se, else
+// in the global CSR scratch); the multi-kernel path below skips them.
 struct SmallCfg {
   int sn, se, slot;  // node / edge capacity of a warp slot, slot bytes
 };
-__host__ __device__ inline bool is_small(int N, int E, const SmallCfg& sc) {
-  return N <= sc.sn && E <= sc.se;
+__host__ __device__ inline bool is_small(int N, int /*E*/, const SmallCfg& sc) {
+  return N <= sc.sn;
 }
 
 __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
@@ -60,9 +63,9 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
   int64_t carry_rows = 0, carry_tiles = 0, carry_q = 0, carry_f = 0;
   for (int base = 0; base < G; base += blockDim.x) {
     const int g = base + threadIdx.x;
-    int64_t rows = 0, tiles = 0, q = 0, fl = 0;
+    int64_t rows = 0, tiles = 0, q = 0, fl = 0, n = 0;
     if (g < G) {
-      const int64_t n = d.node_ptr[g + 1] - d.node_ptr[g];
+      n = d.node_ptr[g + 1] - d.node_ptr[g];
       const int64_t e = d.edge_ptr[g + 1] - d.edge_ptr[g];
       int st = PREDTOP_OK;
       if (n < 1 || n > max_nodes || n > PREDTOP_MAX_NODES) st = PREDTOP_ERR_TOO_LARGE;
@@ -86,7 +89,13 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
     if (g < G) d.tile_off[g] = carry_tiles + ex;
     carry_tiles += tot;
     ex = block_excl_scan<int64_t>(q, &tot, sh64);
-    if (g < G) d.qtile_off[g] = (int32_t)(carry_q + ex);
+    if (g < G) {
+      // attention work items (graph, 128-row q-tile), written for every graph
+      // with rows here, so a graph that a later kernel marks RANGE / SELF_LOOP /
+      // CYCLE still leaves valid items (attention skips it by its status)
+      d.qtile_off[g] = (int32_t)(carry_q + ex);
+      for (int qt = 0; qt < q; ++qt) d.work[carry_q + ex + qt] = make_int2(g, qt);
+    }
     carry_q += tot;
     ex = block_excl_scan<int64_t>(fl, &tot, sh64);
     if (g < G) d.bflag_off[g] = carry_f + ex;
@@ -507,16 +516,6 @@ __global__ void __launch_bounds__(256) k_classify(DagDev d, SmallCfg sc) {
   if (threadIdx.x == 0) d.pairs[g] = (int64_t)s_pairs;
 }
 
-__global__ void k_work(DagDev d, SmallCfg sc) {
-  const int g = blockIdx.x;
-  const int st = d.status[g];
-  if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
-  const int N = (int)(d.node_ptr[g + 1] - d.node_ptr[g]);
-  if (is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
-  const int T = (N + 127) / 128;
-  for (int qt = threadIdx.x; qt < T; qt += blockDim.x) d.work[d.qtile_off[g] + qt] = make_int2(g, qt);
-}
-
 
 // ---------------------------------------------------------------------------
 // Fused small-graph path: one warp per graph does K1 + K2 + K3 in shared
@@ -557,8 +556,9 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
   unsigned char* slot = sm_small + (size_t)warp * sc.slot;
   int* indeg = reinterpret_cast<int*>(slot);
   int* soff = indeg + sc.sn;        // N+1
-  int* succ = soff + sc.sn + 1;     // E
-  int* topo = succ + sc.se;         // N
+  // E successors: shared slot when they fit, else the global CSR scratch
+  int* succ = E <= sc.se ? soff + sc.sn + 1 : d.succ + e0;
+  int* topo = soff + sc.sn + 1 + sc.se;  // N
   int* lptr = topo + sc.sn;         // N+1 (first the fill cursor)
   int* tcnt = lptr + sc.sn + 1;     // 16 tile counts (T <= 4)
   int* ctr = tcnt + 16;             // Kahn queue tail
@@ -799,7 +799,6 @@ __global__ void __launch_bounds__(128) k_dag_small(DagDev d, int G, SmallCfg sc)
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) pairs += __shfl_xor_sync(0xffffffffu, pairs, o);
   if (lane == 0) d.pairs[g] = pairs;
-  for (int qt = lane; qt < T; qt += 32) d.work[d.qtile_off[g] + qt] = make_int2(g, qt);
   DTR(4);
 }
 
@@ -855,13 +854,9 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
   const predtop_batch_desc& b = dag->desc;
   const DagDev& d = dag->d;
   const int G = b.num_graphs;
-  PT_CUDA_TRY(cudaMemsetAsync(d.tile_cnt, 0, sizeof(int32_t) * (size_t)dag->tiles_bound, st));
-{
-    ProfScope _p(PK_DAG_META, st);
-    k_meta<<<1, 1024, 0, st>>>(d, G, b.max_nodes);
-    PT_LAUNCH_CHECK();
-  }
-  // small-graph capacity: graphs up to 512 nodes (and <= 4 edges/node) run fused
+  // small-graph capacity: graphs up to 512 nodes run fused (k_dag_small);
+  // when the batch's max_nodes is within it, the multi-kernel path is not
+  // launched at all
   SmallCfg sc{0, 0, 0};
   if (b.max_nodes <= 512) {
     sc.sn = b.max_nodes;
@@ -869,27 +864,25 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
     const size_t ib = align_up((size_t)4 * (4 * (size_t)sc.sn + 2 + sc.se + 24), 16);
     sc.slot = (int)align_up(ib + (size_t)sc.sn * 2 * ceil_div(sc.sn, 128) * 8, 16);
   }
-  const bool all_small_possible = sc.sn > 0;
-  if (all_small_possible) {
-    static int attr_small = 0;
-    if (attr_small < 4 * sc.slot) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_dag_small, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       std::max(4 * sc.slot, 48 * 1024)));
-      attr_small = std::max(4 * sc.slot, 48 * 1024);
-    }
+  const bool all_small = sc.sn > 0;
+  if (!all_small)
+    PT_CUDA_TRY(cudaMemsetAsync(d.tile_cnt, 0, sizeof(int32_t) * (size_t)dag->tiles_bound, st));
+{
+    ProfScope _p(PK_DAG_META, st);
+    k_meta<<<1, 1024, 0, st>>>(d, G, b.max_nodes);
+    PT_LAUNCH_CHECK();
+  }
+  if (all_small) {
+    PT_SMEM_ATTR(k_dag_small, 4 * sc.slot);
     ProfScope _p(PK_DAG_SMALL, st);
     k_dag_small<<<(unsigned)ceil_div(G, 4), 128, 4 * sc.slot, st>>>(d, G, sc);
     PT_LAUNCH_CHECK();
-  }
+  } else {
 {
     // in-degrees and the Kahn queue in shared memory when the largest graph fits
     const int smem_nodes = b.max_nodes <= 26 * 1024 ? b.max_nodes : 0;
     const int dsm = 2 * 4 * smem_nodes;
-    static int attr_depth = 0;
-    if (dsm > 48 * 1024 && dsm > attr_depth) {
-      PT_CUDA_TRY(cudaFuncSetAttribute(k_depth, cudaFuncAttributeMaxDynamicSharedMemorySize, dsm));
-      attr_depth = dsm;
-    }
+    PT_SMEM_ATTR(k_depth, dsm);
     ProfScope _p(PK_DAG_DEPTH, st);
     k_depth<<<G, 256, dsm, st>>>(d, sc, smem_nodes);
     PT_LAUNCH_CHECK();
@@ -901,12 +894,7 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
   int64_t want = maxN * Wmax * 8 + 4 * (4 * maxN + 8) + 16;  // R slice + CSR (E ~ 2N)
   int smem = (int)std::min<int64_t>(want, 200 * 1024);
   smem = (int)align_up((size_t)smem, 1024);
-  static bool attr_done = false;
-  if (!attr_done) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_closure, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     200 * 1024));
-    attr_done = true;
-  }
+  PT_SMEM_ATTR(k_closure, 200 * 1024);
   int64_t cw = std::max<int64_t>(1, std::min<int64_t>(Wmax, (int64_t)smem / (8 * maxN)));
   int64_t slices = ceil_div(Wmax, cw);
   if ((int64_t)smem < 8 * maxN) slices = std::min<int64_t>(ceil_div(Wmax, 2), 65535);  // global mode
@@ -928,11 +916,7 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
     k_classify<<<G, 256, 0, st>>>(d, sc);
     PT_LAUNCH_CHECK();
   }
-{
-    ProfScope _p(PK_DAG_WORK, st);
-    k_work<<<G, 128, 0, st>>>(d, sc);
-    PT_LAUNCH_CHECK();
-  }
+  }  // multi-kernel path
   {
     ProfScope _p(PK_DAG_FLAGS, st);
     const int64_t items = ceil_div(b.max_nodes, 16) * ceil_div(b.max_nodes, 64);

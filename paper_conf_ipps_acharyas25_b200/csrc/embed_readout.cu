@@ -42,7 +42,7 @@ template <int D>
 __global__ void __launch_bounds__(256) k_embed(const float* __restrict__ WT, const float* __restrict__ b,
                                                const predtop_node_feat* __restrict__ feats,
                                                const int32_t* __restrict__ depth,
-                                               const float* __restrict__ pe, int64_t n_tot,
+                                               const float* __restrict__ pe, int pe_rows, int64_t n_tot,
                                                float* __restrict__ x32, __half* __restrict__ x16) {
   constexpr int PER = D / 32;  // columns per lane
   const int lane = threadIdx.x & 31;
@@ -50,8 +50,9 @@ __global__ void __launch_bounds__(256) k_embed(const float* __restrict__ WT, con
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t v = warp0; v < n_tot; v += nwarps) {
     const predtop_node_feat f = feats[v];
-    int dep = depth[v];
-    if (dep < 0) dep = 0;  // invalid graph: latency is NaN anyway
+    // a graph with an error status (latency NaN) may hold no depth at all
+    // (TOO_LARGE / INVALID_ARG graphs are never built): clamp into the table
+    const int dep = min(max(depth[v], 0), pe_rows - 1);
     float l[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) l[j] = log1pf((float)f.dims[j]);
@@ -80,10 +81,11 @@ predtop_status embed_launch(const predtop_model_s* m, const predtop_dag_s* dag, 
   const int64_t n = dag->desc.total_nodes;
   const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 8), 148 * 16));
   const DagDev& d = dag->d;
+  const int pe_rows = std::min<int>(dag->desc.max_nodes, PREDTOP_MAX_NODES);
   ProfScope _p(PK_EMBED, st);
 #define PT_EMBED(D)                                                                  \
   case D:                                                                            \
-    k_embed<D><<<blocks, 256, 0, st>>>(m->W_inT, m->b_in, d.feats, d.depth, pe, n, x32, x16); \
+    k_embed<D><<<blocks, 256, 0, st>>>(m->W_inT, m->b_in, d.feats, d.depth, pe, pe_rows, n, x32, x16); \
     break;
   switch (m->cfg.d_model) {
     PT_EMBED(32)

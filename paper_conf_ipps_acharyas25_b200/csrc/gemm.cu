@@ -383,22 +383,13 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (warp == 1) sm100::tmem_dealloc<NCOLS>(tmem);
 }
 
-int g_num_sms = 0;
 
 template <int BN, int KCH, int EPI>
 predtop_status launch_t(const Maps& maps, const GemmArgs& a, cudaStream_t st) {
   using C = Cfg<BN, KCH, EPI>;
-  static bool attr_done = false;  // once per instantiation (one device per process)
-  if (!attr_done) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_gemm<BN, KCH, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     C::SMEM));
-    attr_done = true;
-  }
-  if (!g_num_sms) {
-    int dev = 0;
-    PT_CUDA_TRY(cudaGetDevice(&dev));
-    PT_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
-  }
+  PT_SMEM_ATTR((k_gemm<BN, KCH, EPI>), C::SMEM);
+  const int g_num_sms = num_sms();
+  if (!g_num_sms) return PREDTOP_ERR_CUDA;
   const int64_t tiles = ceil_div(a.M, 128) * (a.N / BN);
   const int grid = (int)std::min<int64_t>(tiles, g_num_sms);
   k_gemm<BN, KCH, EPI><<<grid, kThreads, C::SMEM, st>>>(maps, a);

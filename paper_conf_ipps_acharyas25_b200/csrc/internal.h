@@ -200,9 +200,6 @@ predtop_status search_launch(int64_t P, int L, int K, const int32_t* dev, int D,
 // ---- layer.cu (fused O-proj + LN1 + FFN + LN2)
 bool layer_tail_supported(int d, int dff);
 bool layer_tail2_supported(int d, int dff);
-bool layer_tail3_supported(int d, int dff);
-predtop_status layer_tail3_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
-                                  __half* x16, int M, cudaStream_t st);
 predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
                                   __half* x16, int M, cudaStream_t st);
 predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* att, float* x32,

@@ -416,21 +416,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail(const __grid_constan
   if (warp == 1) sm100::tmem_dealloc<C::TMEM_COLS>(tmem);
 }
 
-int g_sms = 0;
 
 template <int D>
 predtop_status launch_d(const TailMaps& mp, const TailArgs& a, cudaStream_t st) {
   using C = TailCfg<D>;
-  static bool attr_done = false;
-  if (!attr_done) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_layer_tail<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
-    attr_done = true;
-  }
-  if (!g_sms) {
-    int dev = 0;
-    PT_CUDA_TRY(cudaGetDevice(&dev));
-    PT_CUDA_TRY(cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev));
-  }
+  PT_SMEM_ATTR(k_layer_tail<D>, C::SMEM);
+  const int g_sms = num_sms();
+  if (!g_sms) return PREDTOP_ERR_CUDA;
   const int grid = (int)std::min<int64_t>(ceil_div(a.M, 128), g_sms);
   k_layer_tail<D><<<grid, kThreads, C::SMEM, st>>>(mp, a);
   PT_LAUNCH_CHECK();

@@ -550,7 +550,6 @@ __global__ void __launch_bounds__(kThreads, 2) k_layer_tail2(const __grid_consta
   if (warp == 1) sm100::tmem_dealloc<TMEM_COLS>(tmem);
 }
 
-int g_sms2 = 0;
 
 }  // namespace
 
@@ -573,16 +572,9 @@ predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half*
   mp.w1 = L.tm_1h;
   mp.w2 = L.tm_2;
   Tail2Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
-  static bool attr_done = false;
-  if (!attr_done) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_layer_tail2, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM));
-    attr_done = true;
-  }
-  if (!g_sms2) {
-    int dev = 0;
-    PT_CUDA_TRY(cudaGetDevice(&dev));
-    PT_CUDA_TRY(cudaDeviceGetAttribute(&g_sms2, cudaDevAttrMultiProcessorCount, dev));
-  }
+  PT_SMEM_ATTR(k_layer_tail2, SMEM);
+  const int g_sms2 = num_sms();
+  if (!g_sms2) return PREDTOP_ERR_CUDA;
   const int grid = (int)std::min<int64_t>(ceil_div(M, 128), 2 * g_sms2);
   k_layer_tail2<<<grid, kThreads, SMEM, st>>>(mp, a);
   PT_LAUNCH_CHECK();

@@ -236,16 +236,9 @@ predtop_status search_launch(int64_t P, int L, int K, const int32_t* dev, int D,
   a.C = (int64_t)K * a.NT;
   a.Tc = reinterpret_cast<double*>(ws);
   const size_t fbytes = (size_t)(L + 1) * (D + 1) * sizeof(double);
-  static size_t attr_cand = 0, attr_pick = 0;
   const size_t cand_smem = 4 * fbytes, pick_smem = fbytes + align_up((size_t)(L + 1) * (D + 1) * 2, 16);
-  if (cand_smem > 48 * 1024 && cand_smem > attr_cand) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_search_cand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cand_smem));
-    attr_cand = cand_smem;
-  }
-  if (pick_smem > 48 * 1024 && pick_smem > attr_pick) {
-    PT_CUDA_TRY(cudaFuncSetAttribute(k_search_pick, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pick_smem));
-    attr_pick = pick_smem;
-  }
+  PT_SMEM_ATTR(k_search_cand, cand_smem);
+  PT_SMEM_ATTR(k_search_pick, pick_smem);
   const int64_t warps = P * a.C;
   const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(warps, 4), 148 * 16));
   {

@@ -18,3 +18,25 @@ def oracle_mod():
     import oracle
     oracle.build()
     return oracle
+
+
+@pytest.fixture(scope="session")
+def parity_log():
+    """record(name, **fields): append one JSON line of measured GPU-vs-oracle
+    errors to $PREDTOP_PARITY_LOG (default gpurun_out/parity_log.jsonl, which
+    gpurun brings back; profiles/parity_r02.json is the tracked copy)."""
+    import json
+    import time
+    path = os.environ.get("PREDTOP_PARITY_LOG", os.path.join(ROOT, "gpurun_out", "parity_log.jsonl"))
+
+    def record(name, **fields):
+        try:
+            os.makedirs(os.path.dirname(path), exist_ok=True)
+            with open(path, "a") as f:
+                f.write(json.dumps(dict(test=name, when=time.strftime("%Y-%m-%dT%H:%M:%S"),
+                                        **{k: (float(v) if hasattr(v, "dtype") else v)
+                                           for k, v in fields.items()})) + "\n")
+        except OSError:
+            pass
+    return record
+

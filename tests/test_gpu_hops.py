@@ -98,16 +98,13 @@ def test_negative_hops_rejected(pt):
         pt.Dag(pt.DeviceBatch.from_host(b), hops=-1)
 
 
-@pytest.mark.parametrize("sparse", ["0", "1"])
 @pytest.mark.parametrize("name, batch_fn, k", [
     ("gpt", lambda: synth.stage_batch("gpt", 16), 2),
     ("gpt", lambda: synth.stage_batch("gpt", 16, first_graph=16), 6),
     ("moe", lambda: synth.stage_batch("moe", 2), 3),
 ])
-def test_forward_parity(pt, oracle_mod, name, batch_fn, k, sparse, monkeypatch):
-    """sparse = "1": the opt-in gather kernel (k_attn_sparse) takes the graphs
-    of density <= 1/5, the block-sparse MMA kernel the others."""
-    monkeypatch.setenv("PREDTOP_ATTN_SPARSE", sparse)
+def test_forward_parity(pt, oracle_mod, name, batch_fn, k):
+    """k-hop masks through the block-sparse attention kernel."""
     cfg = dict(synth.MODEL_CONFIGS[name])
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
     model = pt.Model(cfg, blob)

@@ -241,3 +241,25 @@ def test_invalid_graph_gives_nan(oracle_mod):
     f = np.zeros(3, synth.FEAT_DTYPE)
     st, y, _ = oracle_mod.forward(cfg, blob, 3, np.array([0, 1, 2]), np.array([1, 2, 0]), f)
     assert st == oracle_mod.CYCLE and math.isnan(y)
+
+
+def test_row_block_evaluation_is_the_same_layer(oracle_mod):
+    """oracle.layer_rows / forward_rows (the 16k path: one graph's layers
+    evaluated row block by row block on several threads) compose the same
+    orc_qkv_rows / orc_attention_rows / orc_layer_post_rows that orc_layer
+    is built from, so they reproduce orc_layer / orc_forward bit for bit, for
+    any row subset and any thread count."""
+    from paper_conf_ipps_acharyas25_b200 import synth
+    cfg = synth.MODEL_CONFIGS["paper"]
+    blob = synth.pack_weights(cfg, synth.model_weights(cfg))
+    b = synth.stage_batch("gpt", 2, first_graph=9)
+    for g in range(2):
+        n, s, d, f = b.graph(g)
+        st, y, taps = oracle_mod.forward(cfg, blob, n, s, d, f, taps=True)
+        st2, y2, taps2 = oracle_mod.forward_rows(cfg, blob, n, s, d, f, threads=3, taps=True)
+        assert st == st2 == 0 and y == y2
+        np.testing.assert_array_equal(taps, taps2)
+        M = oracle_mod.mask(n, oracle_mod.reach(n, s, d))
+        rows = [0, 1, 2, 40, 41, n - 1]
+        np.testing.assert_array_equal(oracle_mod.layer_rows(cfg, blob, 2, n, M, taps[2], rows=rows, threads=2),
+                                      oracle_mod.layer(cfg, blob, 2, n, M, taps[2])[rows])
