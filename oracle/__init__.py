@@ -234,6 +234,52 @@ def forward_batch(model_cfg, blob, batch, graphs: Optional[Sequence[int]] = None
         return np.asarray(list(ex.map(one, gs)), np.float64)
 
 
+def head_condition(model_cfg, blob, n, x_final) -> float:
+    """Condition scale of the head's last dot product (reading R10):
+    sum_i |w_o,i * h2_i| with h2 = ReLU(H_2 ReLU(H_1 g + c_1) + c_2) and g
+    the pooled final embeddings (Eqn 2).  It is the magnitude of the
+    terms that cancel in y - c_o = w_o . h2, so |dy| / head_condition is the
+    normwise relative error of the computed (bias-free) part (reading R22);
+    dividing by |y - c_o| instead is ill-conditioned where the terms cancel.
+    Test metadata only: numpy on the oracle's own fp64 taps, the blob's head
+    weights in the include/predtop.h order (H_1, c_1, H_2, c_2, w_o, c_o last)."""
+    d = model_cfg["d_model"]
+    b = np.asarray(blob, np.float64)
+    tail = b[len(b) - (2 * d * d + 3 * d + 1):]
+    H1 = tail[:d * d].reshape(d, d)
+    c1 = tail[d * d:d * d + d]
+    H2 = tail[d * d + d:2 * d * d + d].reshape(d, d)
+    c2 = tail[2 * d * d + d:2 * d * d + 2 * d]
+    wo = tail[2 * d * d + 2 * d:2 * d * d + 3 * d]
+    g = np.asarray(x_final, np.float64).sum(0)
+    if model_cfg.get("pool", 0) == 1:
+        g = g / n
+    h1 = np.maximum(H1 @ g + c1, 0.0)
+    h2 = np.maximum(H2 @ h1 + c2, 0.0)
+    return float(np.abs(wo * h2).sum())
+
+
+def forward_batch_cond(model_cfg, blob, batch, graphs: Optional[Sequence[int]] = None,
+                       threads: Optional[int] = None, hops: int = 0):
+    """(latency, head_condition) of every listed graph: forward_batch plus the
+    condition scale of each graph's bias-free output (from its final taps)."""
+    gs = list(range(batch.num_graphs)) if graphs is None else list(graphs)
+    threads = threads or (os.cpu_count() or 1)
+    lib()
+
+    def one(g):
+        n, s, d, f = batch.graph(g)
+        _, y, t = forward(model_cfg, blob, n, s, d, f, taps=True, hops=hops)
+        return y, head_condition(model_cfg, blob, n, t[-1])
+
+    if threads <= 1 or len(gs) <= 1:
+        out = [one(g) for g in gs]
+    else:
+        with ThreadPoolExecutor(threads) as ex:
+            out = list(ex.map(one, gs))
+    return np.asarray([o[0] for o in out], np.float64), np.asarray([o[1] for o in out], np.float64)
+
+
 # ---- one large graph, row block by row block --------------------------------
 def _ranges(rows, threads):
     """Split a sorted row list into <= ~4*threads contiguous runs."""

@@ -16,10 +16,6 @@ TOL = 2e-3
 U16 = 2.0 ** -11
 
 
-def _c_o(cfg):
-    return float(synth.model_weights(cfg)["c_o"][0])
-
-
 @pytest.fixture(scope="module")
 def pt():
     from paper_conf_ipps_acharyas25_b200 import build, predtop
@@ -60,8 +56,8 @@ def test_latency_parity(pt, oracle_mod, parity_log, name, batch_fn):
     cfg, blob, model = _model(pt, name)
     batch = batch_fn()
     y, _ = _gpu_latency(pt, model, batch)
-    want = oracle_mod.forward_batch(cfg, blob, batch)
-    st = rel_err_stats(y, want, _c_o(cfg))
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch)
+    st = rel_err_stats(y, want, cond)
     parity_log(f"latency_parity[{name}]", **st)
     print(f"{name}: {st}")
     assert np.isfinite(y).all()
@@ -220,8 +216,8 @@ def test_full_gpt_config_sampled(pt, oracle_mod, parity_log):
     y, _ = _gpu_latency(pt, model, batch)
     assert np.isfinite(y).all()
     sample = list(range(0, 1024, 16)) + [1023]
-    want = oracle_mod.forward_batch(cfg, blob, batch, graphs=sample)
-    st = rel_err_stats(y[sample], want, _c_o(cfg))
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch, graphs=sample)
+    st = rel_err_stats(y[sample], want, cond)
     parity_log("full_gpt_sampled", **st)
     print(f"gpt full: {st}")
     assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
@@ -237,8 +233,8 @@ def test_full_moe_config_sampled(pt, oracle_mod, parity_log):
     y, _ = _gpu_latency(pt, model, batch)
     assert np.isfinite(y).all()
     sample = list(range(0, 512, 16)) + [511]  # 33 graphs
-    want = oracle_mod.forward_batch(cfg, blob, batch, graphs=sample)
-    st = rel_err_stats(y[sample], want, _c_o(cfg))
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch, graphs=sample)
+    st = rel_err_stats(y[sample], want, cond)
     parity_log("full_moe_sampled", **st)
     print(f"moe full: {st}")
     assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
@@ -275,9 +271,9 @@ def test_16k_forward_parity(pt, oracle_mod, parity_log):
     dag = pt.Dag(pt.DeviceBatch.from_host(b))
     y = model.forward(dag).cpu().numpy().astype(np.float64)
     n, s_, d_, f_ = b.graph(0)
-    st_, want, _ = oracle_mod.forward_rows(cfg, blob, n, s_, d_, f_)
+    st_, want, taps16 = oracle_mod.forward_rows(cfg, blob, n, s_, d_, f_, taps=True)
     assert st_ == 0
-    st = rel_err_stats(y, [want], _c_o(cfg))
+    st = rel_err_stats(y, [want], [oracle_mod.head_condition(cfg, blob, n, taps16[-1])])
     parity_log("16k_forward", **st, y=float(y[0]), want=want)
     print(f"16k: y {y[0]:.6f} oracle {want:.6f} {st}")
     assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
@@ -315,9 +311,9 @@ def test_sweep_chunk_4096(pt, oracle_mod, parity_log):
     lo, hi, key = next(c for c in sh.chunks if c[1] - c[0] == 4096)
     idx = sorted(set(synth.CounterRng(4096, 1).permutation(4096)[:63].tolist()) | {4095})
     gs = [pool[(key[0] + i) % len(pool)] for i in idx]
-    want = oracle_mod.forward_batch(cfg, blob, synth.pack_graphs(gs))
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, synth.pack_graphs(gs))
     got = lat[lo:hi][idx].astype(np.float64)
-    st = rel_err_stats(got, want, _c_o(cfg))
+    st = rel_err_stats(got, want, cond)
     parity_log("sweep_chunk_4096", **st)
     print(f"sweep chunk: {st}")
     assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL

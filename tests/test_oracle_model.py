@@ -263,3 +263,22 @@ def test_row_block_evaluation_is_the_same_layer(oracle_mod):
         rows = [0, 1, 2, 40, 41, n - 1]
         np.testing.assert_array_equal(oracle_mod.layer_rows(cfg, blob, 2, n, M, taps[2], rows=rows, threads=2),
                                       oracle_mod.layer(cfg, blob, 2, n, M, taps[2])[rows])
+
+
+@pytest.mark.parametrize("pool", [0, 1])
+def test_head_condition_bounds_bias_free_output(oracle_mod, pool):
+    """oracle.head_condition (reading R22) is the absolute sum of the terms of
+    y - c_o = w_o . h2: it bounds |y - c_o| (triangle inequality), and equals
+    it when every w_o,i >= 0 (h2 >= 0 after the ReLU), on the oracle readout."""
+    cfg = _cfg("gpt", pool=pool)
+    w, blob = _blob(cfg)
+    n = 29
+    x = synth.CounterRng(3, 3).uniform_array(n * cfg["d_model"]).reshape(n, -1) * 2 - 1
+    c_o = float(w["c_o"][0])
+    y = oracle_mod.readout(cfg, blob, n, x)
+    assert oracle_mod.head_condition(cfg, blob, n, x) >= abs(y - c_o) * (1 - 1e-12)
+    w2 = dict(w)
+    w2["w_o"] = np.abs(w["w_o"])
+    blob2 = synth.pack_weights(cfg, w2)
+    y2 = oracle_mod.readout(cfg, blob2, n, x)
+    assert oracle_mod.head_condition(cfg, blob2, n, x) == pytest.approx(y2 - c_o, rel=1e-12)
