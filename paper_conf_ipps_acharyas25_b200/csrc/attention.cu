@@ -24,8 +24,8 @@
 // At d_h = 16/32 the kernel is bound by the exponentials and the issue slots
 // around them, not by the tensor pipe: QK^T and PV are 2*d_h flops per score
 // each.  The S accumulator fragment is the P operand fragment, so S and P
-// never leave registers; see DESIGN.md "K6".  attention_tc.cu holds an
-// opt-in tcgen05/TMEM variant.
+// never leave registers; see DESIGN.md "K6".  This kernel serves d_h = 16;
+// d_h = 32 runs on the tcgen05/TMEM kernel of attention_tc.cu.
 #include "internal.h"
 #include "sm100.cuh"
 
@@ -478,10 +478,14 @@ predtop_status attention_launch(const predtop_dag_s* dag, int d, int H, const __
     return PREDTOP_ERR_TOO_LARGE;
   }
   ProfScope _p(PK_ATTN, st);
-  // PREDTOP_ATTN_TC=1: the tcgen05/TMEM variant (attention_tc.cu); measured
-  // slower than this kernel on the GPT workload, so opt-in
+  // tcgen05/TMEM kernel (attention_tc.cu) at d_h = 32, where this kernel's
+  // mma.sync QK^T + PV demand equals the MUFU rate; this kernel at d_h = 16.
+  // PREDTOP_ATTN_TC=1 / =0 forces one or the other (parity tests, A/B runs).
   const char* tc = getenv("PREDTOP_ATTN_TC");
-  if (tc && tc[0] == '1' && attention_tc_supported(dag, d, H)) return attention_tc_launch(dag, d, H, qkv, out, st);
+  bool use_tc = dh == 32;
+  if (tc && tc[0] == '1') use_tc = true;
+  if (tc && tc[0] == '0') use_tc = false;
+  if (use_tc && attention_tc_supported(dag, d, H)) return attention_tc_launch(dag, d, H, qkv, out, st);
   if (dh == 16) return launch_dh<16>(dag, d, H, qkv, out, st, (unsigned)blocks);
   if (dh == 32) return launch_dh<32>(dag, d, H, qkv, out, st, (unsigned)blocks);
   set_error("unsupported head dim %d", dh);

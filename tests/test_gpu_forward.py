@@ -65,22 +65,26 @@ def test_latency_parity(pt, oracle_mod, parity_log, name, batch_fn):
     assert st["max_rel_nobias"] <= TOL
 
 
-@pytest.mark.parametrize("name, batch_fn", [
-    ("paper", lambda: synth.stage_batch("gpt", 12, seed=11)),
-    ("gpt", lambda: synth.stage_batch("gpt", 24)),
-    ("gpt", lambda: synth.tiny_batch()),
+@pytest.mark.parametrize("name, batch_fn, tc", [
+    ("paper", lambda: synth.stage_batch("gpt", 12, seed=11), "1"),
+    ("gpt", lambda: synth.stage_batch("gpt", 24), "1"),
+    ("gpt", lambda: synth.tiny_batch(), "1"),
+    ("moe", lambda: synth.stage_batch("moe", 3, first_graph=20), "0"),
 ])
-def test_latency_parity_tcgen05_attention(pt, oracle_mod, name, batch_fn, monkeypatch):
-    """The opt-in tcgen05/TMEM attention kernel (attention_tc.cu, d_h = 16)."""
-    monkeypatch.setenv("PREDTOP_ATTN_TC", "1")
+def test_latency_parity_attention_kernel_choice(pt, oracle_mod, parity_log, name, batch_fn, tc, monkeypatch):
+    """The attention kernel that is NOT the default for the head dim:
+    PREDTOP_ATTN_TC=1 runs the tcgen05/TMEM kernel (attention_tc.cu) at
+    d_h = 16, =0 the mma.sync kernel (attention.cu) at d_h = 32."""
+    monkeypatch.setenv("PREDTOP_ATTN_TC", tc)
     cfg, blob, model = _model(pt, name)
     batch = batch_fn()
     y, _ = _gpu_latency(pt, model, batch)
-    want = oracle_mod.forward_batch(cfg, blob, batch)
-    err = _rel(y, want)
-    print(f"{name} (tcgen05 attention): max rel err {err.max():.3e}")
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch)
+    st = rel_err_stats(y, want, cond)
+    parity_log(f"latency_parity_attn_tc={tc}[{name}]", **st)
+    print(f"{name} (PREDTOP_ATTN_TC={tc}): {st}")
     assert np.isfinite(y).all()
-    assert err.max() <= TOL
+    assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
 
 
 @pytest.mark.parametrize("name, batch_fn", [
