@@ -3,35 +3,41 @@
 //     O_h = softmax(Q_h K_h^T / sqrt(d_h) + M) V_h,  M(u,v) = 0 iff bit M[u][v]
 //     of M = R | R^T | I is set (DAGRA), else -inf.
 //
-// One CTA = one (graph, 128-row query tile, head); four CTAs per SM (128 TMEM
-// columns each, 16 softmax warps per SM to hide the TMEM/MUFU latencies).
-// Every query row is one TMEM lane, so a softmax thread owns a whole row: no
-// shuffles, 32 independent exponentials per key chunk.
+// One CTA = one (graph, 128-row query tile, head); two CTAs per SM (256 TMEM
+// columns each), 8 softmax warps per CTA.  Each query row is one TMEM lane;
+// the two softmax warps of a lane quarter split every 64-key chunk into key
+// halves, so a softmax thread owns (row, 32 keys of the chunk): no shuffles.
 //
-//   warp 0      TMA producer: the Q tile, then K and V of every 32-key chunk
+//   warp 0      TMA producer: the Q tile, then K and V of every 64-key chunk
 //               of the graph's head through a kKV-stage ring (SW64 boxes at
 //               d_h = 32, SW32 at d_h = 16)
 //   warp 1      TMEM owner + MMA issuer (one thread):
-//                 S_b  = Q K_c^T + Qm_b One^T   SS-MMA, M=128 N=32: q.k - m
-//                 O   += P_b V_c                TS-MMA (A = P in TMEM), V is
-//                                               the MN-major B operand as TMA
-//                                               wrote it (no transpose)
-//   warps 2..5  softmax (row = TMEM lane): mask bits -> -inf, exp2, P as fp16
-//               written over S_b (tcgen05.st), row sums l in registers
-//               (fp32), then O / l -> fp16 rows.
+//                 S_b  = Q K_c^T + Qm One^T     SS-MMA, M=128 N=64: q.k - m
+//                 [O | l] += P_b [V_c | 1]      TS-MMA (A = P in TMEM), N =
+//                                               d_h + 16: V is the MN-major B
+//                                               operand as TMA wrote it (no
+//                                               transpose), a constant ones
+//                                               atom LBO bytes after it gives
+//                                               the row sums l
+//   warps 2..9  softmax: mask bit -> -inf, exp2, P as fp16 written over the
+//               thread's own half of S_b (tcgen05.st), then O / l -> fp16.
 //
-// TMEM (128 columns): S_0 | S_1 | S_2 (32 each, P in the first 16 of its S)
-// | O (d_h).  QK^T of chunk c+3 is issued right after PV of chunk c, so the
-// tensor core runs two chunks ahead of the softmax.
+// TMEM (256 columns): S_0 | S_1 | S_2 (64 each) | O (d_h) | l (16).  P of
+// keys 0-31 of a chunk sits in columns [0,16) of its S, keys 32-63 in
+// [32,48): each half is written only by the threads that read that half of
+// S.  QK^T of chunk c+3 is issued right after PV of chunk c, so the tensor
+// core runs two chunks (128 keys) ahead of the softmax.
 //
-// Online softmax in log2 units (Q pre-scaled by log2(e)/sqrt(d_h) in the QKV
-// epilogue).  The reference m of a row starts at its diagonal score (M
-// includes I, so the row max is >= it) and only moves when some P of a chunk
-// exceeds 2^12 (or overflows fp16): then m moves to the chunk max (fp16-
-// rounded; it enters the MMA as the fp16 operand Qm) and O, l are rescaled in
-// TMEM once the previous PV has completed (rare).  S_b was computed with the
-// m held in Qm_b when its QK^T was issued (mu_b); a row whose m moved since
-// corrects by m - mu_b.
+// Softmax in log2 units (Q pre-scaled by log2(e)/sqrt(d_h) in the QKV
+// epilogue) against a FIXED per-row reference m = the row's diagonal score
+// (allowed: M includes I), rounded to fp16 (it enters the MMA as the fp16
+// operand Qm, so the MMA returns s - m).  P = exp2(s - m) is rounded to fp16
+// in range while s - m <= 12 (P <= 4096); a row where some allowed score
+// exceeds its diagonal by more than that (never seen with the synthetic
+// models; possible with peaked trained attention) is recomputed exactly at
+// the end by its softmax thread on the CUDA cores (fp32 two-pass softmax over
+// the row, from the same fp16 q/k/v; rare path).  No per-chunk rescaling, so
+// the two key-half threads of a row never need to agree on a moving maximum.
 #include <algorithm>
 
 #include "internal.h"
@@ -42,26 +48,32 @@ namespace predtop {
 namespace {
 
 constexpr int kRows = 128;   // query rows per CTA (TMEM lanes)
-constexpr int kCh = 32;      // keys per chunk (S columns)
+constexpr int kCh = 64;      // keys per chunk (S columns)
 constexpr int kSBuf = 3;     // S/P buffers in TMEM
-constexpr int kKV = 8;       // K/V ring stages
-constexpr int kThreads = 192;
-constexpr float kPMax = 4096.f;  // P above this (or inf) moves the reference m
+#ifndef PREDTOP_ATTN_KV
+#define PREDTOP_ATTN_KV 6
+#endif
+constexpr int kKV = PREDTOP_ATTN_KV;  // K/V ring stages
+static_assert(kKV > kSBuf && kKV <= 2 * kSBuf, "K/V stages are released through s_full (see the producer)");
+constexpr int kSoftWarps = 8;
+constexpr int kThreads = 64 + 32 * kSoftWarps;
+constexpr float kPMax = 4096.f;  // P above this (or inf, NaN) sends the row to the exact path
 
 template <int DH>
 struct TcCfg {
   static constexpr int RB = DH * 2;        // bytes per Q/K/V row = swizzle width (32 or 64)
   static constexpr int QB = kRows * RB;    // Q tile
   static constexpr int KB = kCh * RB;      // one K (or V) chunk
-  static constexpr int STAGE = 2 * KB;     // K | V
-  static constexpr int QM = kRows * 32;    // Qm_b: [128][16] fp16, SW32, column 0 = -m
-  static constexpr int ONE = kCh * 32;     // One: [32][16] fp16, SW32, column 0 = 1
+  static constexpr int STAGE = 3 * KB;     // K | V | ones (the l columns of the PV operand)
+  static constexpr int QM = kRows * 32;    // Qm: [128][16] fp16, SW32, column 0 = -m
+  static constexpr int ONE = kCh * 32;     // One: [64][16] fp16, SW32, column 0 = 1
   static constexpr int TO = kSBuf * kCh;   // TMEM column of O
-  static constexpr int BYTES = 1024 + QB + kKV * STAGE + kSBuf * QM + ONE;
-  // > 228/5 KB: at most four CTAs per SM, so the 128-column TMEM
-  // allocations never wait for each other
-  static constexpr int SMEM = BYTES > 47 * 1024 ? BYTES : 47 * 1024;
-  static_assert(TO + DH <= 128, "TMEM budget");
+  static constexpr int TL = TO + DH;       // TMEM column of l
+  static constexpr int BYTES = 1024 + QB + kKV * STAGE + QM + ONE;
+  // > 228/3 KB: at most two CTAs per SM, so the 256-column TMEM allocations
+  // never wait for each other
+  static constexpr int SMEM = BYTES > 80 * 1024 ? BYTES : 80 * 1024;
+  static_assert(TL + 16 <= 256, "TMEM budget");
 };
 
 #ifdef PREDTOP_ATTN_MMA_SPIN
@@ -70,33 +82,91 @@ struct TcCfg {
 #define MMA_WAIT sm100::mbar_wait_sleep
 #endif
 
+#ifdef PREDTOP_TRACE
+// debug timeline of one CTA (clock64 at pipeline events, tools/attn_trace.py)
+__device__ unsigned long long g_at[8][64];
+#define ATR(k, i) \
+  do {            \
+    if (blockIdx.x == 3001 && (i) < 64) g_at[k][i] = clock64(); \
+  } while (0)
+#else
+#define ATR(k, i) \
+  do {            \
+  } while (0)
+#endif
+
 __device__ __forceinline__ float ex2f(float x) {
   float y;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
 
-// bit of key k (0..63 of a 64-key mask word) in the stored layout
-// (internal.h mask_pos)
-__device__ __forceinline__ bool key_bit(uint32_t lo, uint32_t hi, int k) {
-  const int p = mask_pos(k);
-  return p < 32 ? ((lo >> p) & 1u) : ((hi >> (p - 32)) & 1u);
+// mbarrier helpers on precomputed shared-space addresses (the chunk loop does
+// not re-derive them)
+__device__ __forceinline__ void bar_wait(uint32_t addr, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n}" ::"r"(addr),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bar_arrive(uint32_t addr) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(addr) : "memory");
+}
+
+// Exact row on the CUDA cores (rare path): fp32 scores from the fp16 q, k
+// (log2 units), two passes over the allowed keys (max, then sum and P.V).
+template <int DH>
+__device__ __noinline__ void exact_row(const __half* __restrict__ qkv, int64_t n0, int N, int row, int h,
+                                       int dmodel, const uint64_t* __restrict__ Mrow, __half* __restrict__ outrow) {
+  float q[DH];
+  const __half* qr = qkv + (n0 + row) * 3 * dmodel + h * DH;
+#pragma unroll
+  for (int j = 0; j < DH; ++j) q[j] = __half2float(qr[j]);
+  auto allowed = [&](int k) { return ((Mrow[k >> 6] >> mask_pos(k & 63)) & 1ull) != 0ull; };
+  auto score = [&](int k) {
+    const __half* kr = qkv + (n0 + k) * 3 * dmodel + dmodel + h * DH;
+    float s = 0.f;
+#pragma unroll
+    for (int j = 0; j < DH; ++j) s = fmaf(q[j], __half2float(kr[j]), s);
+    return s;
+  };
+  float mx = -INFINITY;
+  for (int k = 0; k < N; ++k)
+    if (allowed(k)) mx = fmaxf(mx, score(k));
+  float l = 0.f, o[DH];
+#pragma unroll
+  for (int j = 0; j < DH; ++j) o[j] = 0.f;
+  for (int k = 0; k < N; ++k) {
+    if (!allowed(k)) continue;
+    const float p = exp2f(score(k) - mx);
+    l += p;
+    const __half* vr = qkv + (n0 + k) * 3 * dmodel + 2 * dmodel + h * DH;
+#pragma unroll
+    for (int j = 0; j < DH; ++j) o[j] = fmaf(p, __half2float(vr[j]), o[j]);
+  }
+  const float inv = 1.f / l;
+#pragma unroll
+  for (int j = 0; j < DH; ++j) outrow[j] = __float2half_rn(o[j] * inv);
 }
 
 template <int DH>
-__global__ void __launch_bounds__(kThreads, 4)
-    k_attn_tc(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tm, DagDev d, int G, int H, int dmodel,
-              const __half* __restrict__ qkv, __half* __restrict__ out) {
+__global__ void __launch_bounds__(kThreads, 2)
+    k_attn_tc(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tm, DagDev d, int G,
+              int H, int dmodel, const __half* __restrict__ qkv, __half* __restrict__ out) {
   using C = TcCfg<DH>;
   extern __shared__ unsigned char dsm[];
   unsigned char* base = sm100::align1024(dsm);
   unsigned char* sQ = base;                      // [128][DH], swizzled
-  unsigned char* sKV = sQ + C::QB;               // stage s: K at s*STAGE, V at +KB
-  unsigned char* sQm = sKV + kKV * C::STAGE;     // Qm_b at b*QM
-  unsigned char* sOne = sQm + kSBuf * C::QM;
-  __shared__ __align__(8) uint64_t q_full, init_done, kv_full[kKV], kv_empty[kKV], s_full[kSBuf],
-      p_ready[kSBuf], pv_done[2], o_full;
+  unsigned char* sKV = sQ + C::QB;               // stage s: K at s*STAGE, V at +KB, ones at +2KB
+  unsigned char* sQm = sKV + kKV * C::STAGE;
+  unsigned char* sOne = sQm + C::QM;
+  __shared__ __align__(8) uint64_t q_full, init_done, kv_full[kKV], s_full[kSBuf],
+      p_ready[kSBuf], o_full;
   __shared__ uint32_t tmem_slot;
+  __shared__ int row_exact[kRows];  // rows sent to the exact path
 
   const int h = blockIdx.x % H;
   const int widx = blockIdx.x / H;
@@ -126,19 +196,17 @@ __global__ void __launch_bounds__(kThreads, 4)
 #pragma unroll
     for (int s = 0; s < kKV; ++s) {
       sm100::mbar_init(&kv_full[s], 1);
-      sm100::mbar_init(&kv_empty[s], 1);
     }
 #pragma unroll
     for (int b = 0; b < kSBuf; ++b) {
       sm100::mbar_init(&s_full[b], 1);
-      sm100::mbar_init(&p_ready[b], 4);
+      sm100::mbar_init(&p_ready[b], kSoftWarps);
     }
-    sm100::mbar_init(&pv_done[0], 1);
-    sm100::mbar_init(&pv_done[1], 1);
     sm100::mbar_init(&o_full, 1);
     sm100::fence_mbar_init();
   }
-  if (warp == 1) sm100::tmem_alloc<128>(&tmem_slot);
+  if (threadIdx.x < kRows) row_exact[threadIdx.x] = 0;
+  if (warp == 1) sm100::tmem_alloc<256>(&tmem_slot);
   sm100::tc_fence_before();
   __syncthreads();
   sm100::tc_fence_after();
@@ -146,233 +214,229 @@ __global__ void __launch_bounds__(kThreads, 4)
 
   if (warp == 0) {
     if (lane == 0) {  // -------------------------------------------- TMA
-      const int r0 = (int)(n0 + qt * kRows);
       sm100::mbar_arrive_expect_tx(&q_full, (uint32_t)C::QB);
-      sm100::tma_load_2d(sQ, &tq, &q_full, h * DH, r0);
+      sm100::tma_load_2d(sQ, &tq, &q_full, h * DH, (int)(n0 + qt * kRows));
+      // stage of chunk c - kKV is free once PV(c - kKV) completed, which the
+      // commit of QK(c - kKV + kSBuf) (issued after it) implies: no separate
+      // "empty" barrier.  kKV <= 2 kSBuf keeps the parity unambiguous (the
+      // next phase of that s_full needs the chunk loaded here).
+      int s = 0;
       for (int c = 0; c < nch; ++c) {
-        const int s = c % kKV;
-        if (c >= kKV) sm100::mbar_wait_sleep(&kv_empty[s], ((c / kKV) - 1) & 1);
+        if (c >= kKV) {
+          // a parity wait is only unambiguous once the barrier has reached
+          // the phase before: the first time round, QK(0..kSBuf-1) first
+          if (c == kKV)
+            for (int i = 0; i < kSBuf; ++i) sm100::mbar_wait_sleep(&s_full[i], 0u);
+          const int j = c - kKV + kSBuf;  // QK(j) commit => PV(c - kKV) done
+          sm100::mbar_wait_sleep(&s_full[j % kSBuf], (uint32_t)(j / kSBuf) & 1u);
+        }
         unsigned char* st = sKV + s * C::STAGE;
-        sm100::mbar_arrive_expect_tx(&kv_full[s], (uint32_t)C::STAGE);
+        sm100::mbar_arrive_expect_tx(&kv_full[s], (uint32_t)(2 * C::KB));  // K and V (not the ones)
         sm100::tma_load_2d(st, &tm, &kv_full[s], dmodel + h * DH, (int)(n0 + c * kCh));
         sm100::tma_load_2d(st + C::KB, &tm, &kv_full[s], 2 * dmodel + h * DH, (int)(n0 + c * kCh));
+        if (++s == kKV) s = 0;
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {  // -------------------------------------------- MMA issuer
       constexpr uint32_t id_qk = sm100::make_idesc_f16(128, kCh);
-      constexpr uint32_t id_pv = sm100::make_idesc_f16(128, DH) | (1u << 16);  // B (V) MN-major
-      const uint32_t aQ = sm100::smem_u32(sQ), aKV = sm100::smem_u32(sKV);
-      const uint32_t aQm = sm100::smem_u32(sQm), aOne = sm100::smem_u32(sOne);
+      constexpr uint32_t id_pv = sm100::make_idesc_f16(128, DH + 16) | (1u << 16);  // B [V|1] MN-major
+      // descriptors precomputed once; a byte offset o advances the start
+      // address field by o >> 4 (shared addresses < 256 KB: no carry out)
+      const uint32_t aKV = sm100::smem_u32(sKV);
+      const uint64_t dQ = sm100::make_sdesc<C::RB>(sm100::smem_u32(sQ));
+      const uint64_t dK = sm100::make_sdesc<C::RB>(aKV);
+      const uint64_t dV = sm100::make_sdesc_lbo<C::RB>(aKV + C::KB, C::KB);
+      const uint64_t dQm = sm100::make_sdesc<32>(sm100::smem_u32(sQm));
+      const uint64_t dOne = sm100::make_sdesc<32>(sm100::smem_u32(sOne));
+      const uint32_t sfull0 = sm100::smem_u32(&s_full[0]), kvfull0 = sm100::smem_u32(&kv_full[0]);
+      int qs = 0, qb = 0;  // stage / S buffer of the next QK^T
+      uint32_t qph = 0;    // kv_full parity of stage qs (flips per ring pass)
       auto qk = [&](int c) {
-        const int s = c % kKV, b = c % kSBuf;
-        sm100::mbar_wait_sleep(&kv_full[s], (c / kKV) & 1);
+        bar_wait(kvfull0 + 8 * qs, qph);
+        ATR(3, c);
         sm100::tc_fence_after();
-        const uint32_t tS = tmem + kCh * b;
+        const uint32_t tS = tmem + kCh * qb;
+        const uint64_t off = (uint64_t)((qs * C::STAGE) >> 4);
 #pragma unroll
         for (int ks = 0; ks < DH / 16; ++ks)
-          sm100::mma_f16_ss(tS, sm100::make_sdesc<C::RB>(aQ + 32 * ks),
-                            sm100::make_sdesc<C::RB>(aKV + s * C::STAGE + 32 * ks), id_qk, ks > 0 ? 1u : 0u);
-        sm100::mma_f16_ss(tS, sm100::make_sdesc<32>(aQm + b * C::QM), sm100::make_sdesc<32>(aOne), id_qk, 1u);
-        sm100::mma_commit(&s_full[b]);
+          sm100::mma_f16_ss(tS, dQ + 2 * ks, dK + off + 2 * ks, id_qk, ks > 0 ? 1u : 0u);
+        sm100::mma_f16_ss(tS, dQm, dOne, id_qk, 1u);
+        ATR(4, c);
+        sm100::mma_commit_addr(sfull0 + 8 * qb);
+        ATR(5, c);
+        if (++qs == kKV) {
+          qs = 0;
+          qph ^= 1u;
+        }
+        if (++qb == kSBuf) qb = 0;
       };
       sm100::mbar_wait_sleep(&q_full, 0);
       sm100::mbar_wait_sleep(&init_done, 0);
       sm100::tc_fence_after();
       for (int c = 0; c < nch && c < kSBuf; ++c) qk(c);
+      int s = 0, b = 0;
+      uint32_t pph = 0;
       for (int c = 0; c < nch; ++c) {
-        const int s = c % kKV, b = c % kSBuf;
-        MMA_WAIT(&p_ready[b], (c / kSBuf) & 1);
+        MMA_WAIT(&p_ready[b], pph);
+        ATR(0, c);
         sm100::tc_fence_after();
         const uint32_t tP = tmem + kCh * b;
-        const uint32_t aV = aKV + s * C::STAGE + C::KB;
+        const uint64_t off = (uint64_t)((s * C::STAGE) >> 4);
 #pragma unroll
         for (int kk = 0; kk < kCh / 16; ++kk) {
           const uint32_t acc = (c > 0 || kk > 0) ? 1u : 0u;
-          // 16 keys = two 8-row core groups of the MN-major V tile
-          sm100::mma_f16_ts(tmem + C::TO, tP + 8 * kk, sm100::make_sdesc<C::RB>(aV + kk * 16 * C::RB), id_pv, acc);
+          // 16 keys = two 8-row core groups of the MN-major V tile; P of keys
+          // 16kk.. at column 8kk (first key half) or 32 + 8(kk-2) (second)
+          const uint32_t tA = tP + (kk < 2 ? 8 * kk : 32 + 8 * (kk - 2));
+          sm100::mma_f16_ts(tmem + C::TO, tA, dV + off + (uint64_t)((kk * 16 * C::RB) >> 4), id_pv, acc);
         }
-        sm100::mma_commit(&kv_empty[s]);
-        sm100::mma_commit(&pv_done[c & 1]);
+        ATR(1, c);
         if (c + kSBuf < nch) qk(c + kSBuf);
+        if (++s == kKV) s = 0;
+        if (++b == kSBuf) {
+          b = 0;
+          pph ^= 1u;
+        }
       }
       sm100::mma_commit(&o_full);
     }
   } else {
     // ---------------------------------------------------------- softmax
-    const int t = threadIdx.x - 64;  // 0..127
-    const int q4 = warp & 3;         // TMEM lane quarter this warp may access
+    const int t = threadIdx.x - 64;        // 0..255
+    const int hf = t >> 7;                 // key half of every chunk
+    const int q4 = warp & 3;               // TMEM lane quarter this warp may access
     const int r = 32 * q4 + lane;
     const int row = qt * kRows + r;
     const bool valid = row < N;
     const bool warp_dead = qt * kRows + 32 * q4 >= N;
     const uint32_t lrow = (uint32_t)(32 * q4) << 16;
     const uint64_t* Mrow = d.M + d.row_off[g] + (int64_t)(valid ? row : 0) * W;
-    // one 64-bit mask word covers two chunks: chunk c uses the keys
-    // 32(c&1)..32(c&1)+31 of word c>>1, i.e. the low (c even) or high (c odd)
-    // byte of each 16-bit field of the stored layout (internal.h mask_pos:
-    // mask_pos(k + 32) = mask_pos(k) + 8)
-    uint64_t wword = valid ? __ldg(Mrow) : 0ull;
     // (1) reference m = the diagonal score q_row . k_row (fp32 from the fp16
     // operands), rounded to fp16: it enters the QK^T MMA as the fp16 Qm entry
-    float m = 0.f;
-    if (valid) {
-      const uint4* qr = reinterpret_cast<const uint4*>(qkv + (n0 + row) * 3 * dmodel + h * DH);
-      const uint4* kr = reinterpret_cast<const uint4*>(qkv + (n0 + row) * 3 * dmodel + dmodel + h * DH);
+    if (hf == 0) {
+      float m = 0.f;
+      if (valid) {
+        const uint4* qr = reinterpret_cast<const uint4*>(qkv + (n0 + row) * 3 * dmodel + h * DH);
+        const uint4* kr = reinterpret_cast<const uint4*>(qkv + (n0 + row) * 3 * dmodel + dmodel + h * DH);
 #pragma unroll
-      for (int j = 0; j < DH / 8; ++j) {
-        const uint4 a = __ldg(qr + j), bq = __ldg(kr + j);
-        const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, bw[4] = {bq.x, bq.y, bq.z, bq.w};
+        for (int j = 0; j < DH / 8; ++j) {
+          const uint4 a = __ldg(qr + j), bq = __ldg(kr + j);
+          const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, bw[4] = {bq.x, bq.y, bq.z, bq.w};
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const float2 x = __half22float2(*reinterpret_cast<const __half2*>(&aw[i]));
-          const float2 y = __half22float2(*reinterpret_cast<const __half2*>(&bw[i]));
-          m = fmaf(x.x, y.x, m);
-          m = fmaf(x.y, y.y, m);
+          for (int i = 0; i < 4; ++i) {
+            const float2 x = __half22float2(*reinterpret_cast<const __half2*>(&aw[i]));
+            const float2 y = __half22float2(*reinterpret_cast<const __half2*>(&bw[i]));
+            m = fmaf(x.x, y.x, m);
+            m = fmaf(x.y, y.y, m);
+          }
         }
       }
-    }
-    m = __half2float(__float2half_rn(m));
-    // Qm_b = [-m 0 ... 0] (SW32 K-major: 16-byte chunk j of row x sits at
-    // x*32 + 16*(j ^ ((x >> 2) & 1))); One = [1 0 ... 0] per key
-    const int qm_off = r * 32 + 16 * ((r >> 2) & 1);
-    {
+      // Qm = [-m 0 ... 0] (SW32 K-major: 16-byte chunk j of row x sits at
+      // x*32 + 16*(j ^ ((x >> 2) & 1)))
       const uint32_t nm = (uint32_t)__half_as_ushort(__float2half_rn(-m));
-#pragma unroll
-      for (int b = 0; b < kSBuf; ++b) {
-        unsigned char* q = sQm + b * C::QM + r * 32;
-        *reinterpret_cast<uint4*>(q + 16 * ((r >> 2) & 1)) = make_uint4(nm, 0u, 0u, 0u);
-        *reinterpret_cast<uint4*>(q + 16 - 16 * ((r >> 2) & 1)) = make_uint4(0u, 0u, 0u, 0u);
-      }
-      if (t < kCh) {
-        const int o0 = 16 * ((t >> 2) & 1);
-        *reinterpret_cast<uint4*>(sOne + t * 32 + o0) = make_uint4(0x3C00u, 0u, 0u, 0u);
-        *reinterpret_cast<uint4*>(sOne + t * 32 + 16 - o0) = make_uint4(0u, 0u, 0u, 0u);
-      }
-      sm100::fence_proxy_async();
-      sm100::named_bar<128>(1);
-      if (t == 0) sm100::mbar_arrive(&init_done);
+      unsigned char* qrow = sQm + r * 32;
+      *reinterpret_cast<uint4*>(qrow + 16 * ((r >> 2) & 1)) = make_uint4(nm, 0u, 0u, 0u);
+      *reinterpret_cast<uint4*>(qrow + 16 - 16 * ((r >> 2) & 1)) = make_uint4(0u, 0u, 0u, 0u);
+    } else if (t - 128 < kCh) {  // One = [1 0 ... 0] per key
+      const int k = t - 128, o0 = 16 * ((k >> 2) & 1);
+      *reinterpret_cast<uint4*>(sOne + k * 32 + o0) = make_uint4(0x3C00u, 0u, 0u, 0u);
+      *reinterpret_cast<uint4*>(sOne + k * 32 + 16 - o0) = make_uint4(0u, 0u, 0u, 0u);
     }
-    // (2) chunks.  S_b = q.k - mu_b, mu_b = the m held in Qm_b when QK^T of
-    // S_b was issued (read back from Qm_b: m is fp16, so exact).  l: two
-    // fp32 partial sums of the unrounded exponentials.
-    float l0 = 0.f, l1 = 0.f;
+    // the ones atom of every K/V stage (constant; the TMA never writes it)
+    for (int i = t; i < kKV * (C::KB / 16); i += 32 * kSoftWarps) {
+      *reinterpret_cast<uint4*>(sKV + (i / (C::KB / 16)) * C::STAGE + 2 * C::KB + (i % (C::KB / 16)) * 16) =
+          make_uint4(0x3C003C00u, 0x3C003C00u, 0x3C003C00u, 0x3C003C00u);
+    }
+    sm100::fence_proxy_async();
+    sm100::named_bar<32 * kSoftWarps>(1);
+    if (t == 0) sm100::mbar_arrive(&init_done);
+    // (2) chunks.  The 64-bit mask word c covers chunk c; this thread's 32
+    // keys are the low (hf = 0) or high (hf = 1) byte of each 16-bit field of
+    // the stored layout (internal.h mask_pos: mask_pos(k + 32) = mask_pos(k) + 8).
+    const uint32_t sfull0 = sm100::smem_u32(&s_full[0]), pready0 = sm100::smem_u32(&p_ready[0]);
+    const uint32_t tS0 = tmem + 32 * hf + lrow;
+    // mask words two chunks ahead (L2 latency)
+    uint64_t wnext = valid ? __ldg(Mrow) : 0ull, wnext2 = (valid && nch > 1) ? __ldg(Mrow + 1) : 0ull;
+    __half2 mx2 = __float2half2_rn(0.f);
     int b = 0;
+    uint32_t ph = 0;  // phase parity of buffer b's barriers
 #pragma unroll 1
     for (int c = 0; c < nch; ++c) {
-      const uint64_t w = ((c & 1) ? (wword >> 8) : wword) & 0x00FF00FF00FF00FFull;
-      if ((c & 1) && 2 * ((c >> 1) + 1) < nch && valid) wword = __ldg(Mrow + (c >> 1) + 1);
-      sm100::mbar_wait(&s_full[b], (c / kSBuf) & 1);
+      const uint64_t w = (wnext >> (8 * hf)) & 0x00FF00FF00FF00FFull;
+      wnext = wnext2;
+      if (c + 2 < nch && valid) wnext2 = __ldg(Mrow + c + 2);
+      bar_wait(sfull0 + 8 * b, ph);
+      if (lane == 0 && warp == 2) ATR(6, c);
       sm100::tc_fence_after();
       if (!warp_dead) {
-        const uint32_t tS = tmem + kCh * b + lrow;
-        __half* qm = reinterpret_cast<__half*>(sQm + b * C::QM + qm_off);
-        uint32_t p[kCh / 2];
+        const uint32_t tS = tS0 + kCh * b;
+        uint32_t p[16];
         if (__any_sync(0xffffffffu, w != 0ull)) {
-          float s[kCh];
-          sm100::tmem_ld<kCh>(tS, s);
-          const float fix = m + __half2float(*qm);  // m - mu_b
-          if (__any_sync(0xffffffffu, fix != 0.f)) {
-#pragma unroll
-            for (int k = 0; k < kCh; ++k) s[k] -= fix;
-          }
+          float s[32];
+          sm100::tmem_ld<32>(tS, s);
           const uint32_t wl = (uint32_t)w, wh = (uint32_t)(w >> 32);
 #pragma unroll
-          for (int k = 0; k < kCh; ++k) s[k] = key_bit(wl, wh, k) ? s[k] : -INFINITY;
-          __half2 mx2 = __float2half2_rn(0.f);
-          const float lb0 = l0, lb1 = l1;  // sums before this chunk (rare path)
-#pragma unroll
-          for (int i = 0; i < kCh / 2; ++i) {
-            const float e0 = ex2f(s[2 * i]), e1 = ex2f(s[2 * i + 1]);
-            p[i] = sm100::pack_half2(e0, e1);
-            if (i & 1) {
-              l1 += e0 + e1;
-            } else {
-              l0 += e0 + e1;
-            }
-            mx2 = __hmax2(mx2, *reinterpret_cast<const __half2*>(&p[i]));
+          for (int k = 0; k < 32; ++k) {
+            const int pos = mask_pos(k);
+            const bool on = pos < 32 ? ((wl >> pos) & 1u) : ((wh >> (pos - 32)) & 1u);
+            s[k] = on ? s[k] : -INFINITY;
           }
-          const float pm = fmaxf(__low2float(mx2), __high2float(mx2));
-          const bool over = !(pm <= kPMax);
-          if (__any_sync(0xffffffffu, over)) {
-            // rare: move m to the chunk maximum and rescale O (TMEM) and l
-            // once PV of chunk c-1 (the last writer of O) has completed.
-            // s_full(c) implies PV(c-3) completed, so the pv_done parity is
-            // unambiguous.
-            float mx = -INFINITY;
 #pragma unroll
-            for (int k = 0; k < kCh; ++k) mx = fmaxf(mx, s[k]);
-            const float mn = over ? __half2float(__float2half_rn(m + mx)) : m;
-            const float dl = mn - m;
-            m = mn;
-#pragma unroll
-            for (int k = 0; k < kCh; ++k) s[k] -= dl;
-            const float al = ex2f(-dl);
-            l0 = lb0 * al;
-            l1 = lb1 * al;
-            if (c > 0) {
-              sm100::mbar_wait(&pv_done[(c - 1) & 1], ((c - 1) >> 1) & 1);
-              sm100::tc_fence_after();
-#pragma unroll 1
-              for (int j = 0; j < DH / 16; ++j) {
-                float o[16];
-                sm100::tmem_ld<16>(tmem + C::TO + lrow + 16 * j, o);
-                uint32_t ob[16];
-#pragma unroll
-                for (int i = 0; i < 16; ++i) ob[i] = __float_as_uint(o[i] * al);
-                sm100::tmem_st16(tmem + C::TO + lrow + 16 * j, ob);
-              }
-            }
-#pragma unroll
-            for (int i = 0; i < kCh / 2; ++i) {
-              const float e0 = ex2f(s[2 * i]), e1 = ex2f(s[2 * i + 1]);
-              p[i] = sm100::pack_half2(e0, e1);
-              if (i & 1) {
-                l1 += e0 + e1;
-              } else {
-                l0 += e0 + e1;
-              }
-            }
-            if (m != -__half2float(*qm)) {  // Qm_b for the QK^T of chunk c+3
-              *qm = __float2half_rn(-m);
-            }
-            sm100::fence_proxy_async();
+          for (int i = 0; i < 16; ++i) {
+            p[i] = sm100::pack_half2(ex2f(s[2 * i]), ex2f(s[2 * i + 1]));
+            mx2 = __hmax2_nan(mx2, *reinterpret_cast<const __half2*>(&p[i]));
           }
         } else {
 #pragma unroll
-          for (int i = 0; i < kCh / 2; ++i) p[i] = 0u;
-        }
-        if (m != -__half2float(*qm)) {  // m moved in an earlier chunk: Qm_b catches up
-          *qm = __float2half_rn(-m);
-          sm100::fence_proxy_async();
+          for (int i = 0; i < 16; ++i) p[i] = 0u;
         }
         sm100::tmem_st16(tS, p);
         sm100::tmem_wait_st();
         sm100::tc_fence_before();
       }
       __syncwarp();
-      if (lane == 0) sm100::mbar_arrive(&p_ready[b]);
-      b = b == kSBuf - 1 ? 0 : b + 1;
+      if (lane == 0) bar_arrive(pready0 + 8 * b);
+      if (lane == 0 && warp == 2) ATR(7, c);
+      if (++b == kSBuf) {
+        b = 0;
+        ph ^= 1u;
+      }
     }
-    // (3) O / l -> fp16
+    {
+      const float pm = fmaxf(__low2float(mx2), __high2float(mx2));
+      if (!(pm <= kPMax) && valid) row_exact[r] = 1;  // also NaN
+    }
+    // (3) O / l -> fp16: this thread writes output columns [DH/2 hf, DH/2 (hf+1))
     sm100::mbar_wait(&o_full, 0);
     sm100::tc_fence_after();
     float o[DH];
     sm100::tmem_ld<DH>(tmem + C::TO + lrow, o);
+    float lv[16];
+    sm100::tmem_ld<16>(tmem + C::TL + lrow, lv);
+    sm100::named_bar<32 * kSoftWarps>(1);  // row_exact of both key halves visible
     if (valid) {
-      const float l = l0 + l1;
-      const float inv = l > 0.f ? 1.f / l : 0.f;
-      uint32_t pk[DH / 2];
+      __half* orow = out + (n0 + row) * dmodel + h * DH;
+      if (row_exact[r]) {
+        if (hf == 0) exact_row<DH>(qkv, n0, N, row, h, dmodel, Mrow, orow);
+      } else {
+        const float inv = lv[0] > 0.f ? 1.f / lv[0] : 0.f;
+        uint32_t pk[DH / 4];
 #pragma unroll
-      for (int i = 0; i < DH / 2; ++i) pk[i] = sm100::pack_half2(o[2 * i] * inv, o[2 * i + 1] * inv);
-      uint4* dst = reinterpret_cast<uint4*>(out + (n0 + row) * dmodel + h * DH);
+        for (int i = 0; i < DH / 4; ++i) {
+          const float a0 = hf ? o[DH / 2 + 2 * i] : o[2 * i];
+          const float a1 = hf ? o[DH / 2 + 2 * i + 1] : o[2 * i + 1];
+          pk[i] = sm100::pack_half2(a0 * inv, a1 * inv);
+        }
+        uint4* dst = reinterpret_cast<uint4*>(orow + (DH / 2) * hf);
 #pragma unroll
-      for (int j = 0; j < DH / 8; ++j) dst[j] = make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+        for (int j = 0; j < DH / 16; ++j) dst[j] = make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+      }
     }
   }
   sm100::tc_fence_before();
   __syncthreads();
-  if (warp == 1) sm100::tmem_dealloc<128>(tmem);
+  if (warp == 1) sm100::tmem_dealloc<256>(tmem);
 }
 
 template <int DH>
@@ -410,3 +474,9 @@ predtop_status attention_tc_launch(const predtop_dag_s* dag, int d, int H, const
 }
 
 }  // namespace predtop
+
+#ifdef PREDTOP_TRACE
+extern "C" PREDTOP_API int predtop_debug_attn_trace(unsigned long long* out) {
+  return cudaMemcpyFromSymbol(out, predtop::g_at, sizeof(predtop::g_at)) == cudaSuccess ? 0 : -7;
+}
+#endif

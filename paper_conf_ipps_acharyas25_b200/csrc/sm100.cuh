@@ -136,6 +136,10 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
           smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void mma_commit_addr(uint32_t bar_smem) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar_smem)
+               : "memory");
+}
 // 32 lanes x 32 bit, 16 consecutive columns per thread (thread i <-> lane base+i).
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
   uint32_t r[16];
@@ -247,6 +251,14 @@ __device__ __forceinline__ uint64_t make_sdesc(uint32_t smem_addr) {
   d |= (uint64_t)1 << 46;
   d |= layout << 61;
   return d;
+}
+
+// Same with an explicit leading byte offset: for an MN-major operand LBO is
+// the stride between consecutive swizzle atoms along MN (CuTe canonical
+// layout ((T, n), (8, k)) : ((1, LBO), (T, SBO)) in 16-byte units).
+template <int SW>
+__device__ __forceinline__ uint64_t make_sdesc_lbo(uint32_t smem_addr, uint32_t lbo_bytes) {
+  return (make_sdesc<SW>(smem_addr) & ~(0x3FFFull << 16)) | ((uint64_t)((lbo_bytes >> 4) & 0x3FFF) << 16);
 }
 
 // Instruction descriptor, kind::f16: D fp32, A/B fp16, both K-major.

@@ -324,3 +324,47 @@ def test_sweep_chunk_4096(pt, oracle_mod, parity_log):
     Tw = oracle_mod.plan_T(pp, np.arange(sh.num_stages), mb, lat)
     assert T.cpu().numpy().tobytes() == Tw.tobytes()
     assert int(best.item()) == oracle_mod.argmin(Tw)
+
+
+@pytest.mark.parametrize("name, tc", [("moe", "1"), ("gpt", "1")])
+def test_attention_exact_row_fallback(pt, oracle_mod, parity_log, name, tc, monkeypatch):
+    """tcgen05 attention (attention_tc.cu) with a peaked layer-0 attention:
+    W_q and b_q of layer 0 scaled by 8 (exact in fp16), so on some rows an
+    allowed score exceeds the diagonal (the kernel's fixed reference m) by
+    more than 12 in log2 units and the row takes the exact CUDA-core path.
+    Precondition checked on the oracle's own q, k; result within 2e-3."""
+    monkeypatch.setenv("PREDTOP_ATTN_TC", tc)
+    cfg = dict(synth.MODEL_CONFIGS[name])
+    w = synth.model_weights(cfg)
+    d, H = cfg["d_model"], cfg["num_heads"]
+    dh = d // H
+    w["L0.W_qkv"] = w["L0.W_qkv"].copy()
+    w["L0.b_qkv"] = w["L0.b_qkv"].copy()
+    w["L0.W_qkv"][:d] *= 8.0
+    w["L0.b_qkv"][:d] *= 8.0
+    blob = synth.pack_weights(cfg, w)
+    model = pt.Model(cfg, blob)
+    batch = synth.stage_batch(name, 2, first_graph=3)
+    # precondition on graph 0, layer 0 (oracle fp64 q/k, log2 units)
+    import ctypes
+    n, s_, d_, f_ = batch.graph(0)
+    x0 = oracle_mod.embed(cfg, blob, n, f_, oracle_mod.depth(n, s_, d_))
+    qkv = np.zeros((n, 3 * d))
+    oracle_mod.lib().orc_qkv_rows(ctypes.byref(oracle_mod.cfg(cfg)), oracle_mod._p(np.ascontiguousarray(blob, np.float32)),
+                                  0, 0, n, oracle_mod._p(np.ascontiguousarray(x0)), oracle_mod._p(qkv))
+    A = oracle_mod.bits_to_dense(oracle_mod.mask(n, oracle_mod.reach(n, s_, d_)), n).astype(bool)
+    gap = 0.0
+    for h in range(H):
+        q = qkv[:, h * dh:(h + 1) * dh]
+        k = qkv[:, d + h * dh:d + (h + 1) * dh]
+        S = (q @ k.T) / np.sqrt(dh) / np.log(2.0)
+        S = np.where(A, S, -np.inf)
+        gap = max(gap, float((S.max(1) - np.diag(S)).max()))
+    assert gap > 13.0, gap
+    y, _ = _gpu_latency(pt, model, batch)
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch)
+    st = rel_err_stats(y, want, cond)
+    parity_log(f"attention_exact_row_fallback[{name}]", gap_log2=gap, **st)
+    print(f"{name} peaked attention (max gap {gap:.1f}): {st}")
+    assert np.isfinite(y).all()
+    assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
