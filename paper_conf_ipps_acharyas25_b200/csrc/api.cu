@@ -451,14 +451,13 @@ size_t predtop_stage_forward_workspace(predtop_model model, predtop_dag dag) {
   return carve_fwd(model, dag, nullptr, nullptr);
 }
 
-// The fused layer tail (layer.cu) covers d in {64, 128}; PREDTOP_UNFUSED=1 forces
-// the three-GEMM path (tests compare the two).
+// The fused layer tail covers d in {64, 128} (layer.cu / layer2.cu) and
+// d = 256 (layer256.cu); PREDTOP_UNFUSED=1 forces the three-GEMM path (tests
+// compare the two).
 static bool use_fused_tail(int d, int dff) {
-  static const bool unfused = [] {
-    const char* e = getenv("PREDTOP_UNFUSED");
-    return e && e[0] == '1';
-  }();
-  return !unfused && layer_tail_supported(d, dff);
+  const char* e = getenv("PREDTOP_UNFUSED");
+  const bool unfused = e && e[0] == '1';
+  return !unfused && (layer_tail_supported(d, dff) || layer_tail256_supported(d, dff));
 }
 
 // d = 128: the two-CTA-per-SM tail (layer2.cu); PREDTOP_TAIL_V1=1 selects the
@@ -512,8 +511,9 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     if ((s = attention_launch(dag, d, H, w.qkv, w.att, st)) != PREDTOP_OK) return s;
     if (use_fused_tail(d, f)) {
       ProfScope _p(PK_LAYER_TAIL, st);
-      s = use_tail_v2(d, f) ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
-                            : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
+      s = layer_tail256_supported(d, f) ? layer_tail256_launch(m, l, w.att, w.x32, w.x16, M, st)
+          : use_tail_v2(d, f)           ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
+                                        : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
       if (s != PREDTOP_OK) return s;
       continue;
     }

@@ -205,4 +205,9 @@ predtop_status layer_tail2_launch(const predtop_model_s* m, int l, const __half*
 predtop_status layer_tail_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
                                  __half* x16, int M, cudaStream_t st);
 
+// ---- layer256.cu (fused O-proj + LN1 + FFN + LN2 at d = 256)
+bool layer_tail256_supported(int d, int dff);
+predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __half* att, float* x32,
+                                    __half* x16, int M, cudaStream_t st);
+
 }  // namespace predtop

@@ -1,0 +1,438 @@
+// layer256.cu -- K7 at d = 256 (the MoE config): the post-attention half of
+// the DAG-Transformer layer (Fig. 4; reading R6, post-LN encoder
+// layer of [34]),
+//     h  = LN1(x + att W_o^T + b_o)
+//     x' = LN2(h + ReLU(h W_1^T + b_1) W_2^T + b_2),
+// as ONE persistent tcgen05 kernel per layer, so the d_ff-wide hidden
+// activation never leaves the SM (the three-GEMM path wrote and re-read it
+// through HBM: 2 x 1.6 GB per layer on the MoE batch).
+//
+// One CTA per SM (all 512 TMEM columns), one 128-row tile at a time:
+//   TMEM  acc [0, 256): the O-projection; after LN1 the epilogue writes
+//         h + b_2 back into it (tcgen05.st) so FFN-2 accumulates onto the
+//         residual: acc = h + b_2 + FFN(h), the LN2 input.
+//         acc_f[b] = [256 + 128 b, +128): FFN-1 chunk j (128 hidden units) in
+//         buffer j & 1, turned in place into the fp16 ReLU output P_j that
+//         FFN-2 reads as its A operand from tensor memory (TS-MMA).
+//   SMEM  AH (64 KB, four SW128 K-slices): the att tile (O-projection A
+//         operand), then h (FFN-1 A operand); a 4-unit ring of 32 KB units
+//         (W_o K-slices, the fp32 residual tile, W_1 / W_2 chunk halves, in
+//         consumption order); biases and LN parameters.
+//   warp 0 TMA producer, warp 1 MMA issuer, warps 2..17 epilogue: lane quarter
+//   q = warp % 4 -> rows 32q.., column group cg = (warp - 2) / 4 -> the 64
+//   columns [64 cg, +64) of acc and the 32 hidden units [32 cg, +32) of an
+//   FFN chunk.
+// MMA per tile: O-proj 16 x (N=256, K=16), FFN-1 8 chunks x 16 x (N=128),
+// FFN-2 8 x 8 x (N=256, A in TMEM) = 2.3 x 10^8 MACs... 151 MFLOP per tile.
+#include <algorithm>
+
+#include "internal.h"
+#include "sm100.cuh"
+
+namespace predtop {
+
+namespace {
+
+constexpr int D = 256;
+constexpr int FC = 128;               // FFN chunk (hidden units), two TMEM buffers
+constexpr int RS = 4;                 // ring units
+constexpr int UNIT = 32 * 1024;       // bytes of one ring unit
+constexpr int KSL = 128 * 128;        // one [128 rows x 64 fp16] SW128 K-slice (16 KB)
+constexpr int AHB = 4 * KSL;          // att / h tile
+constexpr int kEpiWarps = 16;
+constexpr int kEpi = 32 * kEpiWarps;
+constexpr int kThreads = 64 + kEpi;
+constexpr int kMaxFF = 2048;
+constexpr int PARAMS = (6 * D + kMaxFF) * 4;
+constexpr int SMEM = 1024 + RS * UNIT + AHB + PARAMS;
+static_assert(SMEM <= 227 * 1024, "one CTA per SM");
+
+struct T256Maps {
+  CUtensorMap att, x32in, wo, w1, w2;
+};
+
+struct T256Args {
+  int M, dff;
+  const float *bo, *g1, *be1, *b1, *b2, *g2, *be2;
+  float eps;
+  float* x32;   // residual stream [M][D] fp32 (read through x32in, then overwritten with x')
+  __half* x16;  // its fp16 shadow [M][D]
+};
+
+__global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_constant__ T256Maps mp, T256Args args) {
+  extern __shared__ unsigned char dsm[];
+  unsigned char* base = sm100::align1024(dsm);
+  unsigned char* ring = base;               // RS x 32 KB
+  unsigned char* sAH = ring + RS * UNIT;    // [4 K-slices][128 rows x 64] fp16, SW128
+  float* sPar = reinterpret_cast<float*>(sAH + AHB);
+  float* p_bo = sPar;
+  float* p_g1 = sPar + D;
+  float* p_be1 = sPar + 2 * D;
+  float* p_b2 = sPar + 3 * D;
+  float* p_g2 = sPar + 4 * D;
+  float* p_be2 = sPar + 5 * D;
+  float* p_b1 = sPar + 6 * D;
+  for (int i = threadIdx.x; i < D; i += blockDim.x) {
+    p_bo[i] = args.bo[i];
+    p_g1[i] = args.g1[i];
+    p_be1[i] = args.be1[i];
+    p_b2[i] = args.b2[i];
+    p_g2[i] = args.g2[i];
+    p_be2[i] = args.be2[i];
+  }
+  for (int i = threadIdx.x; i < args.dff; i += blockDim.x) p_b1[i] = args.b1[i];
+  __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
+  __shared__ __align__(8) uint64_t att_full, ah_free, o_full, o_empty, h_ready, out_full;
+  __shared__ __align__(8) uint64_t f_full[2], p_ready[2];  // per acc_f buffer
+  __shared__ uint32_t tmem_slot;
+  __shared__ float red[2][4][128];
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ntiles = (int)ceil_div(args.M, 128);
+  const int NJ = args.dff / FC;
+  // ring units per tile: W_o 4, x 4, W_1 2 per chunk, W_2 2 per chunk
+  const int UPT = 8 + 4 * NJ;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < RS; ++s) {
+      sm100::mbar_init(&ring_full[s], 1);
+      sm100::mbar_init(&ring_empty[s], 1);
+    }
+    uint64_t* singles[] = {&att_full, &ah_free, &o_full, &o_empty, &h_ready, &out_full, &f_full[0], &f_full[1]};
+    for (uint64_t* b : singles) sm100::mbar_init(b, 1);
+    sm100::mbar_init(&p_ready[0], kEpiWarps);  // one arrival per epilogue warp
+    sm100::mbar_init(&p_ready[1], kEpiWarps);
+    sm100::fence_mbar_init();
+  }
+  if (warp == 1) sm100::tmem_alloc<512>(&tmem_slot);
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::tc_fence_after();
+  const uint32_t tmem = tmem_slot;
+  const uint32_t acc = tmem, acc_f = tmem + D;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ------------------------------------------ TMA producer
+      sm100::tma_prefetch(&mp.att);
+      sm100::tma_prefetch(&mp.x32in);
+      sm100::tma_prefetch(&mp.wo);
+      sm100::tma_prefetch(&mp.w1);
+      sm100::tma_prefetch(&mp.w2);
+      int it = 0;
+      auto unit = [&]() -> unsigned char* {  // claim the next ring unit (expects UNIT bytes)
+        const int s = it % RS;
+        sm100::mbar_wait(&ring_empty[s], ((it / RS) & 1) ^ 1);
+        sm100::mbar_arrive_expect_tx(&ring_full[s], UNIT);
+        return ring + s * UNIT;
+      };
+      int i = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        const int m0 = t * 128;
+        // att tile into AH once FFN-1 of the previous tile has read h
+        if (i > 0) sm100::mbar_wait(&ah_free, (i - 1) & 1);
+        sm100::mbar_arrive_expect_tx(&att_full, AHB);
+        for (int kc = 0; kc < 4; ++kc) sm100::tma_load_2d(sAH + kc * KSL, &mp.att, &att_full, 64 * kc, m0);
+        // W_o K-slices [256 out x 64 in]
+        for (int kc = 0; kc < 4; ++kc) {
+          unsigned char* u = unit();
+          sm100::tma_load_2d(u, &mp.wo, &ring_full[it % RS], 64 * kc, 0);
+          ++it;
+        }
+        // the residual x: unit cg = columns [64cg, +64) as two [128 x 32] fp32 boxes
+        for (int cg = 0; cg < 4; ++cg) {
+          unsigned char* u = unit();
+          sm100::tma_load_2d(u, &mp.x32in, &ring_full[it % RS], 64 * cg, m0);
+          sm100::tma_load_2d(u + KSL, &mp.x32in, &ring_full[it % RS], 64 * cg + 32, m0);
+          ++it;
+        }
+        // FFN weights in MMA order: F1_0 F1_1 F2_0 F1_2 F2_1 ... F2_{NJ-1}.
+        // W_1 chunk j half a: rows [128j, +128) x K-slices {2a, 2a+1};
+        // W_2 chunk j half a: rows [0, 256) x K-slice (2j + a) of the hidden dim
+        auto load_w1 = [&](int j) {
+          for (int a = 0; a < 2; ++a) {
+            unsigned char* u = unit();
+            for (int sub = 0; sub < 2; ++sub)
+              sm100::tma_load_2d(u + sub * KSL, &mp.w1, &ring_full[it % RS], 64 * (2 * a + sub), FC * j);
+            ++it;
+          }
+        };
+        auto load_w2 = [&](int j) {
+          for (int a = 0; a < 2; ++a) {
+            unsigned char* u = unit();
+            sm100::tma_load_2d(u, &mp.w2, &ring_full[it % RS], FC * j + 64 * a, 0);
+            ++it;
+          }
+        };
+        load_w1(0);
+        for (int j = 0; j < NJ; ++j) {
+          if (j + 1 < NJ) load_w1(j + 1);
+          load_w2(j);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ------------------------------------------ MMA issuer
+      constexpr uint32_t id_N256 = sm100::make_idesc_f16(128, 256);
+      constexpr uint32_t id_N128 = sm100::make_idesc_f16(128, FC);
+      const uint32_t aAH = sm100::smem_u32(sAH), aRing = sm100::smem_u32(ring);
+      int it = 0, i = 0;
+      auto unit_wait = [&]() -> uint32_t {
+        const int s = it % RS;
+        sm100::mbar_wait(&ring_full[s], (it / RS) & 1);
+        sm100::tc_fence_after();
+        return aRing + s * UNIT;
+      };
+      auto unit_free = [&]() {
+        sm100::mma_commit(&ring_empty[it % RS]);
+        ++it;
+      };
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        // ---- O-projection: acc = att W_o^T (acc free once LN2 of the previous tile read it)
+        sm100::mbar_wait(&o_empty, (i & 1) ^ 1);
+        sm100::mbar_wait(&att_full, i & 1);
+        sm100::tc_fence_after();
+        for (int kc = 0; kc < 4; ++kc) {
+          const uint32_t b0 = unit_wait();
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            sm100::mma_f16_ss(acc, sm100::make_sdesc<128>(aAH + kc * KSL + kk * 32),
+                              sm100::make_sdesc<128>(b0 + kk * 32), id_N256, (kc | kk) != 0);
+          unit_free();
+        }
+        sm100::mma_commit(&o_full);
+        // the 4 x units belong to the epilogue (it frees them after LN1).
+        // Skipping them here is safe: the next unit_wait (FFN-1, after
+        // h_ready) is on a phase whose predecessor the epilogue consumed
+        it += 4;
+        // ---- FFN: acc holds h + b_2, AH holds h (written by the epilogue after LN1)
+        sm100::mbar_wait(&h_ready, i & 1);
+        sm100::tc_fence_after();
+        auto ffn1 = [&](int j) {
+          const uint32_t dst = acc_f + (uint32_t)((j & 1) * FC);
+          for (int a = 0; a < 2; ++a) {
+            const uint32_t b0 = unit_wait();
+#pragma unroll
+            for (int sub = 0; sub < 2; ++sub)
+#pragma unroll
+              for (int kk = 0; kk < 4; ++kk)
+                sm100::mma_f16_ss(dst, sm100::make_sdesc<128>(aAH + (2 * a + sub) * KSL + kk * 32),
+                                  sm100::make_sdesc<128>(b0 + sub * KSL + kk * 32), id_N128, (a | sub | kk) != 0);
+            unit_free();
+          }
+          sm100::mma_commit(&f_full[j & 1]);
+          if (j == NJ - 1) sm100::mma_commit(&ah_free);  // every FFN-1 MMA (the last readers of h) issued
+        };
+        ffn1(0);
+        for (int j = 0; j < NJ; ++j) {
+          if (j + 1 < NJ) ffn1(j + 1);  // keeps the tensor pipe busy during ReLU_j
+          // FFN-2 chunk j: acc += P_j W_2[:, chunk]^T, P_j from TMEM.  Epilogue
+          // group cg leaves hidden units [32cg, +32) as 16 packed fp16 columns
+          // at 32cg of the buffer: K-step ks sits at 32(ks/2) + 8(ks%2).
+          sm100::mbar_wait(&p_ready[j & 1], ((i * NJ + j) >> 1) & 1);
+          sm100::tc_fence_after();
+          const uint32_t src = acc_f + (uint32_t)((j & 1) * FC);
+          for (int a = 0; a < 2; ++a) {
+            const uint32_t b0 = unit_wait();
+#pragma unroll
+            for (int kk = 0; kk < 4; ++kk) {
+              const int ks = 4 * a + kk;
+              sm100::mma_f16_ts(acc, src + (uint32_t)(32 * (ks / 2) + 8 * (ks % 2)),
+                                sm100::make_sdesc<128>(b0 + kk * 32), id_N256, 1u);
+            }
+            unit_free();
+          }
+        }
+        sm100::mma_commit(&out_full);
+      }
+    }
+  } else {
+    // ------------------------------------------ epilogue warps 2..17
+    const int ew = warp - 2;
+    const int q = warp & 3, cg = ew >> 2;
+    const int r = q * 32 + lane;  // tile row of this thread (TMEM lane)
+    const uint32_t lrow = (uint32_t)(q * 32) << 16;
+    const bool leader = (ew == 0 && lane == 0);
+    int i = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const int m0 = t * 128;
+      const int cbase = i * NJ;
+      // ---- LN1: z = x + acc + b_o, two passes over 16-column pieces (the
+      // residual x stays in its ring unit, acc in TMEM: no 64-value register
+      // array, which would not fit the 96 registers of an 18-warp CTA).
+      // o_full first: the O-projection consumed this tile's W_o units, i.e.
+      // the previous phase of each x unit completed, so the parity wait is
+      // never two phases ahead (it would alias and return at once)
+      sm100::mbar_wait(&o_full, i & 1);
+      const int xit = i * UPT + 4;
+      const int itk = xit + cg;
+      sm100::mbar_wait(&ring_full[itk % RS], (itk / RS) & 1);
+      sm100::tc_fence_after();
+      const unsigned char* xu = ring + (itk % RS) * UNIT;  // columns [64cg, +64): two [128 x 32] fp32 boxes
+      auto z_piece = [&](int k, float (&z)[16]) {           // columns 64cg + 16k ..
+        sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
+        const unsigned char* bx = xu + (k >> 1) * KSL;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          const float4 v = *reinterpret_cast<const float4*>(bx + sm100::swz<128>(r, 4 * (k & 1) + c));
+          const float* bo = p_bo + 64 * cg + 16 * k + 4 * c;
+          z[4 * c] += v.x + bo[0];
+          z[4 * c + 1] += v.y + bo[1];
+          z[4 * c + 2] += v.z + bo[2];
+          z[4 * c + 3] += v.w + bo[3];
+        }
+      };
+      float mean, rstd;
+      {
+        float s = 0.f, sq = 0.f;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          float z[16];
+          z_piece(k, z);
+#pragma unroll
+          for (int e = 0; e < 16; ++e) {
+            s += z[e];
+            sq = fmaf(z[e], z[e], sq);
+          }
+        }
+        red[0][cg][r] = s;
+        red[1][cg][r] = sq;
+        sm100::named_bar<kEpi>(1);
+        mean = ((red[0][0][r] + red[0][1][r]) + (red[0][2][r] + red[0][3][r])) * (1.0f / D);
+        const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
+        rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
+      }
+      // h (fp16) -> AH K-slice cg (the O-projection, which read att there,
+      // completed before o_full); h + b_2 -> acc (FFN-2 accumulates onto it)
+      unsigned char* hs = sAH + cg * KSL;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        float z[16];
+        z_piece(k, z);
+        uint32_t hb[16], hp[8];
+#pragma unroll
+        for (int e = 0; e < 16; ++e) {
+          const int col = 64 * cg + 16 * k + e;
+          z[e] = (z[e] - mean) * rstd * p_g1[col] + p_be1[col];
+          hb[e] = __float_as_uint(z[e] + p_b2[col]);
+        }
+#pragma unroll
+        for (int e = 0; e < 8; ++e) hp[e] = sm100::pack_half2(z[2 * e], z[2 * e + 1]);
+        *reinterpret_cast<uint4*>(hs + sm100::swz<128>(r, 2 * k)) = make_uint4(hp[0], hp[1], hp[2], hp[3]);
+        *reinterpret_cast<uint4*>(hs + sm100::swz<128>(r, 2 * k + 1)) = make_uint4(hp[4], hp[5], hp[6], hp[7]);
+        sm100::tmem_st16(acc + lrow + 64 * cg + 16 * k, hb);
+      }
+      sm100::tmem_wait_st();
+      sm100::fence_proxy_async();  // h writes (and the x reads) before the async proxy
+      sm100::tc_fence_before();
+      sm100::named_bar<kEpi>(1);
+      if (leader) {
+        for (int k = 0; k < 4; ++k) sm100::mbar_arrive(&ring_empty[(xit + k) % RS]);  // x units free
+        sm100::mbar_arrive(&h_ready);
+      }
+      // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 pairs back into acc_f
+      for (int j = 0; j < NJ; ++j) {
+        const int cj = cbase + j;
+        sm100::mbar_wait(&f_full[j & 1], (cj >> 1) & 1);
+        sm100::tc_fence_after();
+        {
+          const uint32_t buf = acc_f + (uint32_t)((j & 1) * FC);
+          float v[32];
+          sm100::tmem_ld<32>(buf + lrow + 32 * cg, v);
+          const float* b1 = p_b1 + j * FC + 32 * cg;
+          uint32_t pk[16];
+#pragma unroll
+          for (int k = 0; k < 16; ++k)
+            pk[k] = sm100::pack_half2(fmaxf(v[2 * k] + b1[2 * k], 0.f), fmaxf(v[2 * k + 1] + b1[2 * k + 1], 0.f));
+          sm100::tmem_st16(buf + lrow + 32 * cg, pk);
+        }
+        sm100::tmem_wait_st();
+        sm100::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) sm100::mbar_arrive(&p_ready[j & 1]);  // this warp's part of P_j is in TMEM
+      }
+      // ---- LN2: z = acc (= h + b_2 + FFN(h)), two passes over 16-column
+      // pieces of TMEM; x' (fp32) and its fp16 shadow go straight from
+      // registers to global memory (the stores drain during the next tile)
+      sm100::mbar_wait(&out_full, i & 1);
+      sm100::tc_fence_after();
+      {
+        float s = 0.f, sq = 0.f;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          float z[16];
+          sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
+#pragma unroll
+          for (int e = 0; e < 16; ++e) {
+            s += z[e];
+            sq = fmaf(z[e], z[e], sq);
+          }
+        }
+        red[0][cg][r] = s;
+        red[1][cg][r] = sq;
+        sm100::named_bar<kEpi>(1);
+        mean = ((red[0][0][r] + red[0][1][r]) + (red[0][2][r] + red[0][3][r])) * (1.0f / D);
+        const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
+        rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
+      }
+      const bool live = m0 + r < args.M;
+      float4* d32 = reinterpret_cast<float4*>(args.x32 + (int64_t)(m0 + r) * D + 64 * cg);
+      uint4* d16 = reinterpret_cast<uint4*>(args.x16 + (int64_t)(m0 + r) * D + 64 * cg);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        float z[16];
+        sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
+#pragma unroll
+        for (int e = 0; e < 16; ++e) {
+          const int col = 64 * cg + 16 * k + e;
+          z[e] = (z[e] - mean) * rstd * p_g2[col] + p_be2[col];
+        }
+        if (live) {
+#pragma unroll
+          for (int c = 0; c < 4; ++c) d32[4 * k + c] = make_float4(z[4 * c], z[4 * c + 1], z[4 * c + 2], z[4 * c + 3]);
+#pragma unroll
+          for (int c = 0; c < 2; ++c)
+            d16[2 * k + c] = make_uint4(sm100::pack_half2(z[8 * c], z[8 * c + 1]), sm100::pack_half2(z[8 * c + 2], z[8 * c + 3]),
+                                        sm100::pack_half2(z[8 * c + 4], z[8 * c + 5]),
+                                        sm100::pack_half2(z[8 * c + 6], z[8 * c + 7]));
+        }
+      }
+      sm100::tc_fence_before();
+      sm100::named_bar<kEpi>(1);  // every epilogue thread has read acc (and red) ...
+      if (leader) sm100::mbar_arrive(&o_empty);  // ... so the next O-projection may overwrite it
+    }
+  }
+  __syncwarp();
+  sm100::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) sm100::tmem_dealloc<512>(tmem);
+}
+
+}  // namespace
+
+bool layer_tail256_supported(int d, int dff) { return d == D && dff % (2 * FC) == 0 && dff <= kMaxFF; }
+
+predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __half* att, float* x32, __half* x16,
+                                    int M, cudaStream_t st) {
+  const int d = m->cfg.d_model, dff = m->cfg.d_ff;
+  if (!layer_tail256_supported(d, dff)) {
+    set_error("layer tail 256 needs d = 256 and d_ff %% 256 == 0, d_ff <= %d", kMaxFF);
+    return PREDTOP_ERR_UNSUPPORTED;
+  }
+  if (M <= 0) return PREDTOP_OK;
+  const LayerDev& L = m->layer[l];
+  T256Maps mp;
+  if (!encode_tma_2d(&mp.att, att, 2, D, M, 64, 128) || !encode_tma_2d(&mp.x32in, x32, 4, D, M, 32, 128) ||
+      !encode_tma_2d(&mp.wo, L.Wo, 2, D, D, 64, 256) || !encode_tma_2d(&mp.w1, L.W1, 2, D, dff, 64, FC) ||
+      !encode_tma_2d(&mp.w2, L.W2, 2, dff, D, 64, 256))
+    return PREDTOP_ERR_CUDA;
+  T256Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
+  PT_SMEM_ATTR(k_layer_tail256, SMEM);
+  const int sms = num_sms();
+  if (!sms) return PREDTOP_ERR_CUDA;
+  const int grid = (int)std::min<int64_t>(ceil_div(M, 128), sms);
+  k_layer_tail256<<<grid, kThreads, SMEM, st>>>(mp, a);
+  PT_LAUNCH_CHECK();
+  return PREDTOP_OK;
+}
+
+}  // namespace predtop

@@ -142,7 +142,7 @@ def test_mean_pool_and_relabelled(pt, oracle_mod):
     ("moe", lambda: synth.stage_batch("moe", 2, first_graph=7)),
 ])
 def test_layer_taps(pt, oracle_mod, parity_log, name, batch_fn):
-    """Node embeddings layer by layer (d = 128 fused tail; d = 256 GEMM path).
+    """Node embeddings layer by layer (d = 128 fused tail layer2.cu; d = 256 fused tail layer256.cu).
     x0 (fp32 embedding) within 1e-4.  Each layer CONDITIONALLY: the oracle
     layer applied to the GPU's own input of that layer, so the check sees one
     layer's rounding, not the accumulated drift.  Budget: the layer output is
@@ -366,5 +366,25 @@ def test_attention_exact_row_fallback(pt, oracle_mod, parity_log, name, tc, monk
     st = rel_err_stats(y, want, cond)
     parity_log(f"attention_exact_row_fallback[{name}]", gap_log2=gap, **st)
     print(f"{name} peaked attention (max gap {gap:.1f}): {st}")
+    assert np.isfinite(y).all()
+    assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
+
+
+@pytest.mark.parametrize("name, batch_fn", [
+    ("moe", lambda: synth.stage_batch("moe", 2, first_graph=40)),
+    ("gpt", lambda: synth.stage_batch("gpt", 6, first_graph=40)),
+])
+def test_latency_parity_unfused_gemm_path(pt, oracle_mod, parity_log, name, batch_fn, monkeypatch):
+    """PREDTOP_UNFUSED=1: the three-GEMM layer path (O-proj + LN GEMM, FFN-1
+    GEMM, FFN-2 + LN GEMM, gemm.cu) instead of the fused layer tail (layer2.cu
+    at d = 128, layer256.cu at d = 256); the fallback for other widths."""
+    monkeypatch.setenv("PREDTOP_UNFUSED", "1")
+    cfg, blob, model = _model(pt, name)
+    batch = batch_fn()
+    y, _ = _gpu_latency(pt, model, batch)
+    want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch)
+    st = rel_err_stats(y, want, cond)
+    parity_log(f"latency_parity_unfused[{name}]", **st)
+    print(f"{name} (unfused GEMM path): {st}")
     assert np.isfinite(y).all()
     assert st["max_rel"] <= TOL and st["max_rel_nobias"] <= TOL
