@@ -14,10 +14,11 @@
 //         acc_f[b] = [256 + 128 b, +128): FFN-1 chunk j (128 hidden units) in
 //         buffer j & 1, turned in place into the fp16 ReLU output P_j that
 //         FFN-2 reads as its A operand from tensor memory (TS-MMA).
-//   SMEM  AH (64 KB, four SW128 K-slices): the att tile (O-projection A
-//         operand), then h (FFN-1 A operand); a 4-unit ring of 32 KB units
-//         (W_o K-slices, the fp32 residual tile, W_1 / W_2 chunk halves, in
-//         consumption order); biases and LN parameters.
+//   SMEM  AH (64 KB, four SW128 K-slices): h (the FFN-1 A operand), and
+//         after FFN-1 the per-warp staging of the x' TMA stores; a 4-unit
+//         ring of 32 KB units (att halves and W_o K-slices, the fp32 residual
+//         tile, W_1 / W_2 chunk halves, in consumption order).  Biases and LN
+//         parameters are read from global memory (L1).
 //   warp 0 TMA producer, warp 1 MMA issuer, warps 2..17 epilogue: lane quarter
 //   q = warp % 4 -> rows 32q.., column group cg = (warp - 2) / 4 -> the 64
 //   columns [64 cg, +64) of acc and the 32 hidden units [32 cg, +32) of an
@@ -42,13 +43,15 @@ constexpr int AHB = 4 * KSL;          // att / h tile
 constexpr int kEpiWarps = 16;
 constexpr int kEpi = 32 * kEpiWarps;
 constexpr int kThreads = 64 + kEpi;
-constexpr int kMaxFF = 2048;
-constexpr int PARAMS = (6 * D + kMaxFF) * 4;
-constexpr int SMEM = 1024 + RS * UNIT + AHB + PARAMS;
+constexpr int kMaxFF = 4096;
+constexpr int STG32 = 32 * 16 * 4;    // per-warp x' staging in AH: [32 rows x 16 fp32] (SW64)
+constexpr int STG16 = 32 * 16 * 2;    //                           [32 rows x 16 fp16] (SW32)
+static_assert(kEpiWarps * (STG32 + STG16) <= AHB, "x' staging lives in the h tile");
+constexpr int SMEM = 1024 + RS * UNIT + AHB;
 static_assert(SMEM <= 227 * 1024, "one CTA per SM");
 
 struct T256Maps {
-  CUtensorMap att, x32in, wo, w1, w2;
+  CUtensorMap att, x32in, wo, w1, w2, x32out, x16out;
 };
 
 struct T256Args {
@@ -64,25 +67,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
   unsigned char* base = sm100::align1024(dsm);
   unsigned char* ring = base;               // RS x 32 KB
   unsigned char* sAH = ring + RS * UNIT;    // [4 K-slices][128 rows x 64] fp16, SW128
-  float* sPar = reinterpret_cast<float*>(sAH + AHB);
-  float* p_bo = sPar;
-  float* p_g1 = sPar + D;
-  float* p_be1 = sPar + 2 * D;
-  float* p_b2 = sPar + 3 * D;
-  float* p_g2 = sPar + 4 * D;
-  float* p_be2 = sPar + 5 * D;
-  float* p_b1 = sPar + 6 * D;
-  for (int i = threadIdx.x; i < D; i += blockDim.x) {
-    p_bo[i] = args.bo[i];
-    p_g1[i] = args.g1[i];
-    p_be1[i] = args.be1[i];
-    p_b2[i] = args.b2[i];
-    p_g2[i] = args.g2[i];
-    p_be2[i] = args.be2[i];
-  }
-  for (int i = threadIdx.x; i < args.dff; i += blockDim.x) p_b1[i] = args.b1[i];
+  unsigned char* sStg = sAH;                // x' staging (per epilogue warp STG32 + STG16), once h is dead
+  // biases and LN parameters stay in global memory (L1-resident, __ldg)
+  const float* __restrict__ p_bo = args.bo;
+  const float* __restrict__ p_g1 = args.g1;
+  const float* __restrict__ p_be1 = args.be1;
+  const float* __restrict__ p_b2 = args.b2;
+  const float* __restrict__ p_g2 = args.g2;
+  const float* __restrict__ p_be2 = args.be2;
+  const float* __restrict__ p_b1 = args.b1;
   __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
-  __shared__ __align__(8) uint64_t att_full, ah_free, o_full, o_empty, h_ready, out_full;
+  __shared__ __align__(8) uint64_t o_full, o_empty, h_ready, out_full;
   __shared__ __align__(8) uint64_t f_full[2], p_ready[2];  // per acc_f buffer
   __shared__ uint32_t tmem_slot;
   __shared__ float red[2][4][128];
@@ -90,15 +85,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ntiles = (int)ceil_div(args.M, 128);
   const int NJ = args.dff / FC;
-  // ring units per tile: W_o 4, x 4, W_1 2 per chunk, W_2 2 per chunk
-  const int UPT = 8 + 4 * NJ;
+  // ring units per tile: att 2 + W_o 4 (order att_a Wo0 Wo1 att_b Wo2 Wo3),
+  // x 4, W_1 2 per chunk, W_2 2 per chunk
+  const int UPT = 10 + 4 * NJ;
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < RS; ++s) {
       sm100::mbar_init(&ring_full[s], 1);
       sm100::mbar_init(&ring_empty[s], 1);
     }
-    uint64_t* singles[] = {&att_full, &ah_free, &o_full, &o_empty, &h_ready, &out_full, &f_full[0], &f_full[1]};
+    uint64_t* singles[] = {&o_full, &o_empty, &h_ready, &out_full, &f_full[0], &f_full[1]};
     for (uint64_t* b : singles) sm100::mbar_init(b, 1);
     sm100::mbar_init(&p_ready[0], kEpiWarps);  // one arrival per epilogue warp
     sm100::mbar_init(&p_ready[1], kEpiWarps);
@@ -128,15 +124,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       int i = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
         const int m0 = t * 128;
-        // att tile into AH once FFN-1 of the previous tile has read h
-        if (i > 0) sm100::mbar_wait(&ah_free, (i - 1) & 1);
-        sm100::mbar_arrive_expect_tx(&att_full, AHB);
-        for (int kc = 0; kc < 4; ++kc) sm100::tma_load_2d(sAH + kc * KSL, &mp.att, &att_full, 64 * kc, m0);
-        // W_o K-slices [256 out x 64 in]
-        for (int kc = 0; kc < 4; ++kc) {
+        // att half a (K-slices 2a, 2a+1: two [128 x 64] boxes), then the two
+        // W_o K-slices [256 out x 64 in] it multiplies
+        for (int a = 0; a < 2; ++a) {
           unsigned char* u = unit();
-          sm100::tma_load_2d(u, &mp.wo, &ring_full[it % RS], 64 * kc, 0);
+          for (int sub = 0; sub < 2; ++sub)
+            sm100::tma_load_2d(u + sub * KSL, &mp.att, &ring_full[it % RS], 64 * (2 * a + sub), m0);
           ++it;
+          for (int sub = 0; sub < 2; ++sub) {
+            unsigned char* w = unit();
+            sm100::tma_load_2d(w, &mp.wo, &ring_full[it % RS], 64 * (2 * a + sub), 0);
+            ++it;
+          }
         }
         // the residual x: unit cg = columns [64cg, +64) as two [128 x 32] fp32 boxes
         for (int cg = 0; cg < 4; ++cg) {
@@ -189,15 +188,20 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
         // ---- O-projection: acc = att W_o^T (acc free once LN2 of the previous tile read it)
         sm100::mbar_wait(&o_empty, (i & 1) ^ 1);
-        sm100::mbar_wait(&att_full, i & 1);
         sm100::tc_fence_after();
-        for (int kc = 0; kc < 4; ++kc) {
-          const uint32_t b0 = unit_wait();
+        for (int a = 0; a < 2; ++a) {
+          const int ia = it;  // the att unit stays until both W_o units of this half are consumed
+          const uint32_t a0 = unit_wait();
+          ++it;
+          for (int sub = 0; sub < 2; ++sub) {
+            const uint32_t b0 = unit_wait();
 #pragma unroll
-          for (int kk = 0; kk < 4; ++kk)
-            sm100::mma_f16_ss(acc, sm100::make_sdesc<128>(aAH + kc * KSL + kk * 32),
-                              sm100::make_sdesc<128>(b0 + kk * 32), id_N256, (kc | kk) != 0);
-          unit_free();
+            for (int kk = 0; kk < 4; ++kk)
+              sm100::mma_f16_ss(acc, sm100::make_sdesc<128>(a0 + sub * KSL + kk * 32),
+                                sm100::make_sdesc<128>(b0 + kk * 32), id_N256, (a | sub | kk) != 0);
+            unit_free();
+          }
+          sm100::mma_commit(&ring_empty[ia % RS]);
         }
         sm100::mma_commit(&o_full);
         // the 4 x units belong to the epilogue (it frees them after LN1).
@@ -220,7 +224,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
             unit_free();
           }
           sm100::mma_commit(&f_full[j & 1]);
-          if (j == NJ - 1) sm100::mma_commit(&ah_free);  // every FFN-1 MMA (the last readers of h) issued
         };
         ffn1(0);
         for (int j = 0; j < NJ; ++j) {
@@ -263,7 +266,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       // the previous phase of each x unit completed, so the parity wait is
       // never two phases ahead (it would alias and return at once)
       sm100::mbar_wait(&o_full, i & 1);
-      const int xit = i * UPT + 4;
+      const int xit = i * UPT + 6;
       const int itk = xit + cg;
       sm100::mbar_wait(&ring_full[itk % RS], (itk / RS) & 1);
       sm100::tc_fence_after();
@@ -274,11 +277,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
           const float4 v = *reinterpret_cast<const float4*>(bx + sm100::swz<128>(r, 4 * (k & 1) + c));
-          const float* bo = p_bo + 64 * cg + 16 * k + 4 * c;
-          z[4 * c] += v.x + bo[0];
-          z[4 * c + 1] += v.y + bo[1];
-          z[4 * c + 2] += v.z + bo[2];
-          z[4 * c + 3] += v.w + bo[3];
+          const float4 bo = __ldg(reinterpret_cast<const float4*>(p_bo + 64 * cg + 16 * k + 4 * c));
+          z[4 * c] += v.x + bo.x;
+          z[4 * c + 1] += v.y + bo.y;
+          z[4 * c + 2] += v.z + bo.z;
+          z[4 * c + 3] += v.w + bo.w;
         }
       };
       float mean, rstd;
@@ -296,13 +299,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         }
         red[0][cg][r] = s;
         red[1][cg][r] = sq;
+        // h overwrites all of AH below: every warp's x' stores of the
+        // previous tile (staged in AH) must have read it (before the barrier)
+        if (lane == 0) sm100::bulk_wait_read0();
+        __syncwarp();
         sm100::named_bar<kEpi>(1);
         mean = ((red[0][0][r] + red[0][1][r]) + (red[0][2][r] + red[0][3][r])) * (1.0f / D);
         const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
         rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
       }
-      // h (fp16) -> AH K-slice cg (the O-projection, which read att there,
-      // completed before o_full); h + b_2 -> acc (FFN-2 accumulates onto it)
+      // h (fp16) -> AH K-slice cg (FFN-1 of the previous tile, the last
+      // reader of its h, completed before that tile's out_full); h + b_2 ->
+      // acc (FFN-2 accumulates onto it)
       unsigned char* hs = sAH + cg * KSL;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
@@ -310,10 +318,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         z_piece(k, z);
         uint32_t hb[16], hp[8];
 #pragma unroll
-        for (int e = 0; e < 16; ++e) {
-          const int col = 64 * cg + 16 * k + e;
-          z[e] = (z[e] - mean) * rstd * p_g1[col] + p_be1[col];
-          hb[e] = __float_as_uint(z[e] + p_b2[col]);
+        for (int c = 0; c < 4; ++c) {
+          const int col = 64 * cg + 16 * k + 4 * c;
+          const float4 g = __ldg(reinterpret_cast<const float4*>(p_g1 + col));
+          const float4 be = __ldg(reinterpret_cast<const float4*>(p_be1 + col));
+          const float4 b2 = __ldg(reinterpret_cast<const float4*>(p_b2 + col));
+          const float gg[4] = {g.x, g.y, g.z, g.w}, bb[4] = {be.x, be.y, be.z, be.w}, b22[4] = {b2.x, b2.y, b2.z, b2.w};
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            z[4 * c + e] = (z[4 * c + e] - mean) * rstd * gg[e] + bb[e];
+            hb[4 * c + e] = __float_as_uint(z[4 * c + e] + b22[e]);
+          }
         }
 #pragma unroll
         for (int e = 0; e < 8; ++e) hp[e] = sm100::pack_half2(z[2 * e], z[2 * e + 1]);
@@ -338,11 +353,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           const uint32_t buf = acc_f + (uint32_t)((j & 1) * FC);
           float v[32];
           sm100::tmem_ld<32>(buf + lrow + 32 * cg, v);
-          const float* b1 = p_b1 + j * FC + 32 * cg;
+          const float4* b1 = reinterpret_cast<const float4*>(p_b1 + j * FC + 32 * cg);
           uint32_t pk[16];
 #pragma unroll
-          for (int k = 0; k < 16; ++k)
-            pk[k] = sm100::pack_half2(fmaxf(v[2 * k] + b1[2 * k], 0.f), fmaxf(v[2 * k + 1] + b1[2 * k + 1], 0.f));
+          for (int k = 0; k < 8; ++k) {
+            const float4 b = __ldg(b1 + k);
+            pk[2 * k] = sm100::pack_half2(fmaxf(v[4 * k] + b.x, 0.f), fmaxf(v[4 * k + 1] + b.y, 0.f));
+            pk[2 * k + 1] = sm100::pack_half2(fmaxf(v[4 * k + 2] + b.z, 0.f), fmaxf(v[4 * k + 3] + b.w, 0.f));
+          }
           sm100::tmem_st16(buf + lrow + 32 * cg, pk);
         }
         sm100::tmem_wait_st();
@@ -374,26 +392,42 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
         rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
       }
-      const bool live = m0 + r < args.M;
-      float4* d32 = reinterpret_cast<float4*>(args.x32 + (int64_t)(m0 + r) * D + 64 * cg);
-      uint4* d16 = reinterpret_cast<uint4*>(args.x16 + (int64_t)(m0 + r) * D + 64 * cg);
-#pragma unroll
+      // pass B: x' piece k (rows 32q.., columns 64cg + 16k ..) -> this warp's
+      // staging (SW64 fp32 / SW32 fp16, the TMA box layouts) -> TMA stores;
+      // the staging is rewritten once the previous piece's stores have read it
+      unsigned char* s32 = sStg + ew * (STG32 + STG16);
+      unsigned char* s16 = s32 + STG32;
+#pragma unroll 1
       for (int k = 0; k < 4; ++k) {
         float z[16];
         sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
 #pragma unroll
-        for (int e = 0; e < 16; ++e) {
-          const int col = 64 * cg + 16 * k + e;
-          z[e] = (z[e] - mean) * rstd * p_g2[col] + p_be2[col];
+        for (int c = 0; c < 4; ++c) {
+          const int col = 64 * cg + 16 * k + 4 * c;
+          const float4 g = __ldg(reinterpret_cast<const float4*>(p_g2 + col));
+          const float4 be = __ldg(reinterpret_cast<const float4*>(p_be2 + col));
+          z[4 * c] = (z[4 * c] - mean) * rstd * g.x + be.x;
+          z[4 * c + 1] = (z[4 * c + 1] - mean) * rstd * g.y + be.y;
+          z[4 * c + 2] = (z[4 * c + 2] - mean) * rstd * g.z + be.z;
+          z[4 * c + 3] = (z[4 * c + 3] - mean) * rstd * g.w + be.w;
         }
-        if (live) {
+        if (lane == 0) sm100::bulk_wait_read0();
+        __syncwarp();
 #pragma unroll
-          for (int c = 0; c < 4; ++c) d32[4 * k + c] = make_float4(z[4 * c], z[4 * c + 1], z[4 * c + 2], z[4 * c + 3]);
+        for (int c = 0; c < 4; ++c)
+          *reinterpret_cast<float4*>(s32 + lane * 64 + 16 * (c ^ ((lane >> 1) & 3))) =
+              make_float4(z[4 * c], z[4 * c + 1], z[4 * c + 2], z[4 * c + 3]);
 #pragma unroll
-          for (int c = 0; c < 2; ++c)
-            d16[2 * k + c] = make_uint4(sm100::pack_half2(z[8 * c], z[8 * c + 1]), sm100::pack_half2(z[8 * c + 2], z[8 * c + 3]),
-                                        sm100::pack_half2(z[8 * c + 4], z[8 * c + 5]),
-                                        sm100::pack_half2(z[8 * c + 6], z[8 * c + 7]));
+        for (int c = 0; c < 2; ++c)
+          *reinterpret_cast<uint4*>(s16 + lane * 32 + 16 * (c ^ ((lane >> 2) & 1))) =
+              make_uint4(sm100::pack_half2(z[8 * c], z[8 * c + 1]), sm100::pack_half2(z[8 * c + 2], z[8 * c + 3]),
+                         sm100::pack_half2(z[8 * c + 4], z[8 * c + 5]), sm100::pack_half2(z[8 * c + 6], z[8 * c + 7]));
+        sm100::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) {
+          sm100::tma_store_2d(&mp.x32out, s32, 64 * cg + 16 * k, m0 + 32 * q);
+          sm100::tma_store_2d(&mp.x16out, s16, 64 * cg + 16 * k, m0 + 32 * q);
+          sm100::bulk_commit();
         }
       }
       sm100::tc_fence_before();
@@ -401,6 +435,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       if (leader) sm100::mbar_arrive(&o_empty);  // ... so the next O-projection may overwrite it
     }
   }
+  if (warp >= 2 && lane == 0) sm100::bulk_wait0();
   __syncwarp();
   sm100::tc_fence_before();
   __syncthreads();
@@ -423,7 +458,8 @@ predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __hal
   T256Maps mp;
   if (!encode_tma_2d(&mp.att, att, 2, D, M, 64, 128) || !encode_tma_2d(&mp.x32in, x32, 4, D, M, 32, 128) ||
       !encode_tma_2d(&mp.wo, L.Wo, 2, D, D, 64, 256) || !encode_tma_2d(&mp.w1, L.W1, 2, D, dff, 64, FC) ||
-      !encode_tma_2d(&mp.w2, L.W2, 2, dff, D, 64, 256))
+      !encode_tma_2d(&mp.w2, L.W2, 2, dff, D, 64, 256) || !encode_tma_2d(&mp.x32out, x32, 4, D, M, 16, 32) ||
+      !encode_tma_2d(&mp.x16out, x16, 2, D, M, 16, 32))
     return PREDTOP_ERR_CUDA;
   T256Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
   PT_SMEM_ATTR(k_layer_tail256, SMEM);
