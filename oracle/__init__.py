@@ -86,6 +86,8 @@ def lib():
             L.orc_prune.restype = i32
             L.orc_plan_search.argtypes = [i32, i32, P, i32, P, i32, P, P, P]
             L.orc_plan_search.restype = dbl
+            L.orc_grad.argtypes = [P, P, i32, i32, P, P, P, dbl, P, P]
+            L.orc_grad.restype = i32
             _lib = L
     return _lib
 
@@ -278,6 +280,71 @@ def forward_batch_cond(model_cfg, blob, batch, graphs: Optional[Sequence[int]] =
         with ThreadPoolExecutor(threads) as ex:
             out = list(ex.map(one, gs))
     return np.asarray([o[0] for o in out], np.float64), np.asarray([o[1] for o in out], np.float64)
+
+
+# ---- training ------------------------------------
+def grad(model_cfg, blob, n, src, dst, feats, dy: float = 1.0, out: Optional[np.ndarray] = None):
+    """(y, grad): latency of one graph and dy * d y / d theta over the weight
+    blob (orc_grad, fp64; accumulated into `out` when given)."""
+    c = cfg(model_cfg)
+    b = np.ascontiguousarray(blob, np.float32)
+    s, d = _i32(src), _i32(dst)
+    g = np.zeros(len(b), np.float64) if out is None else out
+    y = np.zeros(1, np.float64)
+    st = lib().orc_grad(ctypes.byref(c), _p(b), n, len(s), _p(s), _p(d), _p(_feats(feats)), float(dy), _p(y), _p(g))
+    if st != OK:
+        raise ValueError(f"invalid graph (status {st})")
+    return float(y[0]), g
+
+
+def mae_grad(model_cfg, blob, batch, y_true, threads: Optional[int] = None):
+    """Eqn 3: L = (1/N) sum_i |y_hat_i - y_i| over the graphs of a
+    synth.StageBatch, and dL/dtheta = sum_i sign(y_hat_i - y_i)/N * dy_hat_i/dtheta
+    (sign(0) = 0).  Returns (L, grad, y_hat).  Two passes: the forward latencies
+    (forward_batch) fix the signs, then orc_grad per graph."""
+    y_true = np.asarray(y_true, np.float64)
+    N = batch.num_graphs
+    y_hat = forward_batch(model_cfg, blob, batch, threads=threads)
+    loss = float(np.mean(np.abs(y_hat - y_true)))
+    sgn = np.sign(y_hat - y_true) / N
+    threads = threads or (os.cpu_count() or 1)
+    parts = [np.zeros(len(blob), np.float64) for _ in range(min(threads, N))]
+
+    def one(i):
+        g = i % len(parts)
+        n, s, d, f = batch.graph(i)
+        return g, grad(model_cfg, blob, n, s, d, f, dy=sgn[i])[1]
+
+    total = np.zeros(len(blob), np.float64)
+    with ThreadPoolExecutor(threads) as ex:
+        for _, gi in ex.map(one, range(N)):
+            total += gi
+    return loss, total, y_hat
+
+
+def adam_step(param, grad_, m, v, step: int, lr: float, beta1: float = 0.9, beta2: float = 0.999,
+              eps: float = 1e-8):
+    """One Adam update (PyTorch's Adam with its defaults), written out
+    as torch.optim.Adam computes it (no weight decay, amsgrad off), fp64:
+      m = b1 m + (1-b1) g;  v = b2 v + (1-b2) g^2;
+      p -= lr / (1 - b1^t) * m / (sqrt(v) / sqrt(1 - b2^t) + eps).
+    Returns new (param, m, v)."""
+    g = np.asarray(grad_, np.float64)
+    m = beta1 * np.asarray(m, np.float64) + (1.0 - beta1) * g
+    v = beta2 * np.asarray(v, np.float64) + (1.0 - beta2) * g * g
+    bc1 = 1.0 - beta1 ** step
+    bc2 = 1.0 - beta2 ** step
+    denom = np.sqrt(v) / np.sqrt(bc2) + eps
+    p = np.asarray(param, np.float64) - (lr / bc1) * m / denom
+    return p, m, v
+
+
+def cosine_lr(epoch: int, epochs: int, lr0: float = 1e-3) -> float:
+    """Cosine decay: lr0 in the first epoch down to 0 in the last,
+    lr_e = lr0 * (1 + cos(pi * e / (E - 1))) / 2 for e = 0 .. E-1."""
+    if epochs <= 1:
+        return lr0
+    return lr0 * 0.5 * (1.0 + np.cos(np.pi * epoch / (epochs - 1)))
 
 
 # ---- one large graph, row block by row block --------------------------------

@@ -645,3 +645,273 @@ int orc_prune(int n, int e, const int32_t* src, const int32_t* dst, const orc_fe
   free(removed); free(newid); free(seen); free(target); free(stack); free_csr(&succ);
   return ORC_OK;
 }
+
+/* ======================================================================== */
+/* Training: gradient of the predicted    */
+/* latency of ONE stage graph with respect to every weight of the blob,      */
+/* written as the plain reverse of the forward steps above (same order,      */
+/* same readings), fp64.  The MAE loss of Eqn 3 and Adam / cosine LR */
+/* are composed by the caller (oracle/__init__.py).                  */
+/* ======================================================================== */
+
+/* Gradient blob views: the same float order as the weight blob. */
+typedef struct {
+  double *Wqkv, *bqkv, *Wo, *bo, *g1, *be1, *W1, *b1, *W2, *b2, *g2, *be2;
+} orc_glw;
+typedef struct {
+  double *W_in, *b_in, *H1, *c1, *H2, *c2, *w_o, *c_o;
+} orc_gtop;
+
+static orc_glw grad_layer(const orc_cfg* c, double* g, int l) {
+  long d = c->d, f = c->d_ff;
+  double* p = g + d * ORC_F + d + (long)l * layer_floats(c);
+  orc_glw w;
+  w.Wqkv = p; p += 3 * d * d;
+  w.bqkv = p; p += 3 * d;
+  w.Wo = p; p += d * d;
+  w.bo = p; p += d;
+  w.g1 = p; p += d;
+  w.be1 = p; p += d;
+  w.W1 = p; p += f * d;
+  w.b1 = p; p += f;
+  w.W2 = p; p += d * f;
+  w.b2 = p; p += d;
+  w.g2 = p; p += d;
+  w.be2 = p;
+  return w;
+}
+static orc_gtop grad_top(const orc_cfg* c, double* g) {
+  long d = c->d;
+  orc_gtop t;
+  t.W_in = g;
+  t.b_in = g + d * ORC_F;
+  double* p = g + d * ORC_F + d + (long)c->L * layer_floats(c);
+  t.H1 = p; p += d * d;
+  t.c1 = p; p += d;
+  t.H2 = p; p += d * d;
+  t.c2 = p; p += d;
+  t.w_o = p; p += d;
+  t.c_o = p;
+  return t;
+}
+
+/* Reverse of linear(): y[r][o] = b[o] + sum_i W[o][i] x[r][i].
+ * dW[o][i] += sum_r dy[r][o] x[r][i];  db[o] += sum_r dy[r][o];
+ * dx[r][i] += sum_o dy[r][o] W[o][i]   (dx nullable). */
+static void linear_back(int rows, int in, int out, const double* x, const float* W, const double* dy,
+                        double* dW, double* db, double* dx) {
+  for (int r = 0; r < rows; ++r)
+    for (int o = 0; o < out; ++o) {
+      double g = dy[(size_t)r * out + o];
+      if (db) db[o] += g;
+      for (int i = 0; i < in; ++i) {
+        dW[(size_t)o * in + i] += g * x[(size_t)r * in + i];
+        if (dx) dx[(size_t)r * in + i] += g * (double)W[(size_t)o * in + i];
+      }
+    }
+}
+
+/* Reverse of layer_norm(): y = xhat * g + b, xhat = (z - mean) * inv.
+ * dg += sum_r dy*xhat; db += sum_r dy; with gx = dy*g:
+ * dz = inv * (gx - mean(gx) - xhat * mean(gx * xhat))   (dz overwritten). */
+static void layer_norm_back(int rows, int d, const double* z, const float* g, double eps, const double* dy,
+                            double* dg, double* db, double* dz) {
+  double* xh = (double*)malloc(sizeof(double) * (size_t)d);
+  double* gx = (double*)malloc(sizeof(double) * (size_t)d);
+  for (int r = 0; r < rows; ++r) {
+    const double* zr = z + (size_t)r * d;
+    const double* dyr = dy + (size_t)r * d;
+    double mean = 0.0;
+    for (int i = 0; i < d; ++i) mean += zr[i];
+    mean /= d;
+    double var = 0.0;
+    for (int i = 0; i < d; ++i) var += (zr[i] - mean) * (zr[i] - mean);
+    var /= d;
+    double inv = 1.0 / sqrt(var + eps);
+    double m1 = 0.0, m2 = 0.0;
+    for (int i = 0; i < d; ++i) {
+      xh[i] = (zr[i] - mean) * inv;
+      gx[i] = dyr[i] * (double)g[i];
+      dg[i] += dyr[i] * xh[i];
+      db[i] += dyr[i];
+      m1 += gx[i];
+      m2 += gx[i] * xh[i];
+    }
+    m1 /= d;
+    m2 /= d;
+    for (int i = 0; i < d; ++i) dz[(size_t)r * d + i] = inv * (gx[i] - m1 - xh[i] * m2);
+  }
+  free(xh);
+  free(gx);
+}
+
+/* Reverse of orc_attention_rows over all rows (per head h, Eqn 1):
+ *   S = Q K^T / sqrt(d_h) on allowed pairs, P = softmax_row(S), O = P V.
+ *   dV = P^T dO;  dP = dO V^T;  dS = P * (dP - rowsum(dP * P));
+ *   dQ = dS K / sqrt(d_h);  dK = dS^T Q / sqrt(d_h).
+ * dqkv [n][3d] accumulates. */
+static void attention_back(const orc_cfg* c, int n, const uint64_t* M, const double* qkv, const double* dO,
+                           double* dqkv) {
+  int d = c->d, H = c->H, dh = c->d / c->H;
+  int W = orc_row_words(n);
+  double scale = 1.0 / sqrt((double)dh);
+  double* P = (double*)malloc(sizeof(double) * (size_t)n);
+  double* dP = (double*)malloc(sizeof(double) * (size_t)n);
+  for (int h = 0; h < H; ++h)
+    for (int u = 0; u < n; ++u) {
+      const double* q = qkv + (size_t)u * 3 * d + h * dh;
+      double mx = -INFINITY;
+      for (int v = 0; v < n; ++v) {
+        P[v] = 0.0;
+        if (!bit(M, W, u, v)) continue;
+        const double* k = qkv + (size_t)v * 3 * d + d + h * dh;
+        double acc = 0.0;
+        for (int j = 0; j < dh; ++j) acc += q[j] * k[j];
+        P[v] = acc * scale;
+        if (P[v] > mx) mx = P[v];
+      }
+      double sum = 0.0;
+      for (int v = 0; v < n; ++v)
+        if (bit(M, W, u, v)) { P[v] = exp(P[v] - mx); sum += P[v]; }
+      for (int v = 0; v < n; ++v) P[v] /= sum;
+      const double* dou = dO + (size_t)u * d + h * dh;
+      double rs = 0.0;
+      for (int v = 0; v < n; ++v) {
+        dP[v] = 0.0;
+        if (!bit(M, W, u, v)) continue;
+        const double* vv = qkv + (size_t)v * 3 * d + 2 * d + h * dh;
+        double acc = 0.0;
+        for (int j = 0; j < dh; ++j) acc += dou[j] * vv[j];
+        dP[v] = acc;
+        rs += acc * P[v];
+        double* dvv = dqkv + (size_t)v * 3 * d + 2 * d + h * dh;
+        for (int j = 0; j < dh; ++j) dvv[j] += P[v] * dou[j];
+      }
+      double* dq = dqkv + (size_t)u * 3 * d + h * dh;
+      for (int v = 0; v < n; ++v) {
+        if (!bit(M, W, u, v)) continue;
+        double ds = P[v] * (dP[v] - rs) * scale;
+        const double* k = qkv + (size_t)v * 3 * d + d + h * dh;
+        double* dk = dqkv + (size_t)v * 3 * d + d + h * dh;
+        for (int j = 0; j < dh; ++j) {
+          dq[j] += ds * k[j];
+          dk[j] += ds * q[j];
+        }
+      }
+    }
+  free(P);
+  free(dP);
+}
+
+/* Latency y of one graph (as orc_forward) and grad += dy * dy/dtheta for  */
+/* every weight of the blob (grad: orc_blob_floats doubles, accumulated). */
+int orc_grad(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src, const int32_t* dst,
+             const orc_feat* feats, double dy, double* y, double* grad) {
+  int st = orc_validate(n, e, src, dst);
+  if (st != ORC_OK) { *y = NAN; return st; }
+  int d = c->d, f = c->d_ff, L = c->L, W = orc_row_words(n);
+  size_t nd = (size_t)n * d;
+  int32_t* depth = (int32_t*)malloc(sizeof(int32_t) * (size_t)n);
+  uint64_t* R = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)n * W);
+  uint64_t* Mk = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)n * W);
+  orc_depth(n, e, src, dst, depth);
+  orc_reach(n, e, src, dst, R);
+  orc_mask(n, R, Mk);
+  /* ---- forward with every intermediate kept */
+  double* F = (double*)malloc(sizeof(double) * (size_t)n * ORC_F);
+  orc_features(n, feats, F);
+  double* xs = (double*)malloc(sizeof(double) * nd * (L + 1));     /* layer inputs / outputs */
+  double* qkv = (double*)malloc(sizeof(double) * nd * 3 * L);
+  double* att = (double*)malloc(sizeof(double) * nd * L);
+  double* z1 = (double*)malloc(sizeof(double) * nd * L);
+  double* hh = (double*)malloc(sizeof(double) * nd * L);
+  double* up = (double*)malloc(sizeof(double) * (size_t)n * f * L); /* pre-ReLU */
+  double* uu = (double*)malloc(sizeof(double) * (size_t)n * f * L);
+  double* z2 = (double*)malloc(sizeof(double) * nd * L);
+  orc_embed(c, blob, n, feats, depth, xs);
+  for (int l = 0; l < L; ++l) {
+    orc_lw w = layer_weights(c, blob, l);
+    const double* x = xs + nd * l;
+    double* q = qkv + nd * 3 * l;
+    linear(n, d, 3 * d, x, w.Wqkv, w.bqkv, q);
+    orc_attention_rows(c, n, Mk, q, 0, n, att + nd * l);
+    linear(n, d, d, att + nd * l, w.Wo, w.bo, z1 + nd * l);
+    for (size_t i = 0; i < nd; ++i) z1[nd * l + i] += x[i];
+    layer_norm(n, d, z1 + nd * l, w.g1, w.be1, c->ln_eps, hh + nd * l);
+    linear(n, d, f, hh + nd * l, w.W1, w.b1, up + (size_t)n * f * l);
+    for (size_t i = 0; i < (size_t)n * f; ++i) {
+      double v = up[(size_t)n * f * l + i];
+      uu[(size_t)n * f * l + i] = v > 0.0 ? v : 0.0;
+    }
+    linear(n, f, d, uu + (size_t)n * f * l, w.W2, w.b2, z2 + nd * l);
+    for (size_t i = 0; i < nd; ++i) z2[nd * l + i] += hh[nd * l + i];
+    layer_norm(n, d, z2 + nd * l, w.g2, w.be2, c->ln_eps, xs + nd * (l + 1));
+  }
+  /* readout forward (orc_readout, intermediates kept) */
+  orc_top t = top_weights(c, blob);
+  const double* xL = xs + nd * L;
+  double* g = (double*)calloc((size_t)d, sizeof(double));
+  double* a1 = (double*)malloc(sizeof(double) * (size_t)d);
+  double* a2 = (double*)malloc(sizeof(double) * (size_t)d);
+  double* r1 = (double*)malloc(sizeof(double) * (size_t)d);
+  double* r2 = (double*)malloc(sizeof(double) * (size_t)d);
+  for (int v = 0; v < n; ++v)
+    for (int j = 0; j < d; ++j) g[j] += xL[(size_t)v * d + j];
+  if (c->pool == 1)
+    for (int j = 0; j < d; ++j) g[j] /= n;
+  linear(1, d, d, g, t.H1, t.c1, a1);
+  for (int j = 0; j < d; ++j) r1[j] = a1[j] > 0.0 ? a1[j] : 0.0;
+  linear(1, d, d, r1, t.H2, t.c2, a2);
+  for (int j = 0; j < d; ++j) r2[j] = a2[j] > 0.0 ? a2[j] : 0.0;
+  linear(1, d, 1, r2, t.w_o, t.c_o, y);
+  /* ---- backward */
+  orc_gtop gt = grad_top(c, grad);
+  double* dr2 = (double*)calloc((size_t)d, sizeof(double));
+  double* dr1 = (double*)calloc((size_t)d, sizeof(double));
+  double* dg = (double*)calloc((size_t)d, sizeof(double));
+  double dyv = dy;
+  linear_back(1, d, 1, r2, t.w_o, &dyv, gt.w_o, gt.c_o, dr2);
+  for (int j = 0; j < d; ++j) dr2[j] = a2[j] > 0.0 ? dr2[j] : 0.0;
+  linear_back(1, d, d, r1, t.H2, dr2, gt.H2, gt.c2, dr1);
+  for (int j = 0; j < d; ++j) dr1[j] = a1[j] > 0.0 ? dr1[j] : 0.0;
+  linear_back(1, d, d, g, t.H1, dr1, gt.H1, gt.c1, dg);
+  double* dx = (double*)malloc(sizeof(double) * nd);
+  for (int v = 0; v < n; ++v)
+    for (int j = 0; j < d; ++j) dx[(size_t)v * d + j] = c->pool == 1 ? dg[j] / n : dg[j];
+  double* dz = (double*)malloc(sizeof(double) * nd);
+  double* dh = (double*)malloc(sizeof(double) * nd);
+  double* du = (double*)malloc(sizeof(double) * (size_t)n * f);
+  double* da = (double*)malloc(sizeof(double) * nd);
+  double* dq = (double*)malloc(sizeof(double) * nd * 3);
+  for (int l = L - 1; l >= 0; --l) {
+    orc_lw w = layer_weights(c, blob, l);
+    orc_glw gw = grad_layer(c, grad, l);
+    /* x' = LN2(z2) */
+    layer_norm_back(n, d, z2 + nd * l, w.g2, c->ln_eps, dx, gw.g2, gw.be2, dz);
+    /* z2 = h + W2 u + b2 */
+    memcpy(dh, dz, sizeof(double) * nd);
+    memset(du, 0, sizeof(double) * (size_t)n * f);
+    linear_back(n, f, d, uu + (size_t)n * f * l, w.W2, dz, gw.W2, gw.b2, du);
+    /* u = ReLU(W1 h + b1) */
+    for (size_t i = 0; i < (size_t)n * f; ++i)
+      if (!(up[(size_t)n * f * l + i] > 0.0)) du[i] = 0.0;
+    linear_back(n, d, f, hh + nd * l, w.W1, du, gw.W1, gw.b1, dh);
+    /* h = LN1(z1) */
+    layer_norm_back(n, d, z1 + nd * l, w.g1, c->ln_eps, dh, gw.g1, gw.be1, dz);
+    /* z1 = x + W_o a + b_o */
+    memcpy(dx, dz, sizeof(double) * nd);
+    memset(da, 0, sizeof(double) * nd);
+    linear_back(n, d, d, att + nd * l, w.Wo, dz, gw.Wo, gw.bo, da);
+    /* a = attention(qkv) */
+    memset(dq, 0, sizeof(double) * nd * 3);
+    attention_back(c, n, Mk, qkv + nd * 3 * l, da, dq);
+    /* qkv = W_qkv x + b_qkv */
+    linear_back(n, d, 3 * d, xs + nd * l, w.Wqkv, dq, gw.Wqkv, gw.bqkv, dx);
+  }
+  /* x0 = W_in f + b_in + PE(depth): PE has no weights */
+  linear_back(n, ORC_F, d, F, t.W_in, dx, gt.W_in, gt.b_in, NULL);
+  free(depth); free(R); free(Mk); free(F); free(xs); free(qkv); free(att); free(z1); free(hh);
+  free(up); free(uu); free(z2); free(g); free(a1); free(a2); free(r1); free(r2);
+  free(dr2); free(dr1); free(dg); free(dx); free(dz); free(dh); free(du); free(da); free(dq);
+  return ORC_OK;
+}

@@ -84,6 +84,11 @@ int orc_forward(const orc_cfg* c, const float* blob, int n, int e, const int32_t
 int orc_forward_k(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src,
                   const int32_t* dst, const orc_feat* feats, int k, double* y, double* taps);
 
+/* Training: y of one graph and grad += dy * dy/dtheta */
+/* over the whole weight blob (same float order), fp64.                            */
+int orc_grad(const orc_cfg* c, const float* blob, int n, int e, const int32_t* src, const int32_t* dst,
+             const orc_feat* feats, double dy, double* y, double* grad);
+
 void orc_plan_T(int64_t P, const int64_t* plan_ptr, const int32_t* plan_stage,
                 const int32_t* B, const float* t, int64_t num_stages, double* T);
 int64_t orc_argmin(int64_t n, const double* T);

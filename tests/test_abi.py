@@ -45,6 +45,48 @@ def test_sass_is_blackwell_native(libpath):
                                        text=True).stdout
 
 
+def _sass_by_kernel(libpath):
+    """{mangled kernel name: SASS text} from cuobjdump."""
+    sass = subprocess.run(["cuobjdump", "-sass", libpath], capture_output=True, text=True).stdout
+    out, name = {}, None
+    for line in sass.splitlines():
+        m = re.match(r"\s*Function : (\S+)", line)
+        if m:
+            name = m.group(1)
+            out[name] = []
+        elif name:
+            out[name].append(line)
+    return {k: "\n".join(v) for k, v in out.items()}
+
+
+# Hot-path kernels and the Blackwell instructions each must carry (SASS
+# mnemonics of B200_PROFILING.md): tcgen05.mma = UTCHMMA, tcgen05.ld/st =
+# LDTM/STTM, TMA = UTMALDG/UTMASTG.  k_attn (warp-level HMMA) is the d_h = 16
+# attention kernel, kept there because it measured faster than the tcgen05
+# kernel on the short GPT sequences (DESIGN.md K6); it is listed so the
+# exception is explicit.
+HOT_KERNELS = {
+    "k_gemm": ("UTCHMMA", "UTMALDG", "LDTM"),
+    "k_attn_tcILi32": ("UTCHMMA", "UTMALDG", "LDTM", "STTM"),
+    "k_attn_tcILi16": ("UTCHMMA", "UTMALDG", "LDTM", "STTM"),
+    "k_layer_tail2": ("UTCHMMA", "UTMALDG", "LDTM", "STTM", "UTMASTG"),
+    "k_layer_tail256": ("UTCHMMA", "UTMALDG", "LDTM", "STTM", "UTMASTG"),
+    "k_attnILi16": ("HMMA", "UTMALDG"),
+}
+
+
+def test_sass_per_hot_kernel(libpath):
+    """Every hot-path kernel (not just the library as a whole) carries the
+    tensor-core / TMA instructions of its design."""
+    kern = _sass_by_kernel(libpath)
+    for pat, need in HOT_KERNELS.items():
+        hits = [k for k in kern if pat in k]
+        assert hits, f"no kernel matching {pat}"
+        for k in hits:
+            for mn in need:
+                assert mn in kern[k], f"{k} lacks {mn}"
+
+
 def test_host_validation_without_gpu(libpath):
     from paper_conf_ipps_acharyas25_b200 import predtop as pt
     L = pt.lib()
