@@ -387,6 +387,54 @@ PREDTOP_API predtop_status predtop_plan_search(int64_t num_problems, int32_t num
                                                int32_t* stage_end_out, int32_t* stage_choice_out,
                                                void* workspace, size_t ws_bytes, void* cuda_stream);
 
+/* ---------------------------------------------------------------------------
+ * Training (SIV-B6-8; the training phase of P:219)
+ * of one DAG-Transformer on (stage DAG, latency) pairs:
+ *   loss  L = (1/G) sum_g |y_hat_g - y_g|              MAE, Eqn 3
+ *   Adam (beta1 0.9, beta2 0.999, eps 1e-8)    predtop_train_adam
+ *   cosine learning-rate decay 1e-3 -> 0 and early stopping (patience 200,
+ *   P:186) are host logic of the caller (paper_conf_ipps_acharyas25_b200/train.py).
+ * The training path computes in fp32 throughout (forward with every
+ * activation kept, backward, optimizer): fp32 master weights, no fp16
+ * rounding; dense GEMMs through cuBLAS (plain library GEMMs), the masked
+ * attention forward/backward, LayerNorm, pooling/head and loss in this
+ * library's kernels.  Deterministic (no float atomics).
+ *
+ * The state holds four fp32 copies of the weight blob (same order and length
+ * as predtop_model_weight_floats): parameters, gradient, Adam m and v, in
+ * caller-allocated device memory of predtop_train_state_bytes (256-byte
+ * aligned).  Limits: d_model <= 256, d_model / num_heads <= 32, d_ff <= 4096.
+ * ------------------------------------------------------------------------- */
+typedef struct predtop_train_s* predtop_train;
+
+PREDTOP_API size_t predtop_train_state_bytes(const predtop_model_config* cfg);
+/* Uploads weights_host (num_floats = predtop_model_weight_floats) as the fp32
+ * parameters, zeroes gradient and moments.  Synchronous. */
+PREDTOP_API predtop_status predtop_train_create(const predtop_model_config* cfg, const float* weights_host,
+                                                size_t num_floats, void* device_state, size_t state_bytes,
+                                                predtop_train* out);
+PREDTOP_API void predtop_train_destroy(predtop_train tr);
+/* Device workspace bytes for predtop_train_grad on this batch. */
+PREDTOP_API size_t predtop_train_workspace(predtop_train tr, predtop_dag dag);
+/* Forward (fp32, activations kept), MAE loss against y_true[G] (device fp32)
+ * and backward into the state's gradient (overwritten: the gradient of the
+ * batch mean).  loss_out[1], y_pred_out[G] (device fp32) nullable.  Every
+ * graph of the batch must have status OK (build the DAG with the default
+ * synchronous validation); otherwise PREDTOP_ERR_INVALID_ARG. */
+PREDTOP_API predtop_status predtop_train_grad(predtop_train tr, predtop_dag dag, const float* y_true,
+                                              void* workspace, size_t ws_bytes, float* loss_out,
+                                              float* y_pred_out, void* cuda_stream);
+/* One Adam update of the parameters from the state's gradient (step >= 1 is
+ * the bias-correction count), torch.optim.Adam semantics (no weight decay):
+ *   m = b1 m + (1-b1) g,  v = b2 v + (1-b2) g^2,
+ *   p -= lr / (1 - b1^step) * m / (sqrt(v) / sqrt(1 - b2^step) + eps). */
+PREDTOP_API predtop_status predtop_train_adam(predtop_train tr, float lr, int32_t step, float beta1,
+                                              float beta2, float eps, void* cuda_stream);
+/* Device pointers of the state's fp32 blobs (which: 0 parameters, 1
+ * gradient, 2 m, 3 v), e.g. to copy the trained weights out or to compare the
+ * gradient.  NULL for a bad handle or index. */
+PREDTOP_API float* predtop_train_buffer(predtop_train tr, int32_t which);
+
 PREDTOP_API const char* predtop_status_string(predtop_status s);
 PREDTOP_API const char* predtop_last_error(void); /* thread-local */
 PREDTOP_API int predtop_abi_version(void);

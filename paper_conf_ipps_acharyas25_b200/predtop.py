@@ -79,6 +79,13 @@ _SIGS = {
     "predtop_prune_graphs": (_I32, [_P, _P, _P, _P, _P, _P, _P, _I32, _P, _SZ, _P, _P, _P, _P, _I64, _P, _P, _P, _P]),
     "predtop_plan_search_workspace": (_SZ, [_I64, _I32, _I32]),
     "predtop_plan_search": (_I32, [_I64, _I32, _I32, _P, _I32, _P, _I64, _I64, _P, _P, _P, _P, _P, _P, _P, _SZ, _P]),
+    "predtop_train_state_bytes": (_SZ, [_P]),
+    "predtop_train_create": (_I32, [_P, _P, _SZ, _P, _SZ, _P]),
+    "predtop_train_destroy": (None, [_P]),
+    "predtop_train_workspace": (_SZ, [_P, _P]),
+    "predtop_train_grad": (_I32, [_P, _P, _P, _P, _SZ, _P, _P, _P]),
+    "predtop_train_adam": (_I32, [_P, ctypes.c_float, _I32, ctypes.c_float, ctypes.c_float, ctypes.c_float, _P]),
+    "predtop_train_buffer": (_P, [_P, _I32]),
     "predtop_status_string": (ctypes.c_char_p, [_I32]),
     "predtop_last_error": (ctypes.c_char_p, []),
     "predtop_abi_version": (ctypes.c_int, []),
@@ -430,3 +437,65 @@ def prune_graphs(batch: "DeviceBatch", pruned_ops=(OP_RESHAPE, OP_CONVERT_ELEMEN
     sizes = torch.diff(onp).cpu()
     return DeviceBatch(onp, oep, osrc[:ne], odst[:ne], ofe[:nn * FEAT_BYTES],
                        int(sizes.max()) if G else 1)
+
+
+class Trainer:
+    """predtop_train_* over a host fp32 weight blob (synth.pack_weights order):
+    fp32 parameters, gradient and Adam moments on the device."""
+
+    PARAMS, GRAD, M, V = 0, 1, 2, 3
+
+    def __init__(self, cfg: dict, blob: np.ndarray, device="cuda"):
+        self.cfg = ModelConfig(cfg["num_layers"], cfg["d_model"], cfg["num_heads"], cfg["d_ff"],
+                               cfg.get("pool", 0), float(cfg.get("ln_eps", 1e-5)))
+        nb = lib().predtop_train_state_bytes(ctypes.byref(self.cfg))
+        if nb == 0:
+            raise PredtopError(UNSUPPORTED, "unsupported training config")
+        blob = np.ascontiguousarray(blob, np.float32)
+        self.num_params = blob.size
+        self.state = torch.empty(nb, dtype=torch.uint8, device=device)
+        h = ctypes.c_void_p()
+        _check(lib().predtop_train_create(ctypes.byref(self.cfg), blob.ctypes.data_as(ctypes.c_void_p), blob.size,
+                                          _ptr(self.state), nb, ctypes.byref(h)))
+        self.handle = h
+        self.step = 0
+        self._ws = {}
+
+    def buffer(self, which: int) -> torch.Tensor:
+        """View of one state blob (PARAMS, GRAD, M, V) as a float32 tensor."""
+        p = lib().predtop_train_buffer(self.handle, which)
+        off = p - self.state.data_ptr()
+        return self.state[off:off + 4 * self.num_params].view(torch.float32)
+
+    def workspace(self, dag: "Dag") -> torch.Tensor:
+        n = lib().predtop_train_workspace(self.handle, dag.handle)
+        ws = self._ws.get(id(dag))
+        if ws is None or ws.numel() < n:
+            ws = torch.empty(n, dtype=torch.uint8, device=self.state.device)
+            self._ws[id(dag)] = ws
+        return ws
+
+    def grad(self, dag: "Dag", y_true: torch.Tensor, stream=None):
+        """Forward + MAE loss + backward; returns (loss [1], y_pred [G]) device tensors."""
+        ws = self.workspace(dag)
+        loss = torch.empty(1, dtype=torch.float32, device=self.state.device)
+        y = torch.empty(dag.batch.num_graphs, dtype=torch.float32, device=self.state.device)
+        _check(lib().predtop_train_grad(self.handle, dag.handle, _ptr(y_true), _ptr(ws), ws.numel(), _ptr(loss),
+                                        _ptr(y), _stream(stream)))
+        return loss, y
+
+    def adam(self, lr: float, beta1: float = 0.9, beta2: float = 0.999, eps: float = 1e-8, stream=None):
+        self.step += 1
+        _check(lib().predtop_train_adam(self.handle, float(lr), self.step, beta1, beta2, eps, _stream(stream)))
+
+    def weights(self) -> np.ndarray:
+        """The current fp32 parameters as a host blob."""
+        return self.buffer(self.PARAMS).cpu().numpy().copy()
+
+    def __del__(self):
+        try:
+            if self.handle and self.handle.value:
+                lib().predtop_train_destroy(self.handle)
+        except Exception:
+            pass
+
