@@ -158,6 +158,32 @@ def run_reference(args, rank):
     from paper_conf_ipps_acharyas25_b200 import synth
     import oracle
     oracle.build()
+    if args.config == "train":  # the oracle's fp64 MAE gradient (orc_grad) + Adam on mini-batches
+        cfg = dict(synth.MODEL_CONFIGS["paper"])
+        blob = synth.pack_weights(cfg, synth.model_weights(cfg)).astype(np.float64)
+        cores = host_cores()
+        nb = cores
+        batch = synth.stage_batch("gpt", nb)
+        yl = 0.01 * np.diff(batch.node_ptr) + 1.0
+        m, v = np.zeros_like(blob), np.zeros_like(blob)
+        t_total = 0.0
+        for s_ in range(min(args.warmup, 1) + args.steps):
+            t0 = time.perf_counter()
+            _, g, _ = oracle.mae_grad(cfg, blob.astype(np.float32), batch, yl, threads=cores)
+            blob, m, v = oracle.adam_step(blob, g, m, v, s_ + 1, 1e-3)
+            if s_ >= min(args.warmup, 1):
+                t_total += time.perf_counter() - t0
+        value = nb * args.steps / t_total
+        line = {"impl": "reference", "metric": "stage-DAGs trained/sec (forward + MAE + backward + Adam)",
+                "value": value, "unit": "graphs/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": 1000 * t_total / args.steps, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": f"train: mini-batches of {nb} GPT-style stage DAGs, paper model (P:178)"},
+                "cpu_baseline": {"value": value, "unit": "graphs/s", "cores": cores, "kind": "oracle",
+                                 "sample": f"{args.steps} steps x {nb} graphs, fp64 orc_grad + Adam"},
+                "e2e": {"value": value, "unit": "graphs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return
     gcfg = "gpt" if args.config in ("sweep", "search") else args.config  # sweep stages are GPT-style pool graphs
     cfg = synth.MODEL_CONFIGS[gcfg]
     blob = synth.pack_weights(cfg, synth.model_weights(cfg))
@@ -262,7 +288,7 @@ def workload_config(args):
 
 
 # ----------------------------------------------------------------- main leg
-DEFAULT_GRAPHS = {"tiny": 4, "gpt": 1024, "moe": 512, "16k": 1, "sweep": 0, "search": 0}
+DEFAULT_GRAPHS = {"tiny": 4, "gpt": 1024, "moe": 512, "16k": 1, "sweep": 0, "search": 0, "train": 32}
 ALSO_KEYS = ("metric", "value", "unit", "ms_per_step", "steps", "config", "e2e", "gpu_launches", "roofline",
              "cpu_baseline", "parity", "result", "clocks")
 
@@ -1016,6 +1042,98 @@ def run_sweep(args, ctx, pool):
         emit(line, args)
 
 
+def run_train(args, ctx):
+    """training steps of the paper's model (4 DAG-
+    Transformer layers of width 64, mini-batches of 32 stage graphs, MAE loss,
+    Adam) on GPT-style stage DAGs.  One step = predtop_train_grad (fp32
+    forward, loss, backward) + predtop_train_adam on one mini-batch per rank;
+    with N ranks the gradients are averaged by one NCCL all-reduce before
+    Adam (data-parallel training: the one real exchange of this path)."""
+    import torch
+    from paper_conf_ipps_acharyas25_b200 import synth
+    pt, dev, world, rank = ctx.pt, ctx.dev, ctx.world, ctx.rank
+    cfg = dict(synth.MODEL_CONFIGS["paper"])
+    blob = synth.pack_weights(cfg, synth.model_weights(cfg))
+    G = args.graphs
+    host = synth.stage_batch("gpt", G, first_graph=rank * G)
+    # labels: any latency-like targets (throughput does not depend on them)
+    y_host = (0.01 * np.diff(host.node_ptr).astype(np.float32) + 1.0)
+    y_pin = torch.from_numpy(y_host).pin_memory()
+    y = torch.empty(G, dtype=torch.float32, device=dev)
+    y.copy_(y_pin)
+    tr = pt.Trainer(cfg, blob, device=dev)
+    dag = pt.Dag(pt.DeviceBatch.from_host(host, device=dev))
+    grad = tr.buffer(pt.Trainer.GRAD)
+
+    def step():
+        tr.grad(dag, y)
+        if world > 1:
+            if ctx.gloo:
+                g = grad.cpu()
+                ctx.dist.all_reduce(g)
+                grad.copy_(g)
+            else:
+                ctx.dist.all_reduce(grad)
+            grad.mul_(1.0 / world)
+        tr.adam(1e-3)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    l0 = ctx.L.predtop_launch_count()
+    step()
+    torch.cuda.synchronize()
+    launches = ctx.L.predtop_launch_count() - l0
+    with ClockSampler(ctx.dev_index) as clk:
+        ms = ctx.timed(step, args.steps)
+    total_ms = ctx.max_over_ranks(sum(ms))
+    value = world * G * args.steps / (total_ms / 1e3)
+    loss_pin = torch.empty(1, dtype=torch.float32).pin_memory()
+
+    def e2e_step():  # labels in from pinned host memory, loss back, every step
+        y.copy_(y_pin, non_blocking=True)
+        loss, _ = tr.grad(dag, y)
+        if world > 1:
+            if ctx.gloo:
+                g = grad.cpu()
+                ctx.dist.all_reduce(g)
+                grad.copy_(g)
+            else:
+                ctx.dist.all_reduce(grad)
+            grad.mul_(1.0 / world)
+        tr.adam(1e-3)
+        loss_pin.copy_(loss, non_blocking=True)
+
+    e2e_ms = ctx.max_over_ranks(sum(ctx.timed(e2e_step, args.steps)))
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import time
+        import oracle
+        oracle.build()
+        cores = host_cores()
+        n = min(G, max(cores, 16))
+        sub = host.subset(list(range(n)))
+        t0 = time.perf_counter()
+        oracle.mae_grad(cfg, blob, sub, y_host[:n], threads=cores)
+        wall = time.perf_counter() - t0
+        cpu = {"value": n / wall, "unit": "graphs/s", "cores": cores, "kind": "oracle",
+               "sample": f"{n} of the {G} stage graphs: fp64 forward + MAE gradient (orc_grad), {cores} threads, {wall:.1f} s"}
+    if rank == 0:
+        line = {"metric": "stage-DAGs trained/sec (forward + MAE + backward + Adam)", "value": value,
+                "unit": "graphs/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": total_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": f"train: mini-batches of {G} GPT-style stage DAGs (~300 ops) per GPU, paper "
+                                       "model (4 layers, d=64, 4 heads, d_ff=256; P:178), MAE loss, Adam; "
+                                       "data-parallel gradient all-reduce for N > 1",
+                           "graphs_per_gpu": G, "l2": "flushed before every timed step (256 MiB memset, untimed)"},
+                "e2e": {"value": world * G * args.steps / (e2e_ms / 1e3), "unit": "graphs/s",
+                        "h2d_bytes_per_step": 4 * G, "d2h_bytes_per_step": 4},
+                "gpu_launches": int(launches), "cpu_baseline": cpu, "launch_mode": "eager",
+                "clocks": clk.summary()}
+        emit(line, args)
+
+
 def emit(line, args):
     print(json.dumps(line), flush=True)
     if args.profile_json:
@@ -1029,7 +1147,7 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="moe", choices=["tiny", "gpt", "moe", "16k", "sweep", "search"])
+    ap.add_argument("--config", default="moe", choices=["tiny", "gpt", "moe", "16k", "sweep", "search", "train"])
     ap.add_argument("--no-also", action="store_true",
                     help="moe: skip the configs[1] (GPT) measurement reported under 'also'")
     ap.add_argument("--no-extras", action="store_true",
@@ -1075,6 +1193,8 @@ def main():
         run_sweep(args, ctx, pool)
     elif args.config == "search":
         run_search(args, ctx)
+    elif args.config == "train":
+        run_train(args, ctx)
     else:
         line = run_batch(args, ctx)
         if args.config == "moe" and not args.no_also and not args.no_extras:
