@@ -56,8 +56,22 @@ constexpr int kSBuf = 3;     // S/P buffers in TMEM
 constexpr int kKV = PREDTOP_ATTN_KV;  // K/V ring stages
 static_assert(kKV > kSBuf && kKV <= 2 * kSBuf, "K/V stages are released through s_full (see the producer)");
 constexpr int kSoftWarps = 8;
-constexpr int kThreads = 64 + 32 * kSoftWarps;
+// PREDTOP_ATTN_SPLIT=1: QK^T and PV are issued by two threads in
+// two warps (warp 1 and warp 10), so neither issue stream waits for the
+// other's instructions (a tcgen05.mma costs its issuing thread ~75-120 cycles
+// next to busy softmax warps); QK^T(c+3) waits for PV(c) through pv_done.
+// Measured no faster on MoE (14.1 vs 14.0 ms/step), so off by default.
+#ifndef PREDTOP_ATTN_SPLIT
+#define PREDTOP_ATTN_SPLIT 0
+#endif
+constexpr int kSplit = PREDTOP_ATTN_SPLIT;
+constexpr int kThreads = 64 + 32 * kSoftWarps + 32 * kSplit;
+constexpr int kPvWarp = kSplit ? 2 + kSoftWarps : 1;
 constexpr float kPMax = 4096.f;  // P above this (or inf, NaN) sends the row to the exact path
+#ifndef PREDTOP_ATTN_PREFETCH
+#define PREDTOP_ATTN_PREFETCH 64
+#endif
+constexpr int kPrefetch = PREDTOP_ATTN_PREFETCH;  // work items (q-tiles) ahead for the L2 prefetch
 
 template <int DH>
 struct TcCfg {
@@ -69,7 +83,7 @@ struct TcCfg {
   static constexpr int ONE = kCh * 32;     // One: [64][16] fp16, SW32, column 0 = 1
   static constexpr int TO = kSBuf * kCh;   // TMEM column of O
   static constexpr int TL = TO + DH;       // TMEM column of l
-  static constexpr int BYTES = 1024 + QB + kKV * STAGE + QM + ONE;
+  static constexpr int BYTES = 1024 + 2 * QB + kKV * STAGE + QM + ONE;
   // > 228/3 KB: at most two CTAs per SM, so the 256-column TMEM allocations
   // never wait for each other
   static constexpr int SMEM = BYTES > 80 * 1024 ? BYTES : 80 * 1024;
@@ -160,11 +174,12 @@ __global__ void __launch_bounds__(kThreads, 2)
   extern __shared__ unsigned char dsm[];
   unsigned char* base = sm100::align1024(dsm);
   unsigned char* sQ = base;                      // [128][DH], swizzled
-  unsigned char* sKV = sQ + C::QB;               // stage s: K at s*STAGE, V at +KB, ones at +2KB
+  unsigned char* sKd = sQ + C::QB;               // the tile's own K rows (diagonal scores)
+  unsigned char* sKV = sKd + C::QB;              // stage s: K at s*STAGE, V at +KB, ones at +2KB
   unsigned char* sQm = sKV + kKV * C::STAGE;
   unsigned char* sOne = sQm + C::QM;
   __shared__ __align__(8) uint64_t q_full, init_done, kv_full[kKV], s_full[kSBuf],
-      p_ready[kSBuf], o_full;
+      p_ready[kSBuf], pv_done[kSBuf], o_full;
   __shared__ uint32_t tmem_slot;
   __shared__ int row_exact[kRows];  // rows sent to the exact path
 
@@ -189,6 +204,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   const int W = 2 * ((N + 127) / 128);
   const int nch = (N + kCh - 1) / kCh;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) ATR(2, 0);  // CTA start
 
   if (threadIdx.x == 0) {
     sm100::mbar_init(&q_full, 1);
@@ -201,6 +217,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     for (int b = 0; b < kSBuf; ++b) {
       sm100::mbar_init(&s_full[b], 1);
       sm100::mbar_init(&p_ready[b], kSoftWarps);
+      sm100::mbar_init(&pv_done[b], 1);
     }
     sm100::mbar_init(&o_full, 1);
     sm100::fence_mbar_init();
@@ -211,11 +228,29 @@ __global__ void __launch_bounds__(kThreads, 2)
   __syncthreads();
   sm100::tc_fence_after();
   const uint32_t tmem = tmem_slot;
+  if (threadIdx.x == 0) ATR(2, 1);  // barriers + TMEM ready
 
   if (warp == 0) {
     if (lane == 0) {  // -------------------------------------------- TMA
-      sm100::mbar_arrive_expect_tx(&q_full, (uint32_t)C::QB);
+      // L2 prefetch of the q|k|v rows of the tile kPrefetch work items ahead
+      // (one CTA per tile: head 0): its CTAs start ~1.7 waves later and find
+      // Q, the diagonal K rows and the graph's first K/V chunks in L2 instead
+      // of HBM (the prologue was ~3k cycles of TMA latency)
+      if (h == 0 && widx + kPrefetch < d.qtile_off[G]) {
+        const int2 nx = d.work[widx + kPrefetch];
+        if ((unsigned)nx.x < (unsigned)G) {
+          const int64_t a0 = d.node_ptr[nx.x], a1 = d.node_ptr[nx.x + 1];
+          const int64_t r0 = a0 + (int64_t)nx.y * kRows, r1 = min(a1, r0 + kRows);
+          if (r1 > r0) {
+            const char* base = reinterpret_cast<const char*>(qkv + r0 * 3 * dmodel);
+            const uint32_t bytes = (uint32_t)((r1 - r0) * 3 * dmodel * 2);
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(base), "r"(bytes) : "memory");
+          }
+        }
+      }
+      sm100::mbar_arrive_expect_tx(&q_full, (uint32_t)(2 * C::QB));
       sm100::tma_load_2d(sQ, &tq, &q_full, h * DH, (int)(n0 + qt * kRows));
+      sm100::tma_load_2d(sKd, &tq, &q_full, dmodel + h * DH, (int)(n0 + qt * kRows));
       // stage of chunk c - kKV is free once PV(c - kKV) completed, which the
       // commit of QK(c - kKV + kSBuf) (issued after it) implies: no separate
       // "empty" barrier.  kKV <= 2 kSBuf keeps the parity unambiguous (the
@@ -237,8 +272,8 @@ __global__ void __launch_bounds__(kThreads, 2)
         if (++s == kKV) s = 0;
       }
     }
-  } else if (warp == 1) {
-    if (lane == 0) {  // -------------------------------------------- MMA issuer
+  } else if (warp == 1 || warp == kPvWarp) {
+    if (lane == 0) {  // -------------------------------------------- MMA issuer(s)
       constexpr uint32_t id_qk = sm100::make_idesc_f16(128, kCh);
       constexpr uint32_t id_pv = sm100::make_idesc_f16(128, DH + 16) | (1u << 16);  // B [V|1] MN-major
       // descriptors precomputed once; a byte offset o advances the start
@@ -250,6 +285,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       const uint64_t dQm = sm100::make_sdesc<32>(sm100::smem_u32(sQm));
       const uint64_t dOne = sm100::make_sdesc<32>(sm100::smem_u32(sOne));
       const uint32_t sfull0 = sm100::smem_u32(&s_full[0]), kvfull0 = sm100::smem_u32(&kv_full[0]);
+      const uint32_t pvdone0 = sm100::smem_u32(&pv_done[0]);
       int qs = 0, qb = 0;  // stage / S buffer of the next QK^T
       uint32_t qph = 0;    // kv_full parity of stage qs (flips per ring pass)
       auto qk = [&](int c) {
@@ -271,16 +307,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         }
         if (++qb == kSBuf) qb = 0;
       };
-      sm100::mbar_wait_sleep(&q_full, 0);
-      sm100::mbar_wait_sleep(&init_done, 0);
-      sm100::tc_fence_after();
-      for (int c = 0; c < nch && c < kSBuf; ++c) qk(c);
-      int s = 0, b = 0;
-      uint32_t pph = 0;
-      for (int c = 0; c < nch; ++c) {
-        MMA_WAIT(&p_ready[b], pph);
-        ATR(0, c);
-        sm100::tc_fence_after();
+      auto pv = [&](int c, int s, int b) {
         const uint32_t tP = tmem + kCh * b;
         const uint64_t off = (uint64_t)((s * C::STAGE) >> 4);
 #pragma unroll
@@ -291,15 +318,55 @@ __global__ void __launch_bounds__(kThreads, 2)
           const uint32_t tA = tP + (kk < 2 ? 8 * kk : 32 + 8 * (kk - 2));
           sm100::mma_f16_ts(tmem + C::TO, tA, dV + off + (uint64_t)((kk * 16 * C::RB) >> 4), id_pv, acc);
         }
-        ATR(1, c);
-        if (c + kSBuf < nch) qk(c + kSBuf);
-        if (++s == kKV) s = 0;
-        if (++b == kSBuf) {
-          b = 0;
-          pph ^= 1u;
+      };
+      if (warp == 1) {  // QK^T issuer (and, unsplit, PV too)
+        sm100::mbar_wait_sleep(&q_full, 0);
+        sm100::mbar_wait_sleep(&init_done, 0);
+        sm100::tc_fence_after();
+        for (int c = 0; c < nch && c < kSBuf; ++c) qk(c);
+        int s = 0, b = 0;
+        uint32_t pph = 0;
+        for (int c = 0; c < nch; ++c) {
+          if (kSplit) {
+            // S_b is rewritten by QK^T(c+3) once PV(c) has read P_b
+            if (c + kSBuf < nch) {
+              MMA_WAIT(&pv_done[b], pph);
+              sm100::tc_fence_after();
+              qk(c + kSBuf);
+            }
+          } else {
+            MMA_WAIT(&p_ready[b], pph);
+            ATR(0, c);
+            sm100::tc_fence_after();
+            pv(c, s, b);
+            ATR(1, c);
+            if (c + kSBuf < nch) qk(c + kSBuf);
+          }
+          if (++s == kKV) s = 0;
+          if (++b == kSBuf) {
+            b = 0;
+            pph ^= 1u;
+          }
         }
+        if (!kSplit) sm100::mma_commit(&o_full);
+      } else {  // PV issuer
+        int s = 0, b = 0;
+        uint32_t pph = 0;
+        for (int c = 0; c < nch; ++c) {
+          MMA_WAIT(&p_ready[b], pph);
+          ATR(0, c);
+          sm100::tc_fence_after();
+          pv(c, s, b);
+          ATR(1, c);
+          sm100::mma_commit_addr(pvdone0 + 8 * b);
+          if (++s == kKV) s = 0;
+          if (++b == kSBuf) {
+            b = 0;
+            pph ^= 1u;
+          }
+        }
+        sm100::mma_commit(&o_full);
       }
-      sm100::mma_commit(&o_full);
     }
   } else {
     // ---------------------------------------------------------- softmax
@@ -315,13 +382,16 @@ __global__ void __launch_bounds__(kThreads, 2)
     // (1) reference m = the diagonal score q_row . k_row (fp32 from the fp16
     // operands), rounded to fp16: it enters the QK^T MMA as the fp16 Qm entry
     if (hf == 0) {
+      // from the TMA'd Q tile and the tile's own K rows (swizzled rows of
+      // RB bytes: 16-byte chunk j of row x at x*RB + 16*(j ^ swizzle(x)))
       float m = 0.f;
+      sm100::mbar_wait(&q_full, 0);
       if (valid) {
-        const uint4* qr = reinterpret_cast<const uint4*>(qkv + (n0 + row) * 3 * dmodel + h * DH);
-        const uint4* kr = reinterpret_cast<const uint4*>(qkv + (n0 + row) * 3 * dmodel + dmodel + h * DH);
 #pragma unroll
         for (int j = 0; j < DH / 8; ++j) {
-          const uint4 a = __ldg(qr + j), bq = __ldg(kr + j);
+          const int jj = C::RB == 64 ? (j ^ ((r >> 1) & 3)) : (j ^ ((r >> 2) & 1));
+          const uint4 a = *reinterpret_cast<const uint4*>(sQ + r * C::RB + 16 * jj);
+          const uint4 bq = *reinterpret_cast<const uint4*>(sKd + r * C::RB + 16 * jj);
           const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, bw[4] = {bq.x, bq.y, bq.z, bq.w};
 #pragma unroll
           for (int i = 0; i < 4; ++i) {
@@ -351,6 +421,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     sm100::fence_proxy_async();
     sm100::named_bar<32 * kSoftWarps>(1);
     if (t == 0) sm100::mbar_arrive(&init_done);
+    if (t == 0) ATR(2, 2);  // m, Qm, One written
     // (2) chunks.  The 64-bit mask word c covers chunk c; this thread's 32
     // keys are the low (hf = 0) or high (hf = 1) byte of each 16-bit field of
     // the stored layout (internal.h mask_pos: mask_pos(k + 32) = mask_pos(k) + 8).
@@ -408,8 +479,10 @@ __global__ void __launch_bounds__(kThreads, 2)
       if (!(pm <= kPMax) && valid) row_exact[r] = 1;  // also NaN
     }
     // (3) O / l -> fp16: this thread writes output columns [DH/2 hf, DH/2 (hf+1))
+    if (t == 0) ATR(2, 3);  // softmax done
     sm100::mbar_wait(&o_full, 0);
     sm100::tc_fence_after();
+    if (t == 0) ATR(2, 4);  // O complete
     float o[DH];
     sm100::tmem_ld<DH>(tmem + C::TO + lrow, o);
     float lv[16];
@@ -436,6 +509,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   }
   sm100::tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) ATR(2, 5);  // all stored
   if (warp == 1) sm100::tmem_dealloc<256>(tmem);
 }
 

@@ -32,10 +32,12 @@ def main():
     t = np.frombuffer(buf, dtype=np.uint64).reshape(8, 64).astype(np.int64)
     t0 = t[t > 0].min()
     f = lambda x: f"{x - t0:8d}" if x else "       -"
+    print("CTA start / barriers+TMEM / m,Qm written / softmax done / O complete / stored:",
+          " ".join(f(t[2, i]) for i in range(6)))
     print("chunk | mma: pready_seen  pv_issued  kv_empty_commit | qk: kv_full  issued  s_full_commit | w2: s_seen  arrive")
     for c in range(64):
         if t[0, c] or t[3, c]:
-            print(f"{c:4d} | {f(t[0, c])} {f(t[1, c])} {f(t[2, c])} | {f(t[3, c])} {f(t[4, c])} {f(t[5, c])} | "
+            print(f"{c:4d} | {f(t[0, c])} {f(t[1, c])}        - | {f(t[3, c])} {f(t[4, c])} {f(t[5, c])} | "
                   f"{f(t[6, c])} {f(t[7, c])}")
 
 

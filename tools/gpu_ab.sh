@@ -1,0 +1,10 @@
+#!/bin/bash
+# A/B of library variants on the MoE bench: bash tools/gpu_ab.sh <variant> ...
+O=gpurun_out; mkdir -p $O
+timeout 300 python -m pytest tests -m gpu -q -x --timeout 120 -k "moe or exact or tc" > $O/pt_ab.txt 2>&1; echo "pytest rc=$?" >> $O/pt_ab.txt; tail -2 $O/pt_ab.txt
+for v in default "$@"; do
+  if [ "$v" != default ]; then export PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_$v.so; else unset PREDTOP_LIB; fi
+  timeout 240 python bench.py --config moe --no-cpu-baseline --no-also --steps 20 > $O/bench_$v.json 2>$O/bench_$v.err
+  python -c "
+import json; d=json.loads(open('$O/bench_$v.json').read().strip().splitlines()[-1]); print('$v', round(d['value']), {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if v['ms_per_step']>0.3})" || tail -3 $O/bench_$v.err
+done
