@@ -51,7 +51,7 @@ constexpr int kRows = 128;   // query rows per CTA (TMEM lanes)
 constexpr int kCh = 64;      // keys per chunk (S columns)
 constexpr int kSBuf = 3;     // S/P buffers in TMEM
 #ifndef PREDTOP_ATTN_KV
-#define PREDTOP_ATTN_KV 6
+#define PREDTOP_ATTN_KV 5
 #endif
 constexpr int kKV = PREDTOP_ATTN_KV;  // K/V ring stages
 static_assert(kKV > kSBuf && kKV <= 2 * kSBuf, "K/V stages are released through s_full (see the producer)");
@@ -68,10 +68,6 @@ constexpr int kSplit = PREDTOP_ATTN_SPLIT;
 constexpr int kThreads = 64 + 32 * kSoftWarps + 32 * kSplit;
 constexpr int kPvWarp = kSplit ? 2 + kSoftWarps : 1;
 constexpr float kPMax = 4096.f;  // P above this (or inf, NaN) sends the row to the exact path
-#ifndef PREDTOP_ATTN_PREFETCH
-#define PREDTOP_ATTN_PREFETCH 64
-#endif
-constexpr int kPrefetch = PREDTOP_ATTN_PREFETCH;  // work items (q-tiles) ahead for the L2 prefetch
 
 template <int DH>
 struct TcCfg {
@@ -232,22 +228,6 @@ __global__ void __launch_bounds__(kThreads, 2)
 
   if (warp == 0) {
     if (lane == 0) {  // -------------------------------------------- TMA
-      // L2 prefetch of the q|k|v rows of the tile kPrefetch work items ahead
-      // (one CTA per tile: head 0): its CTAs start ~1.7 waves later and find
-      // Q, the diagonal K rows and the graph's first K/V chunks in L2 instead
-      // of HBM (the prologue was ~3k cycles of TMA latency)
-      if (h == 0 && widx + kPrefetch < d.qtile_off[G]) {
-        const int2 nx = d.work[widx + kPrefetch];
-        if ((unsigned)nx.x < (unsigned)G) {
-          const int64_t a0 = d.node_ptr[nx.x], a1 = d.node_ptr[nx.x + 1];
-          const int64_t r0 = a0 + (int64_t)nx.y * kRows, r1 = min(a1, r0 + kRows);
-          if (r1 > r0) {
-            const char* base = reinterpret_cast<const char*>(qkv + r0 * 3 * dmodel);
-            const uint32_t bytes = (uint32_t)((r1 - r0) * 3 * dmodel * 2);
-            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(base), "r"(bytes) : "memory");
-          }
-        }
-      }
       sm100::mbar_arrive_expect_tx(&q_full, (uint32_t)(2 * C::QB));
       sm100::tma_load_2d(sQ, &tq, &q_full, h * DH, (int)(n0 + qt * kRows));
       sm100::tma_load_2d(sKd, &tq, &q_full, dmodel + h * DH, (int)(n0 + qt * kRows));
