@@ -275,10 +275,15 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   const int K = d.hops;
   if (!csr_in_smem && !global_mode && !(K > 0 && K < L - 1)) {
     // Deep graphs whose CSR does not fit next to the slice (e.g. 16k nodes,
-    // ~11k levels): the level loop is latency-bound, so it reads per-node
-    // records (node, degree, first four successors; built by k_depth in topo
-    // order) prefetched four levels ahead into registers, and the level
-    // bounds from a shared-memory copy: no dependent L2 round trip per level.
+    // ~11k levels; for MoE-size graphs the CSR-in-SMEM loop below measured
+    // faster: 1.27 vs 1.64 ms/step).  Level loop over per-node records (node, degree, first four successors;
+    // built by k_depth in topo order) prefetched four levels ahead into
+    // registers, and the level bounds from a shared-memory copy: the loop is
+    // latency-bound (fwd+bwd stage graphs have ~N/3 levels of a few nodes),
+    // so no dependent L2 round trip per level.  Bit columns are independent
+    // (column j of R[v] reads column j of the successors' rows only), so each
+    // warp owns the words j = warp, warp + nwarps, ... of the slice and walks
+    // the levels on its own with warp barriers: no CTA barrier per level.
     uint64_t* Rsm = reinterpret_cast<uint64_t*>(sm);
     const int rs2 = CW;
     const size_t slice_bytes = align_up((size_t)N * CW * 8, 16);
@@ -290,24 +295,25 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
     const int4* rec = d.rec + n0;
     for (int64_t it = tid; it < (int64_t)N * nw; it += nt) Rsm[(it / nw) * rs2 + it % nw] = 0;
     __syncthreads();
-    // the level loop runs on warp 0 alone (levels hold ~1-2 nodes): warp
-    // barriers instead of CTA barriers between levels
-    if (tid >= 32) return;
-    auto first_rec = [&](int l) -> int4 {  // this thread's first item of level l
-      if (l < 0) return make_int4(0, 0, 0, 0);
-      const int b = lp[l], e = lp[l + 1];
-      return tid < (e - b) * nw ? __ldg(rec + b + tid / nw) : make_int4(0, 0, 0, 0);
-    };
-    // level `level` with its prefetched first record r; then r <- the record of
-    // level - 4 (four fixed registers, unrolled by four: no register moves, so
-    // a load is only waited for when its level comes up)
-    auto do_level = [&](int level, int4& r0) {
-      const int lb = lp[level], items = (lp[level + 1] - lb) * nw;
-      if (nw == 1) {  // one word column (the deep-graph case): no index division
-        const uint32_t w0 = (uint32_t)word0;
-        for (int i = tid; i < items; i += 32) {
-          const int4 r = i == tid ? r0 : __ldg(rec + lb + i);
+    const int warp = tid >> 5, lane = tid & 31, nwarps = nt >> 5;
+    const int my_nw = warp < nw ? (nw - warp + nwarps - 1) / nwarps : 0;
+    if (my_nw > 0) {
+      auto first_rec = [&](int l) -> int4 {  // this lane's first item of level l
+        if (l < 0) return make_int4(0, 0, 0, 0);
+        const int b = lp[l], e = lp[l + 1];
+        return lane < (e - b) * my_nw ? __ldg(rec + b + (my_nw == 1 ? lane : lane / my_nw)) : make_int4(0, 0, 0, 0);
+      };
+      // level `level` with its prefetched first record r0; then r0 <- the
+      // record of level - 4 (four fixed registers, unrolled by four: a load is
+      // only waited for when its level comes up)
+      auto do_level = [&](int level, int4& r0) {
+        const int lb = lp[level], items = (lp[level + 1] - lb) * my_nw;
+        for (int i = lane; i < items; i += 32) {
+          const int node_i = my_nw == 1 ? i : i / my_nw;
+          const int4 r = i == lane ? r0 : __ldg(rec + lb + node_i);
           const uint32_t v = (uint32_t)r.x & 0xFFFFu, deg = (uint32_t)r.x >> 16;
+          const int j = warp + (my_nw == 1 ? 0 : (i - node_i * my_nw)) * nwarps;
+          const uint32_t wj = (uint32_t)(word0 + j);
           const uint32_t s4[4] = {(uint32_t)r.y & 0xFFFFu, (uint32_t)r.y >> 16, (uint32_t)r.z & 0xFFFFu,
                                   (uint32_t)r.z >> 16};
           uint64_t acc = 0;
@@ -315,54 +321,30 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
           for (int k = 0; k < 4; ++k)
             if ((uint32_t)k < deg) {
               const uint32_t w = s4[k];
-              acc |= Rsm[(size_t)w * rs2] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
+              acc |= Rsm[(size_t)w * rs2 + j] | ((w >> 6) == wj ? 1ull << (w & 63) : 0ull);
             }
           if (deg > 4) {
             const uint32_t dg = deg == 0xFFFFu ? (uint32_t)(soff[v + 1] - r.w) : deg;
             for (uint32_t k = 4; k < dg; ++k) {
               const uint32_t w = (uint32_t)succ[r.w + k];
-              acc |= Rsm[(size_t)w * rs2] | ((w >> 6) == w0 ? 1ull << (w & 63) : 0ull);
+              acc |= Rsm[(size_t)w * rs2 + j] | ((w >> 6) == wj ? 1ull << (w & 63) : 0ull);
             }
           }
-          Rsm[(size_t)v * rs2] = acc;  // rs2 = CW > 1 when only the last slice is one word wide
+          Rsm[(size_t)v * rs2 + j] = acc;
         }
         r0 = first_rec(level - 4);
         __syncwarp();
-        return;
+      };
+      int4 r0 = first_rec(L - 1), r1 = first_rec(L - 2), r2 = first_rec(L - 3), r3 = first_rec(L - 4);
+      for (int level = L - 1; level >= 0; level -= 4) {
+        do_level(level, r0);
+        if (level >= 1) do_level(level - 1, r1);
+        if (level >= 2) do_level(level - 2, r2);
+        if (level >= 3) do_level(level - 3, r3);
       }
-      for (int it = tid; it < items; it += 32) {
-        const int4 r = it == tid ? r0 : __ldg(rec + lb + it / nw);
-        const int v = r.x & 0xFFFF;
-        int deg = (int)((unsigned)r.x >> 16);
-        if (deg == 0xFFFF) deg = soff[v + 1] - r.w;  // capped in the record
-        const int j = it % nw, word = word0 + j;
-        uint64_t acc = 0;
-        const int s4[4] = {r.y & 0xFFFF, (int)((unsigned)r.y >> 16), r.z & 0xFFFF, (int)((unsigned)r.z >> 16)};
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-          if (k < deg) {
-            const int w = s4[k];
-            acc |= Rsm[(int64_t)w * rs2 + j];
-            if ((w >> 6) == word) acc |= 1ull << (w & 63);
-          }
-        for (int k = 4; k < deg; ++k) {
-          const int w = succ[r.w + k];
-          acc |= Rsm[(int64_t)w * rs2 + j];
-          if ((w >> 6) == word) acc |= 1ull << (w & 63);
-        }
-        Rsm[(int64_t)v * rs2 + j] = acc;
-      }
-      r0 = first_rec(level - 4);
-      __syncwarp();
-    };
-    int4 r0 = first_rec(L - 1), r1 = first_rec(L - 2), r2 = first_rec(L - 3), r3 = first_rec(L - 4);
-    for (int level = L - 1; level >= 0; level -= 4) {
-      do_level(level, r0);
-      if (level >= 1) do_level(level - 1, r1);
-      if (level >= 2) do_level(level - 2, r2);
-      if (level >= 3) do_level(level - 3, r3);
     }
-    for (int64_t it = tid; it < (int64_t)N * nw; it += 32)
+    __syncthreads();
+    for (int64_t it = tid; it < (int64_t)N * nw; it += nt)
       Rg[(it / nw) * W + word0 + it % nw] = Rsm[(it / nw) * rs2 + it % nw];
     return;
   }
@@ -416,23 +398,34 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   } else {
   for (int64_t it = tid; it < (int64_t)N * nw; it += nt) Rs[(it / nw) * rs + it % nw] = 0;
   __syncthreads();
-  for (int level = L - 1; level >= 0; --level) {
-    const int lb = lptr[level], le = lptr[level + 1];
-    const int items = (le - lb) * nw;
-    for (int it = tid; it < items; it += nt) {
-      const int v = topo[lb + it / nw];
-      const int j = it % nw;
-      const int word = word0 + j;
-      uint64_t acc = 0;
-      for (int k = soff[v]; k < soff[v + 1]; ++k) {
-        const int w = succ[k];
-        acc |= Rs[(int64_t)w * rs + j];
-        if ((w >> 6) == word) acc |= 1ull << (w & 63);
+  // Bit columns are independent (R[v] column j only reads column j of the
+  // successors' rows), so each warp owns the words j = warp, warp + nwarps,
+  // ... of the slice and walks the levels on its own with warp barriers: no
+  // CTA barrier per level (the levels of fwd+bwd stage graphs hold a few
+  // nodes, so the loop is latency-bound; 8 independent warps instead of one
+  // CTA-synchronous sweep).
+  const int warp = tid >> 5, lane = tid & 31, nwarps = nt >> 5;
+  const int my_nw = warp < nw ? (nw - warp + nwarps - 1) / nwarps : 0;
+  if (my_nw > 0) {
+    for (int level = L - 1; level >= 0; --level) {
+      const int lb = lptr[level], le = lptr[level + 1];
+      const int items = (le - lb) * my_nw;
+      for (int it = lane; it < items; it += 32) {
+        const int v = topo[lb + it / my_nw];
+        const int j = warp + (it % my_nw) * nwarps;
+        const int word = word0 + j;
+        uint64_t acc = 0;
+        for (int k = soff[v]; k < soff[v + 1]; ++k) {
+          const int w = succ[k];
+          acc |= Rs[(int64_t)w * rs + j];
+          if ((w >> 6) == word) acc |= 1ull << (w & 63);
+        }
+        Rs[(int64_t)v * rs + j] = acc;
       }
-      Rs[(int64_t)v * rs + j] = acc;
+      __syncwarp();
     }
-    __syncthreads();
   }
+  __syncthreads();
   }
   if (!global_mode)
     for (int64_t it = tid; it < (int64_t)N * nw; it += nt)
