@@ -48,14 +48,25 @@ namespace predtop {
 namespace {
 
 constexpr int kRows = 128;   // query rows per CTA (TMEM lanes)
-constexpr int kCh = 64;      // keys per chunk (S columns)
-constexpr int kSBuf = 3;     // S/P buffers in TMEM
+// Geometry: PREDTOP_ATTN_GEO=64 (default): 64-key chunks, 3 S buffers, 8
+// softmax warps (two key halves per row), 256 TMEM columns, 2 CTAs per SM.
+// =32: 32-key chunks, 2 S buffers, 4 softmax warps (one thread per row),
+// 128 TMEM columns, 4 CTAs per SM.
+#ifndef PREDTOP_ATTN_GEO
+#define PREDTOP_ATTN_GEO 64
+#endif
+constexpr int kCh = PREDTOP_ATTN_GEO;          // keys per chunk (S columns)
+constexpr int kSBuf = kCh == 64 ? 3 : 2;       // S/P buffers in TMEM
+constexpr int kSoftWarps = kCh == 64 ? 8 : 4;  // softmax warps (kSoftWarps / 4 threads per row)
+constexpr int kHalves = kSoftWarps / 4;
+constexpr int kTmemCols = kCh == 64 ? 256 : 128;
+constexpr int kMinBlocks = kCh == 64 ? 2 : 4;
 #ifndef PREDTOP_ATTN_KV
-#define PREDTOP_ATTN_KV 5
+#define PREDTOP_ATTN_KV (kSBuf == 3 ? 5 : 4)
 #endif
 constexpr int kKV = PREDTOP_ATTN_KV;  // K/V ring stages
 static_assert(kKV > kSBuf && kKV <= 2 * kSBuf, "K/V stages are released through s_full (see the producer)");
-constexpr int kSoftWarps = 8;
+static_assert(kCh * 4 / kSoftWarps == 32, "every softmax thread owns 32 keys of a chunk");
 // PREDTOP_ATTN_SPLIT=1: QK^T and PV are issued by two threads in
 // two warps (warp 1 and warp 10), so neither issue stream waits for the
 // other's instructions (a tcgen05.mma costs its issuing thread ~75-120 cycles
@@ -80,10 +91,11 @@ struct TcCfg {
   static constexpr int TO = kSBuf * kCh;   // TMEM column of O
   static constexpr int TL = TO + DH;       // TMEM column of l
   static constexpr int BYTES = 1024 + 2 * QB + kKV * STAGE + QM + ONE;
-  // > 228/3 KB: at most two CTAs per SM, so the 256-column TMEM allocations
-  // never wait for each other
-  static constexpr int SMEM = BYTES > 80 * 1024 ? BYTES : 80 * 1024;
-  static_assert(TL + 16 <= 256, "TMEM budget");
+  // > 228/(kMinBlocks+1) KB: at most kMinBlocks CTAs per SM, so the TMEM
+  // allocations never wait for each other
+  static constexpr int FLOOR = (228 / (kMinBlocks + 1) + 2) * 1024;
+  static constexpr int SMEM = BYTES > FLOOR ? BYTES : FLOOR;
+  static_assert(TL + 16 <= kTmemCols, "TMEM budget");
 };
 
 #ifdef PREDTOP_ATTN_MMA_SPIN
@@ -163,7 +175,7 @@ __device__ __noinline__ void exact_row(const __half* __restrict__ qkv, int64_t n
 }
 
 template <int DH>
-__global__ void __launch_bounds__(kThreads, 2)
+__global__ void __launch_bounds__(kThreads, kMinBlocks)
     k_attn_tc(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tm, DagDev d, int G,
               int H, int dmodel, const __half* __restrict__ qkv, __half* __restrict__ out) {
   using C = TcCfg<DH>;
@@ -219,7 +231,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     sm100::fence_mbar_init();
   }
   if (threadIdx.x < kRows) row_exact[threadIdx.x] = 0;
-  if (warp == 1) sm100::tmem_alloc<256>(&tmem_slot);
+  if (warp == 1) sm100::tmem_alloc<kTmemCols>(&tmem_slot);
   sm100::tc_fence_before();
   __syncthreads();
   sm100::tc_fence_after();
@@ -388,8 +400,9 @@ __global__ void __launch_bounds__(kThreads, 2)
       unsigned char* qrow = sQm + r * 32;
       *reinterpret_cast<uint4*>(qrow + 16 * ((r >> 2) & 1)) = make_uint4(nm, 0u, 0u, 0u);
       *reinterpret_cast<uint4*>(qrow + 16 - 16 * ((r >> 2) & 1)) = make_uint4(0u, 0u, 0u, 0u);
-    } else if (t - 128 < kCh) {  // One = [1 0 ... 0] per key
-      const int k = t - 128, o0 = 16 * ((k >> 2) & 1);
+    }
+    for (int k = t; k < kCh; k += 32 * kSoftWarps) {  // One = [1 0 ... 0] per key
+      const int o0 = 16 * ((k >> 2) & 1);
       *reinterpret_cast<uint4*>(sOne + k * 32 + o0) = make_uint4(0x3C00u, 0u, 0u, 0u);
       *reinterpret_cast<uint4*>(sOne + k * 32 + 16 - o0) = make_uint4(0u, 0u, 0u, 0u);
     }
@@ -407,16 +420,20 @@ __global__ void __launch_bounds__(kThreads, 2)
     // the stored layout (internal.h mask_pos: mask_pos(k + 32) = mask_pos(k) + 8).
     const uint32_t sfull0 = sm100::smem_u32(&s_full[0]), pready0 = sm100::smem_u32(&p_ready[0]);
     const uint32_t tS0 = tmem + 32 * hf + lrow;
-    // mask words two chunks ahead (L2 latency)
-    uint64_t wnext = valid ? __ldg(Mrow) : 0ull, wnext2 = (valid && nch > 1) ? __ldg(Mrow + 1) : 0ull;
+    // mask words two chunks ahead (L2 latency).  This thread's 32 keys of
+    // chunk c start at key kCh c + 32 hf: word (kCh c + 32 hf) >> 6, byte
+    // half ((kCh c + 32 hf) >> 5) & 1 of every 16-bit field.
+    auto word_of = [&](int c) -> int { return (kCh * c + 32 * hf) >> 6; };
+    uint64_t wnext = valid ? __ldg(Mrow + word_of(0)) : 0ull,
+             wnext2 = (valid && nch > 1) ? __ldg(Mrow + word_of(1)) : 0ull;
     __half2 mx2 = __float2half2_rn(0.f);
     int b = 0;
     uint32_t ph = 0;  // phase parity of buffer b's barriers
 #pragma unroll 1
     for (int c = 0; c < nch; ++c) {
-      const uint64_t w = (wnext >> (8 * hf)) & 0x00FF00FF00FF00FFull;
+      const uint64_t w = (wnext >> (8 * (((kCh * c + 32 * hf) >> 5) & 1))) & 0x00FF00FF00FF00FFull;
       wnext = wnext2;
-      if (c + 2 < nch && valid) wnext2 = __ldg(Mrow + c + 2);
+      if (c + 2 < nch && valid) wnext2 = __ldg(Mrow + word_of(c + 2));
       bar_wait(sfull0 + 8 * b, ph);
       if (lane == 0 && warp == 2) ATR(6, c);
       sm100::tc_fence_after();
@@ -458,7 +475,8 @@ __global__ void __launch_bounds__(kThreads, 2)
       const float pm = fmaxf(__low2float(mx2), __high2float(mx2));
       if (!(pm <= kPMax) && valid) row_exact[r] = 1;  // also NaN
     }
-    // (3) O / l -> fp16: this thread writes output columns [DH/2 hf, DH/2 (hf+1))
+    // (3) O / l -> fp16: this thread writes output columns [OC hf, OC (hf+1)),
+    // OC = DH / kHalves
     if (t == 0) ATR(2, 3);  // softmax done
     sm100::mbar_wait(&o_full, 0);
     sm100::tc_fence_after();
@@ -474,23 +492,24 @@ __global__ void __launch_bounds__(kThreads, 2)
         if (hf == 0) exact_row<DH>(qkv, n0, N, row, h, dmodel, Mrow, orow);
       } else {
         const float inv = lv[0] > 0.f ? 1.f / lv[0] : 0.f;
-        uint32_t pk[DH / 4];
+        constexpr int OC = DH / kHalves;
+        uint32_t pk[OC / 2];
 #pragma unroll
-        for (int i = 0; i < DH / 4; ++i) {
-          const float a0 = hf ? o[DH / 2 + 2 * i] : o[2 * i];
-          const float a1 = hf ? o[DH / 2 + 2 * i + 1] : o[2 * i + 1];
+        for (int i = 0; i < OC / 2; ++i) {
+          const float a0 = hf ? o[OC + 2 * i] : o[2 * i];
+          const float a1 = hf ? o[OC + 2 * i + 1] : o[2 * i + 1];
           pk[i] = sm100::pack_half2(a0 * inv, a1 * inv);
         }
-        uint4* dst = reinterpret_cast<uint4*>(orow + (DH / 2) * hf);
+        uint4* dst = reinterpret_cast<uint4*>(orow + OC * hf);
 #pragma unroll
-        for (int j = 0; j < DH / 16; ++j) dst[j] = make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+        for (int j = 0; j < OC / 8; ++j) dst[j] = make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
       }
     }
   }
   sm100::tc_fence_before();
   __syncthreads();
   if (threadIdx.x == 0) ATR(2, 5);  // all stored
-  if (warp == 1) sm100::tmem_dealloc<256>(tmem);
+  if (warp == 1) sm100::tmem_dealloc<kTmemCols>(tmem);
 }
 
 template <int DH>

@@ -236,6 +236,11 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_n
   }
 }
 
+#ifndef PREDTOP_REC_AHEAD
+#define PREDTOP_REC_AHEAD 4
+#endif
+constexpr int kRecAhead = PREDTOP_REC_AHEAD;  // closure record prefetch distance (levels)
+
 // K2: closure.  grid = (G, slices); dynamic smem `smem_bytes`.
 __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, SmallCfg sc) {
   extern __shared__ __align__(16) unsigned char sm[];
@@ -332,15 +337,19 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
           }
           Rsm[(size_t)v * rs2 + j] = acc;
         }
-        r0 = first_rec(level - 4);
+        r0 = first_rec(level - kRecAhead);
         __syncwarp();
       };
-      int4 r0 = first_rec(L - 1), r1 = first_rec(L - 2), r2 = first_rec(L - 3), r3 = first_rec(L - 4);
-      for (int level = L - 1; level >= 0; level -= 4) {
-        do_level(level, r0);
-        if (level >= 1) do_level(level - 1, r1);
-        if (level >= 2) do_level(level - 2, r2);
-        if (level >= 3) do_level(level - 3, r3);
+      // records kRecAhead levels ahead (fixed registers, loop unrolled by
+      // kRecAhead): the ~100-cycle level step would otherwise wait for an L2
+      // round trip (600+ cycles) every few levels
+      int4 rr[kRecAhead];
+#pragma unroll
+      for (int i = 0; i < kRecAhead; ++i) rr[i] = first_rec(L - 1 - i);
+      for (int level = L - 1; level >= 0; level -= kRecAhead) {
+#pragma unroll
+        for (int i = 0; i < kRecAhead; ++i)
+          if (level - i >= 0) do_level(level - i, rr[i]);
       }
     }
     __syncthreads();
