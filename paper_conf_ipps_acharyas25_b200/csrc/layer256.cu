@@ -32,6 +32,18 @@
 
 namespace predtop {
 
+#ifdef PREDTOP_TRACE
+__device__ unsigned long long g_l256[16][16];  // CTA 0, tiles 0..15: clock64 at pipeline events
+#define LT(i, k)                                              \
+  do {                                                        \
+    if (blockIdx.x == 0 && (i) < 16) g_l256[i][k] = clock64(); \
+  } while (0)
+#else
+#define LT(i, k) \
+  do {           \
+  } while (0)
+#endif
+
 namespace {
 
 constexpr int D = 256;
@@ -80,7 +92,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
   __shared__ __align__(8) uint64_t o_full, o_empty, h_ready, out_full;
   __shared__ __align__(8) uint64_t f_full[2], p_ready[2];  // per acc_f buffer
   __shared__ uint32_t tmem_slot;
-  __shared__ float red[2][4][128];
+  __shared__ float red[2][4][128];   // LN1 row statistics
+  __shared__ float red2[2][4][128];  // LN2 row statistics (LN1 of the next tile may overlap their reads)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ntiles = (int)ceil_div(args.M, 128);
@@ -187,7 +200,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       };
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
         // ---- O-projection: acc = att W_o^T (acc free once LN2 of the previous tile read it)
+        LT(i, 0);
         sm100::mbar_wait(&o_empty, (i & 1) ^ 1);
+        LT(i, 1);
         sm100::tc_fence_after();
         for (int a = 0; a < 2; ++a) {
           const int ia = it;  // the att unit stays until both W_o units of this half are consumed
@@ -204,12 +219,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           sm100::mma_commit(&ring_empty[ia % RS]);
         }
         sm100::mma_commit(&o_full);
+        LT(i, 2);
         // the 4 x units belong to the epilogue (it frees them after LN1).
         // Skipping them here is safe: the next unit_wait (FFN-1, after
         // h_ready) is on a phase whose predecessor the epilogue consumed
         it += 4;
         // ---- FFN: acc holds h + b_2, AH holds h (written by the epilogue after LN1)
         sm100::mbar_wait(&h_ready, i & 1);
+        LT(i, 3);
         sm100::tc_fence_after();
         auto ffn1 = [&](int j) {
           const uint32_t dst = acc_f + (uint32_t)((j & 1) * FC);
@@ -246,6 +263,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           }
         }
         sm100::mma_commit(&out_full);
+        LT(i, 4);
       }
     }
   } else {
@@ -266,36 +284,37 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       // the previous phase of each x unit completed, so the parity wait is
       // never two phases ahead (it would alias and return at once)
       sm100::mbar_wait(&o_full, i & 1);
+      if (leader) LT(i, 5);
       const int xit = i * UPT + 6;
       const int itk = xit + cg;
       sm100::mbar_wait(&ring_full[itk % RS], (itk / RS) & 1);
+      if (leader) LT(i, 6);
       sm100::tc_fence_after();
       const unsigned char* xu = ring + (itk % RS) * UNIT;  // columns [64cg, +64): two [128 x 32] fp32 boxes
-      auto z_piece = [&](int k, float (&z)[16]) {           // columns 64cg + 16k ..
-        sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
-        const unsigned char* bx = xu + (k >> 1) * KSL;
+      // z = acc + x + b_o for this thread's 64 columns, kept in registers
+      // across the statistics barrier (one TMEM read: all four loads in
+      // flight, one wait)
+      float z[64];
+      sm100::tmem_ld<64>(acc + lrow + 64 * cg, z);
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          const float4 v = *reinterpret_cast<const float4*>(bx + sm100::swz<128>(r, 4 * (k & 1) + c));
-          const float4 bo = __ldg(reinterpret_cast<const float4*>(p_bo + 64 * cg + 16 * k + 4 * c));
-          z[4 * c] += v.x + bo.x;
-          z[4 * c + 1] += v.y + bo.y;
-          z[4 * c + 2] += v.z + bo.z;
-          z[4 * c + 3] += v.w + bo.w;
+      for (int k = 0; k < 2; ++k)
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          const float4 v = *reinterpret_cast<const float4*>(xu + k * KSL + sm100::swz<128>(r, c));
+          const float4 bo = __ldg(reinterpret_cast<const float4*>(p_bo + 64 * cg + 32 * k + 4 * c));
+          float* zz = z + 32 * k + 4 * c;
+          zz[0] += v.x + bo.x;
+          zz[1] += v.y + bo.y;
+          zz[2] += v.z + bo.z;
+          zz[3] += v.w + bo.w;
         }
-      };
       float mean, rstd;
       {
         float s = 0.f, sq = 0.f;
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          float z[16];
-          z_piece(k, z);
-#pragma unroll
-          for (int e = 0; e < 16; ++e) {
-            s += z[e];
-            sq = fmaf(z[e], z[e], sq);
-          }
+        for (int e = 0; e < 64; ++e) {
+          s += z[e];
+          sq = fmaf(z[e], z[e], sq);
         }
         red[0][cg][r] = s;
         red[1][cg][r] = sq;
@@ -314,8 +333,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       unsigned char* hs = sAH + cg * KSL;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
-        float z[16];
-        z_piece(k, z);
+        float* zk = z + 16 * k;
         uint32_t hb[16], hp[8];
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
@@ -326,12 +344,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           const float gg[4] = {g.x, g.y, g.z, g.w}, bb[4] = {be.x, be.y, be.z, be.w}, b22[4] = {b2.x, b2.y, b2.z, b2.w};
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            z[4 * c + e] = (z[4 * c + e] - mean) * rstd * gg[e] + bb[e];
-            hb[4 * c + e] = __float_as_uint(z[4 * c + e] + b22[e]);
+            zk[4 * c + e] = (zk[4 * c + e] - mean) * rstd * gg[e] + bb[e];
+            hb[4 * c + e] = __float_as_uint(zk[4 * c + e] + b22[e]);
           }
         }
 #pragma unroll
-        for (int e = 0; e < 8; ++e) hp[e] = sm100::pack_half2(z[2 * e], z[2 * e + 1]);
+        for (int e = 0; e < 8; ++e) hp[e] = sm100::pack_half2(zk[2 * e], zk[2 * e + 1]);
         *reinterpret_cast<uint4*>(hs + sm100::swz<128>(r, 2 * k)) = make_uint4(hp[0], hp[1], hp[2], hp[3]);
         *reinterpret_cast<uint4*>(hs + sm100::swz<128>(r, 2 * k + 1)) = make_uint4(hp[4], hp[5], hp[6], hp[7]);
         sm100::tmem_st16(acc + lrow + 64 * cg + 16 * k, hb);
@@ -343,6 +361,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       if (leader) {
         for (int k = 0; k < 4; ++k) sm100::mbar_arrive(&ring_empty[(xit + k) % RS]);  // x units free
         sm100::mbar_arrive(&h_ready);
+        LT(i, 8);
       }
       // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 pairs back into acc_f
       for (int j = 0; j < NJ; ++j) {
@@ -371,25 +390,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       // ---- LN2: z = acc (= h + b_2 + FFN(h)), two passes over 16-column
       // pieces of TMEM; x' (fp32) and its fp16 shadow go straight from
       // registers to global memory (the stores drain during the next tile)
+      if (leader) LT(i, 9);
       sm100::mbar_wait(&out_full, i & 1);
+      if (leader) LT(i, 10);
       sm100::tc_fence_after();
+      // the row's 64 values in registers (one TMEM read), so acc is free for
+      // the next tile's O-projection as soon as every thread has read it
+      sm100::tmem_ld<64>(acc + lrow + 64 * cg, z);
+      sm100::tc_fence_before();
       {
         float s = 0.f, sq = 0.f;
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          float z[16];
-          sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
-#pragma unroll
-          for (int e = 0; e < 16; ++e) {
-            s += z[e];
-            sq = fmaf(z[e], z[e], sq);
-          }
+        for (int e = 0; e < 64; ++e) {
+          s += z[e];
+          sq = fmaf(z[e], z[e], sq);
         }
-        red[0][cg][r] = s;
-        red[1][cg][r] = sq;
-        sm100::named_bar<kEpi>(1);
-        mean = ((red[0][0][r] + red[0][1][r]) + (red[0][2][r] + red[0][3][r])) * (1.0f / D);
-        const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
+        red2[0][cg][r] = s;
+        red2[1][cg][r] = sq;
+        sm100::named_bar<kEpi>(1);  // every epilogue thread has read acc (and written red) ...
+        if (leader) sm100::mbar_arrive(&o_empty);  // ... so the next O-projection may overwrite it
+        mean = ((red2[0][0][r] + red2[0][1][r]) + (red2[0][2][r] + red2[0][3][r])) * (1.0f / D);
+        const float ex2 = ((red2[1][0][r] + red2[1][1][r]) + (red2[1][2][r] + red2[1][3][r])) * (1.0f / D);
         rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
       }
       // pass B: x' piece k (rows 32q.., columns 64cg + 16k ..) -> this warp's
@@ -397,31 +418,30 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       // the staging is rewritten once the previous piece's stores have read it
       unsigned char* s32 = sStg + ew * (STG32 + STG16);
       unsigned char* s16 = s32 + STG32;
-#pragma unroll 1
+#pragma unroll
       for (int k = 0; k < 4; ++k) {
-        float z[16];
-        sm100::tmem_ld16(acc + lrow + 64 * cg + 16 * k, z);
+        float* zk = z + 16 * k;
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
           const int col = 64 * cg + 16 * k + 4 * c;
           const float4 g = __ldg(reinterpret_cast<const float4*>(p_g2 + col));
           const float4 be = __ldg(reinterpret_cast<const float4*>(p_be2 + col));
-          z[4 * c] = (z[4 * c] - mean) * rstd * g.x + be.x;
-          z[4 * c + 1] = (z[4 * c + 1] - mean) * rstd * g.y + be.y;
-          z[4 * c + 2] = (z[4 * c + 2] - mean) * rstd * g.z + be.z;
-          z[4 * c + 3] = (z[4 * c + 3] - mean) * rstd * g.w + be.w;
+          zk[4 * c] = (zk[4 * c] - mean) * rstd * g.x + be.x;
+          zk[4 * c + 1] = (zk[4 * c + 1] - mean) * rstd * g.y + be.y;
+          zk[4 * c + 2] = (zk[4 * c + 2] - mean) * rstd * g.z + be.z;
+          zk[4 * c + 3] = (zk[4 * c + 3] - mean) * rstd * g.w + be.w;
         }
         if (lane == 0) sm100::bulk_wait_read0();
         __syncwarp();
 #pragma unroll
         for (int c = 0; c < 4; ++c)
           *reinterpret_cast<float4*>(s32 + lane * 64 + 16 * (c ^ ((lane >> 1) & 3))) =
-              make_float4(z[4 * c], z[4 * c + 1], z[4 * c + 2], z[4 * c + 3]);
+              make_float4(zk[4 * c], zk[4 * c + 1], zk[4 * c + 2], zk[4 * c + 3]);
 #pragma unroll
         for (int c = 0; c < 2; ++c)
           *reinterpret_cast<uint4*>(s16 + lane * 32 + 16 * (c ^ ((lane >> 2) & 1))) =
-              make_uint4(sm100::pack_half2(z[8 * c], z[8 * c + 1]), sm100::pack_half2(z[8 * c + 2], z[8 * c + 3]),
-                         sm100::pack_half2(z[8 * c + 4], z[8 * c + 5]), sm100::pack_half2(z[8 * c + 6], z[8 * c + 7]));
+              make_uint4(sm100::pack_half2(zk[8 * c], zk[8 * c + 1]), sm100::pack_half2(zk[8 * c + 2], zk[8 * c + 3]),
+                         sm100::pack_half2(zk[8 * c + 4], zk[8 * c + 5]), sm100::pack_half2(zk[8 * c + 6], zk[8 * c + 7]));
         sm100::fence_proxy_async();
         __syncwarp();
         if (lane == 0) {
@@ -430,9 +450,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           sm100::bulk_commit();
         }
       }
-      sm100::tc_fence_before();
-      sm100::named_bar<kEpi>(1);  // every epilogue thread has read acc (and red) ...
-      if (leader) sm100::mbar_arrive(&o_empty);  // ... so the next O-projection may overwrite it
+
+      if (leader) LT(i, 11);
     }
   }
   if (warp >= 2 && lane == 0) sm100::bulk_wait0();
@@ -472,3 +491,9 @@ predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __hal
 }
 
 }  // namespace predtop
+
+#ifdef PREDTOP_TRACE
+extern "C" PREDTOP_API int predtop_debug_l256_trace(unsigned long long* out) {
+  return cudaMemcpyFromSymbol(out, predtop::g_l256, sizeof(predtop::g_l256)) == cudaSuccess ? 0 : -7;
+}
+#endif
