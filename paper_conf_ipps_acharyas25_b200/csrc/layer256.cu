@@ -44,6 +44,10 @@ __device__ unsigned long long g_l256[16][16];  // CTA 0, tiles 0..15: clock64 at
   } while (0)
 #endif
 
+#ifndef PREDTOP_L256_STG
+#define PREDTOP_L256_STG 0  // 1: x' leaves through coalesced STG instead of TMA stores (A/B)
+#endif
+
 namespace {
 
 constexpr int D = 256;
@@ -80,13 +84,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
   unsigned char* ring = base;               // RS x 32 KB
   unsigned char* sAH = ring + RS * UNIT;    // [4 K-slices][128 rows x 64] fp16, SW128
   unsigned char* sStg = sAH;                // x' staging (per epilogue warp STG32 + STG16), once h is dead
-  // biases and LN parameters stay in global memory (L1-resident, __ldg)
-  const float* __restrict__ p_bo = args.bo;
-  const float* __restrict__ p_g1 = args.g1;
-  const float* __restrict__ p_be1 = args.be1;
-  const float* __restrict__ p_b2 = args.b2;
-  const float* __restrict__ p_g2 = args.g2;
-  const float* __restrict__ p_be2 = args.be2;
+  // the D-length biases and LN parameters in shared memory (broadcast
+  // reads; through L1 they are evicted by the epilogue's spill traffic and
+  // every LayerNorm piece waits on L2); b_1 (d_ff long, read once per FFN
+  // chunk) stays in global memory
+  __shared__ __align__(16) float sPar[6][D];
+  const float* p_bo = sPar[0];
+  const float* p_g1 = sPar[1];
+  const float* p_be1 = sPar[2];
+  const float* p_b2 = sPar[3];
+  const float* p_g2 = sPar[4];
+  const float* p_be2 = sPar[5];
   const float* __restrict__ p_b1 = args.b1;
   __shared__ __align__(8) uint64_t ring_full[RS], ring_empty[RS];
   __shared__ __align__(8) uint64_t o_full, o_empty, h_ready, out_full;
@@ -273,6 +281,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
     const int r = q * 32 + lane;  // tile row of this thread (TMEM lane)
     const uint32_t lrow = (uint32_t)(q * 32) << 16;
     const bool leader = (ew == 0 && lane == 0);
+    {
+      const float* src[6] = {args.bo, args.g1, args.be1, args.b2, args.g2, args.be2};
+#pragma unroll
+      for (int k = 0; k < 6; ++k)
+        if (ew * 32 + lane < D) sPar[k][ew * 32 + lane] = src[k][ew * 32 + lane];
+      sm100::named_bar<kEpi>(1);
+    }
     int i = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
       const int m0 = t * 128;
@@ -301,7 +316,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
           const float4 v = *reinterpret_cast<const float4*>(xu + k * KSL + sm100::swz<128>(r, c));
-          const float4 bo = __ldg(reinterpret_cast<const float4*>(p_bo + 64 * cg + 32 * k + 4 * c));
+          const float4 bo = (*reinterpret_cast<const float4*>(p_bo + 64 * cg + 32 * k + 4 * c));
           float* zz = z + 32 * k + 4 * c;
           zz[0] += v.x + bo.x;
           zz[1] += v.y + bo.y;
@@ -318,11 +333,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         }
         red[0][cg][r] = s;
         red[1][cg][r] = sq;
+        if (leader) LT(i, 7);
         // h overwrites all of AH below: every warp's x' stores of the
         // previous tile (staged in AH) must have read it (before the barrier)
         if (lane == 0) sm100::bulk_wait_read0();
         __syncwarp();
         sm100::named_bar<kEpi>(1);
+        if (leader) LT(i, 12);
         mean = ((red[0][0][r] + red[0][1][r]) + (red[0][2][r] + red[0][3][r])) * (1.0f / D);
         const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
         rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
@@ -338,9 +355,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
           const int col = 64 * cg + 16 * k + 4 * c;
-          const float4 g = __ldg(reinterpret_cast<const float4*>(p_g1 + col));
-          const float4 be = __ldg(reinterpret_cast<const float4*>(p_be1 + col));
-          const float4 b2 = __ldg(reinterpret_cast<const float4*>(p_b2 + col));
+          const float4 g = (*reinterpret_cast<const float4*>(p_g1 + col));
+          const float4 be = (*reinterpret_cast<const float4*>(p_be1 + col));
+          const float4 b2 = (*reinterpret_cast<const float4*>(p_b2 + col));
           const float gg[4] = {g.x, g.y, g.z, g.w}, bb[4] = {be.x, be.y, be.z, be.w}, b22[4] = {b2.x, b2.y, b2.z, b2.w};
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
@@ -354,6 +371,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         *reinterpret_cast<uint4*>(hs + sm100::swz<128>(r, 2 * k + 1)) = make_uint4(hp[4], hp[5], hp[6], hp[7]);
         sm100::tmem_st16(acc + lrow + 64 * cg + 16 * k, hb);
       }
+      if (leader) LT(i, 13);
       sm100::tmem_wait_st();
       sm100::fence_proxy_async();  // h writes (and the x reads) before the async proxy
       sm100::tc_fence_before();
@@ -408,6 +426,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         red2[0][cg][r] = s;
         red2[1][cg][r] = sq;
         sm100::named_bar<kEpi>(1);  // every epilogue thread has read acc (and written red) ...
+        if (leader) LT(i, 14);
         if (leader) sm100::mbar_arrive(&o_empty);  // ... so the next O-projection may overwrite it
         mean = ((red2[0][0][r] + red2[0][1][r]) + (red2[0][2][r] + red2[0][3][r])) * (1.0f / D);
         const float ex2 = ((red2[1][0][r] + red2[1][1][r]) + (red2[1][2][r] + red2[1][3][r])) * (1.0f / D);
@@ -424,14 +443,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
           const int col = 64 * cg + 16 * k + 4 * c;
-          const float4 g = __ldg(reinterpret_cast<const float4*>(p_g2 + col));
-          const float4 be = __ldg(reinterpret_cast<const float4*>(p_be2 + col));
+          const float4 g = (*reinterpret_cast<const float4*>(p_g2 + col));
+          const float4 be = (*reinterpret_cast<const float4*>(p_be2 + col));
           zk[4 * c] = (zk[4 * c] - mean) * rstd * g.x + be.x;
           zk[4 * c + 1] = (zk[4 * c + 1] - mean) * rstd * g.y + be.y;
           zk[4 * c + 2] = (zk[4 * c + 2] - mean) * rstd * g.z + be.z;
           zk[4 * c + 3] = (zk[4 * c + 3] - mean) * rstd * g.w + be.w;
         }
+#if !PREDTOP_L256_STG
         if (lane == 0) sm100::bulk_wait_read0();
+#endif
         __syncwarp();
 #pragma unroll
         for (int c = 0; c < 4; ++c)
@@ -442,6 +463,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           *reinterpret_cast<uint4*>(s16 + lane * 32 + 16 * (c ^ ((lane >> 2) & 1))) =
               make_uint4(sm100::pack_half2(zk[8 * c], zk[8 * c + 1]), sm100::pack_half2(zk[8 * c + 2], zk[8 * c + 3]),
                          sm100::pack_half2(zk[8 * c + 4], zk[8 * c + 5]), sm100::pack_half2(zk[8 * c + 6], zk[8 * c + 7]));
+#if PREDTOP_L256_STG
+        __syncwarp();
+        // read back transposed: fp32 -> lane (row l/4 + 8 rr, 16-byte chunk
+        // l%4), fp16 -> (row l/2 + 16 rr, chunk l%2): every store instruction
+        // writes whole 64 / 32-byte row segments
+#pragma unroll
+        for (int rr = 0; rr < 4; ++rr) {
+          const int rw = (lane >> 2) + 8 * rr, ch = lane & 3;
+          const float4 v = *reinterpret_cast<const float4*>(s32 + rw * 64 + 16 * (ch ^ ((rw >> 1) & 3)));
+          if (m0 + 32 * q + rw < args.M)
+            *reinterpret_cast<float4*>(args.x32 + (int64_t)(m0 + 32 * q + rw) * D + 64 * cg + 16 * k + 4 * ch) = v;
+        }
+#pragma unroll
+        for (int rr = 0; rr < 2; ++rr) {
+          const int rw = (lane >> 1) + 16 * rr, ch = lane & 1;
+          const uint4 v = *reinterpret_cast<const uint4*>(s16 + rw * 32 + 16 * (ch ^ ((rw >> 2) & 1)));
+          if (m0 + 32 * q + rw < args.M)
+            *reinterpret_cast<uint4*>(args.x16 + (int64_t)(m0 + 32 * q + rw) * D + 64 * cg + 16 * k + 8 * ch) = v;
+        }
+        __syncwarp();
+#else
         sm100::fence_proxy_async();
         __syncwarp();
         if (lane == 0) {
@@ -449,6 +491,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
           sm100::tma_store_2d(&mp.x16out, s16, 64 * cg + 16 * k, m0 + 32 * q);
           sm100::bulk_commit();
         }
+#endif
       }
 
       if (leader) LT(i, 11);

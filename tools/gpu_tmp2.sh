@@ -1,0 +1,2 @@
+PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_stg.so timeout 200 python -m pytest tests -m gpu -q -x --timeout 100 -k "moe" 2>&1 | tail -1
+bash tools/gpu_ab.sh stg 2>&1 | grep -v "^$"

@@ -28,8 +28,8 @@ def main():
     assert pt.lib().predtop_debug_l256_trace(ctypes.cast(buf, ctypes.c_void_p)) == 0
     t = np.frombuffer(buf, dtype=np.uint64).reshape(16, 16).astype(np.int64)
     t0 = t[0, 0]
-    names = ["mma:start", "o_empty", "oproj_issued", "h_ready", "ffn_issued", "epi:o_full", "x_ready", "-",
-             "h_written", "ffn_done", "out_full", "ln2_acc_read"]
+    names = ["mma:start", "o_empty", "oproj_issued", "h_ready", "ffn_issued", "epi:o_full", "x_ready", "ln1_stats",
+             "h_written", "ffn_done", "out_full", "ln2_done", "ln1_bar", "ln1_passB", "ln2_bar"]
     print("tile " + " ".join(f"{n:>12s}" for n in names))
     for i in range(16):
         print(f"{i:4d} " + " ".join(f"{(t[i, k] - t0) if t[i, k] else 0:12d}" for k in range(len(names))))
