@@ -34,11 +34,24 @@ namespace predtop {
 
 #ifdef PREDTOP_TRACE
 __device__ unsigned long long g_l256[16][16];  // CTA 0, tiles 0..15: clock64 at pipeline events
-#define LT(i, k)                                              \
-  do {                                                        \
-    if (blockIdx.x == 0 && (i) < 16) g_l256[i][k] = clock64(); \
+__device__ unsigned long long g_l256w[16][16][8];  // CTA 0, tiles 0..15, epilogue warps: LN events
+__device__ __forceinline__ unsigned long long l256_clk() {  // memory clobber: stays between the loads/stores around it
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%clock64;" : "=l"(t)::"memory");
+  return t;
+}
+#define LT(i, k)                                                 \
+  do {                                                           \
+    if (blockIdx.x == 0 && (i) < 16) g_l256[i][k] = l256_clk(); \
+  } while (0)
+#define LW(i, k)                                                                  \
+  do {                                                                            \
+    if (blockIdx.x == 0 && (i) < 16 && lane == 0) g_l256w[i][ew][k] = l256_clk(); \
   } while (0)
 #else
+#define LW(i, k) \
+  do {           \
+  } while (0)
 #define LT(i, k) \
   do {           \
   } while (0)
@@ -299,11 +312,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       // the previous phase of each x unit completed, so the parity wait is
       // never two phases ahead (it would alias and return at once)
       sm100::mbar_wait(&o_full, i & 1);
-      if (leader) LT(i, 5);
+      if (leader) LT(i, 5); LW(i, 0);
       const int xit = i * UPT + 6;
       const int itk = xit + cg;
       sm100::mbar_wait(&ring_full[itk % RS], (itk / RS) & 1);
-      if (leader) LT(i, 6);
+      if (leader) LT(i, 6); LW(i, 1);
       sm100::tc_fence_after();
       const unsigned char* xu = ring + (itk % RS) * UNIT;  // columns [64cg, +64): two [128 x 32] fp32 boxes
       // z = acc + x + b_o for this thread's 64 columns, kept in registers
@@ -333,13 +346,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         }
         red[0][cg][r] = s;
         red[1][cg][r] = sq;
-        if (leader) LT(i, 7);
+        if (leader) LT(i, 7); LW(i, 2);
         // h overwrites all of AH below: every warp's x' stores of the
         // previous tile (staged in AH) must have read it (before the barrier)
         if (lane == 0) sm100::bulk_wait_read0();
         __syncwarp();
         sm100::named_bar<kEpi>(1);
-        if (leader) LT(i, 12);
+        if (leader) LT(i, 12); LW(i, 3);
         mean = ((red[0][0][r] + red[0][1][r]) + (red[0][2][r] + red[0][3][r])) * (1.0f / D);
         const float ex2 = ((red[1][0][r] + red[1][1][r]) + (red[1][2][r] + red[1][3][r])) * (1.0f / D);
         rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
@@ -371,7 +384,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         *reinterpret_cast<uint4*>(hs + sm100::swz<128>(r, 2 * k + 1)) = make_uint4(hp[4], hp[5], hp[6], hp[7]);
         sm100::tmem_st16(acc + lrow + 64 * cg + 16 * k, hb);
       }
-      if (leader) LT(i, 13);
+      if (leader) LT(i, 13); LW(i, 4);
       sm100::tmem_wait_st();
       sm100::fence_proxy_async();  // h writes (and the x reads) before the async proxy
       sm100::tc_fence_before();
@@ -381,6 +394,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         sm100::mbar_arrive(&h_ready);
         LT(i, 8);
       }
+      LW(i, 5);
       // ---- FFN chunks: ReLU(acc_f + b_1) -> fp16 pairs back into acc_f
       for (int j = 0; j < NJ; ++j) {
         const int cj = cbase + j;
@@ -410,7 +424,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       // registers to global memory (the stores drain during the next tile)
       if (leader) LT(i, 9);
       sm100::mbar_wait(&out_full, i & 1);
-      if (leader) LT(i, 10);
+      if (leader) LT(i, 10); LW(i, 6);
       sm100::tc_fence_after();
       // the row's 64 values in registers (one TMEM read), so acc is free for
       // the next tile's O-projection as soon as every thread has read it
@@ -494,7 +508,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
 #endif
       }
 
-      if (leader) LT(i, 11);
+      if (leader) LT(i, 11); LW(i, 7);
     }
   }
   if (warp >= 2 && lane == 0) sm100::bulk_wait0();
@@ -538,5 +552,8 @@ predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __hal
 #ifdef PREDTOP_TRACE
 extern "C" PREDTOP_API int predtop_debug_l256_trace(unsigned long long* out) {
   return cudaMemcpyFromSymbol(out, predtop::g_l256, sizeof(predtop::g_l256)) == cudaSuccess ? 0 : -7;
+}
+extern "C" PREDTOP_API int predtop_debug_l256_trace_w(unsigned long long* out) {
+  return cudaMemcpyFromSymbol(out, predtop::g_l256w, sizeof(predtop::g_l256w)) == cudaSuccess ? 0 : -7;
 }
 #endif
