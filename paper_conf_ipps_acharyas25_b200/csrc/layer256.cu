@@ -34,7 +34,7 @@ namespace predtop {
 
 #ifdef PREDTOP_TRACE
 __device__ unsigned long long g_l256[16][16];  // CTA 0, tiles 0..15: clock64 at pipeline events
-__device__ unsigned long long g_l256w[16][16][8];  // CTA 0, tiles 0..15, epilogue warps: LN events
+__device__ unsigned long long g_l256w[16][16][12];  // CTA 0, tiles 0..15, epilogue warps: LN events
 __device__ __forceinline__ unsigned long long l256_clk() {  // memory clobber: stays between the loads/stores around it
   unsigned long long t;
   asm volatile("mov.u64 %0, %%clock64;" : "=l"(t)::"memory");
@@ -57,6 +57,9 @@ __device__ __forceinline__ unsigned long long l256_clk() {  // memory clobber: s
   } while (0)
 #endif
 
+#ifndef PREDTOP_L256_OUTW
+#define PREDTOP_L256_OUTW 1  // x' leaves in 128-byte-row boxes (0: 16-column pieces)
+#endif
 #ifndef PREDTOP_L256_STG
 #define PREDTOP_L256_STG 0  // 1: x' leaves through coalesced STG instead of TMA stores (A/B)
 #endif
@@ -76,6 +79,8 @@ constexpr int kMaxFF = 4096;
 constexpr int STG32 = 32 * 16 * 4;    // per-warp x' staging in AH: [32 rows x 16 fp32] (SW64)
 constexpr int STG16 = 32 * 16 * 2;    //                           [32 rows x 16 fp16] (SW32)
 static_assert(kEpiWarps * (STG32 + STG16) <= AHB, "x' staging lives in the h tile");
+constexpr int STGW = 32 * 128;       // PREDTOP_L256_OUTW: one [32 rows x 128 B] SW128 box per warp
+static_assert(kEpiWarps * STGW <= AHB, "x' staging lives in the h tile");
 constexpr int SMEM = 1024 + RS * UNIT + AHB;
 static_assert(SMEM <= 227 * 1024, "one CTA per SM");
 
@@ -440,12 +445,61 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         red2[0][cg][r] = s;
         red2[1][cg][r] = sq;
         sm100::named_bar<kEpi>(1);  // every epilogue thread has read acc (and written red) ...
-        if (leader) LT(i, 14);
+        if (leader) LT(i, 14); LW(i, 8);
         if (leader) sm100::mbar_arrive(&o_empty);  // ... so the next O-projection may overwrite it
         mean = ((red2[0][0][r] + red2[0][1][r]) + (red2[0][2][r] + red2[0][3][r])) * (1.0f / D);
         const float ex2 = ((red2[1][0][r] + red2[1][1][r]) + (red2[1][2][r] + red2[1][3][r])) * (1.0f / D);
         rstd = rsqrtf(fmaxf(ex2 - mean * mean, 0.f) + args.eps);
       }
+#if PREDTOP_L256_OUTW
+      // pass B: normalise the 64 values in place, then three 128-byte-row
+      // TMA boxes through this warp's 4 KB of AH (SW128: conflict-free
+      // writes): x' columns [64cg, +32), [64cg + 32, +32) in fp32, then all
+      // 64 columns in fp16.  Wide rows: the TMA store cost grows with the
+      // number of box rows (16-column pieces took 2.7x as many)
+#pragma unroll
+      for (int c = 0; c < 16; ++c) {
+        const int col = 64 * cg + 4 * c;
+        const float4 g = (*reinterpret_cast<const float4*>(p_g2 + col));
+        const float4 be = (*reinterpret_cast<const float4*>(p_be2 + col));
+        z[4 * c] = (z[4 * c] - mean) * rstd * g.x + be.x;
+        z[4 * c + 1] = (z[4 * c + 1] - mean) * rstd * g.y + be.y;
+        z[4 * c + 2] = (z[4 * c + 2] - mean) * rstd * g.z + be.z;
+        z[4 * c + 3] = (z[4 * c + 3] - mean) * rstd * g.w + be.w;
+      }
+      LW(i, 9);
+      unsigned char* sw = sStg + ew * STGW;
+#pragma unroll
+      for (int p = 0; p < 3; ++p) {
+        if (p > 0) {
+          if (lane == 0) sm100::bulk_wait_read0();
+          __syncwarp();
+          if (p == 1) LW(i, 10);
+          if (p == 2) LW(i, 11);
+        }
+        if (p < 2) {
+#pragma unroll
+          for (int c = 0; c < 8; ++c)
+            *reinterpret_cast<float4*>(sw + sm100::swz<128>(lane, c)) =
+                make_float4(z[32 * p + 4 * c], z[32 * p + 4 * c + 1], z[32 * p + 4 * c + 2], z[32 * p + 4 * c + 3]);
+        } else {
+#pragma unroll
+          for (int c = 0; c < 8; ++c)
+            *reinterpret_cast<uint4*>(sw + sm100::swz<128>(lane, c)) =
+                make_uint4(sm100::pack_half2(z[8 * c], z[8 * c + 1]), sm100::pack_half2(z[8 * c + 2], z[8 * c + 3]),
+                           sm100::pack_half2(z[8 * c + 4], z[8 * c + 5]), sm100::pack_half2(z[8 * c + 6], z[8 * c + 7]));
+        }
+        sm100::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) {
+          if (p < 2)
+            sm100::tma_store_2d(&mp.x32out, sw, 64 * cg + 32 * p, m0 + 32 * q);
+          else
+            sm100::tma_store_2d(&mp.x16out, sw, 64 * cg, m0 + 32 * q);
+          sm100::bulk_commit();
+        }
+      }
+#else
       // pass B: x' piece k (rows 32q.., columns 64cg + 16k ..) -> this warp's
       // staging (SW64 fp32 / SW32 fp16, the TMA box layouts) -> TMA stores;
       // the staging is rewritten once the previous piece's stores have read it
@@ -508,6 +562,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
 #endif
       }
 
+#endif
       if (leader) LT(i, 11); LW(i, 7);
     }
   }
@@ -534,8 +589,9 @@ predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __hal
   T256Maps mp;
   if (!encode_tma_2d(&mp.att, att, 2, D, M, 64, 128) || !encode_tma_2d(&mp.x32in, x32, 4, D, M, 32, 128) ||
       !encode_tma_2d(&mp.wo, L.Wo, 2, D, D, 64, 256) || !encode_tma_2d(&mp.w1, L.W1, 2, D, dff, 64, FC) ||
-      !encode_tma_2d(&mp.w2, L.W2, 2, dff, D, 64, 256) || !encode_tma_2d(&mp.x32out, x32, 4, D, M, 16, 32) ||
-      !encode_tma_2d(&mp.x16out, x16, 2, D, M, 16, 32))
+      !encode_tma_2d(&mp.w2, L.W2, 2, dff, D, 64, 256) ||
+      !encode_tma_2d(&mp.x32out, x32, 4, D, M, PREDTOP_L256_OUTW ? 32 : 16, 32) ||
+      !encode_tma_2d(&mp.x16out, x16, 2, D, M, PREDTOP_L256_OUTW ? 64 : 16, 32))
     return PREDTOP_ERR_CUDA;
   T256Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
   PT_SMEM_ATTR(k_layer_tail256, SMEM);

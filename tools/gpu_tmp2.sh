@@ -1,2 +1,2 @@
-bash tools/gpu_ab.sh xtma 2>&1 | grep -v "^$"
-PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_trace.so timeout 120 python tools/l256_trace.py > gpurun_out/l256_trace.txt 2>&1; sed -n 18,50p gpurun_out/l256_trace.txt
+PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_stg2.so timeout 200 python -m pytest tests -m gpu -q -x --timeout 100 -k "moe" 2>&1 | tail -1
+bash tools/gpu_ab.sh stg2 2>&1 | grep -v "^$"

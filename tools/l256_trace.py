@@ -34,11 +34,11 @@ def main():
     for i in range(16):
         print(f"{i:4d} " + " ".join(f"{(t[i, k] - t0) if t[i, k] else 0:12d}" for k in range(len(names))))
 
-    w = (ctypes.c_ulonglong * (16 * 16 * 8))()
+    w = (ctypes.c_ulonglong * (16 * 16 * 12))()
     pt.lib().predtop_debug_l256_trace_w.argtypes = [ctypes.c_void_p]
     assert pt.lib().predtop_debug_l256_trace_w(ctypes.cast(w, ctypes.c_void_p)) == 0
-    w = np.frombuffer(w, dtype=np.uint64).reshape(16, 16, 8).astype(np.int64) - t0
-    ev = ["o_full", "x_ready", "stats", "bar1", "passB", "h_wr", "out_full", "ln2_end"]
+    w = np.frombuffer(w, dtype=np.uint64).reshape(16, 16, 12).astype(np.int64) - t0
+    ev = ["o_full", "x_ready", "stats", "bar1", "passB", "h_wr", "out_full", "ln2_end", "ln2_bar", "ln2_norm", "ln2_w1", "ln2_w2"]
     for i in range(2, 5):
         print(f"tile {i}: per-warp events (min / median / max over the 16 epilogue warps)")
         for k, n in enumerate(ev):
