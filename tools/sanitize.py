@@ -1,5 +1,5 @@
 """Small end-to-end run of every hot-path kernel for compute-sanitizer:
-tiny + 2 GPT graphs + 1 MoE-size graph through build_dag / stage_forward /
+tiny + 2 GPT graphs + 16 MoE-size graphs (187 layer-tail tiles: CTAs run several tiles) through build_dag / stage_forward /
 plan_latency, plus one training step (memcheck / racecheck / synccheck)."""
 import os
 import sys
@@ -14,7 +14,7 @@ from paper_conf_ipps_acharyas25_b200 import build, predtop as pt, synth  # noqa:
 def main():
     build.build_library()
     for name, batch in [("tiny", synth.tiny_batch()), ("gpt", synth.stage_batch("gpt", 2)),
-                        ("moe", synth.stage_batch("moe", 1))]:
+                        ("moe", synth.stage_batch("moe", 16))]:
         cfg = synth.MODEL_CONFIGS[name]
         model = pt.Model(cfg, synth.pack_weights(cfg, synth.model_weights(cfg)))
         dag = pt.Dag(pt.DeviceBatch.from_host(batch))
