@@ -471,8 +471,10 @@ def roofline(prof, work, cfg, pairs, node_total, clk, step_ms):
     traffic = None
     try:  # DRAM bytes per launch of the dominant kernel from a committed ncu capture
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-            tr = json.load(f).get(dom)
-        if tr and tr.get("config", "gpt") == cfg.get("_name", "gpt"):
+            tdb = json.load(f)
+        name = cfg.get("_name", "gpt")
+        tr = tdb.get(f"{name}/{dom}") or tdb.get(dom)
+        if tr and tr.get("config", "gpt") == name:
             traffic = tr["bytes"]
             roof["traffic_source"] = tr["source"]
             if dom == "attention":  # algorithmic bytes: q,k,v in (3d fp16) + att out (d fp16) per node
