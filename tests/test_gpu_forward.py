@@ -331,7 +331,8 @@ def test_attention_exact_row_fallback(pt, oracle_mod, parity_log, name, tc, monk
     """tcgen05 attention (attention_tc.cu) with a peaked layer-0 attention:
     W_q and b_q of layer 0 scaled by 8 (exact in fp16), so on some rows an
     allowed score exceeds the diagonal (the kernel's fixed reference m) by
-    more than 12 in log2 units and the row takes the exact CUDA-core path.
+    16 or more in log2 units: P overflows fp16, the row sum is not finite and
+    the row takes the exact CUDA-core path.
     Precondition checked on the oracle's own q, k; result within 2e-3."""
     monkeypatch.setenv("PREDTOP_ATTN_TC", tc)
     cfg = dict(synth.MODEL_CONFIGS[name])
@@ -360,7 +361,7 @@ def test_attention_exact_row_fallback(pt, oracle_mod, parity_log, name, tc, monk
         S = (q @ k.T) / np.sqrt(dh) / np.log(2.0)
         S = np.where(A, S, -np.inf)
         gap = max(gap, float((S.max(1) - np.diag(S)).max()))
-    assert gap > 13.0, gap
+    assert gap > 17.0, gap
     y, _ = _gpu_latency(pt, model, batch)
     want, cond = oracle_mod.forward_batch_cond(cfg, blob, batch)
     st = rel_err_stats(y, want, cond)
