@@ -437,26 +437,39 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
       sm100::tc_fence_after();
       if (!warp_dead) {
         const uint32_t tS = tS0 + kCh * b;
-        uint32_t p[16];
         if (__any_sync(0xffffffffu, w != 0ull)) {
           float s[32];
+          uint32_t p[16];
           sm100::tmem_ld<32>(tS, s);
-          const uint32_t wl = (uint32_t)w, wh = (uint32_t)(w >> 32);
+          // the four mask bytes of this key half in one register: byte f
+          // holds keys k with (k >> 1) & 3 == f at bit 2 (k >> 3) + (k & 1),
+          // so the pair (2i, 2i+1) sits at bits 8f + 2q, +1 (f = i & 3,
+          // q = i >> 2).  The mask is applied after the exponential, to the
+          // packed fp16 pair: x0[q] / x1[q] move bit 2q / 2q+1 of every byte to
+          // the byte's sign bit, and one sign-replicating byte permute per pair
+          // builds its 0xFFFF / 0x0000 halves (a masked score's exponential,
+          // inf included, is ANDed away)
+          const uint32_t w32 = __byte_perm((uint32_t)w, (uint32_t)(w >> 32), 0x6420);
+          uint32_t x0[4], x1[4];
 #pragma unroll
-          for (int k = 0; k < 32; ++k) {
-            const int pos = mask_pos(k);
-            const bool on = pos < 32 ? ((wl >> pos) & 1u) : ((wh >> (pos - 32)) & 1u);
-            s[k] = on ? s[k] : -INFINITY;
+          for (int q = 0; q < 4; ++q) {
+            x0[q] = w32 << (7 - 2 * q);
+            x1[q] = w32 << (6 - 2 * q);
           }
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
-            p[i] = sm100::pack_half2(ex2f(s[2 * i]), ex2f(s[2 * i + 1]));
+            const int f = i & 3, q = i >> 2;
+            // selector nibbles (result bytes 0..3): x0 byte f, x0 byte f,
+            // x1 byte f, x1 byte f, each with the sign-replicate bit 8
+            const uint32_t sel = 0xCC88u + 0x1111u * (uint32_t)f;
+            uint32_t m;
+            asm("prmt.b32 %0, %1, %2, %3;" : "=r"(m) : "r"(x0[q]), "r"(x1[q]), "r"(sel));
+            p[i] = sm100::pack_half2(ex2f(s[2 * i]), ex2f(s[2 * i + 1])) & m;
           }
+          sm100::tmem_st16(tS, p);
         } else {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) p[i] = 0u;
+          sm100::tmem_st16_zero(tS);
         }
-        sm100::tmem_st16(tS, p);
         sm100::tmem_wait_st();
         sm100::tc_fence_before();
       }
