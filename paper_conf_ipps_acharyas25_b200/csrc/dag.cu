@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(1024) k_meta(DagDev d, int G, int max_nodes) {
 // shared memory (the per-level atomicSub and the frontier reads are then
 // shared-memory round trips, not L2 ones: a deep graph runs ~11k levels)
 // and the queue is copied to global (topo) at the end.
-__global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_nodes) {
+__global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_nodes, int ecap) {
   extern __shared__ __align__(16) int32_t sm_depth[];
   const int g = blockIdx.x;
   if (d.status[g] != PREDTOP_OK) return;
@@ -187,6 +187,74 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_n
   __syncthreads();
   // Kahn, level synchronous: a node enters level l+1 when its last
   // predecessor (at level l) is retired, so its level is 1 + max pred level.
+  int lb = 0, le = 0, level = 0;
+  if (in_smem && N < 65536 && E <= ecap) {
+    // Warp mode: the CSR as 16-bit arrays in shared memory and ONE warp
+    // walking the levels with warp barriers (ballot + prefix-popcount queue
+    // appends): deep graphs (16k nodes: ~11k levels of one or two nodes)
+    // are a chain of dependent level steps, each a few shared-memory round
+    // trips instead of global loads and two CTA barriers.
+    uint16_t* topo16 = reinterpret_cast<uint16_t*>(sm_depth + smem_nodes);
+    uint16_t* soff16 = topo16 + smem_nodes;
+    uint16_t* succ16 = soff16 + smem_nodes + 1;
+    for (int v = tid; v <= N; v += nt) soff16[v] = (uint16_t)soff[v];
+    for (int e = tid; e < E; e += nt) succ16[e] = (uint16_t)succ[e];
+    __syncthreads();
+    if (tid < 32) {
+      const int lane = tid;
+      const uint32_t lt = (1u << lane) - 1u;
+      int tail = 0;
+      for (int base = 0; base < N; base += 32) {
+        const int v = base + lane;
+        const bool z = v < N && indeg[v] == 0;
+        const uint32_t bal = __ballot_sync(0xffffffffu, z);
+        if (z) {
+          topo16[tail + __popc(bal & lt)] = (uint16_t)v;
+          depth[v] = 0;
+        }
+        tail += __popc(bal);
+      }
+      if (lane == 0) lptr[0] = 0;
+      __syncwarp();
+      int wb = 0, we = tail, wl = 0;
+      while (wb < we) {
+        for (int i0 = wb; i0 < we; i0 += 32) {
+          int k = 0, kend = 0;
+          if (i0 + lane < we) {
+            const int v = topo16[i0 + lane];
+            k = soff16[v];
+            kend = soff16[v + 1];
+          }
+          while (__any_sync(0xffffffffu, k < kend)) {
+            int w = 0;
+            bool ready = false;
+            if (k < kend) {
+              w = succ16[k++];
+              ready = atomicSub(&indeg[w], 1) == 1;
+            }
+            const uint32_t bal = __ballot_sync(0xffffffffu, ready);
+            if (ready) {
+              topo16[tail + __popc(bal & lt)] = (uint16_t)w;
+              depth[w] = wl + 1;
+            }
+            tail += __popc(bal);
+          }
+        }
+        __syncwarp();
+        wb = we;
+        we = tail;
+        ++wl;
+        if (lane == 0) lptr[wl] = wb;
+      }
+      if (lane == 0) { s_tail = we; sh32[0] = wl; }
+    }
+    __syncthreads();
+    le = s_tail;
+    level = sh32[0];
+    for (int i = tid; i < le; i += nt) topo_g[i] = topo16[i];
+    __syncthreads();
+    topo = topo_g;
+  } else {
   for (int v = tid; v < N; v += nt)
     if (indeg[v] == 0) {
       const int p = atomicAdd(&s_tail, 1);
@@ -194,7 +262,7 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_n
       depth[v] = 0;
     }
   __syncthreads();
-  int lb = 0, le = s_tail, level = 0;
+  le = s_tail;
   if (tid == 0) lptr[0] = 0;
   while (lb < le) {
     for (int i = lb + tid; i < le; i += nt) {
@@ -215,9 +283,10 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_n
     if (tid == 0) lptr[level] = lb;
     __syncthreads();
   }
-  if (tid == 0) d.num_levels[g] = level;
   if (in_smem)
     for (int i = tid; i < le; i += nt) topo_g[i] = topo[i];
+  }  // block-synchronous mode
+  if (tid == 0) d.num_levels[g] = level;
   if (le == N) {  // closure records in topo order: node, degree, first four successors inline
     int4* rec = d.rec + n0;
     for (int i = tid; i < N; i += nt) {
@@ -455,6 +524,131 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
     x = (lane & sh) ? ((x & ~m) | ((y >> sh) & m)) : ((x & m) | ((y << sh) & ~m));
   }
   return x;
+}
+
+// K2 for deep graphs (the batch's largest graph has more than kDeepNodes
+// nodes, k = infinity): 16-bit column chains.  Column j of R[v] only reads
+// column j of the successors' rows, so every 16-bit column of R is an
+// independent chain over the levels (deepest first).  A chain keeps its
+// column for all N rows in shared memory (2 N bytes) and is walked by one
+// warp: `cpb` chains per CTA, one CTA per SM, so the 4 W chains of a 16k-node
+// graph (1024) run in ONE wave of 147 CTAs (64-bit column slices of 8 N bytes
+// fit one per SM: two waves).  The walk is a chain of dependent level steps
+// (~N/1.5 levels), so the number of chains in flight is what matters.  Level
+// records (node, degree, first four successors; built by k_depth in topo
+// order) and level bounds are prefetched kRecAhead levels ahead.
+constexpr int kDeepNodes = 6144;
+#ifndef PREDTOP_REC_AHEAD16
+#define PREDTOP_REC_AHEAD16 4
+#endif
+constexpr int kRecAhead16 = PREDTOP_REC_AHEAD16;  // record prefetch distance (levels): ~L2 latency / level step
+__global__ void __launch_bounds__(256) k_closure16(DagDev d, SmallCfg sc, int cpb) {
+  extern __shared__ __align__(16) unsigned char sm_c16[];
+  uint16_t* Rs = reinterpret_cast<uint16_t*>(sm_c16);  // [cpb][N]
+  const int g = blockIdx.x;
+  const int64_t n0 = d.node_ptr[g];
+  const int N = (int)(d.node_ptr[g + 1] - n0);
+  if (is_small(N, (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]), sc)) return;
+  const int st = d.status[g];
+  if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;  // no rows
+  const int W = 2 * ((N + 127) / 128), nch = 4 * W;
+  const int c0 = blockIdx.y * cpb;
+  if (c0 >= nch) return;
+  const int act = min(cpb, nch - c0);
+  uint16_t* R16 = reinterpret_cast<uint16_t*>(d.R + d.row_off[g]);
+  const int tid = threadIdx.x, nt = blockDim.x, warp = tid >> 5, lane = tid & 31;
+  if (st != PREDTOP_OK) {  // device-detected error: rows are defined as zero
+    for (int64_t it = tid; it < (int64_t)N * act; it += nt)
+      R16[(it / act) * nch + c0 + it % act] = 0;
+    return;
+  }
+  for (int64_t it = tid; it < (int64_t)N * act; it += nt) Rs[it] = 0;
+  __syncthreads();
+  if (warp < act) {
+    const int L = d.num_levels[g];
+    const int32_t* lp = d.level_ptr + n0 + g;
+    const int32_t* soff = d.succ_off + n0 + g;
+    const int32_t* succ = d.succ + d.edge_ptr[g];
+    const int4* rec = d.rec + n0;
+    uint16_t* col = Rs + (size_t)warp * N;
+    const uint32_t cj = (uint32_t)(c0 + warp);  // this chain's 16 columns: [16 cj, +16)
+    // Level bounds in registers, 32 levels per batch: lane j of batch q
+    // holds lp[l] and lp[l + 1] of level l = L - 1 - 32 q - j; the batch
+    // after the current one is loaded 32 levels ahead, and a level's bounds
+    // are two shuffles (a global load here would put an L2 round trip on
+    // every level step: the record fetch below depends on them)
+    int q = 0, bc = 0, ec = 0, bn = 0, en = 0;
+    auto load_batch = [&](int qq, int& bb, int& ee) {
+      const int l = L - 1 - 32 * qq - lane;
+      bb = l >= 0 ? __ldg(lp + l) : 0;
+      ee = l >= 0 ? __ldg(lp + l + 1) : 0;
+    };
+    load_batch(0, bc, ec);
+    load_batch(1, bn, en);
+    auto bounds = [&](int l) -> int2 {  // l in batch q or q + 1 (warp-uniform)
+      const int j = L - 1 - l - 32 * q;
+      if (j < 32) return make_int2(__shfl_sync(0xffffffffu, bc, j), __shfl_sync(0xffffffffu, ec, j));
+      return make_int2(__shfl_sync(0xffffffffu, bn, j - 32), __shfl_sync(0xffffffffu, en, j - 32));
+    };
+    // this lane's record of level l, kRecAhead16 levels ahead
+    auto fetch = [&](int l, int4& r, int2& be) {
+      if (l < 0) {
+        r = make_int4(0, 0, 0, 0);
+        be = make_int2(0, 0);
+        return;
+      }
+      be = bounds(l);
+      r = lane < be.y - be.x ? __ldg(rec + be.x + lane) : make_int4(0, 0, 0, 0);
+    };
+    auto do_level = [&](int level, int4& r0, int2& be0) {
+      const int lb = be0.x, items = be0.y - be0.x;
+      for (int i = lane; i < items; i += 32) {
+        const int4 r = i == lane ? r0 : __ldg(rec + lb + i);
+        const uint32_t v = (uint32_t)r.x & 0xFFFFu, deg = (uint32_t)r.x >> 16;
+        const uint32_t s4[4] = {(uint32_t)r.y & 0xFFFFu, (uint32_t)r.y >> 16, (uint32_t)r.z & 0xFFFFu,
+                                (uint32_t)r.z >> 16};
+        uint32_t acc = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          if ((uint32_t)k < deg) {
+            const uint32_t w = s4[k];
+            acc |= col[w] | ((w >> 4) == cj ? 1u << (w & 15) : 0u);
+          }
+        if (deg > 4) {
+          const uint32_t dg = deg == 0xFFFFu ? (uint32_t)(soff[v + 1] - r.w) : deg;
+          for (uint32_t k = 4; k < dg; ++k) {
+            const uint32_t w = (uint32_t)succ[r.w + k];
+            acc |= col[w] | ((w >> 4) == cj ? 1u << (w & 15) : 0u);
+          }
+        }
+        col[v] = (uint16_t)acc;
+      }
+      if (L - 1 - (level - kRecAhead16) - 32 * q >= 64) {  // the prefetch target left batch q + 1
+        bc = bn;
+        ec = en;
+        ++q;
+        load_batch(q + 1, bn, en);
+      }
+      fetch(level - kRecAhead16, r0, be0);
+      __syncwarp();
+    };
+    int4 rr[kRecAhead16];
+    int2 bb[kRecAhead16];
+#pragma unroll
+    for (int i = 0; i < kRecAhead16; ++i) fetch(L - 1 - i, rr[i], bb[i]);
+    for (int level = L - 1; level >= 0; level -= kRecAhead16) {
+#pragma unroll
+      for (int i = 0; i < kRecAhead16; ++i)
+        if (level - i >= 0) do_level(level - i, rr[i], bb[i]);
+    }
+  }
+  __syncthreads();
+  // rows out: consecutive threads write consecutive 16-bit columns of a row
+  for (int64_t it = tid; it < (int64_t)N * act; it += nt) {
+    const int64_t v = it / act;
+    const int k = (int)(it - v * act);
+    R16[v * nch + c0 + k] = Rs[(size_t)k * N + v];
+  }
 }
 
 // K3 (large graphs): M = R | R^T | I in the stored layout and per-tile
@@ -920,18 +1114,32 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
     PT_LAUNCH_CHECK();
   } else {
 {
-    // in-degrees and the Kahn queue in shared memory when the largest graph fits
-    const int smem_nodes = b.max_nodes <= 26 * 1024 ? b.max_nodes : 0;
-    const int dsm = 2 * 4 * smem_nodes;
+    // in-degrees and the Kahn queue in shared memory when the largest graph
+    // fits; warp mode (16-bit CSR in shared memory too) for graphs with at
+    // most `ecap` edges: 8 N + 2 + 2 ecap bytes, ecap <= 4 N within 200 KB
+    const int smem_nodes = b.max_nodes <= 24 * 1024 ? b.max_nodes : 0;
+    int ecap = 0;
+    if (smem_nodes > 0)
+      ecap = (int)std::min<int64_t>(4 * (int64_t)smem_nodes, (200 * 1024 - 8 * (int64_t)smem_nodes - 2) / 2);
+    const int dsm = (int)align_up((size_t)8 * smem_nodes + 2 + 2 * (size_t)std::max(ecap, 0), 16);
     PT_SMEM_ATTR(k_depth, dsm);
     ProfScope _p(PK_DAG_DEPTH, st);
-    k_depth<<<G, 256, dsm, st>>>(d, sc, smem_nodes);
+    k_depth<<<G, 256, dsm, st>>>(d, sc, smem_nodes, std::max(ecap, 0));
     PT_LAUNCH_CHECK();
   }
-  // closure: shared memory for a column slice of all rows of the largest graph
-  // (+ its CSR when it fits); several CTAs per SM for small graphs.
   const int64_t maxN = b.max_nodes;
   const int64_t Wmax = dag->max_words;
+  if (b.hops == 0 && maxN > kDeepNodes) {
+    // deep graphs: 16-bit column chains, `cpb` per CTA, one CTA per SM
+    const int cpb = (int)std::max<int64_t>(1, std::min<int64_t>(8, (227 * 1024 - 64) / (2 * maxN)));
+    const int csm = (int)align_up((size_t)cpb * 2 * (size_t)maxN, 16);
+    PT_SMEM_ATTR(k_closure16, csm);
+    ProfScope _p(PK_DAG_CLOSURE, st);
+    k_closure16<<<dim3(G, (unsigned)ceil_div(4 * Wmax, cpb)), 256, csm, st>>>(d, sc, cpb);
+    PT_LAUNCH_CHECK();
+  } else {
+  // closure: shared memory for a column slice of all rows of the largest graph
+  // (+ its CSR when it fits); several CTAs per SM for small graphs.
   int64_t want = maxN * Wmax * 8 + 4 * (4 * maxN + 8) + 16;  // R slice + CSR (E ~ 2N)
   int smem = (int)std::min<int64_t>(want, 200 * 1024);
   smem = (int)align_up((size_t)smem, 1024);
@@ -944,6 +1152,7 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
     ProfScope _p(PK_DAG_CLOSURE, st);
     k_closure<<<gc, 256, smem, st>>>(d, smem, sc);
     PT_LAUNCH_CHECK();
+  }
   }
 {
     ProfScope _p(PK_DAG_MASK, st);
