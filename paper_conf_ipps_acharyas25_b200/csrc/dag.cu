@@ -537,7 +537,10 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
 // (~N/1.5 levels), so the number of chains in flight is what matters.  Level
 // records (node, degree, first four successors; built by k_depth in topo
 // order) and level bounds are prefetched kRecAhead levels ahead.
-constexpr int kDeepNodes = 6144;
+#ifndef PREDTOP_DEEP_NODES
+#define PREDTOP_DEEP_NODES 6144
+#endif
+constexpr int kDeepNodes = PREDTOP_DEEP_NODES;
 #ifndef PREDTOP_REC_AHEAD16
 #define PREDTOP_REC_AHEAD16 4
 #endif
