@@ -306,6 +306,9 @@ __global__ void __launch_bounds__(256) k_depth(DagDev d, SmallCfg sc, int smem_n
   }
 }
 
+#ifndef PREDTOP_CLOS_REC_SMEM
+#define PREDTOP_CLOS_REC_SMEM 1  // k_closure level loop over shared-memory records (0: over the CSR)
+#endif
 #ifndef PREDTOP_REC_AHEAD
 #define PREDTOP_REC_AHEAD 4
 #endif
@@ -326,7 +329,13 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   // Column slicing: CW words of every row resident in shared memory.
   const int L = d.num_levels[g];
   const int E = (int)(d.edge_ptr[g + 1] - d.edge_ptr[g]);
-  const size_t csr_bytes = align_up((size_t)4 * ((size_t)N + (N + 1) + E + (L + 1)), 16);
+  // finite-k rounds read the CSR; the k = infinity level loop reads the
+  // per-node records (node, degree, first four successors, in topo order;
+  // built by k_depth) and the level bounds
+  const bool kfin = d.hops > 0 && d.hops < L - 1;
+  const bool recs = !kfin && PREDTOP_CLOS_REC_SMEM;
+  const size_t csr_bytes = recs ? align_up((size_t)16 * N + 4 * ((size_t)L + 1), 16)
+                                : align_up((size_t)4 * ((size_t)N + (N + 1) + E + (L + 1)), 16);
   int CW = (int)min((int64_t)W, (int64_t)smem_bytes / (8 * (int64_t)N));
   bool csr_in_smem = false;
   if ((int64_t)smem_bytes > (int64_t)csr_bytes) {
@@ -429,7 +438,17 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   }
   uint64_t* Rs;
   int64_t rs;  // row stride of Rs in words
-  if (csr_in_smem) {
+  const int32_t* soff_g = soff;
+  const int32_t* succ_g = succ;
+  const int4* s_rec = reinterpret_cast<const int4*>(sm);
+  if (csr_in_smem && recs) {
+    int4* rs_ = reinterpret_cast<int4*>(sm);
+    int32_t* s_lptr = reinterpret_cast<int32_t*>(rs_ + N);
+    const int4* rec = d.rec + n0;
+    for (int i = tid; i < N; i += nt) rs_[i] = rec[i];
+    for (int i = tid; i <= L; i += nt) s_lptr[i] = lptr[i];
+    lptr = s_lptr;
+  } else if (csr_in_smem) {
     int32_t* s_topo = (int32_t*)sm;
     int32_t* s_soff = s_topo + N;
     int32_t* s_succ = s_soff + (N + 1);
@@ -485,7 +504,37 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   // CTA-synchronous sweep).
   const int warp = tid >> 5, lane = tid & 31, nwarps = nt >> 5;
   const int my_nw = warp < nw ? (nw - warp + nwarps - 1) / nwarps : 0;
-  if (my_nw > 0) {
+  if (my_nw > 0 && csr_in_smem && recs) {
+    // records in shared memory: one record load, then the successors' words
+    for (int level = L - 1; level >= 0; --level) {
+      const int lb = lptr[level], items = (lptr[level + 1] - lb) * my_nw;
+      for (int it = lane; it < items; it += 32) {
+        const int node_i = my_nw == 1 ? it : it / my_nw;
+        const int j = warp + (my_nw == 1 ? 0 : it - node_i * my_nw) * nwarps;
+        const uint32_t wj = (uint32_t)(word0 + j);
+        const int4 r = s_rec[lb + node_i];
+        const uint32_t v = (uint32_t)r.x & 0xFFFFu, deg = (uint32_t)r.x >> 16;
+        const uint32_t s4[4] = {(uint32_t)r.y & 0xFFFFu, (uint32_t)r.y >> 16, (uint32_t)r.z & 0xFFFFu,
+                                (uint32_t)r.z >> 16};
+        uint64_t acc = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          if ((uint32_t)k < deg) {
+            const uint32_t w = s4[k];
+            acc |= Rs[(int64_t)w * rs + j] | ((w >> 6) == wj ? 1ull << (w & 63) : 0ull);
+          }
+        if (deg > 4) {
+          const uint32_t dg = deg == 0xFFFFu ? (uint32_t)(soff_g[v + 1] - r.w) : deg;
+          for (uint32_t k = 4; k < dg; ++k) {
+            const uint32_t w = (uint32_t)succ_g[r.w + k];
+            acc |= Rs[(int64_t)w * rs + j] | ((w >> 6) == wj ? 1ull << (w & 63) : 0ull);
+          }
+        }
+        Rs[(int64_t)v * rs + j] = acc;
+      }
+      __syncwarp();
+    }
+  } else if (my_nw > 0) {
     for (int level = L - 1; level >= 0; --level) {
       const int lb = lptr[level], le = lptr[level + 1];
       const int items = (le - lb) * my_nw;
