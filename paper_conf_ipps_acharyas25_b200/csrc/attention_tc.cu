@@ -5,8 +5,9 @@
 //
 // One CTA = one (graph, 128-row query tile, head); two CTAs per SM (256 TMEM
 // columns each), 8 softmax warps per CTA.  Each query row is one TMEM lane;
-// the two softmax warps of a lane quarter split every 64-key chunk into key
-// halves, so a softmax thread owns (row, 32 keys of the chunk): no shuffles.
+// the two softmax warps of a lane quarter own the even and the odd 64-key
+// chunks, so a softmax thread owns (row, chunk): no shuffles, and the two
+// warps sharing a scheduler run half a chunk apart.
 //
 //   warp 0      TMA producer: the Q tile, then K and V of every 64-key chunk
 //               of the graph's head through a kKV-stage ring (SW64 boxes at
@@ -19,13 +20,12 @@
 //                                               transpose), a constant ones
 //                                               atom LBO bytes after it gives
 //                                               the row sums l
-//   warps 2..9  softmax: mask bit -> -inf, exp2, P as fp16 written over the
-//               thread's own half of S_b (tcgen05.st), then O / l -> fp16.
+//   warps 2..9  softmax: exp2, P as fp16 masked by the bitset and written
+//               over its own S_b (tcgen05.st), then O / l -> fp16.
 //
 // TMEM (256 columns): S_0 | S_1 | S_2 (64 each) | O (d_h) | l (16).  P of
 // keys 0-31 of a chunk sits in columns [0,16) of its S, keys 32-63 in
-// [32,48): each half is written only by the threads that read that half of
-// S.  QK^T of chunk c+3 is issued right after PV of chunk c, so the tensor
+// [32,48) (each 32-key half is read before it is overwritten).  QK^T of chunk c+3 is issued right after PV of chunk c, so the tensor
 // core runs two chunks (128 keys) ahead of the softmax.
 //
 // Softmax in log2 units (Q pre-scaled by log2(e)/sqrt(d_h) in the QKV
@@ -60,8 +60,16 @@ constexpr int kRows = 128;   // query rows per CTA (TMEM lanes)
 #endif
 constexpr int kCh = PREDTOP_ATTN_GEO;          // keys per chunk (S columns)
 constexpr int kSBuf = kCh == 64 ? 3 : 2;       // S/P buffers in TMEM
-constexpr int kSoftWarps = kCh == 64 ? 8 : 4;  // softmax warps (kSoftWarps / 4 threads per row)
-constexpr int kHalves = kSoftWarps / 4;
+// PREDTOP_ATTN_PAR: 2 (default with 64-key chunks) = each softmax warp owns
+// whole chunks of one parity; 3 = twelve softmax warps, one per (lane
+// quarter, S buffer) (measured equal to 2); 0 = two warps split every chunk
+// into key halves (1-2 % slower on MoE: the two warps of a lane quarter run in
+// lockstep on the same S buffer)
+#ifndef PREDTOP_ATTN_PAR
+#define PREDTOP_ATTN_PAR (PREDTOP_ATTN_GEO == 64 ? 2 : 0)
+#endif
+constexpr int kPar = PREDTOP_ATTN_PAR;
+constexpr int kSoftWarps = kPar == 3 ? 12 : kCh == 64 ? 8 : 4;  // softmax warps (kSoftWarps / 4 threads per row)
 constexpr int kTmemCols = kCh == 64 ? 256 : 128;
 constexpr int kMinBlocks = kCh == 64 ? 2 : 4;
 #ifndef PREDTOP_ATTN_KV
@@ -69,7 +77,9 @@ constexpr int kMinBlocks = kCh == 64 ? 2 : 4;
 #endif
 constexpr int kKV = PREDTOP_ATTN_KV;  // K/V ring stages
 static_assert(kKV > kSBuf && kKV <= 2 * kSBuf, "K/V stages are released through s_full (see the producer)");
-static_assert(kCh * 4 / kSoftWarps == 32, "every softmax thread owns 32 keys of a chunk");
+static_assert(kPar || kCh * 4 / kSoftWarps == 32, "every softmax thread owns 32 keys of a chunk");
+static_assert(kPar == 0 || (kCh == 64 && (kPar == 2 || kPar == kSBuf)), "chunk ownership strides");
+constexpr int kOutSplit = kCh == 64 ? 2 : 1;  // threads per row writing the output
 // PREDTOP_ATTN_SPLIT=1: QK^T and PV are issued by two threads in
 // two warps (warp 1 and warp 10), so neither issue stream waits for the
 // other's instructions (a tcgen05.mma costs its issuing thread ~75-120 cycles
@@ -81,6 +91,12 @@ static_assert(kCh * 4 / kSoftWarps == 32, "every softmax thread owns 32 keys of 
 constexpr int kSplit = PREDTOP_ATTN_SPLIT;
 constexpr int kThreads = 64 + 32 * kSoftWarps + 32 * kSplit;
 constexpr int kPvWarp = kSplit ? 2 + kSoftWarps : 1;
+// mask words are loaded kMpf chunks ahead of their use
+#ifndef PREDTOP_ATTN_MPF
+#define PREDTOP_ATTN_MPF 2
+#endif
+constexpr int kMpf = PREDTOP_ATTN_MPF;
+
 
 template <int DH>
 struct TcCfg {
@@ -189,7 +205,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
 #pragma unroll
     for (int b = 0; b < kSBuf; ++b) {
       sm100::mbar_init(&s_full[b], 1);
-      sm100::mbar_init(&p_ready[b], kSoftWarps);
+      sm100::mbar_init(&p_ready[b], kPar ? 4 : kSoftWarps);
       sm100::mbar_init(&pv_done[b], 1);
     }
     sm100::mbar_init(&o_full, 1);
@@ -383,58 +399,105 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
     // keys are the low (hf = 0) or high (hf = 1) byte of each 16-bit field of
     // the stored layout (internal.h mask_pos: mask_pos(k + 32) = mask_pos(k) + 8).
     const uint32_t sfull0 = sm100::smem_u32(&s_full[0]), pready0 = sm100::smem_u32(&p_ready[0]);
+    // P of one 32-key half: exponentials, fp16 pairs, mask (w: this half's
+    // four mask bytes in the low byte of every 16-bit field)
+    auto half = [&](uint32_t tS, uint64_t w) {
+      if (__any_sync(0xffffffffu, w != 0ull)) {
+        float s[32];
+        uint32_t p[16];
+        sm100::tmem_ld<32>(tS, s);
+        // the four mask bytes of this key half in one register: byte f
+        // holds keys k with (k >> 1) & 3 == f at bit 2 (k >> 3) + (k & 1),
+        // so the pair (2i, 2i+1) sits at bits 8f + 2q, +1 (f = i & 3,
+        // q = i >> 2).  The mask is applied after the exponential, to the
+        // packed fp16 pair: x0[q] / x1[q] move bit 2q / 2q+1 of every byte to
+        // the byte's sign bit, and one sign-replicating byte permute per pair
+        // builds its 0xFFFF / 0x0000 halves (a masked score's exponential,
+        // inf included, is ANDed away)
+        const uint32_t w32 = __byte_perm((uint32_t)w, (uint32_t)(w >> 32), 0x6420);
+        uint32_t x0[4], x1[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          x0[q] = w32 << (7 - 2 * q);
+          x1[q] = w32 << (6 - 2 * q);
+        }
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const int f = i & 3, q = i >> 2;
+          // selector nibbles (result bytes 0..3): x0 byte f, x0 byte f,
+          // x1 byte f, x1 byte f, each with the sign-replicate bit 8
+          const uint32_t sel = 0xCC88u + 0x1111u * (uint32_t)f;
+          uint32_t m;
+          asm("prmt.b32 %0, %1, %2, %3;" : "=r"(m) : "r"(x0[q]), "r"(x1[q]), "r"(sel));
+          p[i] = sm100::pack_half2(ex2f(s[2 * i]), ex2f(s[2 * i + 1])) & m;
+        }
+        sm100::tmem_st16(tS, p);
+      } else {
+        sm100::tmem_st16_zero(tS);
+      }
+    };
+#ifdef PREDTOP_ATTN_MASK_ONES
+    constexpr uint64_t kOnes = 0x00FF00FF00FF00FFull;  // timing diagnostic only: every pair allowed
+#endif
+#if PREDTOP_ATTN_PAR
+    // chunk ownership: warp (q4, hf) owns ALL 64 keys of the chunks c with
+    // c % kPar == hf, so the warps of a lane quarter run staggered instead of
+    // in lockstep on the same S buffer
+    const uint32_t tR = tmem + lrow;
+    uint64_t wq[kMpf];
+#pragma unroll
+    for (int i = 0; i < kMpf; ++i) wq[i] = (valid && hf + kPar * i < nch) ? __ldg(Mrow + hf + kPar * i) : 0ull;
+#pragma unroll 1
+    for (int c = hf; c < nch; c += kPar) {
+      const int b = c % kSBuf;
+      const uint32_t ph = (uint32_t)(c / kSBuf) & 1u;
+#ifdef PREDTOP_ATTN_MASK_ONES
+      const uint64_t w = kOnes;
+#else
+      const uint64_t w = wq[0];
+#endif
+#pragma unroll
+      for (int i = 0; i + 1 < kMpf; ++i) wq[i] = wq[i + 1];
+      if (c + kPar * kMpf < nch && valid) wq[kMpf - 1] = __ldg(Mrow + c + kPar * kMpf);
+      bar_wait(sfull0 + 8 * b, ph);
+      if (lane == 0 && warp == 2) ATR(6, c);
+      sm100::tc_fence_after();
+      if (!warp_dead) {
+        half(tR + kCh * b, w & 0x00FF00FF00FF00FFull);
+        half(tR + kCh * b + 32, (w >> 8) & 0x00FF00FF00FF00FFull);
+        sm100::tmem_wait_st();
+        sm100::tc_fence_before();
+      }
+      __syncwarp();
+      if (lane == 0) bar_arrive(pready0 + 8 * b);
+      if (lane == 0 && warp == 2) ATR(7, c);
+    }
+#else
     const uint32_t tS0 = tmem + 32 * hf + lrow;
     // mask words two chunks ahead (L2 latency).  This thread's 32 keys of
     // chunk c start at key kCh c + 32 hf: word (kCh c + 32 hf) >> 6, byte
     // half ((kCh c + 32 hf) >> 5) & 1 of every 16-bit field.
     auto word_of = [&](int c) -> int { return (kCh * c + 32 * hf) >> 6; };
-    uint64_t wnext = valid ? __ldg(Mrow + word_of(0)) : 0ull,
-             wnext2 = (valid && nch > 1) ? __ldg(Mrow + word_of(1)) : 0ull;
+    uint64_t wq[kMpf];
+#pragma unroll
+    for (int i = 0; i < kMpf; ++i) wq[i] = (valid && i < nch) ? __ldg(Mrow + word_of(i)) : 0ull;
     int b = 0;
     uint32_t ph = 0;  // phase parity of buffer b's barriers
 #pragma unroll 1
     for (int c = 0; c < nch; ++c) {
-      const uint64_t w = (wnext >> (8 * (((kCh * c + 32 * hf) >> 5) & 1))) & 0x00FF00FF00FF00FFull;
-      wnext = wnext2;
-      if (c + 2 < nch && valid) wnext2 = __ldg(Mrow + word_of(c + 2));
+#ifdef PREDTOP_ATTN_MASK_ONES
+      const uint64_t w = kOnes;
+#else
+      const uint64_t w = (wq[0] >> (8 * (((kCh * c + 32 * hf) >> 5) & 1))) & 0x00FF00FF00FF00FFull;
+#endif
+#pragma unroll
+      for (int i = 0; i + 1 < kMpf; ++i) wq[i] = wq[i + 1];
+      if (c + kMpf < nch && valid) wq[kMpf - 1] = __ldg(Mrow + word_of(c + kMpf));
       bar_wait(sfull0 + 8 * b, ph);
       if (lane == 0 && warp == 2) ATR(6, c);
       sm100::tc_fence_after();
       if (!warp_dead) {
-        const uint32_t tS = tS0 + kCh * b;
-        if (__any_sync(0xffffffffu, w != 0ull)) {
-          float s[32];
-          uint32_t p[16];
-          sm100::tmem_ld<32>(tS, s);
-          // the four mask bytes of this key half in one register: byte f
-          // holds keys k with (k >> 1) & 3 == f at bit 2 (k >> 3) + (k & 1),
-          // so the pair (2i, 2i+1) sits at bits 8f + 2q, +1 (f = i & 3,
-          // q = i >> 2).  The mask is applied after the exponential, to the
-          // packed fp16 pair: x0[q] / x1[q] move bit 2q / 2q+1 of every byte to
-          // the byte's sign bit, and one sign-replicating byte permute per pair
-          // builds its 0xFFFF / 0x0000 halves (a masked score's exponential,
-          // inf included, is ANDed away)
-          const uint32_t w32 = __byte_perm((uint32_t)w, (uint32_t)(w >> 32), 0x6420);
-          uint32_t x0[4], x1[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            x0[q] = w32 << (7 - 2 * q);
-            x1[q] = w32 << (6 - 2 * q);
-          }
-#pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            const int f = i & 3, q = i >> 2;
-            // selector nibbles (result bytes 0..3): x0 byte f, x0 byte f,
-            // x1 byte f, x1 byte f, each with the sign-replicate bit 8
-            const uint32_t sel = 0xCC88u + 0x1111u * (uint32_t)f;
-            uint32_t m;
-            asm("prmt.b32 %0, %1, %2, %3;" : "=r"(m) : "r"(x0[q]), "r"(x1[q]), "r"(sel));
-            p[i] = sm100::pack_half2(ex2f(s[2 * i]), ex2f(s[2 * i + 1])) & m;
-          }
-          sm100::tmem_st16(tS, p);
-        } else {
-          sm100::tmem_st16_zero(tS);
-        }
+        half(tS0 + kCh * b, w);
         sm100::tmem_wait_st();
         sm100::tc_fence_before();
       }
@@ -446,8 +509,9 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
         ph ^= 1u;
       }
     }
-    // (3) O / l -> fp16: this thread writes output columns [OC hf, OC (hf+1)),
-    // OC = DH / kHalves
+#endif
+    // (3) O / l -> fp16: threads hf < kOutSplit write output columns
+    // [OC hf, OC (hf+1)), OC = DH / kOutSplit
     if (t == 0) ATR(2, 3);  // softmax done
     sm100::mbar_wait(&o_full, 0);
     sm100::tc_fence_after();
@@ -456,7 +520,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
     sm100::tmem_ld<DH>(tmem + C::TO + lrow, o);
     float lv[16];
     sm100::tmem_ld<16>(tmem + C::TL + lrow, lv);
-    if (valid) {
+    if (valid && hf < kOutSplit) {
       __half* orow = out + (n0 + row) * dmodel + h * DH;
       // a P that overflowed fp16 (s - m >= 16: inf) or a NaN score leaves l
       // non-finite; both key-half threads read the same l, so they agree
@@ -464,7 +528,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
         if (hf == 0) exact_row<DH>(qkv, n0, N, row, h, dmodel, Mrow, orow);
       } else {
         const float inv = lv[0] > 0.f ? 1.f / lv[0] : 0.f;
-        constexpr int OC = DH / kHalves;
+        constexpr int OC = DH / kOutSplit;
         uint32_t pk[OC / 2];
 #pragma unroll
         for (int i = 0; i < OC / 2; ++i) {

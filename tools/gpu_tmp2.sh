@@ -1,8 +1,13 @@
-timeout 900 python -m pytest tests/test_gpu_dag.py tests/test_gpu_hops.py tests/test_gpu_prune.py -m gpu -q -x --timeout 300 2>&1 | tail -2
-timeout 300 python -m pytest tests -m gpu -q -x --timeout 200 -k "16k or moe or invalid" 2>&1 | tail -2
-timeout 200 python bench.py --config moe --no-cpu-baseline --no-also --steps 20 > gpurun_out/bench_moe.json 2>gpurun_out/bench_moe.err
-python -c "
-import json; d=json.loads(open('gpurun_out/bench_moe.json').read().strip().splitlines()[-1]); print(round(d['value']), {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if v['ms_per_step']>0.05})" || tail -3 gpurun_out/bench_moe.err
-timeout 300 python bench.py --config 16k --no-cpu-baseline --no-also --steps 5 > gpurun_out/bench_16k.json 2>gpurun_out/bench_16k.err
-python -c "
-import json; d=json.loads(open('gpurun_out/bench_16k.json').read().strip().splitlines()[-1]); print(d['value'], d['ms_per_step'], {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if v['ms_per_step']>0.05})" || tail -3 gpurun_out/bench_16k.err
+# A/B of attention variants: parity subset with each variant lib, then MoE bench x2
+O=gpurun_out; mkdir -p $O
+for v in "$@"; do
+  PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_$v.so timeout 300 python -m pytest tests -m gpu -q -x --timeout 120 -k "moe or exact or tc or forward" > $O/pt_$v.txt 2>&1; echo "$v pytest rc=$?"; tail -1 $O/pt_$v.txt
+done
+for i in 1 2; do
+for v in default "$@"; do
+  if [ "$v" != default ]; then export PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_$v.so; else unset PREDTOP_LIB; fi
+  timeout 240 python bench.py --config moe --no-cpu-baseline --no-also --steps 20 > $O/bench_$v.json 2>$O/bench_$v.err
+  python -c "
+import json; d=json.loads(open('$O/bench_$v.json').read().strip().splitlines()[-1]); print('$v', round(d['value']), {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if v['ms_per_step']>1})" || tail -3 $O/bench_$v.err
+done
+done
