@@ -38,40 +38,94 @@ predtop_status pe_table_launch(float* pe, int rows, int d, cudaStream_t st) {
   return PREDTOP_OK;
 }
 
+// A lane's PER columns of a D-wide fp32 row: groups of four at columns
+// 4 lane + 128 j (each 16-byte vector instruction of the warp covers 512
+// contiguous bytes), or PER < 4 consecutive columns at PER lane.
+template <int PER>
+__device__ __forceinline__ int col_of(int lane, int k) {
+  if constexpr (PER >= 4) return 128 * (k / 4) + 4 * lane + (k % 4);
+  else return PER * lane + k;
+}
+template <int PER>
+__device__ __forceinline__ void ld_cols(const float* __restrict__ row, int lane, float (&a)[PER]) {
+  if constexpr (PER % 4 == 0) {
+#pragma unroll
+    for (int j = 0; j < PER / 4; ++j) {
+      const float4 v = __ldg(reinterpret_cast<const float4*>(row + 128 * j + 4 * lane));
+      a[4 * j] = v.x, a[4 * j + 1] = v.y, a[4 * j + 2] = v.z, a[4 * j + 3] = v.w;
+    }
+  } else if constexpr (PER == 2) {
+    const float2 v = __ldg(reinterpret_cast<const float2*>(row + 2 * lane));
+    a[0] = v.x, a[1] = v.y;
+  } else {
+#pragma unroll
+    for (int k = 0; k < PER; ++k) a[k] = __ldg(row + PER * lane + k);
+  }
+}
+
 template <int D>
 __global__ void __launch_bounds__(256) k_embed(const float* __restrict__ WT, const float* __restrict__ b,
                                                const predtop_node_feat* __restrict__ feats,
                                                const int32_t* __restrict__ depth,
                                                const float* __restrict__ pe, int pe_rows, int64_t n_tot,
                                                float* __restrict__ x32, __half* __restrict__ x16) {
-  constexpr int PER = D / 32;  // columns per lane
+  // one warp per node, PER = D / 32 columns per lane (col_of: vector loads of
+  // the W_in^T rows and the PE row, coalesced vector stores)
+  constexpr int PER = D / 32;
   const int lane = threadIdx.x & 31;
   const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  float bias[PER];
+  ld_cols<PER>(b, lane, bias);
   for (int64_t v = warp0; v < n_tot; v += nwarps) {
     const predtop_node_feat f = feats[v];
     // a graph with an error status (latency NaN) may hold no depth at all
     // (TOO_LARGE / INVALID_ARG graphs are never built): clamp into the table
     const int dep = min(max(depth[v], 0), pe_rows - 1);
-    float l[4];
+    float acc[PER], t[PER];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) l[j] = log1pf((float)f.dims[j]);
-    const float* rop = f.op < PREDTOP_NUM_OPS ? WT + (size_t)f.op * D : nullptr;
-    const float* rdt = f.dtype < PREDTOP_NUM_DTYPES ? WT + (size_t)(68 + f.dtype) * D : nullptr;
-    const float* rkd = f.kind < PREDTOP_NUM_KINDS ? WT + (size_t)(76 + f.kind) * D : nullptr;
-    const float* rpe = pe + (size_t)dep * D;
+    for (int k = 0; k < PER; ++k) acc[k] = bias[k];
+    if (f.op < PREDTOP_NUM_OPS) {
+      ld_cols<PER>(WT + (size_t)f.op * D, lane, t);
 #pragma unroll
-    for (int k = 0; k < PER; ++k) {
-      const int c = k * 32 + lane;
-      float acc = b[c];
-      if (rop) acc += rop[c];
+      for (int k = 0; k < PER; ++k) acc[k] += t[k];
+    }
 #pragma unroll
-      for (int j = 0; j < 4; ++j) acc += l[j] * WT[(size_t)(64 + j) * D + c];
-      if (rdt) acc += rdt[c];
-      if (rkd) acc += rkd[c];
-      acc += rpe[c];
-      x32[v * D + c] = acc;
-      x16[v * D + c] = __float2half_rn(acc);
+    for (int j = 0; j < 4; ++j) {
+      const float l = log1pf((float)f.dims[j]);
+      ld_cols<PER>(WT + (size_t)(64 + j) * D, lane, t);
+#pragma unroll
+      for (int k = 0; k < PER; ++k) acc[k] += l * t[k];
+    }
+    if (f.dtype < PREDTOP_NUM_DTYPES) {
+      ld_cols<PER>(WT + (size_t)(68 + f.dtype) * D, lane, t);
+#pragma unroll
+      for (int k = 0; k < PER; ++k) acc[k] += t[k];
+    }
+    if (f.kind < PREDTOP_NUM_KINDS) {
+      ld_cols<PER>(WT + (size_t)(76 + f.kind) * D, lane, t);
+#pragma unroll
+      for (int k = 0; k < PER; ++k) acc[k] += t[k];
+    }
+    ld_cols<PER>(pe + (size_t)dep * D, lane, t);
+#pragma unroll
+    for (int k = 0; k < PER; ++k) acc[k] += t[k];
+    float* o32 = x32 + v * D;
+    __half* o16 = x16 + v * D;
+    if constexpr (PER % 4 == 0) {
+#pragma unroll
+      for (int j = 0; j < PER / 4; ++j) {
+        const int c = 128 * j + 4 * lane;
+        *reinterpret_cast<float4*>(o32 + c) = make_float4(acc[4 * j], acc[4 * j + 1], acc[4 * j + 2], acc[4 * j + 3]);
+        __half2 h[2] = {__floats2half2_rn(acc[4 * j], acc[4 * j + 1]), __floats2half2_rn(acc[4 * j + 2], acc[4 * j + 3])};
+        *reinterpret_cast<uint2*>(o16 + c) = *reinterpret_cast<const uint2*>(h);
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < PER; ++k) {
+        o32[col_of<PER>(lane, k)] = acc[k];
+        o16[col_of<PER>(lane, k)] = __float2half_rn(acc[k]);
+      }
     }
   }
 }
