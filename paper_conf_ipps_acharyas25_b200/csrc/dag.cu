@@ -717,12 +717,14 @@ constexpr int kMC = 32;           // 64-bit words per column chunk
 constexpr int kMA = 2 * kMC + 1;  // padded row stride (32-bit words) of the row tile
 constexpr int kMB = 5;            // padded row stride (32-bit words) of the strip
 constexpr size_t kMaskSmem = (size_t)4 * (128 * kMA + 64 * kMC * kMB + 128);
-__global__ void __launch_bounds__(256) k_mask2(DagDev d, SmallCfg sc) {
+__global__ void __launch_bounds__(256) k_mask2(DagDev d, SmallCfg sc, int rb) {
   extern __shared__ __align__(16) unsigned char sm_mask[];
   uint32_t* sA = reinterpret_cast<uint32_t*>(sm_mask);       // [128][kMA]
   uint32_t* sB = sA + 128 * kMA;                               // [64 kMC][kMB]
   int* s_cnt = reinterpret_cast<int*>(sB + 64 * kMC * kMB);  // [T <= 128]
-  const int g = blockIdx.x, a = blockIdx.y;
+  // row blocks of one graph are consecutive CTAs, so the graph's R column
+  // strips, which every row block reads, are re-read from L2, not DRAM
+  const int a = (int)(blockIdx.x % (unsigned)rb), g = (int)(blockIdx.x / (unsigned)rb);  // rb row blocks per graph
   const int st = d.status[g];
   if (st == PREDTOP_ERR_TOO_LARGE || st == PREDTOP_ERR_INVALID_ARG) return;
   const int64_t n0 = d.node_ptr[g];
@@ -1209,7 +1211,13 @@ predtop_status dag_build_launch(predtop_dag_s* dag, cudaStream_t st) {
 {
     ProfScope _p(PK_DAG_MASK, st);
     PT_SMEM_ATTR(k_mask2, (int)kMaskSmem);
-    k_mask2<<<dim3(G, (unsigned)ceil_div(maxN, 128)), 256, kMaskSmem, st>>>(d, sc);
+    // 1D grid of G x rb CTAs, the row blocks of a graph consecutive
+    const int64_t rb = ceil_div(maxN, 128);
+    if ((int64_t)G * rb > 0x7fffffff) {
+      set_error("mask grid too large");
+      return PREDTOP_ERR_TOO_LARGE;
+    }
+    k_mask2<<<(unsigned)(G * rb), 256, kMaskSmem, st>>>(d, sc, (int)rb);
     PT_LAUNCH_CHECK();
   }
 {
