@@ -381,11 +381,14 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
     __syncthreads();
     const int warp = tid >> 5, lane = tid & 31, nwarps = nt >> 5;
     const int my_nw = warp < nw ? (nw - warp + nwarps - 1) / nwarps : 0;
+    // i / my_nw as a multiply-high by ceil(2^32 / my_nw) (exact for i < 2^32 / my_nw)
+    const uint32_t inv_nw = my_nw > 1 ? (uint32_t)((0xFFFFFFFFull + (uint64_t)my_nw) / (uint64_t)my_nw) : 0u;
     if (my_nw > 0) {
       auto first_rec = [&](int l) -> int4 {  // this lane's first item of level l
         if (l < 0) return make_int4(0, 0, 0, 0);
         const int b = lp[l], e = lp[l + 1];
-        return lane < (e - b) * my_nw ? __ldg(rec + b + (my_nw == 1 ? lane : lane / my_nw)) : make_int4(0, 0, 0, 0);
+        return lane < (e - b) * my_nw ? __ldg(rec + b + (my_nw == 1 ? lane : (int)__umulhi((uint32_t)lane, inv_nw)))
+                                      : make_int4(0, 0, 0, 0);
       };
       // level `level` with its prefetched first record r0; then r0 <- the
       // record of level - 4 (four fixed registers, unrolled by four: a load is
@@ -393,7 +396,7 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
       auto do_level = [&](int level, int4& r0) {
         const int lb = lp[level], items = (lp[level + 1] - lb) * my_nw;
         for (int i = lane; i < items; i += 32) {
-          const int node_i = my_nw == 1 ? i : i / my_nw;
+          const int node_i = my_nw == 1 ? i : (int)__umulhi((uint32_t)i, inv_nw);
           const int4 r = i == lane ? r0 : __ldg(rec + lb + node_i);
           const uint32_t v = (uint32_t)r.x & 0xFFFFu, deg = (uint32_t)r.x >> 16;
           const int j = warp + (my_nw == 1 ? 0 : (i - node_i * my_nw)) * nwarps;
@@ -504,12 +507,16 @@ __global__ void __launch_bounds__(256) k_closure(DagDev d, int smem_bytes, Small
   // CTA-synchronous sweep).
   const int warp = tid >> 5, lane = tid & 31, nwarps = nt >> 5;
   const int my_nw = warp < nw ? (nw - warp + nwarps - 1) / nwarps : 0;
+  // it / my_nw as a multiply-high by ceil(2^32 / my_nw) (exact for it <
+  // 2^32 / my_nw, far above N * my_nw): a runtime integer division is a ~20-instruction dependent chain
+  // inside the latency-bound level step
+  const uint32_t inv_nw = my_nw > 1 ? (uint32_t)((0xFFFFFFFFull + (uint64_t)my_nw) / (uint64_t)my_nw) : 0u;
   if (my_nw > 0 && csr_in_smem && recs) {
     // records in shared memory: one record load, then the successors' words
     for (int level = L - 1; level >= 0; --level) {
       const int lb = lptr[level], items = (lptr[level + 1] - lb) * my_nw;
       for (int it = lane; it < items; it += 32) {
-        const int node_i = my_nw == 1 ? it : it / my_nw;
+        const int node_i = my_nw == 1 ? it : (int)__umulhi((uint32_t)it, inv_nw);
         const int j = warp + (my_nw == 1 ? 0 : it - node_i * my_nw) * nwarps;
         const uint32_t wj = (uint32_t)(word0 + j);
         const int4 r = s_rec[lb + node_i];
