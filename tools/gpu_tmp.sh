@@ -1,8 +1,11 @@
-# GEMM epilogue (32-column steps) check: forward/unfused gpu tests, MoE + GPT bench x2
+# attention early-TMA A/B: parity subset with the variant, MoE bench default vs variant x2
 O=gpurun_out; mkdir -p $O
-timeout 900 python -m pytest tests -m gpu -q -x --timeout 300 -k "forward or unfused or moe or gemm or tap" > $O/pt_g.txt 2>&1; echo "pytest rc=$?"; tail -1 $O/pt_g.txt
-for c in moe gpt moe gpt; do
-  timeout 240 python bench.py --config $c --no-cpu-baseline --no-also --steps 20 > $O/bench_e.json 2>$O/bench_e.err
+PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_pipe.so timeout 600 python -m pytest tests -m gpu -q -x --timeout 120 -k "moe or exact or tc or forward" > $O/pt_new.txt 2>&1; echo "pytest rc=$?"; tail -1 $O/pt_new.txt
+for i in 1 2; do
+for v in default pipe; do
+  if [ "$v" != default ]; then export PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_$v.so; else unset PREDTOP_LIB; fi
+  timeout 240 python bench.py --config moe --no-cpu-baseline --no-also --steps 20 > $O/bench_$v.json 2>$O/bench_$v.err
   python -c "
-import json; d=json.loads(open('$O/bench_e.json').read().strip().splitlines()[-1]); print('$c', round(d['value'],1), {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if k in ('gemm_qkv','attention','layer_tail')})" || tail -3 $O/bench_e.err
+import json; d=json.loads(open('$O/bench_$v.json').read().strip().splitlines()[-1]); print('$v', round(d['value']), {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if v['ms_per_step']>1})" || tail -3 $O/bench_$v.err
+done
 done
