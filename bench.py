@@ -1040,7 +1040,7 @@ def run_sweep(args, ctx, pool):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         host = synth.pack_graphs(list(pool[:1024]))
-        v, cores, n, wall = oracle_rate(cfg, blob, host)
+        v, cores, n, wall, _ = oracle_rate(cfg, blob, host)
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": f"first {n} pool stage graphs, fp64 C oracle, {cores} threads, {wall:.1f} s"}
     if rank == 0:
