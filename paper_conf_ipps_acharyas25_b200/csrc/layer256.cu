@@ -60,6 +60,9 @@ __device__ __forceinline__ unsigned long long l256_clk() {  // memory clobber: s
 #ifndef PREDTOP_L256_OUTW
 #define PREDTOP_L256_OUTW 1  // x' leaves in 128-byte-row boxes (0: 16-column pieces)
 #endif
+#ifndef PREDTOP_L256_PF
+#define PREDTOP_L256_PF 1  // L2 prefetch of the next tile's x and att during this tile's FFN (0: off)
+#endif
 #ifndef PREDTOP_L256_STG
 #define PREDTOP_L256_STG 0  // 1: x' leaves through coalesced STG instead of TMA stores (A/B)
 #endif
@@ -201,10 +204,25 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
             ++it;
           }
         };
+        // PREDTOP_L256_PF: the next tile's residual x (8 boxes, 128 KB fp32)
+        // and att (4 boxes, 64 KB) prefetched into L2, spread over this
+        // tile's FFN chunks behind their weight loads: the ring frees their
+        // units only after the O-projection, and from HBM at one SM's share of
+        // the bandwidth the x tile alone cost ~5k cycles of LN1 wait
+        const bool pf = PREDTOP_L256_PF && t + (int)gridDim.x < ntiles;
+        const int m1 = (t + (int)gridDim.x) * 128;
+        int pfb = 0;
+        auto prefetch_upto = [&](int nb) {
+          for (; pfb < nb; ++pfb) {
+            if (pfb < D / 32) sm100::tma_prefetch_l2_2d(&mp.x32in, 32 * pfb, m1);
+            else sm100::tma_prefetch_l2_2d(&mp.att, 64 * (pfb - D / 32), m1);
+          }
+        };
         load_w1(0);
         for (int j = 0; j < NJ; ++j) {
           if (j + 1 < NJ) load_w1(j + 1);
           load_w2(j);
+          if (pf) prefetch_upto(((j + 1) * (D / 32 + 4)) / NJ);
         }
       }
     }

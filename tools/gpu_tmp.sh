@@ -1,8 +1,8 @@
-# attention early-TMA A/B: parity subset with the variant, MoE bench default vs variant x2
+# variant A/B: parity subset with the variant, MoE bench default vs variant x2
 O=gpurun_out; mkdir -p $O
-PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_pipe.so timeout 600 python -m pytest tests -m gpu -q -x --timeout 120 -k "moe or exact or tc or forward" > $O/pt_new.txt 2>&1; echo "pytest rc=$?"; tail -1 $O/pt_new.txt
+PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_pf.so timeout 600 python -m pytest tests -m gpu -q -x --timeout 120 -k "moe or forward or tail" > $O/pt_new.txt 2>&1; echo "pytest rc=$?"; tail -1 $O/pt_new.txt
 for i in 1 2; do
-for v in default pipe; do
+for v in default pf; do
   if [ "$v" != default ]; then export PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_$v.so; else unset PREDTOP_LIB; fi
   timeout 240 python bench.py --config moe --no-cpu-baseline --no-also --steps 20 > $O/bench_$v.json 2>$O/bench_$v.err
   python -c "
