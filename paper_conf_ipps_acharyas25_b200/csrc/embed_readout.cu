@@ -64,7 +64,7 @@ __device__ __forceinline__ void ld_cols(const float* __restrict__ row, int lane,
 }
 
 template <int D>
-__global__ void __launch_bounds__(256) k_embed(const float* __restrict__ WT, const float* __restrict__ b,
+__global__ void __launch_bounds__(256, 4) k_embed(const float* __restrict__ WT, const float* __restrict__ b,
                                                const predtop_node_feat* __restrict__ feats,
                                                const int32_t* __restrict__ depth,
                                                const float* __restrict__ pe, int pe_rows, int64_t n_tot,
@@ -77,11 +77,23 @@ __global__ void __launch_bounds__(256) k_embed(const float* __restrict__ WT, con
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   float bias[PER];
   ld_cols<PER>(b, lane, bias);
+  // the next node's features and depth are loaded one iteration ahead (the
+  // row gathers depend on them: two dependent round trips per node otherwise)
+  predtop_node_feat fn{};
+  int dn = 0;
+  if (warp0 < n_tot) {
+    fn = feats[warp0];
+    dn = depth[warp0];
+  }
   for (int64_t v = warp0; v < n_tot; v += nwarps) {
-    const predtop_node_feat f = feats[v];
+    const predtop_node_feat f = fn;
     // a graph with an error status (latency NaN) may hold no depth at all
     // (TOO_LARGE / INVALID_ARG graphs are never built): clamp into the table
-    const int dep = min(max(depth[v], 0), pe_rows - 1);
+    const int dep = min(max(dn, 0), pe_rows - 1);
+    if (v + nwarps < n_tot) {
+      fn = feats[v + nwarps];
+      dn = depth[v + nwarps];
+    }
     float acc[PER], t[PER];
 #pragma unroll
     for (int k = 0; k < PER; ++k) acc[k] = bias[k];
