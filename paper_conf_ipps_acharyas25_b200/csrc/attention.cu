@@ -259,7 +259,7 @@ template <int DH, bool RESIDENT, int NW = 8>
 __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_MINB16
                                            : (DH == 16 ? 4 : PREDTOP_ATTN_MINB32) * (8 / NW))
     k_attn(const __grid_constant__ CUtensorMap tkv, DagDev d, int G, int H, int dmodel,
-           const __half* __restrict__ qkv, __half* __restrict__ out) {
+           const __half* __restrict__ qkv, __half* __restrict__ out, int nmax) {
   using A = Attn<DH>;
   constexpr int kStageChunks = stage_chunks<DH>();
   extern __shared__ __align__(16) unsigned char dsm_attn[];
@@ -273,6 +273,7 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   if ((unsigned)g >= (unsigned)G || d.status[g] != PREDTOP_OK) return;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
+  if (N > nmax) return;  // a larger graph: the tcgen05 kernel's (attention_tc.cu)
   const int rbase = qt * 128 + part * NW * 16;  // first query row of this CTA
   if (rbase >= N) return;
   const int W = 2 * ((N + 127) / 128);
@@ -436,15 +437,20 @@ __global__ void __launch_bounds__(NW * 32, (DH == 16 && NW == 4) ? PREDTOP_ATTN_
   }
 }
 
+// d_h = 16: graphs above this many nodes take the tcgen05 kernel
+constexpr int kTc16Min = 384;
+
 template <int DH>
 predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
-                         cudaStream_t st, unsigned blocks) {
+                         cudaStream_t st, unsigned blocks, int nmax) {
   constexpr int CH_BYTES = kChunk * DH * 2;  // one K or V chunk
   const int G = dag->desc.num_graphs;
-  const int maxch = (int)ceil_div(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), kChunk);
+  // the shared-memory path is sized by the largest graph THIS launch handles
+  const int nbig = std::min(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), nmax);
+  const int maxch = (int)ceil_div(nbig, kChunk);
   const int resident_bytes = 2 * maxch * CH_BYTES + 1024;
   // the 4-warp resident kernel also stages its 64 mask rows (W words each)
-  const int wmax = 2 * (int)ceil_div(std::min(dag->desc.max_nodes, PREDTOP_MAX_NODES), 128);
+  const int wmax = 2 * (int)ceil_div(nbig, 128);
   const int resident4_bytes = 2 * maxch * CH_BYTES + 64 * wmax * 8 + 256;
   CUtensorMap tkv;
   if (!encode_tma_2d(&tkv, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kChunk))
@@ -454,14 +460,14 @@ predtop_status launch_dh(const predtop_dag_s* dag, int d, int H, const __half* q
   if (half_tiles && resident4_bytes <= 28 * 1024) {
     // 4-warp CTAs (half q-tiles), up to 8 per SM (28 KB + 1 KB static each)
     PT_SMEM_ATTR((k_attn<DH, true, 4>), 28 * 1024);
-    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, true, 4><<<2 * blocks, 128, resident4_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, nmax);
   } else if (resident_bytes + 128 * wmax * 8 <= 100 * 1024) {
     PT_SMEM_ATTR((k_attn<DH, true>), 100 * 1024);
-    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, true><<<blocks, 256, resident_bytes + 128 * wmax * 8, st>>>(tkv, dag->d, G, H, d, qkv, out, nmax);
   } else {
     constexpr int stream_bytes = 2 * kStages * stage_chunks<DH>() * CH_BYTES + 1024;
     PT_SMEM_ATTR((k_attn<DH, false>), stream_bytes);
-    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out);
+    k_attn<DH, false><<<blocks, 256, stream_bytes, st>>>(tkv, dag->d, G, H, d, qkv, out, nmax);
   }
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;
@@ -479,17 +485,31 @@ predtop_status attention_launch(const predtop_dag_s* dag, int d, int H, const __
   }
   ProfScope _p(PK_ATTN, st);
   // tcgen05/TMEM kernel (attention_tc.cu) at d_h = 32, where this kernel's
-  // mma.sync QK^T + PV demand equals the MUFU rate; this kernel at d_h = 16.
-  // PREDTOP_ATTN_TC=1 / =0 forces one or the other (parity tests, A/B runs).
+  // mma.sync QK^T + PV demand equals the MUFU rate.  At d_h = 16 the split is
+  // per graph: graphs of more than kTc16Min nodes go to the tcgen05 kernel
+  // (its per-CTA prologue is amortised over >= 12 key chunks), smaller ones
+  // to this kernel, each launch skipping the other's graphs; a batch without
+  // large graphs (the GPT config) launches this kernel only.
+  // PREDTOP_ATTN_TC=1 / =0 forces one kernel for every graph (parity tests,
+  // A/B runs); PREDTOP_ATTN_TC16_MIN overrides the split size.
   const char* tc = getenv("PREDTOP_ATTN_TC");
-  bool use_tc = dh == 32;
-  if (tc && tc[0] == '1') use_tc = true;
-  if (tc && tc[0] == '0') use_tc = false;
-  if (use_tc && attention_tc_supported(dag, d, H)) return attention_tc_launch(dag, d, H, qkv, out, st);
-  if (dh == 16) return launch_dh<16>(dag, d, H, qkv, out, st, (unsigned)blocks);
-  if (dh == 32) return launch_dh<32>(dag, d, H, qkv, out, st, (unsigned)blocks);
-  set_error("unsupported head dim %d", dh);
-  return PREDTOP_ERR_UNSUPPORTED;
+  const char* t16 = getenv("PREDTOP_ATTN_TC16_MIN");
+  const int tc16_min = t16 ? atoi(t16) : kTc16Min;
+  int nsplit = dh == 32 ? 0 : (dag->desc.max_nodes > tc16_min ? tc16_min : INT_MAX);  // k_attn takes N <= nsplit
+  if (tc && tc[0] == '1') nsplit = 0;
+  if (tc && tc[0] == '0') nsplit = INT_MAX;
+  if (dh != 16 && dh != 32) {
+    set_error("unsupported head dim %d", dh);
+    return PREDTOP_ERR_UNSUPPORTED;
+  }
+  if (nsplit < INT_MAX && attention_tc_supported(dag, d, H)) {
+    predtop_status s = attention_tc_launch(dag, d, H, qkv, out, st, nsplit + 1);
+    if (s != PREDTOP_OK || nsplit == 0) return s;
+  } else {
+    nsplit = INT_MAX;
+  }
+  if (dh == 16) return launch_dh<16>(dag, d, H, qkv, out, st, (unsigned)blocks, nsplit);
+  return launch_dh<32>(dag, d, H, qkv, out, st, (unsigned)blocks, nsplit);
 }
 
 }  // namespace predtop

@@ -159,7 +159,7 @@ __device__ __forceinline__ void bar_arrive(uint32_t addr) {
 template <int DH>
 __global__ void __launch_bounds__(kThreads, kMinBlocks)
     k_attn_tc(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tm, DagDev d, int G,
-              int H, int dmodel, const __half* __restrict__ qkv, __half* __restrict__ out) {
+              int H, int dmodel, const __half* __restrict__ qkv, __half* __restrict__ out, int nmin) {
   using C = TcCfg<DH>;
   extern __shared__ unsigned char dsm[];
   unsigned char* base = sm100::align1024(dsm);
@@ -180,6 +180,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
   if ((unsigned)g >= (unsigned)G) return;
   const int64_t n0 = d.node_ptr[g];
   const int N = (int)(d.node_ptr[g + 1] - n0);
+  if (N < nmin) return;  // a smaller graph: the mma.sync kernel's (attention.cu)
   if (d.status[g] != PREDTOP_OK) {
     // an invalid graph (latency NaN) still gets finite zero rows, so no NaN
     // reaches a neighbouring graph's K/V chunk in the next layer
@@ -550,14 +551,14 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks)
 
 template <int DH>
 predtop_status launch_tc(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out, cudaStream_t st,
-                         unsigned blocks) {
+                         unsigned blocks, int nmin) {
   using C = TcCfg<DH>;
   PT_SMEM_ATTR(k_attn_tc<DH>, C::SMEM);
   CUtensorMap tq, tm;
   if (!encode_tma_2d(&tq, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kRows) ||
       !encode_tma_2d(&tm, qkv, 2, (uint64_t)3 * d, (uint64_t)dag->desc.total_nodes, DH, kCh))
     return PREDTOP_ERR_CUDA;
-  k_attn_tc<DH><<<blocks, kThreads, C::SMEM, st>>>(tq, tm, dag->d, dag->desc.num_graphs, H, d, qkv, out);
+  k_attn_tc<DH><<<blocks, kThreads, C::SMEM, st>>>(tq, tm, dag->d, dag->desc.num_graphs, H, d, qkv, out, nmin);
   PT_LAUNCH_CHECK();
   return PREDTOP_OK;
 }
@@ -570,14 +571,14 @@ bool attention_tc_supported(const predtop_dag_s* dag, int d, int H) {
 }
 
 predtop_status attention_tc_launch(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
-                                   cudaStream_t st) {
+                                   cudaStream_t st, int nmin) {
   const int64_t blocks = std::max<int64_t>(1, dag->qtiles_bound) * H;
   if (blocks > 0x7fffffff) {
     set_error("too many attention work items");
     return PREDTOP_ERR_TOO_LARGE;
   }
-  if (d / H == 32) return launch_tc<32>(dag, d, H, qkv, out, st, (unsigned)blocks);
-  if (d / H == 16) return launch_tc<16>(dag, d, H, qkv, out, st, (unsigned)blocks);
+  if (d / H == 32) return launch_tc<32>(dag, d, H, qkv, out, st, (unsigned)blocks, nmin);
+  if (d / H == 16) return launch_tc<16>(dag, d, H, qkv, out, st, (unsigned)blocks, nmin);
   set_error("unsupported head dim %d", d / H);
   return PREDTOP_ERR_UNSUPPORTED;
 }

@@ -170,8 +170,9 @@ predtop_status pe_table_launch(float* pe, int max_depth, int d, cudaStream_t st)
 predtop_status embed_launch(const predtop_model_s* m, const predtop_dag_s* dag, const float* pe,
                             float* x32, __half* x16, cudaStream_t st);
 bool attention_tc_supported(const predtop_dag_s* dag, int d, int H);
+// graphs with at least nmin nodes (0: all)
 predtop_status attention_tc_launch(const predtop_dag_s* dag, int d, int H, const __half* qkv, __half* out,
-                                   cudaStream_t st);
+                                   cudaStream_t st, int nmin = 0);
 predtop_status attention_launch(const predtop_dag_s* dag, int d, int H, const __half* qkv,
                                 __half* out, cudaStream_t st);
 predtop_status readout_launch(const predtop_model_s* m, const predtop_dag_s* dag, const float* x32,

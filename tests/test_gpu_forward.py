@@ -105,11 +105,16 @@ def test_latency_parity_tail_v1(pt, oracle_mod, name, batch_fn, monkeypatch):
     assert err.max() <= TOL
 
 
+@pytest.mark.parametrize("tc", ["0", None])
 @pytest.mark.parametrize("name, n", [("paper", 1700), ("moe", 800)])
-def test_latency_parity_streaming_attention(pt, oracle_mod, name, n):
+def test_latency_parity_streaming_attention(pt, oracle_mod, name, n, tc, monkeypatch):
     """Graphs whose K/V do not fit shared memory (d_h = 16: N > 1536; d_h =
-    32: N > 768) take the two-buffer TMA streaming path of the attention
-    kernel; plus a small graph in the same batch."""
+    32: N > 768) take the two-buffer TMA streaming path of the mma.sync
+    attention kernel when it is forced (PREDTOP_ATTN_TC=0); by default the
+    large graph goes to the tcgen05 kernel and the small one (90 nodes, d_h =
+    16) to the mma.sync kernel: the per-graph split of one batch."""
+    if tc is not None:
+        monkeypatch.setenv("PREDTOP_ATTN_TC", tc)
     rng = synth.CounterRng(7, n)
     s, d = synth.random_dag(n, 2.5 / n, rng)
     s2, d2 = synth.random_dag(90, 0.05, rng)
