@@ -92,6 +92,14 @@ __device__ __forceinline__ void bulk_wait_read0() {
   asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read_n() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+#ifndef PREDTOP_GEMM_BOXPIPE
+#define PREDTOP_GEMM_BOXPIPE 1  // 0: one bulk group per tile, waited for as a whole before restaging
+#endif
+constexpr bool kBoxPipe = PREDTOP_GEMM_BOXPIPE;
 __device__ __forceinline__ void bulk_wait_read1() {
   asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
 }
@@ -201,18 +209,29 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int acc = local & 1;
         unsigned char* stage = st16 + (C::DBUF ? (local & 1) * (128 * BN * 2) : 0);
         // this warp's stores of the tile that last used this staging buffer
-        // (local-2 double-buffered, local-1 otherwise) have read it
-        if (lane == 0) {
-          if (C::DBUF) bulk_wait_read1();
-          else bulk_wait_read0();
+        // (local-2 double-buffered, local-1 otherwise) have read it.  Single
+        // staging buffer with kBoxPipe: every box is its own bulk group and is
+        // waited for just before it is rewritten (the box stores of tile i
+        // drain while tile i+1's first boxes are staged)
+        if (!kBoxPipe || C::DBUF) {
+          if (lane == 0) {
+            if (C::DBUF) bulk_wait_read1();
+            else bulk_wait_read0();
+          }
+          __syncwarp();
         }
-        __syncwarp();
         sm100::mbar_wait(&tfull[acc], (local >> 1) & 1);
         sm100::tc_fence_after();
         const uint32_t t_row = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * BN);
         float v[16];
+        constexpr bool kPipe = kBoxPipe && !C::DBUF;
+        constexpr int kNB = BN / 64;  // this warp's 32-column boxes
 #pragma unroll 1
         for (int c = cbeg; c < cend; c += 16) {
+          if (kPipe && c % 32 == 0) {
+            if (lane == 0) bulk_wait_read_n<kNB - 1>();  // this box of the previous tile has been read
+            __syncwarp();
+          }
           sm100::tmem_ld16(t_row + c, v);
           const float4* b4 = reinterpret_cast<const float4*>(args.bias + n0 + c);
           float bb[16];
@@ -235,16 +254,26 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int ch = (c % 32) / 8;
           *reinterpret_cast<uint4*>(box + swz<64>(r, ch)) = make_uint4(p[0], p[1], p[2], p[3]);
           *reinterpret_cast<uint4*>(box + swz<64>(r, ch + 1)) = make_uint4(p[4], p[5], p[6], p[7]);
+          if (kPipe && c % 32 == 16) {  // box complete: store it as its own bulk group
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0) {
+              tma_store_2d(&maps.out16w, stage + (c / 32) * (128 * 64) + q * 32 * 64, n0 + c - 16, m0 + 32 * q);
+              bulk_commit();
+            }
+          }
         }
         sm100::tc_fence_before();
         mbar_arrive(&tempty[acc]);  // accumulator may be overwritten now
-        fence_proxy_async();         // staging writes -> visible to the TMA (async proxy)
-        __syncwarp();
-        if (lane == 0) {
-          // rows 32q.. of each of this warp's boxes: 32 rows x 64 B, contiguous
-          for (int c = cbeg; c < cend; c += 32)
-            tma_store_2d(&maps.out16w, stage + (c / 32) * (128 * 64) + q * 32 * 64, n0 + c, m0 + 32 * q);
-          bulk_commit();
+        if (!kPipe) {
+          fence_proxy_async();  // staging writes -> visible to the TMA (async proxy)
+          __syncwarp();
+          if (lane == 0) {
+            // rows 32q.. of each of this warp's boxes: 32 rows x 64 B, contiguous
+            for (int c = cbeg; c < cend; c += 32)
+              tma_store_2d(&maps.out16w, stage + (c / 32) * (128 * 64) + q * 32 * 64, n0 + c, m0 + 32 * q);
+            bulk_commit();
+          }
         }
       }
       if (lane == 0) bulk_wait0();
