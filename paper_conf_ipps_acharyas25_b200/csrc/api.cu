@@ -511,7 +511,9 @@ static predtop_status forward_impl(predtop_model m, predtop_dag dag, void* ws, s
     if ((s = attention_launch(dag, d, H, w.qkv, w.att, st)) != PREDTOP_OK) return s;
     if (use_fused_tail(d, f)) {
       ProfScope _p(PK_LAYER_TAIL, st);
-      s = layer_tail256_supported(d, f) ? layer_tail256_launch(m, l, w.att, w.x32, w.x16, M, st)
+      // after the last layer only the fp32 stream is read (readout, x_out):
+      // the d = 256 tail skips its fp16 shadow there
+      s = layer_tail256_supported(d, f) ? layer_tail256_launch(m, l, w.att, w.x32, l == last_layer ? nullptr : w.x16, M, st)
           : use_tail_v2(d, f)           ? layer_tail2_launch(m, l, w.att, w.x32, w.x16, M, st)
                                         : layer_tail_launch(m, l, w.att, w.x32, w.x16, M, st);
       if (s != PREDTOP_OK) return s;

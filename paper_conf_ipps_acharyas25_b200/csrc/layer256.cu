@@ -489,6 +489,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
       unsigned char* sw = sStg + ew * STGW;
 #pragma unroll
       for (int p = 0; p < 3; ++p) {
+        if (p == 2 && args.x16 == nullptr) break;  // last layer: no fp16 shadow
         if (p > 0) {
           if (lane == 0) sm100::bulk_wait_read0();
           __syncwarp();
@@ -565,7 +566,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         for (int rr = 0; rr < 2; ++rr) {
           const int rw = (lane >> 1) + 16 * rr, ch = lane & 1;
           const uint4 v = *reinterpret_cast<const uint4*>(s16 + rw * 32 + 16 * (ch ^ ((rw >> 2) & 1)));
-          if (m0 + 32 * q + rw < args.M)
+          if (m0 + 32 * q + rw < args.M && args.x16 != nullptr)
             *reinterpret_cast<uint4*>(args.x16 + (int64_t)(m0 + 32 * q + rw) * D + 64 * cg + 16 * k + 8 * ch) = v;
         }
         __syncwarp();
@@ -574,7 +575,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_layer_tail256(const __grid_cons
         __syncwarp();
         if (lane == 0) {
           sm100::tma_store_2d(&mp.x32out, s32, 64 * cg + 16 * k, m0 + 32 * q);
-          sm100::tma_store_2d(&mp.x16out, s16, 64 * cg + 16 * k, m0 + 32 * q);
+          if (args.x16 != nullptr) sm100::tma_store_2d(&mp.x16out, s16, 64 * cg + 16 * k, m0 + 32 * q);
           sm100::bulk_commit();
         }
 #endif
@@ -609,7 +610,8 @@ predtop_status layer_tail256_launch(const predtop_model_s* m, int l, const __hal
       !encode_tma_2d(&mp.wo, L.Wo, 2, D, D, 64, 256) || !encode_tma_2d(&mp.w1, L.W1, 2, D, dff, 64, FC) ||
       !encode_tma_2d(&mp.w2, L.W2, 2, dff, D, 64, 256) ||
       !encode_tma_2d(&mp.x32out, x32, 4, D, M, PREDTOP_L256_OUTW ? 32 : 16, 32) ||
-      !encode_tma_2d(&mp.x16out, x16, 2, D, M, PREDTOP_L256_OUTW ? 64 : 16, 32))
+      // x16 == nullptr (the last layer: nothing reads the fp16 shadow) skips its stores
+      !encode_tma_2d(&mp.x16out, x16 ? (const void*)x16 : (const void*)x32, 2, D, M, PREDTOP_L256_OUTW ? 64 : 16, 32))
     return PREDTOP_ERR_CUDA;
   T256Args a{M, dff, L.bo, L.g1, L.be1, L.b1, L.b2, L.g2, L.be2, m->cfg.ln_eps, x32, x16};
   PT_SMEM_ATTR(k_layer_tail256, SMEM);

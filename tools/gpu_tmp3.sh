@@ -1,1 +1,11 @@
-timeout 900 python -m pytest tests/test_gpu_dag.py tests/test_gpu_hops.py tests/test_gpu_prune.py tests/test_gpu_forward.py -m gpu -q -x --timeout 300 > gpurun_out/pt_dag.txt 2>&1; echo "rc=$?" >> gpurun_out/pt_dag.txt
+# A/B of the working tree (default) against HEAD (libpredtop_head.so): forward/moe tests on the default, MoE bench x2
+O=gpurun_out; mkdir -p $O
+timeout 600 python -m pytest tests -m gpu -q -x --timeout 200 -k "forward or moe or tap" > $O/pt_new.txt 2>&1; echo "pytest rc=$?"; tail -1 $O/pt_new.txt
+for i in 1 2; do
+for v in default head; do
+  if [ "$v" != default ]; then export PREDTOP_LIB=$PWD/paper_conf_ipps_acharyas25_b200/lib/libpredtop_$v.so; else unset PREDTOP_LIB; fi
+  timeout 240 python bench.py --config moe --no-cpu-baseline --no-also --steps 20 > $O/bench_$v.json 2>$O/bench_$v.err
+  python -c "
+import json; d=json.loads(open('$O/bench_$v.json').read().strip().splitlines()[-1]); print('$v', round(d['value']), {k: round(v['ms_per_step'],3) for k,v in d['kernels'].items() if v['ms_per_step']>1})" || tail -3 $O/bench_$v.err
+done
+done
