@@ -181,8 +181,17 @@ __global__ void __launch_bounds__(D) k_readout(const float* __restrict__ x32,
     return;
   }
   const int64_t n0 = node_ptr[g], n1 = node_ptr[g + 1];
-  float s = 0.f;
-  for (int64_t v = n0; v < n1; ++v) s += x32[v * D + c];  // Eqn 2, node order
+  // Eqn 2: eight interleaved partial sums (node v into partial (v - n0) % 8,
+  // combined pairwise in a fixed order: deterministic, and eight independent
+  // row loads in flight per thread instead of one dependent add chain)
+  float ps[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  int64_t v = n0;
+  for (; v + 8 <= n1; v += 8) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) ps[k] += __ldg(x32 + (v + k) * D + c);
+  }
+  for (int k = 0; v < n1; ++v, ++k) ps[k] += __ldg(x32 + v * D + c);
+  float s = ((ps[0] + ps[1]) + (ps[2] + ps[3])) + ((ps[4] + ps[5]) + (ps[6] + ps[7]));
   if (pool_mean) s /= (float)(n1 - n0);
   sg[c] = s;
   __syncthreads();
